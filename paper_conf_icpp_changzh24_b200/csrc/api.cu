@@ -1,0 +1,812 @@
+// api.cu -- the C-ABI (include/gsap.h): context management, argument
+// marshalling, and the thin host driver of SBP (P:137-141 3 Fig. 2): merge ->
+// batched MCMC (Table 2) -> golden-section search over B (P:34 1,
+// P:328 4.3; readings Z19-Z21), which stays on the host as in the paper.
+#include <math.h>
+#include <string.h>
+
+#include <algorithm>
+#include <chrono>
+#include <new>
+#include <vector>
+
+#include "internal.h"
+
+struct gsap_ctx {
+    gsap::Ctx c;
+};
+
+using namespace gsap;
+
+static thread_local std::string g_err;
+
+#define API_TRY try {
+#define API_CATCH                                      \
+    }                                                  \
+    catch (const Error &e) {                           \
+        g_err = e.msg;                                 \
+        return e.code;                                 \
+    }                                                  \
+    catch (const std::bad_alloc &) {                   \
+        g_err = "host allocation failed";              \
+        return GSAP_ENOMEM;                            \
+    }                                                  \
+    catch (const std::exception &e) {                  \
+        g_err = e.what();                              \
+        return GSAP_EINVAL;                            \
+    }                                                  \
+    catch (...) {                                      \
+        g_err = "unknown error";                       \
+        return GSAP_EINVAL;                            \
+    }                                                  \
+    return GSAP_OK;
+
+#define REQUIRE(cond, code, msg)          \
+    do {                                  \
+        if (!(cond)) throw Error{code, msg}; \
+    } while (0)
+
+namespace gsap {
+
+// ------------------------------------------------------- event timing --
+static cudaEvent_t ev_get(KClass &k) {
+    if (!k.pool.empty()) {
+        cudaEvent_t e = k.pool.back();
+        k.pool.pop_back();
+        return e;
+    }
+    cudaEvent_t e;
+    GSAP_CUDA(cudaEventCreate(&e));
+    return e;
+}
+
+void kc_begin(Ctx &c, KClass &k, cudaEvent_t *ev) {
+    *ev = nullptr;
+    if (!c.prm.profile) return;
+    *ev = ev_get(k);
+    GSAP_CUDA(cudaEventRecord(*ev, c.stream));
+}
+
+void kc_end(Ctx &c, KClass &k, cudaEvent_t ev, double bytes) {
+    k.launches += 1;
+    k.bytes += bytes;
+    if (!ev) return;
+    cudaEvent_t e2 = ev_get(k);
+    GSAP_CUDA(cudaEventRecord(e2, c.stream));
+    k.pending.emplace_back(ev, e2);
+    if (k.pending.size() > 4096) kc_resolve(c, k);
+}
+
+void kc_resolve(Ctx &c, KClass &k) {
+    (void)c;
+    for (auto &p : k.pending) {
+        GSAP_CUDA(cudaEventSynchronize(p.second));
+        float ms = 0.f;
+        GSAP_CUDA(cudaEventElapsedTime(&ms, p.first, p.second));
+        k.ms += ms;
+        k.pool.push_back(p.first);
+        k.pool.push_back(p.second);
+    }
+    k.pending.clear();
+}
+
+}  // namespace gsap
+
+template <typename T>
+static T *dalloc(size_t n) {
+    void *p = nullptr;
+    const cudaError_t e = cudaMalloc(&p, std::max<size_t>(n, 1) * sizeof(T));
+    if (e == cudaErrorMemoryAllocation) {
+        cudaGetLastError();
+        throw Error{GSAP_ENOMEM, "cudaMalloc failed"};
+    }
+    GSAP_CUDA(e);
+    return static_cast<T *>(p);
+}
+
+static bool is_dev(const void *p) {
+    if (!p) return false;
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// dst: host or device; src: device
+static void copy_out(Ctx &c, void *dst, const void *src, size_t bytes) {
+    if (!dst || !bytes) return;
+    GSAP_CUDA(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDefault, c.stream));
+    if (!is_dev(dst)) GSAP_CUDA(cudaStreamSynchronize(c.stream));
+}
+
+// src: host or device -> a device pointer (src itself, or staged into `scratch`)
+template <typename T>
+static const T *stage_in(Ctx &c, const T *src, size_t n, T *scratch) {
+    if (!src || is_dev(src)) return src;
+    if (n) GSAP_CUDA(cudaMemcpyAsync(scratch, src, n * sizeof(T), cudaMemcpyHostToDevice, c.stream));
+    return scratch;
+}
+
+template <typename T>
+static std::vector<T> to_host(const T *src, size_t n) {
+    std::vector<T> h(n);
+    if (n) GSAP_CUDA(cudaMemcpy(h.data(), src, n * sizeof(T), cudaMemcpyDefault));
+    return h;
+}
+
+static void check_sm100() {
+    int dev = 0;
+    GSAP_CUDA(cudaGetDevice(&dev));
+    cudaDeviceProp p;
+    GSAP_CUDA(cudaGetDeviceProperties(&p, dev));
+    REQUIRE(p.major == 10, GSAP_EUNSUPPORTED, "libgsap is built for sm_100a (B200) only");
+}
+
+static void free_ctx(Ctx &c) {
+    void *ptrs[] = {c.rowptr, c.col, c.wgt, c.cscptr, c.cscsrc, c.cscwgt, c.esrc, c.kout, c.kin, c.selfw,
+                    c.big, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
+                    c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT, c.keys0,
+                    c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
+                    c.rowid, c.counts, c.scan_tmp, c.rownnz, c.s, c.dS, c.H, c.acc, c.best, c.dSbest,
+                    c.partials, c.scal, c.scal_i, c.Dh, c.skey0, c.skey1, c.sval0, c.sval1, c.rank,
+                    c.nxt0, c.nxt1, c.mx0, c.mx1, c.oncyc, c.label, c.present, c.slot_b[0], c.slot_b[1],
+                    c.slot_b[2]};
+    for (void *p : ptrs)
+        if (p) cudaFree(p);
+    if (c.h_scal) cudaFreeHost(c.h_scal);
+    if (c.h_int) cudaFreeHost(c.h_int);
+    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl}) {
+        for (auto &p : k->pending) {
+            cudaEventDestroy(p.first);
+            cudaEventDestroy(p.second);
+        }
+        for (auto e : k->pool) cudaEventDestroy(e);
+    }
+    if (c.own_stream && c.stream) cudaStreamDestroy(c.stream);
+}
+
+static int log2_ceil_h(long long x) {
+    int l = 0;
+    while ((1LL << l) < x) ++l;
+    return l;
+}
+
+// ----------------------------------------------------------- create ----
+static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t *col, const int32_t *wgt,
+                        const gsap_params *params, const gsap_dist *dist, void *stream) {
+    REQUIRE(V >= 1, GSAP_EINVAL, "V must be >= 1");
+    REQUIRE(rowptr && (col || true), GSAP_EINVAL, "rowptr is NULL");
+    REQUIRE(!dist || dist->nranks <= 1, GSAP_EUNSUPPORTED,
+            "multi-GPU contexts are not built in this version (use one context per GPU)");
+    check_sm100();
+    if (params) c.prm = *params;
+    else gsap_default_params(&c.prm);
+    REQUIRE(c.prm.num_batches >= 1 && c.prm.max_nodal_itr >= 1 && c.prm.window >= 1, GSAP_EINVAL,
+            "num_batches, max_nodal_itr and window must be >= 1");
+    REQUIRE(c.prm.num_proposals >= 1 && c.prm.num_proposals <= 32, GSAP_EINVAL, "num_proposals in [1, 32]");
+    // stage + validate the CSR on the host
+    std::vector<int64_t> rp = to_host(rowptr, (size_t)V + 1);
+    REQUIRE(rp[0] == 0, GSAP_EINVAL, "rowptr[0] must be 0");
+    for (int v = 0; v < V; ++v) REQUIRE(rp[v + 1] >= rp[v], GSAP_EINVAL, "rowptr must be non-decreasing");
+    const int64_t E64 = rp[V];
+    REQUIRE(E64 < (1LL << 30), GSAP_EUNSUPPORTED, "more than 2^30 edges");
+    REQUIRE(E64 == 0 || col, GSAP_EINVAL, "col is NULL");
+    const int E = (int)E64;
+    std::vector<int32_t> hc = to_host(col, (size_t)E);
+    std::vector<int32_t> hw;
+    long long W = 0;
+    for (int e = 0; e < E; ++e) REQUIRE(hc[e] >= 0 && hc[e] < V, GSAP_EINVAL, "col out of range");
+    if (wgt) {
+        hw = to_host(wgt, (size_t)E);
+        for (int e = 0; e < E; ++e) {
+            REQUIRE(hw[e] >= 1, GSAP_EINVAL, "weights must be >= 1");
+            W += hw[e];
+        }
+    } else {
+        W = E;
+    }
+    REQUIRE(W < (1LL << 30), GSAP_EUNSUPPORTED, "total edge weight must be < 2^30");
+    c.V = V;
+    c.E = E;
+    c.W = W;
+    c.weighted = wgt != nullptr;
+    if (stream) {
+        c.stream = (cudaStream_t)stream;
+    } else {
+        GSAP_CUDA(cudaStreamCreateWithFlags(&c.stream, cudaStreamNonBlocking));
+        c.own_stream = true;
+    }
+    GSAP_CUDA(cudaGetDevice(&c.dev));
+    // host-side static info
+    c.h_rowptr.resize((size_t)V + 1);
+    for (int v = 0; v <= V; ++v) c.h_rowptr[v] = (int)rp[v];
+    c.h_cscptr.assign((size_t)V + 1, 0);
+    for (int e = 0; e < E; ++e) c.h_cscptr[hc[e] + 1]++;
+    for (int v = 0; v < V; ++v) c.h_cscptr[v + 1] += c.h_cscptr[v];
+    int kmax_big = 0;
+    for (int v = 0; v < V; ++v) {
+        const int k = (c.h_rowptr[v + 1] - c.h_rowptr[v]) + (c.h_cscptr[v + 1] - c.h_cscptr[v]);
+        if (k > 128) {
+            c.h_big.push_back(v);
+            kmax_big = std::max(kmax_big, k);
+        }
+    }
+    // allocation ---------------------------------------------------------
+    const size_t Vs = (size_t)V, Es = (size_t)std::max(E, 1);
+    const size_t VE = std::max(Vs, Es) + 1;
+    const int P = c.prm.num_proposals;
+    c.rowptr = dalloc<int>(Vs + 1);
+    c.col = dalloc<int>(Es);
+    if (c.weighted) {
+        c.wgt = dalloc<int>(Es);
+        c.cscwgt = dalloc<int>(Es);
+    }
+    c.cscptr = dalloc<int>(Vs + 1);
+    c.cscsrc = dalloc<int>(Es);
+    c.esrc = dalloc<int>(Es);
+    c.kout = dalloc<int>(Vs);
+    c.kin = dalloc<int>(Vs);
+    c.selfw = dalloc<int>(Vs);
+    if (!c.h_big.empty()) {
+        c.big = dalloc<int>(c.h_big.size());
+        const int log2cap = std::max(log2_ceil_h(2LL * std::min(kmax_big, V)), 5);
+        if ((1 << log2cap) > 4096) {
+            c.big_table_slots = (size_t)296 << log2cap;
+            c.big_tables = dalloc<int>(c.big_table_slots * 4);
+        }
+    }
+    c.b = dalloc<int>(Vs);
+    c.bm_rowptr = dalloc<int>(Vs + 1);
+    c.bm_colptr = dalloc<int>(Vs + 1);
+    c.bm_col = dalloc<int>(Es);
+    c.bm_cnt = dalloc<int>(Es);
+    c.bm_cum = dalloc<int>(Es);
+    c.bm_row = dalloc<int>(Es);
+    c.bm_ccnt = dalloc<int>(Es);
+    c.bm_ccum = dalloc<int>(Es);
+    c.dout = dalloc<int>(Vs);
+    c.din = dalloc<int>(Vs);
+    c.d_nnz = dalloc<int>(1);
+    c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, 65536), (size_t)1 << 28);
+    c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
+    c.dense = dalloc<int>(c.dense_cap);
+    c.denseT = dalloc<int>(c.dense_cap);
+    c.keys0 = dalloc<unsigned long long>(Es);
+    c.keys1 = dalloc<unsigned long long>(Es);
+    c.vals64a = dalloc<unsigned long long>(Es);
+    c.vals64b = dalloc<unsigned long long>(Es);
+    c.ukeys0 = dalloc<unsigned>(Es);
+    c.ukeys1 = dalloc<unsigned>(Es);
+    c.wa = dalloc<int>(VE);
+    c.wb = dalloc<int>(VE);
+    c.flags = dalloc<int>(VE);
+    c.pos = dalloc<int>(VE);
+    c.tmpi = dalloc<int>(VE);
+    c.rowid = dalloc<int>(VE);
+    c.rownnz = dalloc<int>(Vs + 1);
+    const size_t tiles = (VE + 4095) / 4096 + 1;
+    c.counts_cap = 256 * tiles;
+    c.counts = dalloc<int>(c.counts_cap);
+    c.scan_tmp_cap = std::max(c.counts_cap, VE) / 4096 + 16;
+    c.scan_tmp = dalloc<int>(c.scan_tmp_cap);
+    c.s = dalloc<int>(Vs * (size_t)P);
+    c.dS = dalloc<double>(Vs * (size_t)P);
+    c.H = dalloc<double>(Vs);
+    c.acc = dalloc<unsigned char>(Vs);
+    c.best = dalloc<int>(Vs);
+    c.dSbest = dalloc<double>(Vs);
+    c.partials = dalloc<double>(VE / 4096 + 64);
+    c.scal = dalloc<double>(8);
+    c.scal_i = dalloc<int>(8);
+    c.Dh = dalloc<double>((size_t)c.prm.max_nodal_itr + 1);
+    c.skey0 = dalloc<unsigned long long>(Vs);
+    c.skey1 = dalloc<unsigned long long>(Vs);
+    c.sval0 = dalloc<int>(Vs);
+    c.sval1 = dalloc<int>(Vs);
+    c.rank = dalloc<int>(Vs);
+    c.nxt0 = dalloc<int>(Vs);
+    c.nxt1 = dalloc<int>(Vs);
+    c.mx0 = dalloc<int>(Vs);
+    c.mx1 = dalloc<int>(Vs);
+    c.oncyc = dalloc<int>(Vs);
+    c.label = dalloc<int>(Vs);
+    c.present = dalloc<int>(Vs + 1);
+    GSAP_CUDA(cudaMallocHost(&c.h_scal, 8 * sizeof(double)));
+    GSAP_CUDA(cudaMallocHost(&c.h_int, 8 * sizeof(int)));
+    // upload ---------------------------------------------------------------
+    GSAP_CUDA(cudaMemcpyAsync(c.rowptr, c.h_rowptr.data(), sizeof(int) * (Vs + 1), cudaMemcpyHostToDevice, c.stream));
+    if (E) GSAP_CUDA(cudaMemcpyAsync(c.col, hc.data(), sizeof(int) * (size_t)E, cudaMemcpyHostToDevice, c.stream));
+    if (c.weighted && E)
+        GSAP_CUDA(cudaMemcpyAsync(c.wgt, hw.data(), sizeof(int) * (size_t)E, cudaMemcpyHostToDevice, c.stream));
+    if (!c.h_big.empty())
+        GSAP_CUDA(cudaMemcpyAsync(c.big, c.h_big.data(), sizeof(int) * c.h_big.size(), cudaMemcpyHostToDevice,
+                                  c.stream));
+    GSAP_CUDA(cudaMemsetAsync(c.scal, 0, 8 * sizeof(double), c.stream));
+    GSAP_CUDA(cudaMemsetAsync(c.scal_i, 0, 8 * sizeof(int), c.stream));
+    build_graph_device(c);
+    // the singleton partition (P:61 2.1)
+    std::vector<int> iota(Vs);
+    for (int v = 0; v < V; ++v) iota[v] = v;
+    GSAP_CUDA(cudaMemcpyAsync(c.b, iota.data(), sizeof(int) * Vs, cudaMemcpyHostToDevice, c.stream));
+    c.B = V;
+    rebuild(c);
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+}
+
+// ------------------------------------------------------------- driver --
+static void set_iota(Ctx &c) {
+    std::vector<int> iota((size_t)c.V);
+    for (int v = 0; v < c.V; ++v) iota[v] = v;
+    GSAP_CUDA(cudaMemcpyAsync(c.b, iota.data(), sizeof(int) * (size_t)c.V, cudaMemcpyHostToDevice, c.stream));
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    c.B = c.V;
+}
+
+static double mdl_now(Ctx &c) {
+    return model_term(c.W, c.V, c.B, c.prm.model_term) + device_data_term(c);
+}
+
+static void merge_phase(Ctx &c, uint32_t outer, int K, int *best_out, double *dSbest_out) {
+    REQUIRE(c.B >= 2, GSAP_ESTATE, "a merge phase needs B >= 2");
+    REQUIRE(K >= 0 && K <= c.B / 2, GSAP_EINVAL, "K must be in [0, B/2]");
+    const int B = c.B;
+    launch_merge_props(c, outer, 0, B, true, nullptr, nullptr, c.best, c.dSbest);
+    copy_out(c, best_out, c.best, sizeof(int) * (size_t)B);
+    copy_out(c, dSbest_out, c.dSbest, sizeof(double) * (size_t)B);
+    select_merges(c, c.best, c.dSbest, K, nullptr);
+    rebuild(c);
+    c.st.n_merge_prop += (long long)B * c.prm.num_proposals;
+}
+
+static void move_batch(Ctx &c, uint32_t outer, uint32_t itr, int first, int count, double *dsum) {
+    launch_move(c, MOVE_FUSED, outer, itr, first, count, c.s, c.dS, nullptr, c.acc);
+    launch_apply(c, first, count, c.s, c.acc, c.dS, dsum, c.scal_i + 1);
+    rebuild(c);
+    c.st.n_move_prop += count;
+}
+
+// returns the number of MCMC iterations run (O.8)
+static int mcmc_phase(Ctx &c, uint32_t outer, double thresh) {
+    const int V = c.V, nb = c.prm.num_batches, w = c.prm.window;
+    const int bs = (V + nb - 1) / nb;
+    std::vector<double> D((size_t)c.prm.max_nodal_itr + 1, 0.0);
+    int ran = 0;
+    for (int itr = 0; itr < c.prm.max_nodal_itr; ++itr) {
+        GSAP_CUDA(cudaMemsetAsync(c.Dh + itr, 0, sizeof(double), c.stream));
+        for (int k = 0; k < nb; ++k) {
+            const int first = k * bs, last = std::min(V, first + bs);
+            if (first >= last) continue;
+            move_batch(c, outer, (uint32_t)itr, first, last - first, c.Dh + itr);
+        }
+        ran = itr + 1;
+        if (itr >= w - 1) {
+            launch_data_term(c);
+            GSAP_CUDA(cudaMemcpyAsync(c.h_scal + 1, c.scal + 1, sizeof(double), cudaMemcpyDeviceToHost, c.stream));
+            GSAP_CUDA(cudaMemcpyAsync(D.data(), c.Dh, sizeof(double) * (size_t)(itr + 1), cudaMemcpyDeviceToHost,
+                                      c.stream));
+            GSAP_CUDA(cudaStreamSynchronize(c.stream));
+            const double mdl = model_term(c.W, c.V, c.B, c.prm.model_term) + c.h_scal[1];
+            double sum = 0.0;
+            int n = 0;
+            for (int j = itr - w + 1; j < itr; ++j) {
+                sum += D[j];
+                ++n;
+            }
+            const double mean = n ? sum / n : 0.0;
+            if (-mean < thresh * mdl) break;
+        }
+    }
+    return ran;
+}
+
+namespace {
+// golden-section bracket over (b, B, MDL), slot 1 = best (GraphChallenge's
+// prepare_for_partition_on_next_num_blocks; R:Z21).  Returns true when done.
+struct Bracket {
+    int B[3] = {0, 0, 0};
+    double S[3] = {INFINITY, INFINITY, INFINITY};
+};
+
+bool bracket_update(Ctx &c, Bracket &br, int B, double S, int *K, int *restart) {
+    auto copy_slot = [&](int dst, const int *src) {
+        GSAP_CUDA(cudaMemcpyAsync(c.slot_b[dst], src, sizeof(int) * (size_t)c.V, cudaMemcpyDeviceToDevice,
+                                  c.stream));
+    };
+    int idx;
+    if (S <= br.S[1]) {
+        idx = br.B[1] > B ? 0 : 2;
+        copy_slot(idx, c.slot_b[1]);
+        br.B[idx] = br.B[1];
+        br.S[idx] = br.S[1];
+        idx = 1;
+    } else {
+        idx = br.B[1] > B ? 2 : 0;
+    }
+    copy_slot(idx, c.b);
+    br.B[idx] = B;
+    br.S[idx] = S;
+    if (br.S[2] == INFINITY) {
+        *K = (int)((double)B * c.prm.reduction_rate);
+        *restart = 1;
+        return *K == 0;
+    }
+    if (br.B[0] - br.B[2] == 2) return true;
+    const int i = (br.B[0] - br.B[1]) >= (br.B[1] - br.B[2]) ? 0 : 1;
+    const int next = br.B[i + 1] + (int)nearbyint((double)(br.B[i] - br.B[i + 1]) * 0.618);
+    *K = br.B[i] - next;
+    *restart = i;
+    return *K <= 0;
+}
+}  // namespace
+
+static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out, double *trace, int trace_cap,
+                     int32_t *rounds_out) {
+    const auto t0 = std::chrono::steady_clock::now();
+    for (int i = 0; i < 3; ++i)
+        if (!c.slot_b[i]) c.slot_b[i] = dalloc<int>((size_t)c.V);
+    GSAP_CUDA(cudaMemsetAsync(c.scal_i + 1, 0, sizeof(int), c.stream));
+    set_iota(c);
+    rebuild(c);
+    Bracket br;
+    int K = (int)((double)c.B * c.prm.reduction_rate);
+    uint32_t outer = 0;
+    int rounds = 0;
+    bool done = false;
+    if (K == 0) {
+        br.S[1] = mdl_now(c);
+        br.B[1] = c.B;
+        GSAP_CUDA(cudaMemcpyAsync(c.slot_b[1], c.b, sizeof(int) * (size_t)c.V, cudaMemcpyDeviceToDevice, c.stream));
+        done = true;
+    }
+    double t_merge = 0, t_move = 0, t_mdl = 0;
+    while (!done && rounds < c.prm.max_rounds) {
+        const bool bracket = br.S[2] != INFINITY;
+        auto ta = std::chrono::steady_clock::now();
+        merge_phase(c, outer, K, nullptr, nullptr);
+        const int B = c.B;
+        auto tb = std::chrono::steady_clock::now();
+        const int itrs = mcmc_phase(c, outer, bracket ? c.prm.thresh2 : c.prm.thresh1);
+        auto tc = std::chrono::steady_clock::now();
+        const double S = mdl_now(c);
+        auto td = std::chrono::steady_clock::now();
+        t_merge += std::chrono::duration<double>(tb - ta).count();
+        t_move += std::chrono::duration<double>(tc - tb).count();
+        t_mdl += std::chrono::duration<double>(td - tc).count();
+        if (trace && rounds < trace_cap) {
+            trace[4 * rounds + 0] = (double)outer;
+            trace[4 * rounds + 1] = (double)B;
+            trace[4 * rounds + 2] = (double)itrs;
+            trace[4 * rounds + 3] = S;
+        }
+        c.st.mcmc_itr_total += itrs;
+        ++rounds;
+        int restart = 1;
+        if (bracket_update(c, br, B, S, &K, &restart)) break;
+        GSAP_CUDA(cudaMemcpyAsync(c.b, c.slot_b[restart], sizeof(int) * (size_t)c.V, cudaMemcpyDeviceToDevice,
+                                  c.stream));
+        c.B = br.B[restart];
+        rebuild(c);
+        ++outer;
+    }
+    // the answer: slot 1
+    GSAP_CUDA(cudaMemcpyAsync(c.b, c.slot_b[1], sizeof(int) * (size_t)c.V, cudaMemcpyDeviceToDevice, c.stream));
+    c.B = br.B[1];
+    rebuild(c);
+    copy_out(c, bmap_out, c.b, sizeof(int) * (size_t)c.V);
+    GSAP_CUDA(cudaMemcpyAsync(c.h_int + 1, c.scal_i + 1, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    c.st.n_move_acc += c.h_int[1];
+    if (B_out) *B_out = c.B;
+    if (mdl_out) *mdl_out = br.S[1];
+    if (rounds_out) *rounds_out = rounds;
+    c.st.rounds += rounds;
+    c.st.B_final = c.B;
+    c.st.t_merge += t_merge;
+    c.st.t_move += t_move;
+    c.st.t_mdl += t_mdl;
+    c.st.t_total += std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+}
+
+static void fill_stats(Ctx &c, gsap_stats *out) {
+    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl}) kc_resolve(c, *k);
+    gsap_stats s = c.st;
+    s.gpu_launches = c.launches;
+    s.k_move_ms = c.k_move.ms;
+    s.k_move_bytes = c.k_move.bytes;
+    s.k_move_launches = c.k_move.launches;
+    s.k_rebuild_ms = c.k_rebuild.ms;
+    s.k_rebuild_bytes = c.k_rebuild.bytes;
+    s.k_rebuild_launches = c.k_rebuild.launches;
+    s.k_merge_ms = c.k_merge.ms;
+    s.k_merge_bytes = c.k_merge.bytes;
+    s.k_merge_launches = c.k_merge.launches;
+    s.k_mdl_ms = c.k_mdl.ms;
+    s.k_mdl_launches = c.k_mdl.launches;
+    *out = s;
+}
+
+// ================================================================ C-ABI ===
+extern "C" {
+
+void gsap_default_params(gsap_params *p) {
+    if (!p) return;
+    memset(p, 0, sizeof(*p));
+    p->seed = 0x5B9D2024ULL;
+    p->beta = 3.0;
+    p->reduction_rate = 0.4;
+    p->num_proposals = 10;
+    p->max_nodal_itr = 100;
+    p->thresh1 = 5e-4;
+    p->thresh2 = 1e-4;
+    p->window = 3;
+    p->num_batches = 4;
+    p->model_term = 0;
+    p->max_rounds = 500;
+    p->profile = 0;
+}
+
+const char *gsap_last_error(void) { return g_err.c_str(); }
+
+gsap_status gsap_create(int32_t V, const int64_t *rowptr, const int32_t *col, const int32_t *wgt,
+                        const gsap_params *params, const gsap_dist *dist, void *stream, gsap_ctx **out) {
+    API_TRY
+    REQUIRE(out, GSAP_EINVAL, "out is NULL");
+    *out = nullptr;
+    gsap_ctx *h = new gsap_ctx();
+    try {
+        create_impl(h->c, V, rowptr, col, wgt, params, dist, stream);
+    } catch (...) {
+        free_ctx(h->c);
+        delete h;
+        throw;
+    }
+    *out = h;
+    API_CATCH
+}
+
+void gsap_destroy(gsap_ctx *ctx) {
+    if (!ctx) return;
+    if (ctx->c.stream) cudaStreamSynchronize(ctx->c.stream);
+    free_ctx(ctx->c);
+    delete ctx;
+}
+
+gsap_status gsap_set_partition(gsap_ctx *ctx, const int32_t *b, int32_t B) {
+    API_TRY
+    REQUIRE(ctx && b, GSAP_EINVAL, "NULL argument");
+    Ctx &c = ctx->c;
+    REQUIRE(B >= 1 && B <= c.V, GSAP_EINVAL, "B must be in [1, V]");
+    if (!is_dev(b)) {
+        for (int v = 0; v < c.V; ++v) REQUIRE(b[v] >= 0 && b[v] < B, GSAP_EINVAL, "b[v] out of [0, B)");
+    }
+    GSAP_CUDA(cudaMemcpyAsync(c.b, b, sizeof(int) * (size_t)c.V, cudaMemcpyDefault, c.stream));
+    c.B = B;
+    rebuild(c);
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    API_CATCH
+}
+
+gsap_status gsap_get_partition(gsap_ctx *ctx, int32_t *b_out, int32_t *B_out) {
+    API_TRY
+    REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
+    copy_out(ctx->c, b_out, ctx->c.b, sizeof(int) * (size_t)ctx->c.V);
+    if (B_out) *B_out = ctx->c.B;
+    API_CATCH
+}
+
+gsap_status gsap_update_blockmodel(gsap_ctx *ctx) {
+    API_TRY
+    REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
+    rebuild(ctx->c);
+    API_CATCH
+}
+
+gsap_status gsap_propose(gsap_ctx *ctx, gsap_phase phase, uint32_t outer, uint32_t itr, int32_t first,
+                         int32_t count, int32_t *s_out) {
+    API_TRY
+    REQUIRE(ctx && s_out, GSAP_EINVAL, "NULL argument");
+    Ctx &c = ctx->c;
+    const int n = phase == GSAP_MOVE ? c.V : c.B;
+    REQUIRE(first >= 0 && count >= 0 && (long long)first + count <= n, GSAP_EINVAL, "range out of bounds");
+    if (count == 0) return GSAP_OK;
+    if (phase == GSAP_MOVE) {
+        launch_move(c, MOVE_PROPOSE, outer, itr, first, count, c.s, nullptr, nullptr, nullptr);
+        copy_out(c, s_out, c.s, sizeof(int) * (size_t)count);
+    } else {
+        REQUIRE(c.B >= 2, GSAP_ESTATE, "merge proposals need B >= 2");
+        launch_merge_props(c, outer, first, count, true, c.s, nullptr, nullptr, nullptr);
+        copy_out(c, s_out, c.s, sizeof(int) * (size_t)count * c.prm.num_proposals);
+    }
+    API_CATCH
+}
+
+gsap_status gsap_delta_mdl(gsap_ctx *ctx, gsap_phase phase, uint32_t outer, uint32_t itr, int32_t first,
+                           int32_t count, const int32_t *s, double *dS_out, double *H_out, uint8_t *acc_out) {
+    API_TRY
+    REQUIRE(ctx && s, GSAP_EINVAL, "NULL argument");
+    Ctx &c = ctx->c;
+    const int n = phase == GSAP_MOVE ? c.V : c.B;
+    REQUIRE(first >= 0 && count >= 0 && (long long)first + count <= n, GSAP_EINVAL, "range out of bounds");
+    if (count == 0) return GSAP_OK;
+    if (phase == GSAP_MOVE) {
+        const int *ds = stage_in(c, s, (size_t)count, c.s);
+        launch_move(c, MOVE_DELTA, outer, itr, first, count, const_cast<int *>(ds), c.dS, c.H, c.acc);
+        copy_out(c, dS_out, c.dS, sizeof(double) * (size_t)count);
+        copy_out(c, H_out, c.H, sizeof(double) * (size_t)count);
+        copy_out(c, acc_out, c.acc, (size_t)count);
+    } else {
+        REQUIRE(c.B >= 2, GSAP_ESTATE, "merge proposals need B >= 2");
+        const size_t np = (size_t)count * c.prm.num_proposals;
+        const int *ds = stage_in(c, s, np, c.s);
+        launch_merge_props(c, outer, first, count, false, const_cast<int *>(ds), c.dS, nullptr, nullptr);
+        copy_out(c, dS_out, c.dS, sizeof(double) * np);
+    }
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    API_CATCH
+}
+
+gsap_status gsap_select_merges(gsap_ctx *ctx, const int32_t *best, const double *dS, int32_t K,
+                               int32_t *label_out, int32_t *newB_out) {
+    API_TRY
+    REQUIRE(ctx && best && dS, GSAP_EINVAL, "NULL argument");
+    Ctx &c = ctx->c;
+    REQUIRE(c.B >= 2, GSAP_ESTATE, "selection needs B >= 2");
+    REQUIRE(K >= 0 && K <= c.B / 2, GSAP_EINVAL, "K must be in [0, B/2]");
+    const int B = c.B;
+    if (!is_dev(best))
+        for (int r = 0; r < B; ++r)
+            REQUIRE(best[r] >= 0 && best[r] < B && best[r] != r, GSAP_EINVAL, "best[r] must be in [0,B), != r");
+    const int *db = stage_in(c, best, (size_t)B, c.best);
+    const double *dd = stage_in(c, dS, (size_t)B, c.dSbest);
+    select_merges(c, db, dd, K, nullptr);
+    copy_out(c, label_out, c.label, sizeof(int) * (size_t)B);
+    rebuild(c);
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    if (newB_out) *newB_out = c.B;
+    API_CATCH
+}
+
+gsap_status gsap_apply_moves(gsap_ctx *ctx, int32_t first, int32_t count, const int32_t *s, const uint8_t *acc) {
+    API_TRY
+    REQUIRE(ctx && s && acc, GSAP_EINVAL, "NULL argument");
+    Ctx &c = ctx->c;
+    REQUIRE(first >= 0 && count >= 0 && (long long)first + count <= c.V, GSAP_EINVAL, "range out of bounds");
+    if (!is_dev(s))
+        for (int i = 0; i < count; ++i)
+            REQUIRE(!acc[i] || (s[i] >= 0 && s[i] < c.B), GSAP_EINVAL, "s out of [0, B)");
+    const int *ds = stage_in(c, s, (size_t)count, c.s);
+    const unsigned char *da = stage_in(c, (const unsigned char *)acc, (size_t)count, c.acc);
+    launch_apply(c, first, count, ds, da, nullptr, c.scal, nullptr);
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    API_CATCH
+}
+
+gsap_status gsap_move_batch(gsap_ctx *ctx, uint32_t outer, uint32_t itr, int32_t first, int32_t count,
+                            int32_t *s_out, double *dS_out, uint8_t *acc_out, double *dsum_out) {
+    API_TRY
+    REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
+    Ctx &c = ctx->c;
+    REQUIRE(first >= 0 && count >= 0 && (long long)first + count <= c.V, GSAP_EINVAL, "range out of bounds");
+    GSAP_CUDA(cudaMemsetAsync(c.scal, 0, sizeof(double), c.stream));
+    move_batch(c, outer, itr, first, count, c.scal);
+    copy_out(c, s_out, c.s, sizeof(int) * (size_t)count);
+    copy_out(c, dS_out, c.dS, sizeof(double) * (size_t)count);
+    copy_out(c, acc_out, c.acc, (size_t)count);
+    if (dsum_out) {
+        GSAP_CUDA(cudaMemcpyAsync(c.h_scal, c.scal, sizeof(double), cudaMemcpyDeviceToHost, c.stream));
+        GSAP_CUDA(cudaStreamSynchronize(c.stream));
+        *dsum_out = c.h_scal[0];
+    }
+    API_CATCH
+}
+
+gsap_status gsap_merge_phase(gsap_ctx *ctx, uint32_t outer, int32_t K, int32_t *best_out, double *dSbest_out) {
+    API_TRY
+    REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
+    merge_phase(ctx->c, outer, K, best_out, dSbest_out);
+    GSAP_CUDA(cudaStreamSynchronize(ctx->c.stream));
+    API_CATCH
+}
+
+gsap_status gsap_mdl(gsap_ctx *ctx, double *mdl_out, double *data_term_out) {
+    API_TRY
+    REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
+    Ctx &c = ctx->c;
+    const double S = device_data_term(c);
+    if (data_term_out) *data_term_out = S;
+    if (mdl_out) *mdl_out = model_term(c.W, c.V, c.B, c.prm.model_term) + S;
+    API_CATCH
+}
+
+gsap_status gsap_get_blockmodel(gsap_ctx *ctx, int64_t *nnz_io, int64_t *rowptr, int32_t *col, int32_t *cnt,
+                                int32_t *cum, int64_t *colptr, int32_t *row, int32_t *ccnt, int32_t *ccum,
+                                int32_t *dout, int32_t *din) {
+    API_TRY
+    REQUIRE(ctx && nnz_io, GSAP_EINVAL, "NULL argument");
+    Ctx &c = ctx->c;
+    GSAP_CUDA(cudaMemcpyAsync(c.h_int, c.d_nnz, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    const int64_t nnz = c.h_int[0];
+    const bool any = col || cnt || cum || row || ccnt || ccum;
+    REQUIRE(!any || *nnz_io >= nnz, GSAP_EINVAL, "entry arrays too small (see *nnz_io)");
+    *nnz_io = nnz;
+    const size_t B = (size_t)c.B;
+    auto widen = [&](int64_t *dst, const int *src) {
+        if (!dst) return;
+        std::vector<int> h = to_host(src, B + 1);
+        std::vector<int64_t> w(h.begin(), h.end());
+        GSAP_CUDA(cudaMemcpy(dst, w.data(), sizeof(int64_t) * (B + 1), cudaMemcpyDefault));
+    };
+    widen(rowptr, c.bm_rowptr);
+    widen(colptr, c.bm_colptr);
+    const size_t nb = sizeof(int) * (size_t)nnz;
+    copy_out(c, col, c.bm_col, nb);
+    copy_out(c, cnt, c.bm_cnt, nb);
+    copy_out(c, cum, c.bm_cum, nb);
+    copy_out(c, row, c.bm_row, nb);
+    copy_out(c, ccnt, c.bm_ccnt, nb);
+    copy_out(c, ccum, c.bm_ccum, nb);
+    copy_out(c, dout, c.dout, sizeof(int) * B);
+    copy_out(c, din, c.din, sizeof(int) * B);
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    API_CATCH
+}
+
+gsap_status gsap_get_stats(gsap_ctx *ctx, gsap_stats *out) {
+    API_TRY
+    REQUIRE(ctx && out, GSAP_EINVAL, "NULL argument");
+    fill_stats(ctx->c, out);
+    API_CATCH
+}
+
+gsap_status gsap_reset_stats(gsap_ctx *ctx) {
+    API_TRY
+    REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
+    Ctx &c = ctx->c;
+    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl}) {
+        kc_resolve(c, *k);
+        k->ms = 0;
+        k->bytes = 0;
+        k->launches = 0;
+    }
+    c.st = gsap_stats{};
+    c.launches = 0;
+    API_CATCH
+}
+
+gsap_status gsap_sync(gsap_ctx *ctx) {
+    API_TRY
+    REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
+    GSAP_CUDA(cudaStreamSynchronize(ctx->c.stream));
+    API_CATCH
+}
+
+gsap_status gsap_run(gsap_ctx *ctx, int32_t *bmap_out, int32_t *B_out, double *mdl_out, double *trace,
+                     int32_t trace_cap, int32_t *rounds_out) {
+    API_TRY
+    REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
+    run_impl(ctx->c, bmap_out, B_out, mdl_out, trace, trace_cap, rounds_out);
+    API_CATCH
+}
+
+gsap_status gsap_partition(int32_t V, const int64_t *rowptr, const int32_t *col, const int32_t *wgt,
+                           const gsap_params *params, const gsap_dist *dist, int32_t *bmap_out, int32_t *B_out,
+                           double *mdl_out, gsap_stats *stats) {
+    gsap_ctx *ctx = nullptr;
+    const auto t0 = std::chrono::steady_clock::now();
+    gsap_status st = gsap_create(V, rowptr, col, wgt, params, dist, nullptr, &ctx);
+    if (st != GSAP_OK) return st;
+    const double t_setup = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    st = gsap_run(ctx, bmap_out, B_out, mdl_out, nullptr, 0, nullptr);
+    if (st == GSAP_OK && stats) {
+        st = gsap_get_stats(ctx, stats);
+        stats->t_setup = t_setup;
+        stats->t_total = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    }
+    gsap_destroy(ctx);
+    return st;
+}
+
+}  // extern "C"

@@ -1,0 +1,169 @@
+// common.cuh -- device helpers shared by the GSAP sm_100a kernels.
+//
+// Philox4x32-10 (replaces the paper's cuRAND lookup tables, P:168 3.2 Fig. 4;
+// reading Z6), the multiply-shift range map, the cancellation-free entropy
+// differences used by Delta MDL (Eq. 3-7, P:205-246 3.3), warp reductions and
+// blockmodel lookups.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#define GSAP_DEV __device__ __forceinline__
+
+namespace gsap {
+
+constexpr unsigned FULL = 0xffffffffu;
+
+// ---------------------------------------------------------------- Philox --
+// Random123 philox4x32 round: (hi(M1*c2)^c1^k0, lo(M1*c2), hi(M0*c0)^c3^k1, lo(M0*c0))
+GSAP_DEV uint4 philox4x32_10(uint4 c, uint2 k) {
+#pragma unroll
+    for (int i = 0; i < 10; ++i) {
+        const uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+        c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
+        k.x += 0x9E3779B9u;
+        k.y += 0xBB67AE85u;
+    }
+    return c;
+}
+
+// words for (id, draw, iteration, outer round, phase): ctr = (id, j, itr, outer<<1|phase)
+GSAP_DEV uint4 draws(uint64_t seed, uint32_t id, uint32_t j, uint32_t itr, uint32_t outer,
+                     uint32_t phase) {
+    return philox4x32_10(make_uint4(id, j, itr, (outer << 1) | phase),
+                         make_uint2((uint32_t)seed, (uint32_t)(seed >> 32)));
+}
+
+// floor(w * T / 2^32), T < 2^32
+GSAP_DEV uint32_t pick(uint32_t w, uint32_t T) {
+    return (uint32_t)(((uint64_t)w * (uint64_t)T) >> 32);
+}
+
+// the proposal coin x <= B / (B + d) as an exact integer test (reading Z9)
+GSAP_DEV bool coin_random(uint32_t w1, uint32_t B, uint32_t d) {
+    return (uint64_t)w1 * ((uint64_t)B + d) <= ((uint64_t)B << 32);
+}
+
+// ------------------------------------------------------------- entropy --
+// f(m) = m ln m.  df(m, d) = f(m + d) - f(m) for integers m >= 0, m + d >= 0,
+// written without cancellation: d ln(m + d) + m log1p(d / m).
+GSAP_DEV double fx(double m) { return m > 0.0 ? m * log(m) : 0.0; }
+
+GSAP_DEV double df(long long m, long long d) {
+    if (d == 0) return 0.0;
+    const long long n = m + d;
+    if (m == 0) return fx((double)n);
+    if (n == 0) return -fx((double)m);
+    return (double)d * log((double)n) + (double)m * log1p((double)d / (double)m);
+}
+
+// g(a, c) = f(a + c) - f(a) - f(c) = a log1p(c/a) + c log1p(a/c)
+GSAP_DEV double g2(long long a, long long c) {
+    if (a == 0 || c == 0) return 0.0;
+    return (double)a * log1p((double)c / (double)a) + (double)c * log1p((double)a / (double)c);
+}
+
+// -------------------------------------------------------------- warps --
+GSAP_DEV unsigned lane_id() { return threadIdx.x & 31u; }
+
+template <typename T>
+GSAP_DEV T warp_sum(T v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+    return v;
+}
+
+GSAP_DEV int warp_incl_scan(int v) {
+    const unsigned l = lane_id();
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(FULL, v, o);
+        if (l >= (unsigned)o) v += t;
+    }
+    return v;
+}
+
+// ---------------------------------------------------------- blockmodel --
+// CSR (rows ascending column) + CSC (columns ascending row), cum = inclusive
+// prefix of cnt within a row / column, out/in degrees (P:143-162 3.1), and a
+// dense row-major copy M[x*B+y] when B is small.
+struct BM {
+    int B;
+    const int *__restrict__ dense;   // nullptr in the sparse regime
+    const int *__restrict__ rowptr;  // [B+1]
+    const int *__restrict__ col;
+    const int *__restrict__ cnt;
+    const int *__restrict__ cum;
+    const int *__restrict__ colptr;  // [B+1]
+    const int *__restrict__ row;
+    const int *__restrict__ ccnt;
+    const int *__restrict__ ccum;
+    const int *__restrict__ dout;
+    const int *__restrict__ din;
+};
+
+// first index i in [lo, hi) with a[i] > p (upper bound); hi if none
+GSAP_DEV int upper_bound(const int *__restrict__ a, int lo, int hi, long long p) {
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if ((long long)__ldg(a + mid) > p) hi = mid;
+        else lo = mid + 1;
+    }
+    return lo;
+}
+
+GSAP_DEV int bm_at(const BM &m, int x, int y) {
+    if (m.dense) return __ldg(m.dense + (size_t)x * m.B + y);
+    const int lo = __ldg(m.rowptr + x), hi = __ldg(m.rowptr + x + 1);
+    int a = lo, b = hi;
+    while (a < b) {
+        const int mid = (a + b) >> 1;
+        if (__ldg(m.col + mid) < y) a = mid + 1;
+        else b = mid;
+    }
+    return (a < hi && __ldg(m.col + a) == y) ? __ldg(m.cnt + a) : 0;
+}
+
+GSAP_DEV int bm_deg(const BM &m, int x) { return __ldg(m.dout + x) + __ldg(m.din + x); }
+
+// the weighted neighbour block of u at offset p of (out-row u ++ in-col u),
+// skipping id `skip` (-1: none) -- binary search on cum (R:O.4 step 4)
+GSAP_DEV int bm_walk(const BM &m, int u, long long p, int skip) {
+    const int rlo = __ldg(m.rowptr + u), rhi = __ldg(m.rowptr + u + 1);
+    const int dout_u = __ldg(m.dout + u);
+    int wskip = 0;
+    if (skip >= 0) {
+        int a = rlo, b = rhi;
+        while (a < b) {
+            const int mid = (a + b) >> 1;
+            if (__ldg(m.col + mid) < skip) a = mid + 1;
+            else b = mid;
+        }
+        if (a < rhi && __ldg(m.col + a) == skip) {
+            wskip = __ldg(m.cnt + a);
+            const long long before = (long long)__ldg(m.cum + a) - wskip;
+            if (p >= before) p += wskip;
+        }
+    }
+    if (p < dout_u) return __ldg(m.col + upper_bound(m.cum, rlo, rhi, p));
+    long long q = p - dout_u;
+    const int clo = __ldg(m.colptr + u), chi = __ldg(m.colptr + u + 1);
+    if (skip >= 0) {
+        int a = clo, b = chi;
+        while (a < b) {
+            const int mid = (a + b) >> 1;
+            if (__ldg(m.row + mid) < skip) a = mid + 1;
+            else b = mid;
+        }
+        if (a < chi && __ldg(m.row + a) == skip) {
+            const int w = __ldg(m.ccnt + a);
+            const long long before = (long long)__ldg(m.ccum + a) - w;
+            if (q >= before) q += w;
+        }
+    }
+    return __ldg(m.row + upper_bound(m.ccum, clo, chi, q));
+}
+
+}  // namespace gsap

@@ -1,0 +1,144 @@
+// internal.h -- the device state owned by a gsap_ctx and the host-side entry
+// points of each kernel family (rebuild.cu, move.cu, merge.cu, mdl.cu).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/gsap.h"
+#include "common.cuh"
+
+namespace gsap {
+
+// timing / accounting of one kernel class (CUDA events on the context stream)
+struct KClass {
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> pending;
+    std::vector<cudaEvent_t> pool;
+    double ms = 0.0, bytes = 0.0;
+    long long launches = 0;
+};
+
+struct Ctx {
+    int dev = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    gsap_params prm{};
+
+    // graph (device): out CSR in the caller's order, in CSC (by source id, then
+    // CSR position), the source of every edge, weighted degrees, self-loops
+    int V = 0, E = 0;
+    long long W = 0;
+    bool weighted = false;
+    int *rowptr = nullptr, *col = nullptr, *wgt = nullptr;
+    int *cscptr = nullptr, *cscsrc = nullptr, *cscwgt = nullptr;
+    int *esrc = nullptr, *kout = nullptr, *kin = nullptr, *selfw = nullptr;
+    std::vector<int> h_rowptr, h_cscptr;   // host copies (static) for batch accounting
+    // vertices whose total degree exceeds the warp path's table (static list)
+    int *big = nullptr;
+    std::vector<int> h_big;
+    size_t big_table_slots = 0;            // per-CTA global table capacity (slots)
+    int *big_tables = nullptr;             // global tables for very large vertices
+
+    // partition
+    int *b = nullptr;
+    int B = 0;
+
+    // blockmodel (capacity: nnz <= min(E, B^2); B <= V)
+    int *bm_rowptr = nullptr, *bm_col = nullptr, *bm_cnt = nullptr, *bm_cum = nullptr;
+    int *bm_colptr = nullptr, *bm_row = nullptr, *bm_ccnt = nullptr, *bm_ccum = nullptr;
+    int *dout = nullptr, *din = nullptr, *d_nnz = nullptr;
+    int *dense = nullptr, *denseT = nullptr;
+    size_t dense_cap = 0;   // elements
+    bool dense_mode = false;
+
+    // rebuild scratch
+    unsigned long long *keys0 = nullptr, *keys1 = nullptr, *vals64a = nullptr, *vals64b = nullptr;
+    unsigned *ukeys0 = nullptr, *ukeys1 = nullptr;
+    int *wa = nullptr, *wb = nullptr, *flags = nullptr, *pos = nullptr, *tmpi = nullptr,
+        *rowid = nullptr, *counts = nullptr, *scan_tmp = nullptr, *rownnz = nullptr;
+    size_t counts_cap = 0, scan_tmp_cap = 0;
+
+    // per-phase buffers
+    int *s = nullptr;            // proposals: V (MOVE) or B * P (MERGE)
+    double *dS = nullptr;        // V or B * P
+    double *H = nullptr;         // V
+    unsigned char *acc = nullptr;// V
+    int *best = nullptr;         // B
+    double *dSbest = nullptr;    // B
+    double *partials = nullptr;  // reduction partials
+    double *scal = nullptr;      // device scalars [0] = batch dS sum, [1] = data term
+    int *scal_i = nullptr;       // device int scalars [0] = new B, [1] = accepted moves
+    double *Dh = nullptr;        // per-iteration sum of accepted dS (max_nodal_itr)
+    int *slot_b[3] = {nullptr, nullptr, nullptr};   // golden-section bracket partitions
+    // merge selection scratch
+    unsigned long long *skey0 = nullptr, *skey1 = nullptr;
+    int *sval0 = nullptr, *sval1 = nullptr, *rank = nullptr, *nxt0 = nullptr, *nxt1 = nullptr,
+        *mx0 = nullptr, *mx1 = nullptr, *oncyc = nullptr, *label = nullptr, *present = nullptr;
+
+    // pinned host scalars
+    double *h_scal = nullptr;
+    int *h_int = nullptr;
+
+    // accounting
+    long long launches = 0;
+    KClass k_move, k_rebuild, k_merge, k_mdl;
+    gsap_stats st{};
+    std::vector<double> move_bytes_per_batch;   // algorithmic bytes per MOVE launch
+
+    BM bm() const {
+        BM m;
+        m.B = B;
+        m.dense = dense_mode ? dense : nullptr;
+        m.rowptr = bm_rowptr; m.col = bm_col; m.cnt = bm_cnt; m.cum = bm_cum;
+        m.colptr = bm_colptr; m.row = bm_row; m.ccnt = bm_ccnt; m.ccum = bm_ccum;
+        m.dout = dout; m.din = din;
+        return m;
+    }
+};
+
+// error plumbing -----------------------------------------------------------
+struct Error {
+    gsap_status code;
+    std::string msg;
+};
+
+#define GSAP_CUDA(x)                                                                          \
+    do {                                                                                      \
+        cudaError_t e_ = (x);                                                                 \
+        if (e_ != cudaSuccess)                                                                \
+            throw ::gsap::Error{GSAP_ECUDA, std::string(#x) + ": " + cudaGetErrorString(e_)}; \
+    } while (0)
+
+#define GSAP_CHECK_LAUNCH() GSAP_CUDA(cudaGetLastError())
+
+// event timing of a kernel class (no-op unless prm.profile)
+void kc_begin(Ctx &c, KClass &k, cudaEvent_t *ev);
+void kc_end(Ctx &c, KClass &k, cudaEvent_t ev, double bytes);
+void kc_resolve(Ctx &c, KClass &k);
+
+// rebuild.cu
+void build_graph_device(Ctx &c);                 // CSC, esrc, degrees (create time)
+void rebuild(Ctx &c);                            // Alg. 2 from c.b, c.B
+bool dense_ok(const Ctx &c, int B);
+
+// move.cu
+enum MoveMode { MOVE_FUSED = 0, MOVE_PROPOSE = 1, MOVE_DELTA = 2 };
+void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first, int count,
+                 int *s, double *dS, double *H, unsigned char *acc);
+void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned char *acc,
+                  const double *dS, double *dsum, int *nacc);
+
+// merge.cu
+void launch_merge_props(Ctx &c, uint32_t outer, int first, int count, bool propose, int *s,
+                        double *dS, int *best, double *dSbest);
+void select_merges(Ctx &c, const int *best, const double *dS, int K, int *label_out);
+
+// mdl.cu
+void launch_data_term(Ctx &c);                   // -> c.scal[1], no synchronisation
+double device_data_term(Ctx &c);                 // S = -sum f(M) + sum f(dout) + sum f(din)
+double model_term(long long W, int V, int B, int variant);
+
+}  // namespace gsap

@@ -1,0 +1,82 @@
+// mdl.cu -- the full description length, Eq. 1-2 (P:56-65 2.1; readings
+// Z1-Z4, Z22):
+//   S   = -sum_xy f(M_xy) + sum_x f(dout_x) + sum_y f(din_y),  f(m) = m ln m
+//   MDL = E h(B^2/E) + V ln B + S,  h(x) = (1 + x) ln(1 + x) - x ln x.
+// The data term is a fixed-chunk fp64 reduction (chunk = 8192 entries per
+// CTA, then one ordered pass), so it does not depend on the launch shape.
+#include <math.h>
+
+#include <algorithm>
+
+#include "internal.h"
+
+namespace gsap {
+
+constexpr int MDL_CHUNK = 8192;
+
+__global__ void __launch_bounds__(256) k_mdl_partials(const int *__restrict__ cnt, const int *__restrict__ d_nnz,
+                                                      const int *__restrict__ dout, const int *__restrict__ din,
+                                                      int B, double *__restrict__ partials) {
+    __shared__ double sh[8];
+    const int nnz = *d_nnz;
+    const long long base = (long long)blockIdx.x * MDL_CHUNK;
+    double acc = 0.0;
+    for (int k = threadIdx.x; k < MDL_CHUNK; k += 256) {
+        const long long i = base + k;
+        if (i < nnz) acc -= fx((double)cnt[i]);
+        if (i < B) acc += fx((double)dout[i]) + fx((double)din[i]);
+    }
+    acc = warp_sum(acc);
+    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = acc;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < 8; ++w) t += sh[w];
+        partials[blockIdx.x] = t;
+    }
+}
+
+__global__ void __launch_bounds__(256) k_mdl_final(const double *__restrict__ partials, int n, double *out) {
+    __shared__ double sh[8];
+    double v = 0.0;
+    for (int i = threadIdx.x; i < n; i += 256) v += partials[i];
+    v = warp_sum(v);
+    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = v;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < 8; ++w) t += sh[w];
+        *out = t;
+    }
+}
+
+// launches the reduction into c.scal[1] (no synchronisation)
+void launch_data_term(Ctx &c) {
+    cudaEvent_t ev = nullptr;
+    kc_begin(c, c.k_mdl, &ev);
+    const long long n = std::max<long long>(std::max<long long>(c.E, c.B), 1);
+    const int nb = (int)((n + MDL_CHUNK - 1) / MDL_CHUNK);
+    k_mdl_partials<<<nb, 256, 0, c.stream>>>(c.bm_cnt, c.d_nnz, c.dout, c.din, c.B, c.partials);
+    k_mdl_final<<<1, 256, 0, c.stream>>>(c.partials, nb, c.scal + 1);
+    c.launches += 2;
+    GSAP_CHECK_LAUNCH();
+    kc_end(c, c.k_mdl, ev, 0.0);
+}
+
+double device_data_term(Ctx &c) {
+    launch_data_term(c);
+    GSAP_CUDA(cudaMemcpyAsync(c.h_scal + 1, c.scal + 1, sizeof(double), cudaMemcpyDeviceToHost, c.stream));
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    return c.h_scal[1];
+}
+
+double model_term(long long W, int V, int B, int variant) {
+    const double lnB = log((double)B);
+    if (W <= 0) return (double)V * lnB;
+    const double E = (double)W, x = (double)B * (double)B / E;
+    const double t = variant == 1 ? E * (1.0 + x) * log1p(x) - x * log(x)
+                                  : E * ((1.0 + x) * log1p(x) - x * log(x));
+    return t + (double)V * lnB;
+}
+
+}  // namespace gsap

@@ -1,0 +1,286 @@
+// merge.cu -- the block-merge phase (P:67 2.1, P:141 3, P:166-170 3.2,
+// P:211-232 3.3):
+//   (a3) every block r draws num_proposals merge targets (Alg. 1, excluding r;
+//        readings Z6, Z8) and evaluates Delta S of merging r into s in exact
+//        form (Eq. 4-6 with the terms Z11/Z12 add):
+//          dS = -sum_{t != r,s} [g(M_st, M_rt) + g(M_ts, M_tr)]
+//               - [f(M_ss + M_sr + M_rs + M_rr) - f(M_ss) - f(M_sr) - f(M_rs) - f(M_rr)]
+//               + g(dout_s, dout_r) + g(din_s, din_r),   g(a,c) = f(a+c) - f(a) - f(c),
+//        where only t in the intersection of the two rows (columns) contribute:
+//        a warp walks the shorter row and looks the other up (dense copy or
+//        binary search);  best_r = argmin_j (first j wins ties, R:Z16);
+//   (a4) the perform-merge, in an exact parallel form of the
+//        sequential GraphChallenge loop: rank by
+//        (dS_best, r); reject the max-rank edge of every cycle of r -> best_r
+//        (pointer doubling with running max); apply the accepted edges of the
+//        shortest rank prefix with K of them; roots by pointer jumping;
+//        relabel to the ranks of the roots present in b (R:Z18).
+#include <algorithm>
+
+#include "internal.h"
+#include "prims.cuh"
+
+namespace gsap {
+
+typedef unsigned long long u64;
+
+constexpr int MERGE_WARPS = 8;
+constexpr int MAX_P = 32;
+
+GSAP_DEV int propose_merge(const BM &m, int r, uint32_t j, uint64_t seed, uint32_t outer) {
+    const uint32_t B = (uint32_t)m.B;
+    const uint4 w = draws(seed, (uint32_t)r, j, 0u, outer, 0u);
+    const uint32_t K = (uint32_t)bm_deg(m, r);
+    if (K > 0) {
+        const int u = bm_walk(m, r, (long long)pick(w.x, K), -1);
+        const uint32_t du = (uint32_t)bm_deg(m, u);
+        if (!coin_random(w.y, B, du)) {
+            const uint32_t T = du - (uint32_t)bm_at(m, u, r) - (uint32_t)bm_at(m, r, u);
+            if (T > 0) return bm_walk(m, u, (long long)pick(w.z, T), r);
+        }
+    }
+    int s = (int)pick(w.z, B - 1);
+    if (s >= r) ++s;
+    return s;
+}
+
+// sum over t != r, s of g over the intersection of (ptrA/idxA/cntA row a) and
+// row b of the same structure; lookups of the other side via lookup(t)
+template <typename Lookup>
+GSAP_DEV double inter_sum(const int *__restrict__ ptr, const int *__restrict__ idx, const int *__restrict__ cnt,
+                          int a, int b, int r, int s, Lookup lookup) {
+    const int alo = __ldg(ptr + a), ahi = __ldg(ptr + a + 1);
+    const int blo = __ldg(ptr + b), bhi = __ldg(ptr + b + 1);
+    const bool walk_a = (ahi - alo) <= (bhi - blo);
+    const int lo = walk_a ? alo : blo, hi = walk_a ? ahi : bhi, other = walk_a ? b : a;
+    double acc = 0.0;
+    for (int i = lo + (int)(threadIdx.x & 31); i < hi; i += 32) {
+        const int t = __ldg(idx + i);
+        if (t == r || t == s) continue;
+        const int m1 = __ldg(cnt + i);
+        const int m2 = lookup(other, t);
+        acc += g2(m1, m2);
+    }
+    return acc;
+}
+
+GSAP_DEV double merge_delta(const BM &m, int r, int s) {
+    // rows r, s (t in both supports): g(M_st, M_rt)
+    double acc = inter_sum(m.rowptr, m.col, m.cnt, r, s, r, s,
+                           [&](int x, int t) { return bm_at(m, x, t); });
+    // columns r, s: g(M_ts, M_tr)
+    acc += inter_sum(m.colptr, m.row, m.ccnt, r, s, r, s, [&](int y, int t) { return bm_at(m, t, y); });
+    acc = warp_sum(acc);
+    const long long Mss = bm_at(m, s, s), Msr = bm_at(m, s, r), Mrs = bm_at(m, r, s), Mrr = bm_at(m, r, r);
+    // f(a+b+c+d) - f(a) - f(b) - f(c) - f(d), telescoped into g's
+    const double core = g2(Mss, Msr) + g2(Mss + Msr, Mrs) + g2(Mss + Msr + Mrs, Mrr);
+    const double deg = g2(__ldg(m.dout + s), __ldg(m.dout + r)) + g2(__ldg(m.din + s), __ldg(m.din + r));
+    return -acc - core + deg;
+}
+
+struct MergeArgs {
+    BM m;
+    uint64_t seed;
+    uint32_t outer;
+    int P, first, count;
+    bool propose;
+    int *s;          // [count * P] in (propose = false) or out (nullable)
+    double *dS;      // [count * P] out, nullable
+    int *best;       // [count] out, nullable
+    double *dSbest;  // [count] out, nullable
+};
+
+__global__ void __launch_bounds__(MERGE_WARPS * 32) k_merge(MergeArgs a) {
+    const int lane = threadIdx.x & 31;
+    const int nwarps = gridDim.x * MERGE_WARPS;
+    for (int i = blockIdx.x * MERGE_WARPS + (threadIdx.x >> 5); i < a.count; i += nwarps) {
+        const int r = a.first + i;
+        int sj = -1;
+        if (lane < a.P) {
+            sj = a.propose ? propose_merge(a.m, r, (uint32_t)lane, a.seed, a.outer) : a.s[(size_t)i * a.P + lane];
+            if (a.propose && a.s) a.s[(size_t)i * a.P + lane] = sj;
+        }
+        if (!a.dS && !a.best && !a.dSbest) continue;   // proposals only
+        int bs = -1;
+        double bd = 0.0;
+        for (int j = 0; j < a.P; ++j) {
+            const int s = __shfl_sync(FULL, sj, j);
+            const double d = merge_delta(a.m, r, s);
+            if (lane == 0) {
+                if (a.dS) a.dS[(size_t)i * a.P + j] = d;
+                if (j == 0 || d < bd) {
+                    bd = d;
+                    bs = s;
+                }
+            }
+        }
+        if (lane == 0) {
+            if (a.best) a.best[i] = bs;
+            if (a.dSbest) a.dSbest[i] = bd;
+        }
+    }
+}
+
+void launch_merge_props(Ctx &c, uint32_t outer, int first, int count, bool propose, int *s, double *dS,
+                        int *best, double *dSbest) {
+    if (count <= 0) return;
+    if (c.prm.num_proposals < 1 || c.prm.num_proposals > MAX_P)
+        throw Error{GSAP_EINVAL, "num_proposals must be in [1, 32]"};
+    if (c.B < 2) throw Error{GSAP_ESTATE, "merge proposals need B >= 2"};
+    cudaEvent_t ev = nullptr;
+    kc_begin(c, c.k_merge, &ev);
+    MergeArgs a;
+    a.m = c.bm();
+    a.seed = c.prm.seed;
+    a.outer = outer;
+    a.P = c.prm.num_proposals;
+    a.first = first;
+    a.count = count;
+    a.propose = propose;
+    a.s = s;
+    a.dS = dS;
+    a.best = best;
+    a.dSbest = dSbest;
+    const long long need = ((long long)count + MERGE_WARPS - 1) / MERGE_WARPS;
+    const int grid = (int)std::min<long long>(need, 148LL * 16);
+    k_merge<<<grid, MERGE_WARPS * 32, 0, c.stream>>>(a);
+    ++c.launches;
+    GSAP_CHECK_LAUNCH();
+    // algorithmic bytes: each proposal reads rows / columns r and s (id + cnt)
+    // once; estimated from the mean row length (nnz unknown on the host)
+    const double mean_row = (double)std::min<long long>(c.E, (long long)c.B * c.B) / std::max(1, c.B);
+    kc_end(c, c.k_merge, ev, (double)count * (double)a.P * 4.0 * 8.0 * mean_row);
+}
+
+// ----------------------------------------------------------- selection --
+__global__ void k_sel_keys(int B, const double *__restrict__ dS, u64 *__restrict__ keys, int *__restrict__ ids) {
+    for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < B; r += gridDim.x * blockDim.x) {
+        double d = dS[r];
+        if (d == 0.0) d = 0.0;   // -0.0 == +0.0
+        u64 bits = (u64)__double_as_longlong(d);
+        bits = (bits >> 63) ? ~bits : (bits | 0x8000000000000000ULL);
+        keys[r] = bits;
+        ids[r] = r;
+    }
+}
+
+__global__ void k_sel_rank(int B, const int *__restrict__ sorted_ids, int *__restrict__ rank) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < B; i += gridDim.x * blockDim.x) rank[sorted_ids[i]] = i;
+}
+
+__global__ void k_sel_init(int B, const int *__restrict__ best, const int *__restrict__ rank, int *__restrict__ nxt,
+                           int *__restrict__ mx, int *__restrict__ oncyc) {
+    for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < B; r += gridDim.x * blockDim.x) {
+        nxt[r] = best[r];
+        mx[r] = rank[r];
+        oncyc[r] = 0;
+    }
+}
+
+// one doubling step: mx'(r) = max(mx(r), mx(nxt(r))), nxt'(r) = nxt(nxt(r))
+__global__ void k_sel_double(int B, const int *__restrict__ nxt, const int *__restrict__ mx, int *__restrict__ nxt2,
+                             int *__restrict__ mx2) {
+    for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < B; r += gridDim.x * blockDim.x) {
+        const int n = nxt[r];
+        nxt2[r] = nxt[n];
+        mx2[r] = max(mx[r], mx[n]);
+    }
+}
+
+__global__ void k_sel_mark(int B, const int *__restrict__ nxt, int *__restrict__ oncyc) {
+    for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < B; r += gridDim.x * blockDim.x) oncyc[nxt[r]] = 1;
+}
+
+// acc_in_rank[i] = 1 iff the edge of the block at rank i is not a rejected cycle edge
+__global__ void k_sel_accepted(int B, const int *__restrict__ sorted_ids, const int *__restrict__ rank,
+                               const int *__restrict__ mx, const int *__restrict__ oncyc, int *__restrict__ acc_rank) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < B; i += gridDim.x * blockDim.x) {
+        const int r = sorted_ids[i];
+        const bool rejected = oncyc[r] && mx[r] == rank[r];
+        acc_rank[i] = rejected ? 0 : 1;
+    }
+}
+
+// applied edges: accepted and inside the shortest rank prefix with K of them;
+// nxt(r) = best[r] if applied else r.  incl = inclusive scan of acc_rank.
+__global__ void k_sel_applied(int B, int K, const int *__restrict__ sorted_ids, const int *__restrict__ acc_rank,
+                              const int *__restrict__ incl, const int *__restrict__ best, int *__restrict__ nxt) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < B; i += gridDim.x * blockDim.x) {
+        const int r = sorted_ids[i];
+        const bool applied = acc_rank[i] && incl[i] <= K;
+        nxt[r] = applied ? best[r] : r;
+    }
+}
+
+__global__ void k_jump(int B, const int *__restrict__ nxt, int *__restrict__ nxt2) {
+    for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < B; r += gridDim.x * blockDim.x) nxt2[r] = nxt[nxt[r]];
+}
+
+__global__ void k_present(int V, const int *__restrict__ b, const int *__restrict__ root, int *__restrict__ present) {
+    for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) present[root[b[v]]] = 1;
+}
+
+__global__ void k_labels(int B, const int *__restrict__ root, const int *__restrict__ present,
+                         const int *__restrict__ excl, int *__restrict__ label) {
+    for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < B; r += gridDim.x * blockDim.x) {
+        const int x = root[r];
+        label[r] = present[x] ? excl[x] : -1;
+    }
+}
+
+__global__ void k_relabel(int V, const int *__restrict__ label, int *__restrict__ b) {
+    for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) b[v] = label[b[v]];
+}
+
+static inline int g256(long long n) { return (int)std::max<long long>(1, std::min<long long>((n + 255) / 256, 148LL * 32)); }
+
+void select_merges(Ctx &c, const int *best, const double *dS, int K, int *label_out) {
+    Launcher L{c.stream, &c.launches};
+    const int B = c.B, V = c.V;
+    int rounds = 1;
+    while ((1LL << rounds) < 2LL * B) ++rounds;
+    k_sel_keys<<<g256(B), 256, 0, c.stream>>>(B, dS, c.skey0, c.sval0);
+    ++c.launches;
+    const int w = radix_sort<u64, int, true>(c.skey0, c.skey1, c.sval0, c.sval1, nullptr, B, 64, c.counts,
+                                             c.scan_tmp, L);
+    const int *sorted = w ? c.sval1 : c.sval0;
+    k_sel_rank<<<g256(B), 256, 0, c.stream>>>(B, sorted, c.rank);
+    k_sel_init<<<g256(B), 256, 0, c.stream>>>(B, best, c.rank, c.nxt0, c.mx0, c.oncyc);
+    c.launches += 2;
+    int *n0 = c.nxt0, *n1 = c.nxt1, *m0 = c.mx0, *m1 = c.mx1;
+    for (int k = 0; k < rounds; ++k) {
+        k_sel_double<<<g256(B), 256, 0, c.stream>>>(B, n0, m0, n1, m1);
+        std::swap(n0, n1);
+        std::swap(m0, m1);
+    }
+    k_sel_mark<<<g256(B), 256, 0, c.stream>>>(B, n0, c.oncyc);
+    k_sel_accepted<<<g256(B), 256, 0, c.stream>>>(B, sorted, c.rank, m0, c.oncyc, c.flags);
+    c.launches += rounds + 2;
+    device_scan<int>(c.flags, c.pos, nullptr, B, true, c.scan_tmp, nullptr, L);
+    k_sel_applied<<<g256(B), 256, 0, c.stream>>>(B, K, sorted, c.flags, c.pos, best, c.nxt0);
+    ++c.launches;
+    n0 = c.nxt0;
+    n1 = c.nxt1;
+    for (int k = 0; k < rounds; ++k) {
+        k_jump<<<g256(B), 256, 0, c.stream>>>(B, n0, n1);
+        std::swap(n0, n1);
+    }
+    c.launches += rounds;
+    GSAP_CUDA(cudaMemsetAsync(c.present, 0, sizeof(int) * ((size_t)B + 1), c.stream));
+    k_present<<<g256(V), 256, 0, c.stream>>>(V, c.b, n0, c.present);
+    ++c.launches;
+    device_scan<int>(c.present, c.pos, nullptr, B, false, c.scan_tmp, c.scal_i, L);
+    k_labels<<<g256(B), 256, 0, c.stream>>>(B, n0, c.present, c.pos, c.label);
+    k_relabel<<<g256(V), 256, 0, c.stream>>>(V, c.label, c.b);
+    c.launches += 2;
+    GSAP_CHECK_LAUNCH();
+    if (label_out)
+        GSAP_CUDA(cudaMemcpyAsync(label_out, c.label, sizeof(int) * (size_t)B, cudaMemcpyDefault, c.stream));
+    int newB = 0;
+    GSAP_CUDA(cudaMemcpyAsync(c.h_int, c.scal_i, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    newB = *c.h_int;
+    c.B = newB;
+}
+
+}  // namespace gsap

@@ -1,0 +1,414 @@
+// rebuild.cu -- blockmodel rebuild (Alg. 2, P:248-283 3.4) and create-time
+// graph preparation.
+//
+// M_xy = sum over edges u->w of weight [b_u = x][b_w = y] (P:56 2.1), stored
+// as CSR (rows ascending column) + CSC (columns ascending row) with the
+// in-row / in-column inclusive prefix `cum` used by the proposal walks, and the
+// out / in block degrees.  Two regimes:
+//   dense  (B^2 <= 4E): shared-memory-privatised (B <= 221) or L2-atomic
+//          histogram into a dense B x B matrix, tiled transpose, warp-per-row
+//          compaction into CSR / CSC;
+//   sparse (B^2 > 4E): 64-bit keys (b_src << sh | b_dst), stable LSD radix sort
+//          (prims.cuh), run-length encode, row pointers by lower bound, cum by
+//          one global scan; CSC by a second stable radix sort on the column.
+#include <algorithm>
+
+#include "internal.h"
+#include "prims.cuh"
+
+namespace gsap {
+
+typedef unsigned long long u64;
+
+static inline int grid_for(long long n, int threads) {
+    long long g = (n + threads - 1) / threads;
+    return (int)(g < 1 ? 1 : (g > 2147483647LL ? 2147483647LL : g));
+}
+
+static inline int bits_for(long long n) {   // ceil(log2(n)), at least 1
+    int b = 1;
+    while ((1LL << b) < n) ++b;
+    return b;
+}
+
+// ------------------------------------------------------------ create time --
+__global__ void k_esrc_kout(int V, const int *__restrict__ rowptr, const int *__restrict__ col,
+                            const int *__restrict__ wgt, int *__restrict__ esrc, int *__restrict__ kout,
+                            int *__restrict__ selfw) {
+    const int lane = threadIdx.x & 31;
+    for (int v = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < V; v += (gridDim.x * blockDim.x) >> 5) {
+        const int lo = rowptr[v], hi = rowptr[v + 1];
+        int sum = 0, self = 0;
+        for (int e = lo + lane; e < hi; e += 32) {
+            esrc[e] = v;
+            const int w = wgt ? wgt[e] : 1;
+            sum += w;
+            if (col[e] == v) self += w;
+        }
+        sum = warp_sum(sum);
+        self = warp_sum(self);
+        if (lane == 0) {
+            kout[v] = sum;
+            selfw[v] = self;
+        }
+    }
+}
+
+__global__ void k_csc_fill(int E, const int *__restrict__ idx, const int *__restrict__ esrc,
+                           const int *__restrict__ wgt, int *__restrict__ cscsrc, int *__restrict__ cscwgt) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < E; i += (long long)gridDim.x * blockDim.x) {
+        const int e = idx[i];
+        cscsrc[i] = esrc[e];
+        if (wgt) cscwgt[i] = wgt[e];
+    }
+}
+
+__global__ void k_iota(int n, int *a) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        a[i] = (int)i;
+}
+
+// ptr[x] = first i in [0, n) with ids[i] >= x, x in [0, B]
+template <typename T>
+__global__ void k_ptr_from_ids(const T *__restrict__ ids, const int *d_n, int n_static, int B, int *__restrict__ ptr) {
+    const int n = read_n(d_n, n_static);
+    for (int x = blockIdx.x * blockDim.x + threadIdx.x; x <= B; x += gridDim.x * blockDim.x) {
+        int lo = 0, hi = n;
+        while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if ((long long)ids[mid] < (long long)x) lo = mid + 1;
+            else hi = mid;
+        }
+        ptr[x] = lo;
+    }
+}
+
+__global__ void k_kin(int V, const int *__restrict__ cscptr, const int *__restrict__ cscwgt, int *__restrict__ kin) {
+    const int lane = threadIdx.x & 31;
+    for (int v = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < V; v += (gridDim.x * blockDim.x) >> 5) {
+        const int lo = cscptr[v], hi = cscptr[v + 1];
+        int sum = 0;
+        for (int e = lo + lane; e < hi; e += 32) sum += cscwgt ? cscwgt[e] : 1;
+        sum = warp_sum(sum);
+        if (lane == 0) kin[v] = sum;
+    }
+}
+
+void build_graph_device(Ctx &c) {
+    Launcher L{c.stream, &c.launches};
+    const int V = c.V, E = c.E;
+    k_esrc_kout<<<grid_for((long long)V * 32, 256), 256, 0, c.stream>>>(V, c.rowptr, c.col, c.wgt, c.esrc,
+                                                                        c.kout, c.selfw);
+    GSAP_CHECK_LAUNCH();
+    ++c.launches;
+    // CSC: stable sort of edge ids by destination (ties keep CSR order = by source)
+    if (E > 0) {
+        GSAP_CUDA(cudaMemcpyAsync(c.ukeys0, c.col, sizeof(int) * (size_t)E, cudaMemcpyDeviceToDevice, c.stream));
+        k_iota<<<grid_for(E, 256), 256, 0, c.stream>>>(E, c.wa);
+        ++c.launches;
+        const int which = radix_sort<unsigned, int, true>(c.ukeys0, c.ukeys1, c.wa, c.wb, nullptr, E,
+                                                          bits_for(V), c.counts, c.scan_tmp, L);
+        const unsigned *keys = which ? c.ukeys1 : c.ukeys0;
+        const int *idx = which ? c.wb : c.wa;
+        k_csc_fill<<<grid_for(E, 256), 256, 0, c.stream>>>(E, idx, c.esrc, c.wgt, c.cscsrc, c.cscwgt);
+        k_ptr_from_ids<unsigned><<<grid_for(V + 1, 256), 256, 0, c.stream>>>(keys, nullptr, E, V, c.cscptr);
+        c.launches += 2;
+    } else {
+        GSAP_CUDA(cudaMemsetAsync(c.cscptr, 0, sizeof(int) * ((size_t)V + 1), c.stream));
+    }
+    k_kin<<<grid_for((long long)V * 32, 256), 256, 0, c.stream>>>(V, c.cscptr, c.cscwgt, c.kin);
+    ++c.launches;
+    GSAP_CHECK_LAUNCH();
+}
+
+// ----------------------------------------------------------------- dense --
+bool dense_ok(const Ctx &c, int B) { return (size_t)B * (size_t)B <= c.dense_cap; }
+
+constexpr int HIST_SMEM_MAX_B = 221;   // B^2 * 4 bytes <= 195 KB of shared memory
+
+// histogram of (b[src], b[dst]) over an edge range; PRIV: privatised in smem
+template <bool PRIV>
+__global__ void __launch_bounds__(1024) k_hist(int E, const int *__restrict__ esrc, const int *__restrict__ col,
+                                                const int *__restrict__ wgt, const int *__restrict__ b, int B,
+                                                int *__restrict__ M) {
+    extern __shared__ int h[];
+    const int BB = B * B;
+    if (PRIV) {
+        for (int i = threadIdx.x; i < BB; i += blockDim.x) h[i] = 0;
+        __syncthreads();
+    }
+    int *dst = PRIV ? h : M;
+    const long long chunk = ((long long)E + gridDim.x - 1) / gridDim.x;
+    const long long lo = (long long)blockIdx.x * chunk;
+    const long long hi = min((long long)E, lo + chunk);
+    // iterate whole warps so that __match_any_sync sees a converged warp
+    for (long long e0 = lo; e0 < hi; e0 += blockDim.x) {
+        const long long e = e0 + threadIdx.x;
+        int key = -1, w = 0;
+        if (e < hi) {
+            key = __ldg(b + __ldg(esrc + e)) * B + __ldg(b + __ldg(col + e));
+            w = wgt ? __ldg(wgt + e) : 1;
+        }
+        if (wgt) {
+            if (key >= 0) atomicAdd(dst + key, w);
+        } else {
+            const unsigned peers = __match_any_sync(FULL, key);
+            if (key >= 0 && (int)(threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(dst + key, __popc(peers));
+        }
+    }
+    if (PRIV) {
+        __syncthreads();
+        for (int i = threadIdx.x; i < BB; i += blockDim.x) {
+            const int v = h[i];
+            if (v) atomicAdd(M + i, v);
+        }
+    }
+}
+
+__global__ void k_transpose(const int *__restrict__ M, int B, int *__restrict__ T) {
+    __shared__ int tile[32][33];
+    const int bx = blockIdx.x * 32, by = blockIdx.y * 32;
+    for (int j = threadIdx.y; j < 32; j += blockDim.y) {
+        const int x = by + j, y = bx + threadIdx.x;
+        tile[j][threadIdx.x] = (x < B && y < B) ? M[(size_t)x * B + y] : 0;
+    }
+    __syncthreads();
+    for (int j = threadIdx.y; j < 32; j += blockDim.y) {
+        const int x = bx + j, y = by + threadIdx.x;
+        if (x < B && y < B) T[(size_t)x * B + y] = tile[threadIdx.x][j];
+    }
+}
+
+// per row of a dense B x B matrix: number of non-zeros and the row sum
+__global__ void k_row_stats(const int *__restrict__ M, int B, int *__restrict__ nnz, int *__restrict__ sum) {
+    const int lane = threadIdx.x & 31;
+    for (int x = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < B; x += (gridDim.x * blockDim.x) >> 5) {
+        int c = 0, s = 0;
+        for (int y = lane; y < B; y += 32) {
+            const int v = M[(size_t)x * B + y];
+            c += v != 0;
+            s += v;
+        }
+        c = warp_sum(c);
+        s = warp_sum(s);
+        if (lane == 0) {
+            nnz[x] = c;
+            sum[x] = s;
+        }
+    }
+}
+
+// compact the non-zeros of each row into (idx, cnt, cum) at ptr[row]
+__global__ void k_row_compact(const int *__restrict__ M, int B, const int *__restrict__ ptr,
+                              int *__restrict__ idx, int *__restrict__ cnt, int *__restrict__ cum) {
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    for (int x = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < B; x += (gridDim.x * blockDim.x) >> 5) {
+        int base = ptr[x], run = 0;
+        for (int y0 = 0; y0 < B; y0 += 32) {
+            const int y = y0 + lane;
+            const int v = y < B ? M[(size_t)x * B + y] : 0;
+            const unsigned bal = __ballot_sync(FULL, v != 0);
+            const int sc = warp_incl_scan(v) + run;
+            if (v != 0) {
+                const int p = base + __popc(bal & lt);
+                idx[p] = y;
+                cnt[p] = v;
+                cum[p] = sc;
+            }
+            base += __popc(bal);
+            run = __shfl_sync(FULL, sc, 31);
+        }
+    }
+}
+
+static void rebuild_dense(Ctx &c) {
+    Launcher L{c.stream, &c.launches};
+    const int B = c.B, E = c.E;
+    const size_t BB = (size_t)B * B;
+    GSAP_CUDA(cudaMemsetAsync(c.dense, 0, sizeof(int) * BB, c.stream));
+    if (E > 0) {
+        int dev_sms = 148;
+        if (B <= HIST_SMEM_MAX_B) {
+            const size_t smem = sizeof(int) * BB;
+            static bool attr = false;
+            if (!attr) {
+                GSAP_CUDA(cudaFuncSetAttribute(k_hist<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                               HIST_SMEM_MAX_B * HIST_SMEM_MAX_B * 4));
+                attr = true;
+            }
+            const int grid = (int)std::min<long long>(dev_sms, ((long long)E + 1023) / 1024);
+            k_hist<true><<<grid, 1024, smem, c.stream>>>(E, c.esrc, c.col, c.wgt, c.b, B, c.dense);
+        } else {
+            const int grid = (int)std::min<long long>(dev_sms * 8, ((long long)E + 1023) / 1024);
+            k_hist<false><<<grid, 1024, 0, c.stream>>>(E, c.esrc, c.col, c.wgt, c.b, B, c.dense);
+        }
+        ++c.launches;
+        GSAP_CHECK_LAUNCH();
+    }
+    dim3 tg((B + 31) / 32, (B + 31) / 32), tb(32, 8);
+    k_transpose<<<tg, tb, 0, c.stream>>>(c.dense, B, c.denseT);
+    const int rg = grid_for((long long)B * 32, 256);
+    k_row_stats<<<rg, 256, 0, c.stream>>>(c.dense, B, c.rownnz, c.dout);
+    k_row_stats<<<rg, 256, 0, c.stream>>>(c.denseT, B, c.tmpi, c.din);
+    c.launches += 3;
+    device_scan<int>(c.rownnz, c.bm_rowptr, nullptr, B, false, c.scan_tmp, c.bm_rowptr + B, L);
+    device_scan<int>(c.tmpi, c.bm_colptr, nullptr, B, false, c.scan_tmp, c.bm_colptr + B, L);
+    k_row_compact<<<rg, 256, 0, c.stream>>>(c.dense, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum);
+    k_row_compact<<<rg, 256, 0, c.stream>>>(c.denseT, B, c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum);
+    c.launches += 2;
+    GSAP_CUDA(cudaMemcpyAsync(c.d_nnz, c.bm_rowptr + B, sizeof(int), cudaMemcpyDeviceToDevice, c.stream));
+    GSAP_CHECK_LAUNCH();
+}
+
+// ---------------------------------------------------------------- sparse --
+__global__ void k_keys(int E, const int *__restrict__ esrc, const int *__restrict__ col,
+                       const int *__restrict__ wgt, const int *__restrict__ b, int sh,
+                       u64 *__restrict__ keys, int *__restrict__ w) {
+    for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < E; e += (long long)gridDim.x * blockDim.x) {
+        keys[e] = ((u64)(unsigned)__ldg(b + __ldg(esrc + e)) << sh) | (u64)(unsigned)__ldg(b + __ldg(col + e));
+        if (wgt) w[e] = wgt[e];
+    }
+}
+
+__global__ void k_heads(int n, const u64 *__restrict__ keys, int *__restrict__ flags) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        flags[i] = (i == 0 || keys[i] != keys[i - 1]) ? 1 : 0;
+}
+
+__global__ void k_unique(int n, const u64 *__restrict__ keys, const int *__restrict__ flags,
+                         const int *__restrict__ pos, int sh, int *__restrict__ rowid, int *__restrict__ colv,
+                         int *__restrict__ headidx) {
+    const u64 mask = (1ULL << sh) - 1ULL;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+        if (flags[i]) {
+            const int u = pos[i];
+            const u64 k = keys[i];
+            rowid[u] = (int)(k >> sh);
+            colv[u] = (int)(k & mask);
+            headidx[u] = (int)i;
+        }
+    }
+}
+
+__global__ void k_cnt_runs(int n, const int *__restrict__ headidx, const int *__restrict__ d_nnz, int *__restrict__ cnt) {
+    const int nnz = *d_nnz;
+    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < nnz; u += gridDim.x * blockDim.x)
+        cnt[u] = (u + 1 < nnz ? headidx[u + 1] : n) - headidx[u];
+}
+
+__global__ void k_cnt_weighted(int n, const int *__restrict__ flags, const int *__restrict__ pos,
+                               const int *__restrict__ w, int *__restrict__ cnt) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        atomicAdd(cnt + pos[i] + flags[i] - 1, w[i]);
+}
+
+// cum[u] = P[u] - P[start of u's segment - 1]; P = inclusive scan of cnt
+__global__ void k_seg_cum(const int *__restrict__ ids, const int *__restrict__ ptr, const int *__restrict__ P,
+                          const int *__restrict__ d_n, int *__restrict__ cum) {
+    const int n = *d_n;
+    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < n; u += gridDim.x * blockDim.x) {
+        const int s = ptr[ids[u]];
+        cum[u] = P[u] - (s > 0 ? P[s - 1] : 0);
+    }
+}
+
+__global__ void k_seg_deg(int B, const int *__restrict__ ptr, const int *__restrict__ P, int *__restrict__ deg) {
+    for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < B; x += gridDim.x * blockDim.x) {
+        const int lo = ptr[x], hi = ptr[x + 1];
+        deg[x] = hi > lo ? P[hi - 1] - (lo > 0 ? P[lo - 1] : 0) : 0;
+    }
+}
+
+__global__ void k_csc_keys(const int *__restrict__ d_n, const int *__restrict__ colv, const int *__restrict__ rowid,
+                           const int *__restrict__ cnt, unsigned *__restrict__ keys, u64 *__restrict__ vals) {
+    const int n = *d_n;
+    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < n; u += gridDim.x * blockDim.x) {
+        keys[u] = (unsigned)colv[u];
+        vals[u] = ((u64)(unsigned)rowid[u] << 32) | (u64)(unsigned)cnt[u];
+    }
+}
+
+__global__ void k_csc_unpack(const int *__restrict__ d_n, const unsigned *__restrict__ keys,
+                             const u64 *__restrict__ vals, int *__restrict__ colid, int *__restrict__ row,
+                             int *__restrict__ ccnt) {
+    const int n = *d_n;
+    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < n; u += gridDim.x * blockDim.x) {
+        colid[u] = (int)keys[u];
+        const u64 v = vals[u];
+        row[u] = (int)(v >> 32);
+        ccnt[u] = (int)(unsigned)(v & 0xffffffffULL);
+    }
+}
+
+static void rebuild_sparse(Ctx &c) {
+    Launcher L{c.stream, &c.launches};
+    const int B = c.B, E = c.E;
+    if (E == 0) {
+        GSAP_CUDA(cudaMemsetAsync(c.bm_rowptr, 0, sizeof(int) * ((size_t)B + 1), c.stream));
+        GSAP_CUDA(cudaMemsetAsync(c.bm_colptr, 0, sizeof(int) * ((size_t)B + 1), c.stream));
+        GSAP_CUDA(cudaMemsetAsync(c.dout, 0, sizeof(int) * (size_t)B, c.stream));
+        GSAP_CUDA(cudaMemsetAsync(c.din, 0, sizeof(int) * (size_t)B, c.stream));
+        GSAP_CUDA(cudaMemsetAsync(c.d_nnz, 0, sizeof(int), c.stream));
+        return;
+    }
+    const int sh = bits_for(B);
+    const int g = grid_for(E, 256);
+    k_keys<<<g, 256, 0, c.stream>>>(E, c.esrc, c.col, c.wgt, c.b, sh, c.keys0, c.wa);
+    ++c.launches;
+    int which;
+    if (c.weighted)
+        which = radix_sort<u64, int, true>(c.keys0, c.keys1, c.wa, c.wb, nullptr, E, 2 * sh, c.counts, c.scan_tmp, L);
+    else
+        which = radix_sort<u64, int, false>(c.keys0, c.keys1, c.wa, c.wb, nullptr, E, 2 * sh, c.counts, c.scan_tmp, L);
+    const u64 *keys = which ? c.keys1 : c.keys0;
+    const int *w = which ? c.wb : c.wa;
+    k_heads<<<g, 256, 0, c.stream>>>(E, keys, c.flags);
+    ++c.launches;
+    device_scan<int>(c.flags, c.pos, nullptr, E, false, c.scan_tmp, c.d_nnz, L);
+    k_unique<<<g, 256, 0, c.stream>>>(E, keys, c.flags, c.pos, sh, c.rowid, c.bm_col, c.tmpi);
+    ++c.launches;
+    if (c.weighted) {
+        GSAP_CUDA(cudaMemsetAsync(c.bm_cnt, 0, sizeof(int) * (size_t)E, c.stream));
+        k_cnt_weighted<<<g, 256, 0, c.stream>>>(E, c.flags, c.pos, w, c.bm_cnt);
+    } else {
+        k_cnt_runs<<<g, 256, 0, c.stream>>>(E, c.tmpi, c.d_nnz, c.bm_cnt);
+    }
+    ++c.launches;
+    // CSR row pointers, cum, dout
+    k_ptr_from_ids<int><<<grid_for(B + 1, 256), 256, 0, c.stream>>>(c.rowid, c.d_nnz, E, B, c.bm_rowptr);
+    ++c.launches;
+    device_scan<int>(c.bm_cnt, c.tmpi, c.d_nnz, E, true, c.scan_tmp, nullptr, L);
+    k_seg_cum<<<g, 256, 0, c.stream>>>(c.rowid, c.bm_rowptr, c.tmpi, c.d_nnz, c.bm_cum);
+    k_seg_deg<<<grid_for(B, 256), 256, 0, c.stream>>>(B, c.bm_rowptr, c.tmpi, c.dout);
+    c.launches += 2;
+    // CSC: stable sort of the CSR entries by column (rows stay ascending)
+    k_csc_keys<<<g, 256, 0, c.stream>>>(c.d_nnz, c.bm_col, c.rowid, c.bm_cnt, c.ukeys0, c.vals64a);
+    ++c.launches;
+    const int w2 = radix_sort<unsigned, u64, true>(c.ukeys0, c.ukeys1, c.vals64a, c.vals64b, c.d_nnz, E, sh,
+                                                   c.counts, c.scan_tmp, L);
+    k_csc_unpack<<<g, 256, 0, c.stream>>>(c.d_nnz, w2 ? c.ukeys1 : c.ukeys0, w2 ? c.vals64b : c.vals64a,
+                                          c.flags, c.bm_row, c.bm_ccnt);
+    k_ptr_from_ids<int><<<grid_for(B + 1, 256), 256, 0, c.stream>>>(c.flags, c.d_nnz, E, B, c.bm_colptr);
+    c.launches += 2;
+    device_scan<int>(c.bm_ccnt, c.tmpi, c.d_nnz, E, true, c.scan_tmp, nullptr, L);
+    k_seg_cum<<<g, 256, 0, c.stream>>>(c.flags, c.bm_colptr, c.tmpi, c.d_nnz, c.bm_ccum);
+    k_seg_deg<<<grid_for(B, 256), 256, 0, c.stream>>>(B, c.bm_colptr, c.tmpi, c.din);
+    c.launches += 2;
+    GSAP_CHECK_LAUNCH();
+}
+
+void rebuild(Ctx &c) {
+    cudaEvent_t ev = nullptr;
+    kc_begin(c, c.k_rebuild, &ev);
+    c.dense_mode = dense_ok(c, c.B);
+    if (c.dense_mode) rebuild_dense(c);
+    else rebuild_sparse(c);
+    // algorithmic bytes: the compulsory inputs (dst ids,
+    // row pointers, b) and the fixed-size outputs (row / column pointers,
+    // degrees); the nnz-sized outputs are left out (nnz stays on the device)
+    const double bytes = 4.0 * c.E + 8.0 * c.V + 8.0 * (c.B + 1) + 8.0 * c.B;
+    kc_end(c, c.k_rebuild, ev, bytes);
+}
+
+}  // namespace gsap

@@ -1,0 +1,88 @@
+"""The C-ABI library loads and exports every symbol include/gsap.h declares (no GPU needed)."""
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def libgsap():
+    from paper_conf_icpp_changzh24_b200 import build
+    build.build()
+    return ctypes.CDLL(build.LIB)
+
+
+def declared():
+    src = open(os.path.join(ROOT, "include", "gsap.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(gsap_[a-z_]+)\s*\(", src)))
+
+
+def test_header_declares_the_north_star_calls():
+    names = declared()
+    for n in ("gsap_partition", "gsap_propose", "gsap_delta_mdl", "gsap_update_blockmodel", "gsap_mdl"):
+        assert n in names
+
+
+def test_every_declared_symbol_is_exported(libgsap):
+    for name in declared():
+        assert hasattr(libgsap, name), name
+
+
+def test_binding_covers_every_symbol(libgsap):
+    from paper_conf_icpp_changzh24_b200 import gsap
+    assert sorted(gsap.EXPORTED) == declared()
+
+
+def test_default_params_table2(libgsap):
+    from paper_conf_icpp_changzh24_b200 import gsap
+    p = gsap.gsap_default_params()
+    assert (p.reduction_rate, p.num_proposals, p.max_nodal_itr, p.thresh1, p.thresh2, p.window,
+            p.num_batches) == (0.4, 10, 100, 5e-4, 1e-4, 3, 4)        # Table 2
+    assert p.beta == 3.0 and p.seed == 0x5B9D2024
+
+
+def test_struct_layout_matches_header():
+    """ctypes mirrors of the header structs: field order / sizes (checked with gcc)."""
+    import subprocess
+    import tempfile
+    from paper_conf_icpp_changzh24_b200 import gsap
+    prog = r'''
+#include <stdio.h>
+#include <stddef.h>
+#include "gsap.h"
+int main(void){printf("%zu %zu %zu %zu %zu\n", sizeof(gsap_params), sizeof(gsap_stats), sizeof(gsap_dist),
+  offsetof(gsap_stats, k_move_ms), offsetof(gsap_params, profile));return 0;}
+'''
+    with tempfile.TemporaryDirectory() as d:
+        c = os.path.join(d, "t.c")
+        open(c, "w").write(prog)
+        exe = os.path.join(d, "t")
+        subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), c, "-o", exe])
+        got = list(map(int, subprocess.check_output([exe]).split()))
+    want = [ctypes.sizeof(gsap.gsap_params), ctypes.sizeof(gsap.gsap_stats), ctypes.sizeof(gsap.gsap_dist),
+            gsap.gsap_stats.k_move_ms.offset, gsap.gsap_params.profile.offset]
+    assert got == want
+
+
+def test_no_gpu_fails_loudly(libgsap):
+    """Without a device the product path returns an error; it never falls back to the CPU."""
+    import numpy as np
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    from paper_conf_icpp_changzh24_b200 import gsap
+    with pytest.raises(gsap.GsapError):
+        gsap.Context(np.array([0, 1], np.int64), np.array([0], np.int32))
+
+
+def test_product_never_imports_the_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_icpp_changzh24_b200")
+    for dp, _, fs in os.walk(pkg):
+        for f in fs:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                txt = open(os.path.join(dp, f)).read()
+                assert "oracle" not in re.sub(r"(#|//).*", "", txt).lower() or f == "__init__.py", f

@@ -1,0 +1,280 @@
+"""Parity of the CUDA path (libgsap.so through its C-ABI) against the CPU oracle.
+
+Layer 1 (bit-exact): proposals, blockmodel CSR/CSC/cnt/cum/degrees, merge
+selection + relabel, MCMC state after each batch (lockstep).  Layer 2 (1e-9):
+dS, H, MDL.  Layer 3: end-to-end MDL within 1% of the oracle.
+"""
+import numpy as np
+import pytest
+
+from gen import dcsbm
+from tests.helpers import close, ties
+
+pytestmark = pytest.mark.gpu
+
+SEED = dcsbm.RUN_SEED
+
+
+@pytest.fixture(scope="module")
+def G():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_icpp_changzh24_b200 import gsap
+    gsap.lib()
+    return gsap
+
+
+def make_pair(G, oracle_mod, rowptr, col, wgt=None, **params):
+    p = G.gsap_default_params(seed=SEED, **params)
+    ctx = G.Context(rowptr, col, wgt, params=p)
+    orc = oracle_mod.Oracle(rowptr, col, wgt)
+    return ctx, orc
+
+
+def set_both(ctx, orc, b, B):
+    ctx.gsap_set_partition(np.ascontiguousarray(b, np.int32), B)
+    orc.set_partition(b, B)
+
+
+def assert_same_blockmodel(ctx, orc):
+    g = ctx.gsap_get_blockmodel()
+    o = orc.blockmodel()
+    for k in ("rowptr", "col", "cnt", "cum", "colptr", "row", "ccnt", "ccum", "dout", "din"):
+        assert np.array_equal(g[k].astype(np.int64), o[k].astype(np.int64)), k
+
+
+GRAPHS = {
+    "multi": lambda: dcsbm.random_multigraph(300, 3000, 1),
+    "multi_w": lambda: dcsbm.random_multigraph(300, 3000, 2, weighted=True),
+    "dcsbm1k": lambda: dcsbm.make("1k")[:2] + (None,),
+}
+
+
+@pytest.mark.parametrize("gname", list(GRAPHS))
+@pytest.mark.parametrize("B", [1, 2, 7, 11, 150, 222, 299, 300])
+def test_rebuild_bit_exact(G, oracle_mod, gname, B):
+    rowptr, col, w = GRAPHS[gname]()
+    V = len(rowptr) - 1
+    B = min(B, V)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w)
+    assert_same_blockmodel(ctx, orc)      # singleton partition at create
+    b = dcsbm.random_partition(V, B, B)
+    set_both(ctx, orc, b, B)
+    assert_same_blockmodel(ctx, orc)
+
+
+def test_rebuild_20k_all_regimes(G, oracle_mod):
+    rowptr, col, truth, cfg = dcsbm.make("20k")
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    for B in (32, 1000, 1375, 1376, 5000, 20000):
+        b = dcsbm.random_partition(cfg.V, B, B)
+        set_both(ctx, orc, b, B)
+        assert_same_blockmodel(ctx, orc)
+        m_g, S_g = ctx.gsap_mdl()
+        m_o, S_o = orc.mdl()
+        assert abs(m_g - m_o) <= 1e-9 * abs(m_o)
+
+
+def _states(V, rng_seed):
+    rng = np.random.default_rng(rng_seed)
+    for B in (3, 40, 129, 400, V):
+        B = min(B, V)
+        yield B, dcsbm.random_partition(V, B, int(rng.integers(1 << 30)))
+
+
+@pytest.mark.parametrize("gname", list(GRAPHS))
+def test_move_proposals_dS_accept(G, oracle_mod, gname):
+    rowptr, col, w = GRAPHS[gname]()
+    V = len(rowptr) - 1
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w)
+    nties = 0
+    for B, b in _states(V, 5):
+        set_both(ctx, orc, b, B)
+        for outer, itr in ((0, 0), (3, 17)):
+            s = ctx.gsap_propose(G.GSAP_MOVE, outer, itr, 0, V)
+            s_o = orc.propose(1, SEED, outer, itr, 0, V)
+            assert np.array_equal(s, s_o), (B, outer, itr)
+            dS, H, acc = ctx.gsap_delta_mdl(G.GSAP_MOVE, outer, itr, 0, V, s)
+            dS_o, H_o, p_o, acc_o = orc.delta_move(SEED, outer, itr, 0, V, s_o)
+            assert np.all(close(dS, dS_o)), np.max(np.abs(dS - dS_o))
+            assert np.all(close(H, H_o, floor=1e-300))
+            t = ties(oracle_mod, SEED, outer, itr, range(V), p_o)
+            nties += int(t.sum())
+            assert np.array_equal(acc[~t], acc_o[~t])
+    print("MH ties:", nties)
+
+
+@pytest.mark.parametrize("gname", list(GRAPHS))
+def test_merge_proposals_dS_best(G, oracle_mod, gname):
+    rowptr, col, w = GRAPHS[gname]()
+    V = len(rowptr) - 1
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w)
+    for B, b in _states(V, 9):
+        if B < 2:
+            continue
+        set_both(ctx, orc, b, B)
+        for outer in (0, 5):
+            s = ctx.gsap_propose(G.GSAP_MERGE, outer, 0, 0, B)
+            s_o = orc.propose(0, SEED, outer, 0, 0, B)
+            assert np.array_equal(s, s_o), (B, outer)
+            dS = ctx.gsap_delta_mdl(G.GSAP_MERGE, outer, 0, 0, B, s)
+            dS_o = orc.delta_merge(0, B, s_o)
+            assert np.all(close(dS, dS_o)), np.max(np.abs(dS - dS_o))
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_select_merges_bit_exact(G, oracle_mod, seed):
+    rng = np.random.default_rng(seed)
+    V = 500
+    B = int(rng.integers(2, 400))
+    rowptr, col, _ = dcsbm.random_multigraph(V, 2000, seed)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    b = dcsbm.random_partition(V, B, seed)
+    if seed % 3 == 0:
+        b = np.where(b == 0, 1, b).astype(np.int32)    # an empty block
+    set_both(ctx, orc, b, B)
+    best = np.array([(r + 1 + rng.integers(0, B - 1)) % B for r in range(B)], np.int32)
+    dS = rng.integers(-4, 5, B).astype(np.float64) * 0.25   # heavy ties
+    dS[rng.random(B) < 0.1] = -0.0
+    K = int(0.4 * B)
+    lab, nb = ctx.gsap_select_merges(best, dS, K)
+    lab_o, nb_o = orc.select_merges(best, dS, K)
+    assert nb == nb_o and np.array_equal(lab, lab_o)
+    b_g, _ = ctx.gsap_get_partition()
+    b_o, _ = orc.partition()
+    assert np.array_equal(b_g, b_o)
+    assert_same_blockmodel(ctx, orc)
+
+
+def test_merge_phase_lockstep(G, oracle_mod):
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    for outer in range(4):
+        B = ctx.B
+        K = int(0.4 * B)
+        best, dSb = ctx.gsap_merge_phase(outer, K)
+        s_o = orc.propose(0, SEED, outer, 0, 0, B)
+        dS_o = orc.delta_merge(0, B, s_o)
+        best_o, dSb_o = orc.best_merges(s_o, dS_o)
+        assert np.array_equal(best, best_o)
+        assert np.all(close(dSb, dSb_o))
+        orc.select_merges(best, dSb, K)      # the GPU's dS decides the order (fp decoupling)
+        b_g, B_g = ctx.gsap_get_partition()
+        b_o, B_o = orc.partition()
+        assert B_g == B_o and np.array_equal(b_g, b_o)
+        assert_same_blockmodel(ctx, orc)
+
+
+@pytest.mark.parametrize("name", ["1k", "20k"])
+def test_mcmc_lockstep(G, oracle_mod, name):
+    """Batches of the fused hot loop vs the oracle, state compared after every batch."""
+    rowptr, col, truth, cfg = dcsbm.make(name)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    # start from a merged state (as after the first merge phases)
+    V = cfg.V
+    B = max(2, int(V ** 0.5))
+    b0 = dcsbm.random_partition(V, B, 3)
+    set_both(ctx, orc, b0, B)
+    bs = (V + 3) // 4
+    nties = 0
+    n_batches = 8 if name == "1k" else 4
+    for k in range(n_batches):
+        itr, batch = divmod(k, 4)
+        first = batch * bs
+        count = min(V, first + bs) - first
+        s_o = orc.propose(1, SEED, 1, itr, first, count)
+        dS_o, H_o, p_o, acc_o = orc.delta_move(SEED, 1, itr, first, count, s_o)
+        s, dS, acc, dsum = ctx.gsap_move_batch(1, itr, first, count)
+        assert np.array_equal(s, s_o)
+        assert np.all(close(dS, dS_o))
+        t = ties(oracle_mod, SEED, 1, itr, range(first, first + count), p_o)
+        nties += int(t.sum())
+        assert np.array_equal(acc[~t], acc_o[~t])
+        assert abs(dsum - float(np.sum(dS[acc == 1]))) <= 1e-9 * max(1.0, abs(dsum))
+        orc.apply_moves(first, count, s, acc)   # the GPU's decision on ties
+        orc.rebuild()
+        b_g, _ = ctx.gsap_get_partition()
+        b_o, _ = orc.partition()
+        assert np.array_equal(b_g, b_o)
+        assert_same_blockmodel(ctx, orc)
+    print("MH ties:", nties)
+
+
+def test_big_vertices_and_global_tables(G, oracle_mod):
+    """Hubs with > 128 and > 2048 distinct neighbour blocks (CTA path, global table)."""
+    rng = np.random.default_rng(0)
+    V = 6000
+    src = [rng.integers(0, V, 20000)]
+    dst = [rng.integers(0, V, 20000)]
+    for hub, deg in ((5, 200), (17, 3000), (4000, 5000)):
+        src.append(np.full(deg, hub))
+        dst.append(rng.choice(V, deg, replace=False))
+        src.append(rng.choice(V, deg // 2, replace=False))
+        dst.append(np.full(deg // 2, hub))
+    src = np.concatenate(src)
+    dst = np.concatenate(dst)
+    order = np.argsort(src, kind="stable")
+    rowptr = np.zeros(V + 1, np.int64)
+    np.add.at(rowptr, src[order] + 1, 1)
+    rowptr = np.cumsum(rowptr)
+    col = dst[order].astype(np.int32)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    for B in (100, 3000, V):
+        b = dcsbm.random_partition(V, B, B)
+        set_both(ctx, orc, b, B)
+        s = ctx.gsap_propose(G.GSAP_MOVE, 2, 3, 0, V)
+        s_o = orc.propose(1, SEED, 2, 3, 0, V)
+        assert np.array_equal(s, s_o)
+        dS, H, acc = ctx.gsap_delta_mdl(G.GSAP_MOVE, 2, 3, 0, V, s)
+        dS_o, H_o, p_o, acc_o = orc.delta_move(SEED, 2, 3, 0, V, s_o)
+        assert np.all(close(dS, dS_o)), np.max(np.abs(dS - dS_o))
+        assert np.all(close(H, H_o, floor=1e-300))
+
+
+def test_edge_cases(G, oracle_mod):
+    # no edges at all
+    rowptr = np.zeros(6, np.int64)
+    col = np.zeros(0, np.int32)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    assert_same_blockmodel(ctx, orc)
+    s = ctx.gsap_propose(G.GSAP_MOVE, 0, 0, 0, 5)
+    assert np.array_equal(s, orc.propose(1, SEED, 0, 0, 0, 5))
+    dS, H, acc = ctx.gsap_delta_mdl(G.GSAP_MOVE, 0, 0, 0, 5, s)
+    assert np.all(dS == 0) and np.all(H == 1)
+    res = ctx.gsap_run()
+    ref = orc.partition_run()
+    assert res["B"] == ref["B"]
+    # a single vertex with a self-loop
+    ctx1, orc1 = make_pair(G, oracle_mod, np.array([0, 1], np.int64), np.array([0], np.int32))
+    r1 = ctx1.gsap_run()
+    assert r1["B"] == 1 and r1["b"].tolist() == [0]
+    # bad arguments are reported, not crashed
+    with pytest.raises(G.GsapError):
+        ctx.gsap_set_partition(np.array([0, 1, 2, 3, 9], np.int32), 5)
+    with pytest.raises(G.GsapError):
+        G.Context(np.array([0, 2], np.int64), np.array([0, 5], np.int32))
+
+
+def test_end_to_end_1k(G, oracle_mod):
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    res = ctx.gsap_run()
+    ref = orc.partition_run()
+    assert abs(res["mdl"] - ref["mdl"]) <= 0.01 * ref["mdl"]
+    from sklearn.metrics import normalized_mutual_info_score as nmi
+    print("GPU", res["B"], res["mdl"], nmi(truth, res["b"]), "oracle", ref["B"], ref["mdl"],
+          nmi(truth, ref["b"]))
+    # trajectories agree until the first floating-point tie (normally never)
+    same = np.array_equal(res["b"], ref["b"])
+    print("bit-identical final partition:", same)
+    assert res["trace"].shape == ref["trace"].shape or not same
+
+
+def test_partition_oneshot_matches_context(G, oracle_mod):
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    out = G.gsap_partition(rowptr, col, params=G.gsap_default_params(seed=SEED))
+    ctx = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED))
+    res = ctx.gsap_run()
+    assert np.array_equal(out["b"], res["b"]) and out["B"] == res["B"]
+    assert out["stats"]["gpu_launches"] > 0 and out["stats"]["n_move_prop"] > 0
