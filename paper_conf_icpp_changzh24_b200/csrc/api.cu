@@ -147,7 +147,8 @@ static void check_sm100() {
 static void free_ctx(Ctx &c) {
     void *ptrs[] = {c.rowptr, c.col, c.wgt, c.cscptr, c.cscsrc, c.cscwgt, c.esrc, c.kout, c.kin, c.selfw,
                     c.big, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
-                    c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT, c.keys0,
+                    c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT, c.rtab,
+                    c.rcp, c.fh, c.fl, c.keys0,
                     c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
                     c.rowid, c.counts, c.scan_tmp, c.rownnz, c.s, c.dS, c.H, c.acc, c.best, c.dSbest,
                     c.partials, c.scal, c.scal_i, c.Dh, c.skey0, c.skey1, c.sval0, c.sval1, c.rank,
@@ -252,7 +253,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     if (!c.h_big.empty()) {
         c.big = dalloc<int>(c.h_big.size());
         const int log2cap = std::max(log2_ceil_h(2LL * std::min(kmax_big, V)), 5);
-        if ((1 << log2cap) > 4096) {
+        if ((1 << log2cap) > 2048) {
             c.big_table_slots = (size_t)296 << log2cap;
             c.big_tables = dalloc<int>(c.big_table_slots * 4);
         }
@@ -272,6 +273,21 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, 65536), (size_t)1 << 28);
     c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
     c.dense = dalloc<int>(c.dense_cap);
+    c.rtab = dalloc<int2>(2 * Es);
+    c.rcp = dalloc<double>(Vs);
+    {   // f-table: f(m) = m ln m in long double, split into double hi + float lo
+        std::vector<double> fh(FT_N);
+        std::vector<float> fl(FT_N);
+        for (int m = 0; m < FT_N; ++m) {
+            const long double f = m > 0 ? (long double)m * logl((long double)m) : 0.0L;
+            fh[m] = (double)f;
+            fl[m] = (float)(f - (long double)fh[m]);
+        }
+        c.fh = dalloc<double>(FT_N);
+        c.fl = dalloc<float>(FT_N);
+        GSAP_CUDA(cudaMemcpy(c.fh, fh.data(), sizeof(double) * FT_N, cudaMemcpyHostToDevice));
+        GSAP_CUDA(cudaMemcpy(c.fl, fl.data(), sizeof(float) * FT_N, cudaMemcpyHostToDevice));
+    }
     c.denseT = dalloc<int>(c.dense_cap);
     c.keys0 = dalloc<unsigned long long>(Es);
     c.keys1 = dalloc<unsigned long long>(Es);
@@ -297,7 +313,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.acc = dalloc<unsigned char>(Vs);
     c.best = dalloc<int>(Vs);
     c.dSbest = dalloc<double>(Vs);
-    c.partials = dalloc<double>(VE / 4096 + 64);
+    c.partials = dalloc<double>(VE / 512 + 64);   // >= max(E, B) / MDL_CHUNK, V / APPLY_CHUNK
     c.scal = dalloc<double>(8);
     c.scal_i = dalloc<int>(8);
     c.Dh = dalloc<double>((size_t)c.prm.max_nodal_itr + 1);
@@ -475,10 +491,11 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
         t_move += std::chrono::duration<double>(tc - tb).count();
         t_mdl += std::chrono::duration<double>(td - tc).count();
         if (trace && rounds < trace_cap) {
-            trace[4 * rounds + 0] = (double)outer;
-            trace[4 * rounds + 1] = (double)B;
-            trace[4 * rounds + 2] = (double)itrs;
-            trace[4 * rounds + 3] = S;
+            trace[5 * rounds + 0] = (double)outer;
+            trace[5 * rounds + 1] = (double)B;
+            trace[5 * rounds + 2] = (double)itrs;
+            trace[5 * rounds + 3] = S;
+            trace[5 * rounds + 4] = std::chrono::duration<double>(td - ta).count();
         }
         c.st.mcmc_itr_total += itrs;
         ++rounds;

@@ -48,21 +48,69 @@ GSAP_DEV bool coin_random(uint32_t w1, uint32_t B, uint32_t d) {
 
 // ------------------------------------------------------------- entropy --
 // f(m) = m ln m.  df(m, d) = f(m + d) - f(m) for integers m >= 0, m + d >= 0,
-// written without cancellation: d ln(m + d) + m log1p(d / m).
+// without cancellation: d ln(m + d) + m log1p(d / m), the second term by its
+// series when |d / m| <= 2^-7; below FT_N both f's come from a double-double
+// table (written on the host in long double), so most terms need no
+// transcendental at all.
+constexpr int FT_N = 1 << 16;
+
 GSAP_DEV double fx(double m) { return m > 0.0 ? m * log(m) : 0.0; }
 
-GSAP_DEV double df(long long m, long long d) {
-    if (d == 0) return 0.0;
+GSAP_DEV double ftab(const double *__restrict__ fh, const float *__restrict__ fl, long long n) {
+    return __ldg(fh + n) + (double)__ldg(fl + n);
+}
+
+GSAP_DEV double df_big(long long m, long long d) {
     const long long n = m + d;
     if (m == 0) return fx((double)n);
     if (n == 0) return -fx((double)m);
-    return (double)d * log((double)n) + (double)m * log1p((double)d / (double)m);
+    const double x = (double)d / (double)m;
+    double tail;
+    if (fabs(x) <= 0.0078125) {
+        // m log1p(x) = d (1 - x/2 + x^2/3 - x^3/4 + x^4/5 - x^5/6 + x^6/7 - x^7/8 + ...)
+        double p = -1.0 / 8.0;
+        p = fma(p, x, 1.0 / 7.0);
+        p = fma(p, x, -1.0 / 6.0);
+        p = fma(p, x, 1.0 / 5.0);
+        p = fma(p, x, -1.0 / 4.0);
+        p = fma(p, x, 1.0 / 3.0);
+        p = fma(p, x, -1.0 / 2.0);
+        tail = fma((double)d * x, p, (double)d);
+    } else {
+        tail = (double)m * log1p(x);
+    }
+    return fma((double)d, log((double)n), tail);
+}
+
+GSAP_DEV double df_t(const double *__restrict__ fh, const float *__restrict__ fl, long long m, long long d) {
+    if (d == 0) return 0.0;
+    const long long n = m + d;
+    if (m < FT_N && n < FT_N)
+        return (__ldg(fh + n) - __ldg(fh + m)) + (double)(__ldg(fl + n) - __ldg(fl + m));
+    return df_big(m, d);
 }
 
 // g(a, c) = f(a + c) - f(a) - f(c) = a log1p(c/a) + c log1p(a/c)
 GSAP_DEV double g2(long long a, long long c) {
     if (a == 0 || c == 0) return 0.0;
     return (double)a * log1p((double)c / (double)a) + (double)c * log1p((double)a / (double)c);
+}
+
+GSAP_DEV double g2_t(const double *__restrict__ fh, const float *__restrict__ fl, long long a, long long c) {
+    if (a == 0 || c == 0) return 0.0;
+    if (a + c < FT_N)
+        return ((__ldg(fh + a + c) - __ldg(fh + a)) - __ldg(fh + c)) +
+               (double)((__ldg(fl + a + c) - __ldg(fl + a)) - __ldg(fl + c));
+    return g2(a, c);
+}
+
+// legacy exact-math form (tests of the table path compare against it)
+GSAP_DEV double df(long long m, long long d) {
+    if (d == 0) return 0.0;
+    const long long n = m + d;
+    if (m == 0) return fx((double)n);
+    if (n == 0) return -fx((double)m);
+    return (double)d * log((double)n) + (double)m * log1p((double)d / (double)m);
 }
 
 // -------------------------------------------------------------- warps --
@@ -92,6 +140,11 @@ GSAP_DEV int warp_incl_scan(int v) {
 struct BM {
     int B;
     const int *__restrict__ dense;   // nullptr in the sparse regime
+    const int2 *__restrict__ rtab;   // sparse regime: per-row open-addressing tables {col, cnt},
+                                     // row x owns slots [2 rowptr[x], 2 rowptr[x+1])
+    const double *__restrict__ fh;   // f(m) = m ln m for m < FT_N, double-double (hi, lo)
+    const float *__restrict__ fl;
+    const double *__restrict__ rcp;  // 1 / (d_x + B) per block
     const int *__restrict__ rowptr;  // [B+1]
     const int *__restrict__ col;
     const int *__restrict__ cnt;
@@ -114,16 +167,50 @@ GSAP_DEV int upper_bound(const int *__restrict__ a, int lo, int hi, long long p)
     return lo;
 }
 
+// ---- per-row hash tables (sparse regime): row x has 2 len(x) slots {col, cnt},
+// col = -1 empty, home slot = multiply-shift of the column, linear probing.
+GSAP_DEV unsigned col_mix(int y) { return (unsigned)y * 0x9E3779B1u; }
+
+GSAP_DEV int rtab_get(const BM &m, int x, int y) {
+    const int lo = __ldg(m.rowptr + x), cap = 2 * (__ldg(m.rowptr + x + 1) - lo);
+    if (cap == 0) return 0;
+    const int2 *__restrict__ t = m.rtab + 2 * (size_t)lo;
+    int sl = (int)pick(col_mix(y), (uint32_t)cap);
+    while (true) {
+        const int2 e = __ldg(t + sl);
+        if (e.x == y) return e.y;
+        if (e.x == -1) return 0;
+        if (++sl == cap) sl = 0;
+    }
+}
+
 GSAP_DEV int bm_at(const BM &m, int x, int y) {
     if (m.dense) return __ldg(m.dense + (size_t)x * m.B + y);
-    const int lo = __ldg(m.rowptr + x), hi = __ldg(m.rowptr + x + 1);
-    int a = lo, b = hi;
-    while (a < b) {
-        const int mid = (a + b) >> 1;
-        if (__ldg(m.col + mid) < y) a = mid + 1;
-        else b = mid;
+    return rtab_get(m, x, y);
+}
+
+// first index i in [lo, hi) with a[i] > p, whole warp (32-ary search: one
+// dependent load per factor 32 of the range); hi if none.  Warp-uniform.
+GSAP_DEV int warp_upper_bound(const int *__restrict__ a, int lo, int hi, long long p) {
+    const int lane = (int)(threadIdx.x & 31);
+    while (hi - lo > 32) {
+        const int step = (hi - lo + 31) >> 5;
+        const int idx = lo + lane * step;
+        const bool gt = idx < hi && (long long)__ldg(a + idx) > p;
+        const unsigned bal = __ballot_sync(FULL, gt);
+        if (bal == 0) {
+            const int last = min(31, (hi - 1 - lo) / step);
+            lo = lo + last * step + 1;
+        } else {
+            const int f = __ffs(bal) - 1;   // a[lo + f*step] > p, a[lo + (f-1)*step] <= p
+            const int nlo = f > 0 ? lo + (f - 1) * step + 1 : lo;
+            hi = lo + f * step + 1;
+            lo = nlo;
+        }
     }
-    return (a < hi && __ldg(m.col + a) == y) ? __ldg(m.cnt + a) : 0;
+    const int idx = lo + lane;
+    const unsigned bal = __ballot_sync(FULL, idx < hi && (long long)__ldg(a + idx) > p);
+    return bal ? lo + __ffs(bal) - 1 : hi;
 }
 
 GSAP_DEV int bm_deg(const BM &m, int x) { return __ldg(m.dout + x) + __ldg(m.din + x); }
@@ -164,6 +251,17 @@ GSAP_DEV int bm_walk(const BM &m, int u, long long p, int skip) {
         }
     }
     return __ldg(m.row + upper_bound(m.ccum, clo, chi, q));
+}
+
+// bm_walk without skipping, whole warp (MOVE proposals)
+GSAP_DEV int bm_walk_warp(const BM &m, int u, long long p) {
+    const int dout_u = __ldg(m.dout + u);
+    if (p < dout_u) {
+        const int i = warp_upper_bound(m.cum, __ldg(m.rowptr + u), __ldg(m.rowptr + u + 1), p);
+        return __ldg(m.col + i);
+    }
+    const int i = warp_upper_bound(m.ccum, __ldg(m.colptr + u), __ldg(m.colptr + u + 1), p - dout_u);
+    return __ldg(m.row + i);
 }
 
 }  // namespace gsap

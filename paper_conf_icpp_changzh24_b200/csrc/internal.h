@@ -51,6 +51,10 @@ struct Ctx {
     int *bm_colptr = nullptr, *bm_row = nullptr, *bm_ccnt = nullptr, *bm_ccum = nullptr;
     int *dout = nullptr, *din = nullptr, *d_nnz = nullptr;
     int *dense = nullptr, *denseT = nullptr;
+    int2 *rtab = nullptr;          // sparse-regime per-row hash tables (2 slots per entry)
+    double *fh = nullptr;          // f-table hi / lo (FT_N entries)
+    float *fl = nullptr;
+    double *rcp = nullptr;         // 1 / (d_x + B), refreshed by every rebuild
     size_t dense_cap = 0;   // elements
     bool dense_mode = false;
 
@@ -92,6 +96,10 @@ struct Ctx {
         BM m;
         m.B = B;
         m.dense = dense_mode ? dense : nullptr;
+        m.rtab = rtab;
+        m.fh = fh;
+        m.fl = fl;
+        m.rcp = rcp;
         m.rowptr = bm_rowptr; m.col = bm_col; m.cnt = bm_cnt; m.cum = bm_cum;
         m.colptr = bm_colptr; m.row = bm_row; m.ccnt = bm_ccnt; m.ccum = bm_ccum;
         m.dout = dout; m.din = din;

@@ -2,7 +2,7 @@
 // Z1-Z4, Z22):
 //   S   = -sum_xy f(M_xy) + sum_x f(dout_x) + sum_y f(din_y),  f(m) = m ln m
 //   MDL = E h(B^2/E) + V ln B + S,  h(x) = (1 + x) ln(1 + x) - x ln x.
-// The data term is a fixed-chunk fp64 reduction (chunk = 8192 entries per
+// The data term is a fixed-chunk fp64 reduction (chunk = 2048 entries per
 // CTA, then one ordered pass), so it does not depend on the launch shape.
 #include <math.h>
 
@@ -12,7 +12,7 @@
 
 namespace gsap {
 
-constexpr int MDL_CHUNK = 8192;
+constexpr int MDL_CHUNK = 2048;
 
 __global__ void __launch_bounds__(256) k_mdl_partials(const int *__restrict__ cnt, const int *__restrict__ d_nnz,
                                                       const int *__restrict__ dout, const int *__restrict__ din,

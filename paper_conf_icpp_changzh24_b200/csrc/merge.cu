@@ -48,7 +48,8 @@ GSAP_DEV int propose_merge(const BM &m, int r, uint32_t j, uint64_t seed, uint32
 // row b of the same structure; lookups of the other side via lookup(t)
 template <typename Lookup>
 GSAP_DEV double inter_sum(const int *__restrict__ ptr, const int *__restrict__ idx, const int *__restrict__ cnt,
-                          int a, int b, int r, int s, Lookup lookup) {
+                          int a, int b, int r, int s, const double *__restrict__ fh, const float *__restrict__ fl,
+                          Lookup lookup) {
     const int alo = __ldg(ptr + a), ahi = __ldg(ptr + a + 1);
     const int blo = __ldg(ptr + b), bhi = __ldg(ptr + b + 1);
     const bool walk_a = (ahi - alo) <= (bhi - blo);
@@ -59,22 +60,24 @@ GSAP_DEV double inter_sum(const int *__restrict__ ptr, const int *__restrict__ i
         if (t == r || t == s) continue;
         const int m1 = __ldg(cnt + i);
         const int m2 = lookup(other, t);
-        acc += g2(m1, m2);
+        acc += g2_t(fh, fl, m1, m2);
     }
     return acc;
 }
 
 GSAP_DEV double merge_delta(const BM &m, int r, int s) {
     // rows r, s (t in both supports): g(M_st, M_rt)
-    double acc = inter_sum(m.rowptr, m.col, m.cnt, r, s, r, s,
+    double acc = inter_sum(m.rowptr, m.col, m.cnt, r, s, r, s, m.fh, m.fl,
                            [&](int x, int t) { return bm_at(m, x, t); });
     // columns r, s: g(M_ts, M_tr)
-    acc += inter_sum(m.colptr, m.row, m.ccnt, r, s, r, s, [&](int y, int t) { return bm_at(m, t, y); });
+    acc += inter_sum(m.colptr, m.row, m.ccnt, r, s, r, s, m.fh, m.fl, [&](int y, int t) { return bm_at(m, t, y); });
     acc = warp_sum(acc);
     const long long Mss = bm_at(m, s, s), Msr = bm_at(m, s, r), Mrs = bm_at(m, r, s), Mrr = bm_at(m, r, r);
     // f(a+b+c+d) - f(a) - f(b) - f(c) - f(d), telescoped into g's
-    const double core = g2(Mss, Msr) + g2(Mss + Msr, Mrs) + g2(Mss + Msr + Mrs, Mrr);
-    const double deg = g2(__ldg(m.dout + s), __ldg(m.dout + r)) + g2(__ldg(m.din + s), __ldg(m.din + r));
+    const double core = g2_t(m.fh, m.fl, Mss, Msr) + g2_t(m.fh, m.fl, Mss + Msr, Mrs) +
+                        g2_t(m.fh, m.fl, Mss + Msr + Mrs, Mrr);
+    const double deg = g2_t(m.fh, m.fl, __ldg(m.dout + s), __ldg(m.dout + r)) +
+                       g2_t(m.fh, m.fl, __ldg(m.din + s), __ldg(m.din + r));
     return -acc - core + deg;
 }
 

@@ -27,8 +27,9 @@ constexpr int WARP_TAB = 256;          // slots per warp table (<= 128 keys)
 constexpr int WARP_TAB_LOG2 = 8;
 constexpr int BIG_THR = 128;           // warp path iff min(k_v, B) <= BIG_THR
 constexpr int MOVE_WARPS = 8;          // warps per CTA, warp kernel
-constexpr int CTA_THREADS = 256;       // big-vertex kernel
-constexpr int CTA_SMEM_SLOTS = 4096;   // shared table of the big-vertex kernel (64 KB)
+constexpr int CTA_THREADS = 256;       // big-vertex role: one CTA per vertex
+constexpr int CTA_SMEM_SLOTS = MOVE_WARPS * WARP_TAB;   // big-vertex shared table (<= 1024 keys)
+constexpr int BIG_CTAS_MAX = 296;      // CTAs of the big-vertex role (grid-stride)
 
 struct MoveArgs {
     int B;
@@ -46,8 +47,9 @@ struct MoveArgs {
     int *s_out;
     double *dS, *H;
     unsigned char *acc;
-    int4 *gtab;                     // global tables (big-vertex kernel), per CTA
+    int4 *gtab;                     // global tables (big-vertex role), per CTA, or nullptr
     int gtab_log2;
+    int nbig_ctas;                  // CTAs [0, nbig_ctas) take the big-vertex role
 };
 
 GSAP_DEV unsigned hash_slot(int t, int log2cap) {
@@ -114,7 +116,7 @@ GSAP_DEV int propose_move(const MoveArgs &a, int v, uint4 w) {
     const int u = __ldg(a.b + n);
     const uint32_t du = (uint32_t)bm_deg(a.m, u);
     if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
-    return bm_walk(a.m, u, (long long)pick(w.z, du), -1);
+    return bm_walk_warp(a.m, u, (long long)pick(w.z, du));
 }
 
 // group-wide sums (deterministic fixed trees)
@@ -173,6 +175,9 @@ GSAP_DEV void eval_move(const MoveArgs &a, int v, int s, uint4 w, int4 *tab, int
     const long long dr2 = dr - kout - kin, ds2 = ds + kout + kin;
     const double Bd = (double)B;
     // phase B: the owner of each unique t adds its terms
+    const double *__restrict__ fh = a.m.fh;
+    const float *__restrict__ fl = a.m.fl;
+    const double *__restrict__ rcp = a.m.rcp;
     double accS = 0.0, pf = 0.0, pb = 0.0;
     for (int j = gt; j < deg; j += G) {
         const bool out = j < nout;
@@ -185,33 +190,38 @@ GSAP_DEV void eval_move(const MoveArgs &a, int v, int s, uint4 w, int4 *tab, int
         const long long ot = e.y, it = e.z;
         const double c = (double)(ot + it);
         if (t == r) {
-            pf += c * (double)(Mrs + Msr + 1) / ((double)dr + Bd);
+            pf += c * (double)(Mrs + Msr + 1) * __ldg(rcp + r);
             pb += c * (double)(2 * Mrr2 + 1) / ((double)dr2 + Bd);
         } else if (t == s) {
-            pf += c * (double)(2 * Mss + 1) / ((double)ds + Bd);
+            pf += c * (double)(2 * Mss + 1) * __ldg(rcp + s);
             pb += c * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd);
         } else {
             const long long Mrt = bm_at(a.m, r, t), Mst = bm_at(a.m, s, t);
             const long long Mtr = bm_at(a.m, t, r), Mts = bm_at(a.m, t, s);
-            const double dt = (double)bm_deg(a.m, t);
-            accS -= df(Mrt, -ot) + df(Mst, ot) + df(Mtr, -it) + df(Mts, it);
-            pf += c * (double)(Mts + Mst + 1) / (dt + Bd);
-            pb += c * (double)(Mtr - it + Mrt - ot + 1) / (dt + Bd);
+            const double rt = __ldg(rcp + t);
+            accS -= df_t(fh, fl, Mrt, -ot) + df_t(fh, fl, Mst, ot) + df_t(fh, fl, Mtr, -it) + df_t(fh, fl, Mts, it);
+            pf += c * (double)(Mts + Mst + 1) * rt;
+            pb += c * (double)(Mtr - it + Mrt - ot + 1) * rt;
         }
     }
-    accS = group_sum<G>(accS, sh);
+    // the 2x2 core, the four degree terms and the self-loop terms, one per thread
+    if (gt < 10) {
+        switch (gt) {
+            case 0: accS -= df_t(fh, fl, Mrr, -(o_r + i_r + l)); break;
+            case 1: accS -= df_t(fh, fl, Mrs, i_r - o_s); break;
+            case 2: accS -= df_t(fh, fl, Msr, o_r - i_s); break;
+            case 3: accS -= df_t(fh, fl, Mss, o_s + i_s + l); break;
+            case 4: accS += df_t(fh, fl, __ldg(a.m.dout + r), -kout); break;
+            case 5: accS += df_t(fh, fl, __ldg(a.m.dout + s), kout); break;
+            case 6: accS += df_t(fh, fl, __ldg(a.m.din + r), -kin); break;
+            case 7: accS += df_t(fh, fl, __ldg(a.m.din + s), kin); break;
+            case 8: if (l > 0) pf += 2.0 * (double)l * (double)(Mrs + Msr + 1) * __ldg(rcp + r); break;
+            default: if (l > 0) pb += 2.0 * (double)l * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd); break;
+        }
+    }
+    const double dS = group_sum<G>(accS, sh);
     pf = group_sum<G>(pf, sh);
     pb = group_sum<G>(pb, sh);
-    // core, degree and self-loop terms
-    double dS = accS;
-    dS -= df(Mrr, -(o_r + i_r + l)) + df(Mrs, i_r - o_s) + df(Msr, o_r - i_s) + df(Mss, o_s + i_s + l);
-    const long long dout_r = __ldg(a.m.dout + r), dout_s = __ldg(a.m.dout + s);
-    const long long din_r = __ldg(a.m.din + r), din_s = __ldg(a.m.din + s);
-    dS += df(dout_r, -kout) + df(dout_s, kout) + df(din_r, -kin) + df(din_s, kin);
-    if (l > 0) {
-        pf += 2.0 * (double)l * (double)(Mrs + Msr + 1) / ((double)dr + Bd);
-        pb += 2.0 * (double)l * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd);
-    }
     const double H = (kout + kin == 0) ? 1.0 : pb / pf;
     const double p = exp(-a.beta * dS) * H;
     const double u = ((double)w.w + 0.5) * (1.0 / 4294967296.0);
@@ -259,17 +269,34 @@ GSAP_DEV void do_vertex(const MoveArgs &a, int mode, int v, int4 *tab, int log2c
     }
 }
 
-// one warp per vertex of [first, first + count); skips the big vertices
+// One launch, two roles: CTAs [0, nbig_ctas) take the vertices of a.list
+// (whose neighbour-block count can exceed 128) one CTA per vertex; the other
+// CTAs take every other vertex of [first, first + count) one warp per vertex.
+// The shared memory is the 8 warp tables, or one CTA table over the same bytes.
 template <bool WEIGHTED>
-__global__ void __launch_bounds__(MOVE_WARPS * 32) k_move_warp(MoveArgs a, int mode) {
-    __shared__ int4 tabs[MOVE_WARPS][WARP_TAB];
+__global__ void __launch_bounds__(MOVE_WARPS * 32, 3) k_move(MoveArgs a, int mode) {
+    __shared__ int4 tabs[MOVE_WARPS * WARP_TAB];
+    __shared__ double sh[MOVE_WARPS];
+    __shared__ int bcast;
     const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    int4 *tab = tabs[wl];
+    if ((int)blockIdx.x < a.nbig_ctas) {
+        int4 *tab = a.gtab ? a.gtab + ((size_t)blockIdx.x << a.gtab_log2) : tabs;
+        const int log2cap = a.gtab_log2;
+        for (int li = blockIdx.x; li < a.list_count; li += a.nbig_ctas) {
+            const int v = a.list[li];
+            tab_clear<CTA_THREADS>(tab, 1 << log2cap, threadIdx.x);
+            __syncthreads();
+            do_vertex<CTA_THREADS, WEIGHTED>(a, mode, v, tab, log2cap, threadIdx.x, sh, &bcast);
+            __syncthreads();
+        }
+        return;
+    }
+    int4 *tab = tabs + wl * WARP_TAB;
     tab_clear<32>(tab, WARP_TAB, lane);
     __syncwarp();
-    const int nwarps = gridDim.x * MOVE_WARPS;
+    const int nwarps = (gridDim.x - a.nbig_ctas) * MOVE_WARPS;
     const bool skip_big = a.B > BIG_THR;
-    for (int i = blockIdx.x * MOVE_WARPS + wl; i < a.count; i += nwarps) {
+    for (int i = (blockIdx.x - a.nbig_ctas) * MOVE_WARPS + wl; i < a.count; i += nwarps) {
         const int v = a.first + i;
         // adjacency entries bound the number of unique neighbour blocks
         if (skip_big &&
@@ -279,23 +306,6 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32) k_move_warp(MoveArgs a, int m
         __syncwarp();
         tab_clear<32>(tab, WARP_TAB, lane);
         __syncwarp();
-    }
-}
-
-// one CTA per big vertex (grid-stride over a.list)
-template <bool WEIGHTED>
-__global__ void __launch_bounds__(CTA_THREADS) k_move_cta(MoveArgs a, int mode) {
-    extern __shared__ int4 stab[];
-    __shared__ double sh[CTA_THREADS / 32];
-    __shared__ int bcast;
-    int4 *tab = a.gtab ? a.gtab + ((size_t)blockIdx.x << a.gtab_log2) : stab;
-    const int log2cap = a.gtab_log2;
-    for (int li = blockIdx.x; li < a.list_count; li += gridDim.x) {
-        const int v = a.list[li];
-        tab_clear<CTA_THREADS>(tab, 1 << log2cap, threadIdx.x);
-        __syncthreads();
-        do_vertex<CTA_THREADS, WEIGHTED>(a, mode, v, tab, log2cap, threadIdx.x, sh, &bcast);
-        __syncthreads();
     }
 }
 
@@ -331,14 +341,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     a.gtab = nullptr;
     a.gtab_log2 = 0;
     const int m = (int)mode;
-    {
-        const long long need = ((long long)count + MOVE_WARPS - 1) / MOVE_WARPS;
-        const int grid = (int)std::min<long long>(need, 148LL * 8);
-        if (c.weighted) k_move_warp<true><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a, m);
-        else k_move_warp<false><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a, m);
-        ++c.launches;
-        GSAP_CHECK_LAUNCH();
-    }
+    a.nbig_ctas = 0;
     if (c.B > BIG_THR && !c.h_big.empty()) {
         // the big vertices inside [first, first + count)
         const auto lo = std::lower_bound(c.h_big.begin(), c.h_big.end(), first);
@@ -353,31 +356,21 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
                 kmax = std::max(kmax, (c.h_rowptr[v + 1] - c.h_rowptr[v]) + (c.h_cscptr[v + 1] - c.h_cscptr[v]));
             }
             const int log2cap = std::max(log2_ceil(2LL * std::min(kmax, c.B)), 5);
-            size_t smem = 0;
-            int grid;
-            if ((1 << log2cap) <= CTA_SMEM_SLOTS) {
-                smem = sizeof(int4) << log2cap;
-                grid = nbig;
-            } else {
-                grid = (int)std::min<long long>(nbig, (long long)(c.big_table_slots >> log2cap));
-                if (grid < 1) throw Error{GSAP_ENOMEM, "big-vertex table too small"};
+            a.gtab_log2 = log2cap;
+            a.nbig_ctas = std::min(nbig, BIG_CTAS_MAX);
+            if ((1 << log2cap) > CTA_SMEM_SLOTS) {
+                if (((size_t)a.nbig_ctas << log2cap) > c.big_table_slots)
+                    throw Error{GSAP_ENOMEM, "big-vertex table too small"};
                 a.gtab = reinterpret_cast<int4 *>(c.big_tables);
             }
-            a.gtab_log2 = log2cap;
-            static bool attr = false;
-            if (!attr) {
-                GSAP_CUDA(cudaFuncSetAttribute(k_move_cta<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                               CTA_SMEM_SLOTS * (int)sizeof(int4)));
-                GSAP_CUDA(cudaFuncSetAttribute(k_move_cta<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                               CTA_SMEM_SLOTS * (int)sizeof(int4)));
-                attr = true;
-            }
-            if (c.weighted) k_move_cta<true><<<grid, CTA_THREADS, smem, c.stream>>>(a, m);
-            else k_move_cta<false><<<grid, CTA_THREADS, smem, c.stream>>>(a, m);
-            ++c.launches;
-            GSAP_CHECK_LAUNCH();
         }
     }
+    const long long need = ((long long)count + MOVE_WARPS - 1) / MOVE_WARPS;
+    const int grid = a.nbig_ctas + (int)std::max<long long>(1, std::min<long long>(need, 148LL * 8));
+    if (c.weighted) k_move<true><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a, m);
+    else k_move<false><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a, m);
+    ++c.launches;
+    GSAP_CHECK_LAUNCH();
     // algorithmic bytes: adjacency ids (+ weights),
     // row / column pointers, b[v], the outputs (s, dS, acc)
     const long long adj = (long long)(c.h_rowptr[first + count] - c.h_rowptr[first]) +
@@ -387,7 +380,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
 }
 
 // ---------------------------------------------------------------- apply --
-constexpr int APPLY_CHUNK = 4096;
+constexpr int APPLY_CHUNK = 1024;
 
 __global__ void __launch_bounds__(256) k_apply(int first, int count, const int *__restrict__ s,
                                                const unsigned char *__restrict__ acc,

@@ -341,6 +341,32 @@ __global__ void k_csc_unpack(const int *__restrict__ d_n, const unsigned *__rest
     }
 }
 
+// per-row hash tables of M used for O(1) lookups in the sparse regime
+__global__ void k_rtab_clear(const int *__restrict__ d_n, int2 *__restrict__ tab) {
+    const long long n = 2LL * *d_n;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        tab[i] = make_int2(-1, 0);
+}
+
+__global__ void k_rtab_insert(const int *__restrict__ d_n, const int *__restrict__ rowid, const int *__restrict__ col,
+                              const int *__restrict__ cnt, const int *__restrict__ rowptr, int2 *__restrict__ tab) {
+    const int n = *d_n;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        const int x = rowid[i], y = col[i];
+        const int lo = rowptr[x], cap = 2 * (rowptr[x + 1] - lo);
+        int2 *t = tab + 2 * (size_t)lo;
+        int sl = (int)pick(col_mix(y), (uint32_t)cap);
+        while (atomicCAS(&t[sl].x, -1, y) != -1)
+            if (++sl == cap) sl = 0;
+        t[sl].y = cnt[i];
+    }
+}
+
+__global__ void k_rcp(int B, const int *__restrict__ dout, const int *__restrict__ din, double *__restrict__ rcp) {
+    for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < B; x += gridDim.x * blockDim.x)
+        rcp[x] = 1.0 / ((double)dout[x] + (double)din[x] + (double)B);
+}
+
 static void rebuild_sparse(Ctx &c) {
     Launcher L{c.stream, &c.launches};
     const int B = c.B, E = c.E;
@@ -395,6 +421,10 @@ static void rebuild_sparse(Ctx &c) {
     k_seg_cum<<<g, 256, 0, c.stream>>>(c.flags, c.bm_colptr, c.tmpi, c.d_nnz, c.bm_ccum);
     k_seg_deg<<<grid_for(B, 256), 256, 0, c.stream>>>(B, c.bm_colptr, c.tmpi, c.din);
     c.launches += 2;
+    // per-row hash tables for O(1) lookups
+    k_rtab_clear<<<grid_for(2LL * E, 256), 256, 0, c.stream>>>(c.d_nnz, c.rtab);
+    k_rtab_insert<<<g, 256, 0, c.stream>>>(c.d_nnz, c.rowid, c.bm_col, c.bm_cnt, c.bm_rowptr, c.rtab);
+    c.launches += 2;
     GSAP_CHECK_LAUNCH();
 }
 
@@ -404,6 +434,8 @@ void rebuild(Ctx &c) {
     c.dense_mode = dense_ok(c, c.B);
     if (c.dense_mode) rebuild_dense(c);
     else rebuild_sparse(c);
+    k_rcp<<<grid_for(c.B, 256), 256, 0, c.stream>>>(c.B, c.dout, c.din, c.rcp);
+    ++c.launches;
     // algorithmic bytes: the compulsory inputs (dst ids,
     // row pointers, b) and the fixed-size outputs (row / column pointers,
     // degrees); the nnz-sized outputs are left out (nnz stays on the device)

@@ -295,8 +295,8 @@ class Context:
         B = C.c_int32(0)
         mdl = C.c_double(0)
         rounds = C.c_int32(0)
-        trace = np.zeros(4 * trace_cap)
+        trace = np.zeros(5 * trace_cap)
         _check(lib().gsap_run(self.h, _ptr(b), C.byref(B), C.byref(mdl), trace.ctypes.data, trace_cap,
                               C.byref(rounds)))
-        tr = trace[:4 * min(rounds.value, trace_cap)].reshape(-1, 4)
+        tr = trace[:5 * min(rounds.value, trace_cap)].reshape(-1, 5)
         return dict(b=b, B=B.value, mdl=mdl.value, trace=tr, rounds=rounds.value)

@@ -272,7 +272,7 @@ def test_end_to_end_1k(G, oracle_mod):
     # trajectories agree until the first floating-point tie (normally never)
     same = np.array_equal(res["b"], ref["b"])
     print("bit-identical final partition:", same)
-    assert res["trace"].shape == ref["trace"].shape or not same
+    assert len(res["trace"]) == len(ref["trace"]) or not same
 
 
 def test_partition_oneshot_matches_context(G, oracle_mod):

@@ -1,0 +1,123 @@
+"""Full-size parity (BASELINE.json configs) on sampled outputs, in the launch
+configuration bench.py times: the GPU computes whole batches; the oracle
+re-computes a sample of them one by one."""
+import numpy as np
+import pytest
+
+from gen import dcsbm
+from helpers import close, ties
+
+pytestmark = pytest.mark.gpu
+SEED = dcsbm.RUN_SEED
+
+
+@pytest.fixture(scope="module")
+def G():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_icpp_changzh24_b200 import gsap
+    gsap.lib()
+    return gsap
+
+
+@pytest.fixture(scope="module")
+def g200k():
+    return dcsbm.make("200k")
+
+
+def _sample_ranges(first, count, n_ranges=8, width=64, seed=0):
+    rng = np.random.default_rng(seed)
+    starts = np.sort(rng.choice(max(count - width, 1), n_ranges, replace=False)) + first
+    return [(int(s), width) for s in starts]
+
+
+@pytest.mark.parametrize("B", [71, 3000, 20000, 200000])
+def test_200k_sampled_move_parity(G, oracle_mod, g200k, B):
+    rowptr, col, truth, cfg = g200k
+    V = cfg.V
+    b = truth.copy() if B == 71 else dcsbm.random_partition(V, B, B)
+    ctx = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED))
+    ctx.gsap_set_partition(b, B)
+    orc = oracle_mod.Oracle(rowptr, col)
+    orc.set_partition(b, B)
+    bs = (V + 3) // 4
+    first, count = bs, bs                       # the second batch of an iteration
+    s = ctx.gsap_propose(G.GSAP_MOVE, 2, 5, first, count)
+    dS, H, acc = ctx.gsap_delta_mdl(G.GSAP_MOVE, 2, 5, first, count, s)
+    nt = 0
+    for (a, w) in _sample_ranges(first, count):
+        i = a - first
+        s_o = orc.propose(1, SEED, 2, 5, a, w)
+        assert np.array_equal(s[i:i + w], s_o)
+        dS_o, H_o, p_o, acc_o = orc.delta_move(SEED, 2, 5, a, w, s_o)
+        assert np.all(close(dS[i:i + w], dS_o))
+        assert np.all(close(H[i:i + w], H_o, floor=1e-300))
+        t = ties(oracle_mod, SEED, 2, 5, range(a, a + w), p_o)
+        nt += int(t.sum())
+        assert np.array_equal(acc[i:i + w][~t], acc_o[~t])
+    m_g, _ = ctx.gsap_mdl()
+    m_o, _ = orc.mdl()
+    assert abs(m_g - m_o) <= 1e-9 * abs(m_o)
+
+
+def test_200k_fused_batch_and_blockmodel(G, oracle_mod, g200k):
+    """The fused batch (move + apply + rebuild) equals the oracle's, state compared exactly."""
+    rowptr, col, truth, cfg = g200k
+    V = cfg.V
+    B = 5000
+    b = dcsbm.random_partition(V, B, 1)
+    ctx = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED))
+    ctx.gsap_set_partition(b, B)
+    orc = oracle_mod.Oracle(rowptr, col)
+    orc.set_partition(b, B)
+    bs = (V + 3) // 4
+    s, dS, acc, dsum = ctx.gsap_move_batch(0, 0, 0, bs)
+    s_o = orc.propose(1, SEED, 0, 0, 0, bs)
+    assert np.array_equal(s, s_o)
+    orc.apply_moves(0, bs, s, acc)
+    orc.rebuild()
+    b_g, _ = ctx.gsap_get_partition()
+    b_o, _ = orc.partition()
+    assert np.array_equal(b_g, b_o)
+    g = ctx.gsap_get_blockmodel()
+    o = orc.blockmodel()
+    for k in ("rowptr", "col", "cnt", "cum", "colptr", "row", "ccnt", "ccum", "dout", "din"):
+        assert np.array_equal(g[k].astype(np.int64), o[k].astype(np.int64)), k
+
+
+def test_200k_merge_phase_sampled(G, oracle_mod, g200k):
+    rowptr, col, truth, cfg = g200k
+    V = cfg.V
+    ctx = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED))
+    orc = oracle_mod.Oracle(rowptr, col)
+    B = V
+    s = ctx.gsap_propose(G.GSAP_MERGE, 0, 0, 0, B)
+    dS = ctx.gsap_delta_mdl(G.GSAP_MERGE, 0, 0, 0, B, s)
+    for (a, w) in _sample_ranges(0, B, seed=3):
+        s_o = orc.propose(0, SEED, 0, 0, a, w)
+        assert np.array_equal(s[a * 10:(a + w) * 10], s_o)
+        assert np.all(close(dS[a * 10:(a + w) * 10], orc.delta_merge(a, w, s_o)))
+    best, dSb = ctx.gsap_merge_phase(0, int(0.4 * B))
+    best_o, dSb_o = orc.best_merges(s, dS)
+    assert np.array_equal(best, best_o)
+    orc.select_merges(best, dSb, int(0.4 * B))
+    b_g, B_g = ctx.gsap_get_partition()
+    b_o, B_o = orc.partition()
+    assert B_g == B_o and np.array_equal(b_g, b_o)
+
+
+def test_200k_end_to_end_properties(G, oracle_mod, g200k):
+    """Full run: the reported MDL is the oracle's MDL of the returned partition; quality band."""
+    from sklearn.metrics import normalized_mutual_info_score as nmi
+    rowptr, col, truth, cfg = g200k
+    ctx = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED))
+    res = ctx.gsap_run()
+    orc = oracle_mod.Oracle(rowptr, col)
+    orc.set_partition(res["b"], res["B"])
+    assert abs(orc.mdl()[0] - res["mdl"]) <= 1e-9 * res["mdl"]
+    # MDL of the planted partition is an upper bound the search should approach
+    orc2 = oracle_mod.Oracle(rowptr, col)
+    orc2.set_partition(truth, cfg.B_planted)
+    print("B", res["B"], "MDL", res["mdl"], "planted MDL", orc2.mdl()[0], "NMI", nmi(truth, res["b"]))
+    assert res["mdl"] <= 1.01 * orc2.mdl()[0]

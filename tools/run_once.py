@@ -27,4 +27,7 @@ for i in range(a.runs):
     print(f"run {i}: {dt:.3f} s B={res['B']} rounds={res['rounds']} launches={st['gpu_launches']} "
           f"move_ms={st['k_move_ms']:.1f} rebuild_ms={st['k_rebuild_ms']:.1f} merge_ms={st['k_merge_ms']:.1f} "
           f"itrs={st['mcmc_itr_total']}", flush=True)
+    if i == 0:
+        for row in res["trace"]:
+            print(f"   outer={int(row[0]):3d} B={int(row[1]):8d} itrs={int(row[2]):3d} MDL={row[3]:.6e} sec={row[4]:.4f}")
     ctx.gsap_reset_stats()
