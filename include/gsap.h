@@ -60,6 +60,7 @@ typedef struct {
     int32_t model_term;       /* 0: E h(B^2/E) (Eq. 2); 1: GraphChallenge variant (R:Z3) */
     int32_t max_rounds;       /* guard on merge+MCMC rounds; default 500 */
     int32_t profile;          /* 1: time kernels with CUDA events (gsap_stats k_*) */
+    int32_t cuda_graphs;      /* 1: capture each MCMC iteration as one CUDA graph (default) */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU */

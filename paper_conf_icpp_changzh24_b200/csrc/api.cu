@@ -60,21 +60,59 @@ static cudaEvent_t ev_get(KClass &k) {
     return e;
 }
 
+static void ev_record(Ctx &c, cudaEvent_t e) {
+    if (c.capturing) GSAP_CUDA(cudaEventRecordWithFlags(e, c.stream, cudaEventRecordExternal));
+    else GSAP_CUDA(cudaEventRecord(e, c.stream));
+}
+
 void kc_begin(Ctx &c, KClass &k, cudaEvent_t *ev) {
     *ev = nullptr;
     if (!c.prm.profile) return;
     *ev = ev_get(k);
-    GSAP_CUDA(cudaEventRecord(*ev, c.stream));
+    ev_record(c, *ev);
 }
 
 void kc_end(Ctx &c, KClass &k, cudaEvent_t ev, double bytes) {
+    if (c.capturing) {   // accounted per graph launch (graph_account)
+        if (ev) {
+            cudaEvent_t e2 = ev_get(k);
+            ev_record(c, e2);
+            c.graph_ev.push_back(GraphEv{&k, ev, e2, bytes});
+        } else {
+            c.graph_ev.push_back(GraphEv{&k, nullptr, nullptr, bytes});
+        }
+        return;
+    }
     k.launches += 1;
     k.bytes += bytes;
     if (!ev) return;
     cudaEvent_t e2 = ev_get(k);
-    GSAP_CUDA(cudaEventRecord(e2, c.stream));
+    ev_record(c, e2);
     k.pending.emplace_back(ev, e2);
     if (k.pending.size() > 4096) kc_resolve(c, k);
+}
+
+// after one (synchronised) launch of a captured graph: account its kernel classes
+static void graph_account(Ctx &c) {
+    for (auto &g : c.graph_ev) {
+        g.k->launches += 1;
+        g.k->bytes += g.bytes;
+        if (g.e0) {
+            float ms = 0.f;
+            GSAP_CUDA(cudaEventElapsedTime(&ms, g.e0, g.e1));
+            g.k->ms += ms;
+        }
+    }
+}
+
+static void graph_release_events(Ctx &c) {
+    for (auto &g : c.graph_ev) {
+        if (g.e0) {
+            g.k->pool.push_back(g.e0);
+            g.k->pool.push_back(g.e1);
+        }
+    }
+    c.graph_ev.clear();
 }
 
 void kc_resolve(Ctx &c, KClass &k) {
@@ -151,7 +189,7 @@ static void free_ctx(Ctx &c) {
                     c.rcp, c.fh, c.fl, c.keys0,
                     c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
                     c.rowid, c.counts, c.scan_tmp, c.rownnz, c.s, c.dS, c.H, c.acc, c.best, c.dSbest,
-                    c.partials, c.scal, c.scal_i, c.Dh, c.skey0, c.skey1, c.sval0, c.sval1, c.rank,
+                    c.partials, c.scal, c.scal_i, c.Dh, c.d_itr, c.skey0, c.skey1, c.sval0, c.sval1, c.rank,
                     c.nxt0, c.nxt1, c.mx0, c.mx1, c.oncyc, c.label, c.present, c.slot_b[0], c.slot_b[1],
                     c.slot_b[2]};
     for (void *p : ptrs)
@@ -317,6 +355,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.scal = dalloc<double>(8);
     c.scal_i = dalloc<int>(8);
     c.Dh = dalloc<double>((size_t)c.prm.max_nodal_itr + 1);
+    c.d_itr = dalloc<unsigned>(1);
     c.skey0 = dalloc<unsigned long long>(Vs);
     c.skey1 = dalloc<unsigned long long>(Vs);
     c.sval0 = dalloc<int>(Vs);
@@ -383,8 +422,84 @@ static void move_batch(Ctx &c, uint32_t outer, uint32_t itr, int first, int coun
     c.st.n_move_prop += count;
 }
 
+static bool converged(Ctx &c, const std::vector<double> &D, int itr, double S, double thresh) {
+    const int w = c.prm.window;
+    if (itr < w - 1) return false;
+    const double mdl = model_term(c.W, c.V, c.B, c.prm.model_term) + S;
+    double sum = 0.0;
+    int n = 0;
+    for (int j = itr - w + 1; j < itr; ++j) {
+        sum += D[j];
+        ++n;
+    }
+    const double mean = n ? sum / n : 0.0;
+    return -mean < thresh * mdl;
+}
+
+// MCMC phase with every iteration (num_batches x (move + apply + rebuild) +
+// the MDL reduction) captured once into a CUDA graph; one graph launch, one
+// 16-byte D2H and one synchronisation per iteration.
+static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh) {
+    const int V = c.V, nb = c.prm.num_batches;
+    const int bs = (V + nb - 1) / nb;
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t exec = nullptr;
+    const long long l0 = c.launches;
+    GSAP_CUDA(cudaStreamBeginCapture(c.stream, cudaStreamCaptureModeThreadLocal));
+    c.capturing = true;
+    try {
+        GSAP_CUDA(cudaMemsetAsync(c.scal, 0, sizeof(double), c.stream));
+        for (int k = 0; k < nb; ++k) {
+            const int first = k * bs, last = std::min(V, first + bs);
+            if (first >= last) continue;
+            launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
+            launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1);
+            rebuild(c);
+        }
+        launch_data_term(c);
+    } catch (...) {
+        c.capturing = false;
+        cudaStreamEndCapture(c.stream, &graph);
+        if (graph) cudaGraphDestroy(graph);
+        graph_release_events(c);
+        throw;
+    }
+    c.capturing = false;
+    GSAP_CUDA(cudaStreamEndCapture(c.stream, &graph));
+    const long long kernels = c.launches - l0;
+    c.launches = l0;
+    GSAP_CUDA(cudaGraphInstantiate(&exec, graph, 0));
+    std::vector<double> D((size_t)c.prm.max_nodal_itr + 1, 0.0);
+    int ran = 0;
+    try {
+        for (int itr = 0; itr < c.prm.max_nodal_itr; ++itr) {
+            c.h_int[2] = itr;
+            GSAP_CUDA(cudaMemcpyAsync(c.d_itr, c.h_int + 2, sizeof(unsigned), cudaMemcpyHostToDevice, c.stream));
+            GSAP_CUDA(cudaGraphLaunch(exec, c.stream));
+            GSAP_CUDA(cudaMemcpyAsync(c.h_scal, c.scal, 2 * sizeof(double), cudaMemcpyDeviceToHost, c.stream));
+            GSAP_CUDA(cudaStreamSynchronize(c.stream));
+            c.launches += kernels;
+            c.st.n_move_prop += V;
+            graph_account(c);
+            D[itr] = c.h_scal[0];
+            ran = itr + 1;
+            if (converged(c, D, itr, c.h_scal[1], thresh)) break;
+        }
+    } catch (...) {
+        cudaGraphExecDestroy(exec);
+        cudaGraphDestroy(graph);
+        graph_release_events(c);
+        throw;
+    }
+    GSAP_CUDA(cudaGraphExecDestroy(exec));
+    GSAP_CUDA(cudaGraphDestroy(graph));
+    graph_release_events(c);
+    return ran;
+}
+
 // returns the number of MCMC iterations run (O.8)
 static int mcmc_phase(Ctx &c, uint32_t outer, double thresh) {
+    if (c.prm.cuda_graphs) return mcmc_phase_graph(c, outer, thresh);
     const int V = c.V, nb = c.prm.num_batches, w = c.prm.window;
     const int bs = (V + nb - 1) / nb;
     std::vector<double> D((size_t)c.prm.max_nodal_itr + 1, 0.0);
@@ -403,15 +518,7 @@ static int mcmc_phase(Ctx &c, uint32_t outer, double thresh) {
             GSAP_CUDA(cudaMemcpyAsync(D.data(), c.Dh, sizeof(double) * (size_t)(itr + 1), cudaMemcpyDeviceToHost,
                                       c.stream));
             GSAP_CUDA(cudaStreamSynchronize(c.stream));
-            const double mdl = model_term(c.W, c.V, c.B, c.prm.model_term) + c.h_scal[1];
-            double sum = 0.0;
-            int n = 0;
-            for (int j = itr - w + 1; j < itr; ++j) {
-                sum += D[j];
-                ++n;
-            }
-            const double mean = n ? sum / n : 0.0;
-            if (-mean < thresh * mdl) break;
+            if (converged(c, D, itr, c.h_scal[1], thresh)) break;
         }
     }
     return ran;
@@ -562,6 +669,7 @@ void gsap_default_params(gsap_params *p) {
     p->model_term = 0;
     p->max_rounds = 500;
     p->profile = 0;
+    p->cuda_graphs = 1;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }

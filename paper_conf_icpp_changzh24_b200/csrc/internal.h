@@ -13,6 +13,14 @@
 
 namespace gsap {
 
+struct KClass;
+// an event pair recorded inside a captured CUDA graph (re-read after every launch)
+struct GraphEv {
+    KClass *k;
+    cudaEvent_t e0, e1;
+    double bytes;
+};
+
 // timing / accounting of one kernel class (CUDA events on the context stream)
 struct KClass {
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> pending;
@@ -86,6 +94,11 @@ struct Ctx {
     double *h_scal = nullptr;
     int *h_int = nullptr;
 
+    // CUDA-graph capture of an MCMC iteration (N1: launch overhead, §5)
+    unsigned *d_itr = nullptr;     // MCMC iteration read by k_move (device scalar)
+    bool capturing = false;
+    std::vector<GraphEv> graph_ev;
+
     // accounting
     long long launches = 0;
     KClass k_move, k_rebuild, k_merge, k_mdl;
@@ -135,7 +148,7 @@ bool dense_ok(const Ctx &c, int B);
 // move.cu
 enum MoveMode { MOVE_FUSED = 0, MOVE_PROPOSE = 1, MOVE_DELTA = 2 };
 void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first, int count,
-                 int *s, double *dS, double *H, unsigned char *acc);
+                 int *s, double *dS, double *H, unsigned char *acc, const unsigned *d_itr = nullptr);
 void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned char *acc,
                   const double *dS, double *dsum, int *nacc);
 

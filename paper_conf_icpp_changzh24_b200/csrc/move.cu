@@ -35,6 +35,7 @@ struct MoveArgs {
     int B;
     uint64_t seed;
     uint32_t outer, itr;
+    const unsigned *itr_ptr;        // if set, the iteration is read from the device
     double beta;
     const int *__restrict__ rowptr, *__restrict__ col, *__restrict__ wgt;
     const int *__restrict__ cscptr, *__restrict__ cscsrc, *__restrict__ cscwgt;
@@ -239,7 +240,8 @@ template <int G, bool WEIGHTED>
 GSAP_DEV void do_vertex(const MoveArgs &a, int mode, int v, int4 *tab, int log2cap, int gt, double *sh,
                         int *bcast) {
     const int i = v - a.first;
-    const uint4 w = draws(a.seed, (uint32_t)v, 0u, a.itr, a.outer, 1u);
+    const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
+    const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
     int s;
     if (mode == MOVE_DELTA) {
         s = a.s_in[i];
@@ -317,7 +319,7 @@ static int log2_ceil(long long x) {
 }
 
 void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first, int count, int *s, double *dS,
-                 double *H, unsigned char *acc) {
+                 double *H, unsigned char *acc, const unsigned *d_itr) {
     if (count <= 0) return;
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_move, &ev);
@@ -326,6 +328,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     a.seed = c.prm.seed;
     a.outer = outer;
     a.itr = itr;
+    a.itr_ptr = d_itr;
     a.beta = c.prm.beta;
     a.rowptr = c.rowptr; a.col = c.col; a.wgt = c.wgt;
     a.cscptr = c.cscptr; a.cscsrc = c.cscsrc; a.cscwgt = c.cscwgt;

@@ -282,3 +282,12 @@ def test_partition_oneshot_matches_context(G, oracle_mod):
     res = ctx.gsap_run()
     assert np.array_equal(out["b"], res["b"]) and out["B"] == res["B"]
     assert out["stats"]["gpu_launches"] > 0 and out["stats"]["n_move_prop"] > 0
+
+
+def test_cuda_graph_path_matches_stream_path(G, oracle_mod):
+    """The captured-iteration path (default) and the per-launch path give the same run."""
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    a = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED, cuda_graphs=1, profile=1)).gsap_run()
+    b = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED, cuda_graphs=0)).gsap_run()
+    assert np.array_equal(a["b"], b["b"]) and a["B"] == b["B"] and a["mdl"] == b["mdl"]
+    assert np.array_equal(a["trace"][:, :4], b["trace"][:, :4])
