@@ -206,7 +206,8 @@ gsap_status gsap_sync(gsap_ctx *ctx);
  * Full SBP on an existing context (gsap_partition without the copy-in):
  * restarts from b = iota.  bmap_out: host or device, nullable.
  * trace (host, nullable): rows of [outer, B after merge, MCMC iterations, MDL,
- * round seconds] per round, at most trace_cap rows; *rounds_out (host, nullable).
+ * round seconds, accepted moves] per round, at most trace_cap rows;
+ * *rounds_out (host, nullable).
  */
 gsap_status gsap_run(gsap_ctx *ctx, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
                      double *trace, int32_t trace_cap, int32_t *rounds_out);

@@ -185,7 +185,7 @@ static void check_sm100() {
 static void free_ctx(Ctx &c) {
     void *ptrs[] = {c.rowptr, c.col, c.wgt, c.cscptr, c.cscsrc, c.cscwgt, c.esrc, c.kout, c.kin, c.selfw,
                     c.big, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
-                    c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT, c.rtab,
+                    c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT, c.rtab, c.ctab,
                     c.rcp, c.fh, c.fl, c.keys0,
                     c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
                     c.rowid, c.counts, c.scan_tmp, c.rownnz, c.s, c.dS, c.H, c.acc, c.best, c.dSbest,
@@ -312,6 +312,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
     c.dense = dalloc<int>(c.dense_cap);
     c.rtab = dalloc<int2>(2 * Es);
+    c.ctab = dalloc<int2>(2 * Es);
     c.rcp = dalloc<double>(Vs);
     {   // f-table: f(m) = m ln m in long double, split into double hi + float lo
         std::vector<double> fh(FT_N);
@@ -586,6 +587,12 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
     double t_merge = 0, t_move = 0, t_mdl = 0;
     while (!done && rounds < c.prm.max_rounds) {
         const bool bracket = br.S[2] != INFINITY;
+        int acc_before = 0;
+        if (trace && rounds < trace_cap) {
+            GSAP_CUDA(cudaMemcpyAsync(c.h_int + 3, c.scal_i + 1, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
+            GSAP_CUDA(cudaStreamSynchronize(c.stream));
+            acc_before = c.h_int[3];
+        }
         auto ta = std::chrono::steady_clock::now();
         merge_phase(c, outer, K, nullptr, nullptr);
         const int B = c.B;
@@ -598,11 +605,14 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
         t_move += std::chrono::duration<double>(tc - tb).count();
         t_mdl += std::chrono::duration<double>(td - tc).count();
         if (trace && rounds < trace_cap) {
-            trace[5 * rounds + 0] = (double)outer;
-            trace[5 * rounds + 1] = (double)B;
-            trace[5 * rounds + 2] = (double)itrs;
-            trace[5 * rounds + 3] = S;
-            trace[5 * rounds + 4] = std::chrono::duration<double>(td - ta).count();
+            GSAP_CUDA(cudaMemcpyAsync(c.h_int + 3, c.scal_i + 1, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
+            GSAP_CUDA(cudaStreamSynchronize(c.stream));
+            trace[6 * rounds + 0] = (double)outer;
+            trace[6 * rounds + 1] = (double)B;
+            trace[6 * rounds + 2] = (double)itrs;
+            trace[6 * rounds + 3] = S;
+            trace[6 * rounds + 4] = std::chrono::duration<double>(td - ta).count();
+            trace[6 * rounds + 5] = (double)(c.h_int[3] - acc_before);
         }
         c.st.mcmc_itr_total += itrs;
         ++rounds;

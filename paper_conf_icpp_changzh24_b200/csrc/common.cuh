@@ -142,6 +142,7 @@ struct BM {
     const int *__restrict__ dense;   // nullptr in the sparse regime
     const int2 *__restrict__ rtab;   // sparse regime: per-row open-addressing tables {col, cnt},
                                      // row x owns slots [2 rowptr[x], 2 rowptr[x+1])
+    const int2 *__restrict__ ctab;   // the same per column of the CSC: {row, cnt}
     const double *__restrict__ fh;   // f(m) = m ln m for m < FT_N, double-double (hi, lo)
     const float *__restrict__ fl;
     const double *__restrict__ rcp;  // 1 / (d_x + B) per block
@@ -171,22 +172,45 @@ GSAP_DEV int upper_bound(const int *__restrict__ a, int lo, int hi, long long p)
 // col = -1 empty, home slot = multiply-shift of the column, linear probing.
 GSAP_DEV unsigned col_mix(int y) { return (unsigned)y * 0x9E3779B1u; }
 
-GSAP_DEV int rtab_get(const BM &m, int x, int y) {
-    const int lo = __ldg(m.rowptr + x), cap = 2 * (__ldg(m.rowptr + x + 1) - lo);
-    if (cap == 0) return 0;
-    const int2 *__restrict__ t = m.rtab + 2 * (size_t)lo;
-    int sl = (int)pick(col_mix(y), (uint32_t)cap);
+// one row's (or column's) table, resolved once and probed many times
+struct Line {
+    const int2 *__restrict__ t;
+    int cap;
+};
+
+GSAP_DEV Line line_of(const int2 *__restrict__ tab, const int *__restrict__ ptr, int x) {
+    const int lo = __ldg(ptr + x);
+    Line L;
+    L.t = tab + 2 * (size_t)lo;
+    L.cap = 2 * (__ldg(ptr + x + 1) - lo);
+    return L;
+}
+
+GSAP_DEV int line_get(const Line &L, int y) {
+    if (L.cap == 0) return 0;
+    int sl = (int)pick(col_mix(y), (uint32_t)L.cap);
     while (true) {
-        const int2 e = __ldg(t + sl);
+        const int2 e = __ldg(L.t + sl);
         if (e.x == y) return e.y;
         if (e.x == -1) return 0;
-        if (++sl == cap) sl = 0;
+        if (++sl == L.cap) sl = 0;
     }
 }
 
+GSAP_DEV Line row_line(const BM &m, int x) { return line_of(m.rtab, m.rowptr, x); }
+GSAP_DEV Line col_line(const BM &m, int y) { return line_of(m.ctab, m.colptr, y); }
+
 GSAP_DEV int bm_at(const BM &m, int x, int y) {
     if (m.dense) return __ldg(m.dense + (size_t)x * m.B + y);
-    return rtab_get(m, x, y);
+    return line_get(row_line(m, x), y);
+}
+
+// M_xy with row x resolved (sparse) / M_yx with column x resolved, dense fallback
+GSAP_DEV int row_at(const BM &m, const Line &L, int x, int y) {
+    return m.dense ? __ldg(m.dense + (size_t)x * m.B + y) : line_get(L, y);
+}
+GSAP_DEV int col_at(const BM &m, const Line &L, int x, int y) {   // M_{y x}
+    return m.dense ? __ldg(m.dense + (size_t)y * m.B + x) : line_get(L, y);
 }
 
 // first index i in [lo, hi) with a[i] > p, whole warp (32-ary search: one

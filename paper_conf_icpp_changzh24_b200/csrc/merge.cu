@@ -44,33 +44,33 @@ GSAP_DEV int propose_merge(const BM &m, int r, uint32_t j, uint64_t seed, uint32
     return s;
 }
 
-// sum over t != r, s of g over the intersection of (ptrA/idxA/cntA row a) and
-// row b of the same structure; lookups of the other side via lookup(t)
-template <typename Lookup>
-GSAP_DEV double inter_sum(const int *__restrict__ ptr, const int *__restrict__ idx, const int *__restrict__ cnt,
-                          int a, int b, int r, int s, const double *__restrict__ fh, const float *__restrict__ fl,
-                          Lookup lookup) {
+// sum over t != r, s of g(M_a t, M_b t) over the intersection of line a and
+// line b (rows of the CSR, or columns of the CSC): walk the shorter line,
+// look the other one up in its hash table (or the dense copy)
+GSAP_DEV double inter_sum(const BM &m, bool cols, int a, int b, int r, int s) {
+    const int *__restrict__ ptr = cols ? m.colptr : m.rowptr;
+    const int *__restrict__ idx = cols ? m.row : m.col;
+    const int *__restrict__ cnt = cols ? m.ccnt : m.cnt;
     const int alo = __ldg(ptr + a), ahi = __ldg(ptr + a + 1);
     const int blo = __ldg(ptr + b), bhi = __ldg(ptr + b + 1);
     const bool walk_a = (ahi - alo) <= (bhi - blo);
     const int lo = walk_a ? alo : blo, hi = walk_a ? ahi : bhi, other = walk_a ? b : a;
+    Line L{};
+    if (!m.dense) L = cols ? col_line(m, other) : row_line(m, other);
     double acc = 0.0;
     for (int i = lo + (int)(threadIdx.x & 31); i < hi; i += 32) {
         const int t = __ldg(idx + i);
         if (t == r || t == s) continue;
         const int m1 = __ldg(cnt + i);
-        const int m2 = lookup(other, t);
-        acc += g2_t(fh, fl, m1, m2);
+        const int m2 = cols ? col_at(m, L, other, t) : row_at(m, L, other, t);
+        acc += g2_t(m.fh, m.fl, m1, m2);
     }
     return acc;
 }
 
 GSAP_DEV double merge_delta(const BM &m, int r, int s) {
-    // rows r, s (t in both supports): g(M_st, M_rt)
-    double acc = inter_sum(m.rowptr, m.col, m.cnt, r, s, r, s, m.fh, m.fl,
-                           [&](int x, int t) { return bm_at(m, x, t); });
-    // columns r, s: g(M_ts, M_tr)
-    acc += inter_sum(m.colptr, m.row, m.ccnt, r, s, r, s, m.fh, m.fl, [&](int y, int t) { return bm_at(m, t, y); });
+    // rows r, s (t in both supports): g(M_st, M_rt); columns r, s: g(M_ts, M_tr)
+    double acc = inter_sum(m, false, r, s, r, s) + inter_sum(m, true, r, s, r, s);
     acc = warp_sum(acc);
     const long long Mss = bm_at(m, s, s), Msr = bm_at(m, s, r), Mrs = bm_at(m, r, s), Mrr = bm_at(m, r, r);
     // f(a+b+c+d) - f(a) - f(b) - f(c) - f(d), telescoped into g's

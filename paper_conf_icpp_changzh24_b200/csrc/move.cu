@@ -29,7 +29,10 @@ constexpr int BIG_THR = 128;           // warp path iff min(k_v, B) <= BIG_THR
 constexpr int MOVE_WARPS = 8;          // warps per CTA, warp kernel
 constexpr int CTA_THREADS = 256;       // big-vertex role: one CTA per vertex
 constexpr int CTA_SMEM_SLOTS = MOVE_WARPS * WARP_TAB;   // big-vertex shared table (<= 1024 keys)
-constexpr int BIG_CTAS_MAX = 296;      // CTAs of the big-vertex role (grid-stride)
+constexpr int BIG_CTAS_MAX = 296;
+#ifndef GSAP_MOVE_MINB
+#define GSAP_MOVE_MINB 3               // CTAs per SM the register budget is sized for
+#endif      // CTAs of the big-vertex role (grid-stride)
 
 struct MoveArgs {
     int B;
@@ -79,61 +82,31 @@ GSAP_DEV int tab_find(const int4 *tab, int log2cap, int t) {
     }
 }
 
-// weighted pick over ids[lo, lo+len) by weights wts; p is reduced by the list
-// total when the pick falls beyond it (returns -1).  Whole warp.
-GSAP_DEV int warp_pick(const int *__restrict__ ids, const int *__restrict__ wts, int lo, int len, long long &p) {
-    const int lane = threadIdx.x & 31;
-    long long carry = 0;
-    for (int base = 0; base < len; base += 32) {
-        const int j = base + lane;
-        const int wv = j < len ? __ldg(wts + lo + j) : 0;
-        const int id = j < len ? __ldg(ids + lo + j) : -1;
-        const int sc = warp_incl_scan(wv);
-        const unsigned bal = __ballot_sync(FULL, j < len && carry + sc > p);
-        if (bal) return __shfl_sync(FULL, id, __ffs(bal) - 1);
-        carry += __shfl_sync(FULL, sc, 31);
-    }
-    p -= carry;
-    return -1;
-}
-
-// (a1) MOVE proposal for v (R:O.4).  Whole warp; result warp-uniform.
-template <bool WEIGHTED>
-GSAP_DEV int propose_move(const MoveArgs &a, int v, uint4 w) {
-    const uint32_t B = (uint32_t)a.B;
-    const uint32_t K = (uint32_t)(__ldg(a.kout + v) + __ldg(a.kin + v));
-    if (K == 0) return (int)pick(w.z, B);
-    const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
-    const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
-    int n;
-    if (!WEIGHTED) {
-        const uint32_t p = pick(w.x, K);
-        n = (int)p < nout ? __ldg(a.col + ro + p) : __ldg(a.cscsrc + ci + (p - nout));
-    } else {
-        long long p = pick(w.x, K);
-        n = warp_pick(a.col, a.wgt, ro, nout, p);
-        if (n < 0) n = warp_pick(a.cscsrc, a.cscwgt, ci, nin, p);
-    }
-    const int u = __ldg(a.b + n);
-    const uint32_t du = (uint32_t)bm_deg(a.m, u);
-    if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
-    return bm_walk_warp(a.m, u, (long long)pick(w.z, du));
-}
-
-// group-wide sums (deterministic fixed trees)
+// group-wide sums of three values (deterministic fixed trees)
 template <int G>
-GSAP_DEV double group_sum(double v, double *sh) {
-    v = warp_sum(v);
-    if (G == 32) return v;
+GSAP_DEV void group_sum3(double &x, double &y, double &z, double *sh) {
+    x = warp_sum(x);
+    y = warp_sum(y);
+    z = warp_sum(z);
+    if (G == 32) return;
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (lane == 0) {
+        sh[w] = x;
+        sh[G / 32 + w] = y;
+        sh[2 * (G / 32) + w] = z;
+    }
     __syncthreads();
-    if (lane == 0) sh[w] = v;
-    __syncthreads();
-    double t = 0.0;
+    double a = 0.0, b = 0.0, c = 0.0;
 #pragma unroll
-    for (int i = 0; i < G / 32; ++i) t += sh[i];
+    for (int i = 0; i < G / 32; ++i) {
+        a += sh[i];
+        b += sh[G / 32 + i];
+        c += sh[2 * (G / 32) + i];
+    }
     __syncthreads();
-    return t;
+    x = a;
+    y = b;
+    z = c;
 }
 
 template <int G>
@@ -142,18 +115,191 @@ GSAP_DEV void group_sync() {
     else __syncthreads();
 }
 
-// (a2) Delta S + Hastings + MH accept for v: r -> s, r != s, on the table
-// `tab` (2^log2cap slots, empty on entry).  gt = thread index in the group.
-template <int G, bool WEIGHTED>
-GSAP_DEV void eval_move(const MoveArgs &a, int v, int s, uint4 w, int4 *tab, int log2cap, int gt,
-                        double *sh, double &dS_out, double &H_out, bool &acc_out) {
-    const int B = a.B;
-    const int r = __ldg(a.b + v);
+// the state of one move r -> s that every term needs
+struct MoveCtx {
+    int v, r, s;
+    long long Mrr, Mrs, Msr, Mss, o_r, i_r, o_s, i_s, kout, kin, l, dr, ds, Mrr2, Mrs2, Msr2, dr2, ds2;
+    double Bd;
+    Line Rr, Rs, Cr, Cs;
+};
+
+// dS / Hastings terms of one unique neighbour block t (out weight ot, in weight it)
+GSAP_DEV void t_terms(const MoveArgs &a, const MoveCtx &q, int t, long long ot, long long it, double &accS,
+                      double &pf, double &pb) {
+    const double *__restrict__ fh = a.m.fh;
+    const float *__restrict__ fl = a.m.fl;
+    const double *__restrict__ rcp = a.m.rcp;
+    const double c = (double)(ot + it);
+    if (t == q.r) {
+        pf += c * (double)(q.Mrs + q.Msr + 1) * __ldg(rcp + q.r);
+        pb += c * (double)(2 * q.Mrr2 + 1) / ((double)q.dr2 + q.Bd);
+    } else if (t == q.s) {
+        pf += c * (double)(2 * q.Mss + 1) * __ldg(rcp + q.s);
+        pb += c * (double)(q.Msr2 + q.Mrs2 + 1) / ((double)q.ds2 + q.Bd);
+    } else {
+        const long long Mrt = row_at(a.m, q.Rr, q.r, t), Mst = row_at(a.m, q.Rs, q.s, t);
+        const long long Mtr = col_at(a.m, q.Cr, q.r, t), Mts = col_at(a.m, q.Cs, q.s, t);
+        const double rt = __ldg(rcp + t);
+        accS -= df_t(fh, fl, Mrt, -ot) + df_t(fh, fl, Mst, ot) + df_t(fh, fl, Mtr, -it) + df_t(fh, fl, Mts, it);
+        pf += c * (double)(Mts + Mst + 1) * rt;
+        pb += c * (double)(Mtr - it + Mrt - ot + 1) * rt;
+    }
+}
+
+// the 2x2 core, the four degree terms and the two self-loop terms: term k of 10
+GSAP_DEV void core_term(const MoveArgs &a, const MoveCtx &q, int k, double &accS, double &pf, double &pb) {
+    const double *__restrict__ fh = a.m.fh;
+    const float *__restrict__ fl = a.m.fl;
+    switch (k) {
+        case 0: accS -= df_t(fh, fl, q.Mrr, -(q.o_r + q.i_r + q.l)); break;
+        case 1: accS -= df_t(fh, fl, q.Mrs, q.i_r - q.o_s); break;
+        case 2: accS -= df_t(fh, fl, q.Msr, q.o_r - q.i_s); break;
+        case 3: accS -= df_t(fh, fl, q.Mss, q.o_s + q.i_s + q.l); break;
+        case 4: accS += df_t(fh, fl, __ldg(a.m.dout + q.r), -q.kout); break;
+        case 5: accS += df_t(fh, fl, __ldg(a.m.dout + q.s), q.kout); break;
+        case 6: accS += df_t(fh, fl, __ldg(a.m.din + q.r), -q.kin); break;
+        case 7: accS += df_t(fh, fl, __ldg(a.m.din + q.s), q.kin); break;
+        case 8:
+            if (q.l > 0) pf += 2.0 * (double)q.l * (double)(q.Mrs + q.Msr + 1) * __ldg(a.m.rcp + q.r);
+            break;
+        default:
+            if (q.l > 0) pb += 2.0 * (double)q.l * (double)(q.Msr2 + q.Mrs2 + 1) / ((double)q.ds2 + q.Bd);
+            break;
+    }
+}
+
+// after phase A: the core values (every thread, redundantly: broadcast loads)
+GSAP_DEV void move_ctx(const MoveArgs &a, int v, int r, int s, const int4 *tab, int log2cap, MoveCtx &q) {
+    q.v = v;
+    q.r = r;
+    q.s = s;
+    if (!a.m.dense) {
+        q.Rr = row_line(a.m, r);
+        q.Rs = row_line(a.m, s);
+        q.Cr = col_line(a.m, r);
+        q.Cs = col_line(a.m, s);
+    }
+    q.Mrr = row_at(a.m, q.Rr, r, r);
+    q.Mrs = row_at(a.m, q.Rr, r, s);
+    q.Msr = row_at(a.m, q.Rs, s, r);
+    q.Mss = row_at(a.m, q.Rs, s, s);
+    const int slr = tab_find(tab, log2cap, r), sls = tab_find(tab, log2cap, s);
+    q.o_r = slr >= 0 ? tab[slr].y : 0;
+    q.i_r = slr >= 0 ? tab[slr].z : 0;
+    q.o_s = sls >= 0 ? tab[sls].y : 0;
+    q.i_s = sls >= 0 ? tab[sls].z : 0;
+    q.kout = __ldg(a.kout + v);
+    q.kin = __ldg(a.kin + v);
+    q.l = __ldg(a.selfw + v);
+    q.dr = bm_deg(a.m, r);
+    q.ds = bm_deg(a.m, s);
+    q.Mrr2 = q.Mrr - q.o_r - q.i_r - q.l;
+    q.Mrs2 = q.Mrs + q.i_r - q.o_s;
+    q.Msr2 = q.Msr + q.o_r - q.i_s;
+    q.dr2 = q.dr - q.kout - q.kin;
+    q.ds2 = q.ds + q.kout + q.kin;
+    q.Bd = (double)a.B;
+}
+
+GSAP_DEV void mh_decide(const MoveArgs &a, const MoveCtx &q, uint4 w, double dS, double pf, double pb,
+                        double &dS_out, double &H_out, bool &acc_out) {
+    const double H = (q.kout + q.kin == 0) ? 1.0 : pb / pf;
+    const double p = exp(-a.beta * dS) * H;
+    const double u = ((double)w.w + 0.5) * (1.0 / 4294967296.0);
+    dS_out = dS;
+    H_out = H;
+    acc_out = u <= p;
+}
+
+// (a2), one warp per vertex: phase A builds the neighbour-block table and
+// compacts the unique blocks into `list` in first-occurrence order; phase B
+// gives each lane whole unique blocks (all lanes busy).  Table left empty.
+template <bool WEIGHTED>
+GSAP_DEV void eval_move_warp(const MoveArgs &a, int v, int r, int s, uint4 w, int4 *tab, int *list,
+                             double &dS_out, double &H_out, bool &acc_out) {
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
     const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
     const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
     const int deg = nout + nin;
-    // phase A: histogram of neighbour blocks
-    for (int j = gt; j < deg; j += G) {
+    int keep[4];
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+        keep[c] = -1;
+        const int j = c * 32 + lane;
+        if (j < deg) {
+            const bool out = j < nout;
+            const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+            if (nb != v) {
+                const int t = __ldg(a.b + nb);
+                const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
+                const int sl = tab_insert(tab, WARP_TAB_LOG2, t);
+                atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
+                atomicMin(&tab[sl].w, j);
+                keep[c] = sl;
+            }
+        }
+    }
+    for (int j = 128 + lane; j < deg; j += 32) {   // only when B <= 128 (<= B keys)
+        const bool out = j < nout;
+        const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+        if (nb == v) continue;
+        const int t = __ldg(a.b + nb);
+        const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
+        const int sl = tab_insert(tab, WARP_TAB_LOG2, t);
+        atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
+        atomicMin(&tab[sl].w, j);
+    }
+    __syncwarp();
+    int nuniq = 0;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+        const int sl = keep[c];
+        const bool own = sl >= 0 && tab[sl].w == c * 32 + lane;
+        const unsigned bal = __ballot_sync(FULL, own);
+        if (own) list[nuniq + __popc(bal & lt)] = sl;
+        nuniq += __popc(bal);
+    }
+    for (int base = 128; base < deg; base += 32) {
+        const int j = base + lane;
+        int sl = -1;
+        if (j < deg) {
+            const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+            if (nb != v) sl = tab_find(tab, WARP_TAB_LOG2, __ldg(a.b + nb));
+        }
+        const bool own = sl >= 0 && tab[sl].w == j;
+        const unsigned bal = __ballot_sync(FULL, own);
+        if (own) list[nuniq + __popc(bal & lt)] = sl;
+        nuniq += __popc(bal);
+    }
+    __syncwarp();
+    MoveCtx q;
+    move_ctx(a, v, r, s, tab, WARP_TAB_LOG2, q);
+    double accS = 0.0, pf = 0.0, pb = 0.0;
+    for (int k = lane; k < nuniq; k += 32) {
+        const int4 e = tab[list[k]];
+        t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
+    }
+    if (lane < 10) core_term(a, q, lane, accS, pf, pb);
+    accS = warp_sum(accS);
+    pf = warp_sum(pf);
+    pb = warp_sum(pb);
+    // leave the table empty: exactly the listed slots were used
+    for (int k = lane; k < nuniq; k += 32) tab[list[k]] = make_int4(-1, 0, 0, 0x7fffffff);
+    __syncwarp();
+    mh_decide(a, q, w, accS, pf, pb, dS_out, H_out, acc_out);
+}
+
+// (a2), one CTA per (big) vertex: every unique block owned by its first
+// adjacency position; threads sum their owned terms in position order.
+template <bool WEIGHTED>
+GSAP_DEV void eval_move_cta(const MoveArgs &a, int v, int r, int s, uint4 w, int4 *tab, int log2cap,
+                            double *sh, double &dS_out, double &H_out, bool &acc_out) {
+    const int gt = threadIdx.x;
+    const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
+    const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
+    const int deg = nout + nin;
+    for (int j = gt; j < deg; j += CTA_THREADS) {
         const bool out = j < nout;
         const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
         if (nb == v) continue;   // the self-loop is carried by selfw
@@ -163,72 +309,20 @@ GSAP_DEV void eval_move(const MoveArgs &a, int v, int s, uint4 w, int4 *tab, int
         atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
         atomicMin(&tab[sl].w, j);
     }
-    group_sync<G>();
-    // 2x2 core (every thread, redundantly: broadcast loads)
-    const long long Mrr = bm_at(a.m, r, r), Mrs = bm_at(a.m, r, s);
-    const long long Msr = bm_at(a.m, s, r), Mss = bm_at(a.m, s, s);
-    const int slr = tab_find(tab, log2cap, r), sls = tab_find(tab, log2cap, s);
-    const long long o_r = slr >= 0 ? tab[slr].y : 0, i_r = slr >= 0 ? tab[slr].z : 0;
-    const long long o_s = sls >= 0 ? tab[sls].y : 0, i_s = sls >= 0 ? tab[sls].z : 0;
-    const long long kout = __ldg(a.kout + v), kin = __ldg(a.kin + v), l = __ldg(a.selfw + v);
-    const long long dr = bm_deg(a.m, r), ds = bm_deg(a.m, s);
-    const long long Mrr2 = Mrr - o_r - i_r - l, Mrs2 = Mrs + i_r - o_s, Msr2 = Msr + o_r - i_s;
-    const long long dr2 = dr - kout - kin, ds2 = ds + kout + kin;
-    const double Bd = (double)B;
-    // phase B: the owner of each unique t adds its terms
-    const double *__restrict__ fh = a.m.fh;
-    const float *__restrict__ fl = a.m.fl;
-    const double *__restrict__ rcp = a.m.rcp;
+    __syncthreads();
+    MoveCtx q;
+    move_ctx(a, v, r, s, tab, log2cap, q);
     double accS = 0.0, pf = 0.0, pb = 0.0;
-    for (int j = gt; j < deg; j += G) {
-        const bool out = j < nout;
-        const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+    for (int j = gt; j < deg; j += CTA_THREADS) {
+        const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
         if (nb == v) continue;
-        const int t = __ldg(a.b + nb);
-        const int sl = tab_find(tab, log2cap, t);
-        const int4 e = tab[sl];
+        const int4 e = tab[tab_find(tab, log2cap, __ldg(a.b + nb))];
         if (e.w != j) continue;
-        const long long ot = e.y, it = e.z;
-        const double c = (double)(ot + it);
-        if (t == r) {
-            pf += c * (double)(Mrs + Msr + 1) * __ldg(rcp + r);
-            pb += c * (double)(2 * Mrr2 + 1) / ((double)dr2 + Bd);
-        } else if (t == s) {
-            pf += c * (double)(2 * Mss + 1) * __ldg(rcp + s);
-            pb += c * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd);
-        } else {
-            const long long Mrt = bm_at(a.m, r, t), Mst = bm_at(a.m, s, t);
-            const long long Mtr = bm_at(a.m, t, r), Mts = bm_at(a.m, t, s);
-            const double rt = __ldg(rcp + t);
-            accS -= df_t(fh, fl, Mrt, -ot) + df_t(fh, fl, Mst, ot) + df_t(fh, fl, Mtr, -it) + df_t(fh, fl, Mts, it);
-            pf += c * (double)(Mts + Mst + 1) * rt;
-            pb += c * (double)(Mtr - it + Mrt - ot + 1) * rt;
-        }
+        t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
     }
-    // the 2x2 core, the four degree terms and the self-loop terms, one per thread
-    if (gt < 10) {
-        switch (gt) {
-            case 0: accS -= df_t(fh, fl, Mrr, -(o_r + i_r + l)); break;
-            case 1: accS -= df_t(fh, fl, Mrs, i_r - o_s); break;
-            case 2: accS -= df_t(fh, fl, Msr, o_r - i_s); break;
-            case 3: accS -= df_t(fh, fl, Mss, o_s + i_s + l); break;
-            case 4: accS += df_t(fh, fl, __ldg(a.m.dout + r), -kout); break;
-            case 5: accS += df_t(fh, fl, __ldg(a.m.dout + s), kout); break;
-            case 6: accS += df_t(fh, fl, __ldg(a.m.din + r), -kin); break;
-            case 7: accS += df_t(fh, fl, __ldg(a.m.din + s), kin); break;
-            case 8: if (l > 0) pf += 2.0 * (double)l * (double)(Mrs + Msr + 1) * __ldg(rcp + r); break;
-            default: if (l > 0) pb += 2.0 * (double)l * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd); break;
-        }
-    }
-    const double dS = group_sum<G>(accS, sh);
-    pf = group_sum<G>(pf, sh);
-    pb = group_sum<G>(pb, sh);
-    const double H = (kout + kin == 0) ? 1.0 : pb / pf;
-    const double p = exp(-a.beta * dS) * H;
-    const double u = ((double)w.w + 0.5) * (1.0 / 4294967296.0);
-    dS_out = dS;
-    H_out = H;
-    acc_out = u <= p;
+    if (gt < 10) core_term(a, q, gt, accS, pf, pb);
+    group_sum3<CTA_THREADS>(accS, pf, pb, sh);
+    mh_decide(a, q, w, accS, pf, pb, dS_out, H_out, acc_out);
 }
 
 template <int G>
@@ -236,38 +330,66 @@ GSAP_DEV void tab_clear(int4 *tab, int slots, int gt) {
     for (int i = gt; i < slots; i += G) tab[i] = make_int4(-1, 0, 0, 0x7fffffff);
 }
 
+// outputs of vertex v (index i = v - first) given its proposal s
 template <int G, bool WEIGHTED>
-GSAP_DEV void do_vertex(const MoveArgs &a, int mode, int v, int4 *tab, int log2cap, int gt, double *sh,
-                        int *bcast) {
+GSAP_DEV void do_vertex(const MoveArgs &a, int v, int4 *tab, int log2cap, int *list, double *sh) {
     const int i = v - a.first;
     const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
     const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
-    int s;
-    if (mode == MOVE_DELTA) {
-        s = a.s_in[i];
-    } else {
-        if (G == 32) {
-            s = propose_move<WEIGHTED>(a, v, w);
-        } else {
-            if ((threadIdx.x >> 5) == 0) {
-                const int sp = propose_move<WEIGHTED>(a, v, w);
-                if (threadIdx.x == 0) *bcast = sp;
-            }
-            __syncthreads();
-            s = *bcast;
-            __syncthreads();
-        }
-        if (a.s_out && gt == 0) a.s_out[i] = s;
-        if (mode == MOVE_PROPOSE) return;
-    }
+    const int s = a.s_in[i];
     const int r = __ldg(a.b + v);
     double dS = 0.0, H = 1.0;
     bool acc = false;
-    if (s != r) eval_move<G, WEIGHTED>(a, v, s, w, tab, log2cap, gt, sh, dS, H, acc);
-    if (gt == 0) {
+    if (s != r) {
+        if (G == 32) eval_move_warp<WEIGHTED>(a, v, r, s, w, tab, list, dS, H, acc);
+        else eval_move_cta<WEIGHTED>(a, v, r, s, w, tab, log2cap, sh, dS, H, acc);
+    }
+    if ((threadIdx.x & (G - 1)) == 0) {
         if (a.dS) a.dS[i] = dS;
         if (a.H) a.H[i] = H;
         if (a.acc) a.acc[i] = acc ? 1 : 0;
+    }
+}
+
+// (a1) one thread per vertex: the proposal chain is a handful of dependent
+// loads, so 32 vertices per warp keep them in flight (R:O.4).
+template <bool WEIGHTED>
+GSAP_DEV int propose_move_thread(const MoveArgs &a, int v, uint4 w) {
+    const uint32_t B = (uint32_t)a.B;
+    const uint32_t K = (uint32_t)(__ldg(a.kout + v) + __ldg(a.kin + v));
+    if (K == 0) return (int)pick(w.z, B);
+    const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
+    const int ci = __ldg(a.cscptr + v);
+    const uint32_t p = pick(w.x, K);
+    int n;
+    if (!WEIGHTED) {
+        n = (int)p < nout ? __ldg(a.col + ro + p) : __ldg(a.cscsrc + ci + (p - nout));
+    } else {
+        long long acc = 0;
+        n = -1;
+        for (int e = 0; e < nout && n < 0; ++e) {
+            acc += __ldg(a.wgt + ro + e);
+            if ((long long)p < acc) n = __ldg(a.col + ro + e);
+        }
+        const int nin = __ldg(a.cscptr + v + 1) - ci;
+        for (int e = 0; e < nin && n < 0; ++e) {
+            acc += __ldg(a.cscwgt + ci + e);
+            if ((long long)p < acc) n = __ldg(a.cscsrc + ci + e);
+        }
+    }
+    const int u = __ldg(a.b + n);
+    const uint32_t du = (uint32_t)bm_deg(a.m, u);
+    if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
+    return bm_walk(a.m, u, (long long)pick(w.z, du), -1);
+}
+
+template <bool WEIGHTED>
+__global__ void __launch_bounds__(256) k_propose(MoveArgs a) {
+    const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < a.count; i += gridDim.x * blockDim.x) {
+        const int v = a.first + i;
+        const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
+        a.s_out[i] = propose_move_thread<WEIGHTED>(a, v, w);
     }
 }
 
@@ -276,24 +398,24 @@ GSAP_DEV void do_vertex(const MoveArgs &a, int mode, int v, int4 *tab, int log2c
 // CTAs take every other vertex of [first, first + count) one warp per vertex.
 // The shared memory is the 8 warp tables, or one CTA table over the same bytes.
 template <bool WEIGHTED>
-__global__ void __launch_bounds__(MOVE_WARPS * 32, 3) k_move(MoveArgs a, int mode) {
+__global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveArgs a) {
     __shared__ int4 tabs[MOVE_WARPS * WARP_TAB];
-    __shared__ double sh[MOVE_WARPS];
-    __shared__ int bcast;
+    __shared__ int lists[MOVE_WARPS * (WARP_TAB / 2)];
+    __shared__ double sh[3 * MOVE_WARPS];
     const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if ((int)blockIdx.x < a.nbig_ctas) {
         int4 *tab = a.gtab ? a.gtab + ((size_t)blockIdx.x << a.gtab_log2) : tabs;
         const int log2cap = a.gtab_log2;
         for (int li = blockIdx.x; li < a.list_count; li += a.nbig_ctas) {
-            const int v = a.list[li];
             tab_clear<CTA_THREADS>(tab, 1 << log2cap, threadIdx.x);
             __syncthreads();
-            do_vertex<CTA_THREADS, WEIGHTED>(a, mode, v, tab, log2cap, threadIdx.x, sh, &bcast);
+            do_vertex<CTA_THREADS, WEIGHTED>(a, a.list[li], tab, log2cap, nullptr, sh);
             __syncthreads();
         }
         return;
     }
     int4 *tab = tabs + wl * WARP_TAB;
+    int *list = lists + wl * (WARP_TAB / 2);
     tab_clear<32>(tab, WARP_TAB, lane);
     __syncwarp();
     const int nwarps = (gridDim.x - a.nbig_ctas) * MOVE_WARPS;
@@ -304,10 +426,7 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, 3) k_move(MoveArgs a, int mod
         if (skip_big &&
             (__ldg(a.rowptr + v + 1) - __ldg(a.rowptr + v)) + (__ldg(a.cscptr + v + 1) - __ldg(a.cscptr + v)) > BIG_THR)
             continue;
-        do_vertex<32, WEIGHTED>(a, mode, v, tab, WARP_TAB_LOG2, lane, nullptr, nullptr);
-        __syncwarp();
-        tab_clear<32>(tab, WARP_TAB, lane);
-        __syncwarp();
+        do_vertex<32, WEIGHTED>(a, v, tab, WARP_TAB_LOG2, list, nullptr);
     }
 }
 
@@ -338,12 +457,22 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     a.count = count;
     a.list = nullptr;
     a.list_count = 0;
-    a.s_in = mode == MOVE_DELTA ? s : nullptr;
-    a.s_out = mode == MOVE_DELTA ? nullptr : s;
+    a.s_in = s;
+    a.s_out = s;
     a.dS = dS; a.H = H; a.acc = acc;
     a.gtab = nullptr;
     a.gtab_log2 = 0;
-    const int m = (int)mode;
+    if (mode != MOVE_DELTA) {   // (a1): thread per vertex
+        const int pg = (int)std::min<long long>(((long long)count + 255) / 256, 148LL * 16);
+        if (c.weighted) k_propose<true><<<pg, 256, 0, c.stream>>>(a);
+        else k_propose<false><<<pg, 256, 0, c.stream>>>(a);
+        ++c.launches;
+        GSAP_CHECK_LAUNCH();
+        if (mode == MOVE_PROPOSE) {
+            kc_end(c, c.k_move, ev, 0.0);
+            return;
+        }
+    }
     a.nbig_ctas = 0;
     if (c.B > BIG_THR && !c.h_big.empty()) {
         // the big vertices inside [first, first + count)
@@ -370,8 +499,8 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     }
     const long long need = ((long long)count + MOVE_WARPS - 1) / MOVE_WARPS;
     const int grid = a.nbig_ctas + (int)std::max<long long>(1, std::min<long long>(need, 148LL * 8));
-    if (c.weighted) k_move<true><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a, m);
-    else k_move<false><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a, m);
+    if (c.weighted) k_move<true><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a);
+    else k_move<false><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a);
     ++c.launches;
     GSAP_CHECK_LAUNCH();
     // algorithmic bytes: adjacency ids (+ weights),

@@ -421,10 +421,12 @@ static void rebuild_sparse(Ctx &c) {
     k_seg_cum<<<g, 256, 0, c.stream>>>(c.flags, c.bm_colptr, c.tmpi, c.d_nnz, c.bm_ccum);
     k_seg_deg<<<grid_for(B, 256), 256, 0, c.stream>>>(B, c.bm_colptr, c.tmpi, c.din);
     c.launches += 2;
-    // per-row hash tables for O(1) lookups
+    // per-row and per-column hash tables for O(1) lookups
     k_rtab_clear<<<grid_for(2LL * E, 256), 256, 0, c.stream>>>(c.d_nnz, c.rtab);
+    k_rtab_clear<<<grid_for(2LL * E, 256), 256, 0, c.stream>>>(c.d_nnz, c.ctab);
     k_rtab_insert<<<g, 256, 0, c.stream>>>(c.d_nnz, c.rowid, c.bm_col, c.bm_cnt, c.bm_rowptr, c.rtab);
-    c.launches += 2;
+    k_rtab_insert<<<g, 256, 0, c.stream>>>(c.d_nnz, c.flags, c.bm_row, c.bm_ccnt, c.bm_colptr, c.ctab);
+    c.launches += 4;
     GSAP_CHECK_LAUNCH();
 }
 
