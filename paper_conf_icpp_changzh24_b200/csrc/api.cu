@@ -188,7 +188,8 @@ static void free_ctx(Ctx &c) {
                     c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT, c.rtab, c.ctab,
                     c.rcp, c.fh, c.fl, c.keys0,
                     c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
-                    c.rowid, c.counts, c.scan_tmp, c.rownnz, c.s, c.dS, c.H, c.acc, c.best, c.dSbest,
+                    c.rowid, c.counts, c.scan_tmp, c.rownnz, c.seg_len, c.seg_off, c.seg_cur, c.seg_nnz,
+                    c.seg_listW, c.seg_listC, c.seg_ctr, c.xl_hp, c.xl_keys, c.s, c.dS, c.H, c.acc, c.best, c.dSbest,
                     c.partials, c.scal, c.scal_i, c.Dh, c.d_itr, c.skey0, c.skey1, c.sval0, c.sval1, c.rank,
                     c.nxt0, c.nxt1, c.mx0, c.mx1, c.oncyc, c.label, c.present, c.slot_b[0], c.slot_b[1],
                     c.slot_b[2]};
@@ -341,6 +342,15 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.tmpi = dalloc<int>(VE);
     c.rowid = dalloc<int>(VE);
     c.rownnz = dalloc<int>(Vs + 1);
+    c.seg_len = dalloc<int>(Vs + 1);
+    c.seg_off = dalloc<int>(Vs + 1);
+    c.seg_cur = dalloc<int>(Vs + 1);
+    c.seg_nnz = dalloc<int>(Vs + 1);
+    c.seg_listW = dalloc<int>(Vs + 1);
+    c.seg_listC = dalloc<int>(Vs + 1);
+    c.seg_ctr = dalloc<int>(4);
+    c.xl_keys = dalloc<unsigned long long>(2 * Es);
+    c.xl_hp = dalloc<int>(2 * Es);
     const size_t tiles = (VE + 4095) / 4096 + 1;
     c.counts_cap = 256 * tiles;
     c.counts = dalloc<int>(c.counts_cap);

@@ -73,6 +73,10 @@ struct Ctx {
     int *wa = nullptr, *wb = nullptr, *flags = nullptr, *pos = nullptr, *tmpi = nullptr,
         *rowid = nullptr, *counts = nullptr, *scan_tmp = nullptr, *rownnz = nullptr;
     size_t counts_cap = 0, scan_tmp_cap = 0;
+    // segmented rebuild scratch (per line: length, offset, cursor, runs; line lists)
+    int *seg_len = nullptr, *seg_off = nullptr, *seg_cur = nullptr, *seg_nnz = nullptr, *seg_listW = nullptr,
+        *seg_listC = nullptr, *seg_ctr = nullptr, *xl_hp = nullptr;
+    unsigned long long *xl_keys = nullptr;   // 2E: long-segment sort scratch
 
     // per-phase buffers
     int *s = nullptr;            // proposals: V (MOVE) or B * P (MERGE)

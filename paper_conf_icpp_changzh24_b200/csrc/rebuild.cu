@@ -15,6 +15,7 @@
 
 #include "internal.h"
 #include "prims.cuh"
+#include "segsort.cuh"
 
 namespace gsap {
 
@@ -367,8 +368,42 @@ __global__ void k_rcp(int B, const int *__restrict__ dout, const int *__restrict
         rcp[x] = 1.0 / ((double)dout[x] + (double)din[x] + (double)B);
 }
 
-static void rebuild_sparse(Ctx &c) {
+// one side of the sparse blockmodel: lines (rows of M from the out-CSR, or
+// columns of M from the in-CSC) by counting sort + per-line segment sort
+template <typename K>
+static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw, int *ptr, int *idx, int *cnt,
+                        int *cum, int *lineid, int *deg, int *total) {
     Launcher L{c.stream, &c.launches};
+    const int B = c.B, V = c.V;
+    K *seg = reinterpret_cast<K *>(c.keys0);
+    GSAP_CUDA(cudaMemsetAsync(c.seg_len, 0, sizeof(int) * (size_t)B, c.stream));
+    GSAP_CUDA(cudaMemsetAsync(c.seg_cur, 0, sizeof(int) * (size_t)B, c.stream));
+    GSAP_CUDA(cudaMemsetAsync(c.seg_ctr, 0, 2 * sizeof(int), c.stream));
+    k_line_len<<<grid_for(V, 256), 256, 0, c.stream>>>(V, gptr, c.b, c.seg_len);
+    ++c.launches;
+    device_scan<int>(c.seg_len, c.seg_off, nullptr, B, false, c.scan_tmp, c.seg_off + B, L);
+    k_line_scatter<K><<<grid_for((long long)V * 32, 256), 256, 0, c.stream>>>(V, gptr, gidx, gw, c.b, c.seg_off,
+                                                                             c.seg_cur, seg);
+    k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, c.seg_off, c.seg_nnz, c.seg_listW, c.seg_listC,
+                                                           c.seg_ctr);
+    const int gw_ = (int)std::min<long long>(((long long)B + SEG_WARPS - 1) / SEG_WARPS, 148LL * 16);
+    k_segsort_warp<K><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(c.seg_off, seg, c.seg_listW, c.seg_ctr, c.wa, c.wb,
+                                                           c.seg_nnz);
+    const int gc = (int)std::min<long long>(std::max(1, B / 4), 148LL * 4);
+    k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(c.seg_off, seg, c.seg_listC, c.seg_ctr, c.wa, c.wb, c.seg_nnz,
+                                               reinterpret_cast<K *>(c.xl_keys), c.xl_hp);
+    k_segsort_xl<K><<<gc, 256, 0, c.stream>>>(c.seg_off, seg, c.seg_listC, c.seg_ctr, bits_for(B), c.wa, c.wb,
+                                              c.seg_nnz, reinterpret_cast<K *>(c.xl_keys), c.xl_hp);
+    c.launches += 5;
+    device_scan<int>(c.seg_nnz, ptr, nullptr, B, false, c.scan_tmp, ptr + B, L);
+    k_line_copy<<<grid_for((long long)B * 32, 256), 256, 0, c.stream>>>(B, c.seg_off, c.seg_nnz, ptr, c.wa, c.wb,
+                                                                       idx, cnt, cum, lineid, deg);
+    ++c.launches;
+    if (total) GSAP_CUDA(cudaMemcpyAsync(total, ptr + B, sizeof(int), cudaMemcpyDeviceToDevice, c.stream));
+    GSAP_CHECK_LAUNCH();
+}
+
+static void rebuild_sparse(Ctx &c) {
     const int B = c.B, E = c.E;
     if (E == 0) {
         GSAP_CUDA(cudaMemsetAsync(c.bm_rowptr, 0, sizeof(int) * ((size_t)B + 1), c.stream));
@@ -378,49 +413,18 @@ static void rebuild_sparse(Ctx &c) {
         GSAP_CUDA(cudaMemsetAsync(c.d_nnz, 0, sizeof(int), c.stream));
         return;
     }
-    const int sh = bits_for(B);
     const int g = grid_for(E, 256);
-    k_keys<<<g, 256, 0, c.stream>>>(E, c.esrc, c.col, c.wgt, c.b, sh, c.keys0, c.wa);
-    ++c.launches;
-    int which;
-    if (c.weighted)
-        which = radix_sort<u64, int, true>(c.keys0, c.keys1, c.wa, c.wb, nullptr, E, 2 * sh, c.counts, c.scan_tmp, L);
-    else
-        which = radix_sort<u64, int, false>(c.keys0, c.keys1, c.wa, c.wb, nullptr, E, 2 * sh, c.counts, c.scan_tmp, L);
-    const u64 *keys = which ? c.keys1 : c.keys0;
-    const int *w = which ? c.wb : c.wa;
-    k_heads<<<g, 256, 0, c.stream>>>(E, keys, c.flags);
-    ++c.launches;
-    device_scan<int>(c.flags, c.pos, nullptr, E, false, c.scan_tmp, c.d_nnz, L);
-    k_unique<<<g, 256, 0, c.stream>>>(E, keys, c.flags, c.pos, sh, c.rowid, c.bm_col, c.tmpi);
-    ++c.launches;
     if (c.weighted) {
-        GSAP_CUDA(cudaMemsetAsync(c.bm_cnt, 0, sizeof(int) * (size_t)E, c.stream));
-        k_cnt_weighted<<<g, 256, 0, c.stream>>>(E, c.flags, c.pos, w, c.bm_cnt);
+        build_lines<u64>(c, c.rowptr, c.col, c.wgt, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.rowid, c.dout,
+                         c.d_nnz);
+        build_lines<u64>(c, c.cscptr, c.cscsrc, c.cscwgt, c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.flags,
+                         c.din, nullptr);
     } else {
-        k_cnt_runs<<<g, 256, 0, c.stream>>>(E, c.tmpi, c.d_nnz, c.bm_cnt);
+        build_lines<unsigned>(c, c.rowptr, c.col, nullptr, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.rowid,
+                              c.dout, c.d_nnz);
+        build_lines<unsigned>(c, c.cscptr, c.cscsrc, nullptr, c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum,
+                              c.flags, c.din, nullptr);
     }
-    ++c.launches;
-    // CSR row pointers, cum, dout
-    k_ptr_from_ids<int><<<grid_for(B + 1, 256), 256, 0, c.stream>>>(c.rowid, c.d_nnz, E, B, c.bm_rowptr);
-    ++c.launches;
-    device_scan<int>(c.bm_cnt, c.tmpi, c.d_nnz, E, true, c.scan_tmp, nullptr, L);
-    k_seg_cum<<<g, 256, 0, c.stream>>>(c.rowid, c.bm_rowptr, c.tmpi, c.d_nnz, c.bm_cum);
-    k_seg_deg<<<grid_for(B, 256), 256, 0, c.stream>>>(B, c.bm_rowptr, c.tmpi, c.dout);
-    c.launches += 2;
-    // CSC: stable sort of the CSR entries by column (rows stay ascending)
-    k_csc_keys<<<g, 256, 0, c.stream>>>(c.d_nnz, c.bm_col, c.rowid, c.bm_cnt, c.ukeys0, c.vals64a);
-    ++c.launches;
-    const int w2 = radix_sort<unsigned, u64, true>(c.ukeys0, c.ukeys1, c.vals64a, c.vals64b, c.d_nnz, E, sh,
-                                                   c.counts, c.scan_tmp, L);
-    k_csc_unpack<<<g, 256, 0, c.stream>>>(c.d_nnz, w2 ? c.ukeys1 : c.ukeys0, w2 ? c.vals64b : c.vals64a,
-                                          c.flags, c.bm_row, c.bm_ccnt);
-    k_ptr_from_ids<int><<<grid_for(B + 1, 256), 256, 0, c.stream>>>(c.flags, c.d_nnz, E, B, c.bm_colptr);
-    c.launches += 2;
-    device_scan<int>(c.bm_ccnt, c.tmpi, c.d_nnz, E, true, c.scan_tmp, nullptr, L);
-    k_seg_cum<<<g, 256, 0, c.stream>>>(c.flags, c.bm_colptr, c.tmpi, c.d_nnz, c.bm_ccum);
-    k_seg_deg<<<grid_for(B, 256), 256, 0, c.stream>>>(B, c.bm_colptr, c.tmpi, c.din);
-    c.launches += 2;
     // per-row and per-column hash tables for O(1) lookups
     k_rtab_clear<<<grid_for(2LL * E, 256), 256, 0, c.stream>>>(c.d_nnz, c.rtab);
     k_rtab_clear<<<grid_for(2LL * E, 256), 256, 0, c.stream>>>(c.d_nnz, c.ctab);

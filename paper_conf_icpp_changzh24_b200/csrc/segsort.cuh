@@ -1,0 +1,324 @@
+// segsort.cuh -- the sparse-regime blockmodel rebuild as a counting sort by
+// line + per-line sort (Alg. 2, §3.4: "sort_by_key ... segsort ...
+// find_subseg_hds ... segreduce"), without a global sort of 64-bit keys:
+//
+//   1. line lengths: len[b[v]] += deg(v)                  (one atomic per vertex)
+//   2. offsets: exclusive scan of len
+//   3. scatter: each vertex appends the blocks of its neighbours to its line's
+//      segment (one atomic per vertex, coalesced writes; the order inside a
+//      segment is arbitrary, the sort below makes it canonical)
+//   4. per segment: sort + run-length encode (a warp for <= 512 entries, a CTA
+//      in shared memory for <= 4096, a CTA in global scratch beyond)
+//   5. compact: line pointers by scan, copy with cum and line sums.
+//
+// Keys are the neighbour block (unweighted, u32) or (block << 32 | weight)
+// (weighted, u64): equal blocks become adjacent and their weights are summed.
+#pragma once
+
+#include "common.cuh"
+
+namespace gsap {
+
+constexpr int SEG_WARP_MAX = 512;    // entries sorted by one warp in shared memory
+constexpr int SEG_WARPS = 8;
+
+// entries one CTA sorts in shared memory (48 KB of static shared memory)
+template <typename K>
+struct SegCta {
+    static constexpr int CAP = sizeof(K) == 8 ? 2048 : 4096;
+};
+
+template <typename K>
+GSAP_DEV int key_col(K k) { return sizeof(K) == 8 ? (int)(k >> 32) : (int)k; }
+template <typename K>
+GSAP_DEV int key_w(K k) { return sizeof(K) == 8 ? (int)(unsigned)(k & 0xffffffffULL) : 1; }
+template <typename K>
+GSAP_DEV K key_max() { return (K)~(K)0; }
+
+template <int NT>
+GSAP_DEV void nt_sync() {
+    if (NT == 32) __syncwarp();
+    else __syncthreads();
+}
+
+// bitonic sort of a[0, n), n a power of two, by NT cooperating threads
+template <typename K, int NT>
+GSAP_DEV void bitonic(K *a, int n, int tid) {
+    for (int k = 2; k <= n; k <<= 1) {
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            for (int i = tid; i < (n >> 1); i += NT) {
+                const int lo = ((i & ~(j - 1)) << 1) | (i & (j - 1));
+                const int hi = lo + j;
+                const bool up = (lo & k) == 0;
+                const K x = a[lo], y = a[hi];
+                if ((x > y) == up) {
+                    a[lo] = y;
+                    a[hi] = x;
+                }
+            }
+            nt_sync<NT>();
+        }
+    }
+}
+
+// run-length encode sorted a[0, L) by NT threads: hp[q] = start of run q;
+// writes (block, summed weight) of run q to ocol/ocnt[q]; returns the run count
+template <typename K, int NT>
+GSAP_DEV int rle_runs(const K *a, int L, int *hp, int *ocol, int *ocnt, int tid, int *sh) {
+    // each thread takes a contiguous chunk so the runs come out in order
+    const int chunk = (L + NT - 1) / NT;
+    const int lo = min(L, tid * chunk), hi = min(L, lo + chunk);
+    int heads = 0;
+    for (int i = lo; i < hi; ++i) heads += (i == 0 || key_col(a[i]) != key_col(a[i - 1])) ? 1 : 0;
+    // exclusive scan of heads over the NT threads
+    int x = heads;
+    const int lane = tid & 31;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(FULL, x, o);
+        if (lane >= o) x += t;
+    }
+    int base = x - heads, total;
+    if (NT == 32) {
+        total = __shfl_sync(FULL, x, 31);
+    } else {
+        const int w = tid >> 5;
+        if (lane == 31) sh[w] = x;
+        __syncthreads();
+        int wb = 0;
+        total = 0;
+        for (int i = 0; i < NT / 32; ++i) {
+            if (i < w) wb += sh[i];
+            total += sh[i];
+        }
+        base += wb;
+        __syncthreads();
+    }
+    for (int i = lo; i < hi; ++i)
+        if (i == 0 || key_col(a[i]) != key_col(a[i - 1])) hp[base++] = i;
+    nt_sync<NT>();
+    for (int q = tid; q < total; q += NT) {
+        const int s = hp[q], e = q + 1 < total ? hp[q + 1] : L;
+        int c;
+        if (sizeof(K) == 8) {
+            c = 0;
+            for (int i = s; i < e; ++i) c += key_w(a[i]);
+        } else {
+            c = e - s;
+        }
+        ocol[q] = key_col(a[s]);
+        ocnt[q] = c;
+    }
+    nt_sync<NT>();
+    return total;
+}
+
+// 1. len[b[v]] += deg(v)
+__global__ void k_line_len(int V, const int *__restrict__ gptr, const int *__restrict__ b, int *__restrict__ len) {
+    for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+        const int d = gptr[v + 1] - gptr[v];
+        if (d) atomicAdd(len + b[v], d);
+    }
+}
+
+// 3. scatter neighbour blocks into their line's segment (warp per vertex)
+template <typename K>
+__global__ void k_line_scatter(int V, const int *__restrict__ gptr, const int *__restrict__ gidx,
+                               const int *__restrict__ gw, const int *__restrict__ b,
+                               const int *__restrict__ off, int *__restrict__ cur, K *__restrict__ seg) {
+    const int lane = threadIdx.x & 31;
+    for (int v = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < V; v += (gridDim.x * blockDim.x) >> 5) {
+        const int lo = __ldg(gptr + v), n = __ldg(gptr + v + 1) - lo;
+        if (n == 0) continue;
+        const int x = __ldg(b + v);
+        int base = 0;
+        if (lane == 0) base = __ldg(off + x) + atomicAdd(cur + x, n);
+        base = __shfl_sync(FULL, base, 0);
+        for (int j = lane; j < n; j += 32) {
+            const int t = __ldg(b + __ldg(gidx + lo + j));
+            if (sizeof(K) == 8) seg[base + j] = (K)(((unsigned long long)(unsigned)t << 32) | (unsigned)__ldg(gw + lo + j));
+            else seg[base + j] = (K)(unsigned)t;
+        }
+    }
+}
+
+// 4a. classify lines by segment length
+__global__ void k_line_classify(int B, const int *__restrict__ off, int *__restrict__ nnz, int *__restrict__ listW,
+                                int *__restrict__ listC, int *__restrict__ counters) {
+    for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < B; x += gridDim.x * blockDim.x) {
+        const int L = off[x + 1] - off[x];
+        if (L == 0) nnz[x] = 0;
+        else if (L <= SEG_WARP_MAX) listW[atomicAdd(counters, 1)] = x;
+        else listC[atomicAdd(counters + 1, 1)] = x;
+    }
+}
+
+// 4b. short segments: one warp each, sorted in shared memory
+template <typename K>
+__global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__restrict__ off, K *__restrict__ seg,
+                                                                 const int *__restrict__ listW,
+                                                                 const int *__restrict__ counters,
+                                                                 int *__restrict__ tcol, int *__restrict__ tcnt,
+                                                                 int *__restrict__ nnz) {
+    __shared__ K keys[SEG_WARPS][SEG_WARP_MAX];
+    __shared__ int hp[SEG_WARPS][SEG_WARP_MAX];
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int n_lines = counters[0];
+    for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
+        const int x = listW[li];
+        const int o = off[x], L = off[x + 1] - o;
+        int n = 1;
+        while (n < L) n <<= 1;
+        for (int i = lane; i < n; i += 32) keys[w][i] = i < L ? seg[o + i] : key_max<K>();
+        __syncwarp();
+        bitonic<K, 32>(keys[w], n, lane);
+        const int u = rle_runs<K, 32>(keys[w], L, hp[w], tcol + o, tcnt + o, lane, nullptr);
+        if (lane == 0) nnz[x] = u;
+    }
+}
+
+// 4c. long segments: one CTA each, in shared memory (<= 4096) or in a global
+// scratch region at 2 * off (Sum of regions <= 2E)
+template <typename K>
+__global__ void __launch_bounds__(256) k_segsort_cta(const int *__restrict__ off, K *__restrict__ seg,
+                                                     const int *__restrict__ listC, const int *__restrict__ counters,
+                                                     int *__restrict__ tcol, int *__restrict__ tcnt,
+                                                     int *__restrict__ nnz, K *__restrict__ gkeys,
+                                                     int *__restrict__ ghp) {
+    constexpr int CAP = SegCta<K>::CAP;
+    __shared__ K skeys[CAP];
+    __shared__ int shp[CAP];
+    __shared__ int sh[8];
+    const int n_lines = counters[1];
+    for (int li = blockIdx.x; li < n_lines; li += gridDim.x) {
+        const int x = listC[li];
+        const int o = off[x], L = off[x + 1] - o;
+        if (L > CAP) continue;   // k_segsort_xl
+        int n = 1;
+        while (n < L) n <<= 1;
+        K *keys = skeys;
+        int *hp = shp;
+        for (int i = threadIdx.x; i < n; i += 256) keys[i] = i < L ? seg[o + i] : key_max<K>();
+        __syncthreads();
+        bitonic<K, 256>(keys, n, threadIdx.x);
+        const int u = rle_runs<K, 256>(keys, L, hp, tcol + o, tcnt + o, threadIdx.x, sh);
+        if (threadIdx.x == 0) nnz[x] = u;
+        __syncthreads();
+    }
+}
+
+// 4d. very long segments (> SegCta::CAP): one CTA each, LSD radix sort of the
+// segment over the key's block bits in global memory (8-bit digits; a tile of
+// 256 keys ranked stably with __match_any_sync per warp + per-warp digit
+// counts), ping-pong between the segment and its scratch region, then RLE.
+template <typename K>
+__global__ void __launch_bounds__(256) k_segsort_xl(const int *__restrict__ off, K *__restrict__ seg,
+                                                    const int *__restrict__ listC, const int *__restrict__ counters,
+                                                    int col_bits, int *__restrict__ tcol, int *__restrict__ tcnt,
+                                                    int *__restrict__ nnz, K *__restrict__ gkeys, int *__restrict__ ghp) {
+    __shared__ int hist[256];
+    __shared__ int base[256];
+    __shared__ int wcnt[8][256];
+    __shared__ int sh[8];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+    const int n_lines = counters[1];
+    const int shift0 = sizeof(K) == 8 ? 32 : 0;
+    for (int li = blockIdx.x; li < n_lines; li += gridDim.x) {
+        const int x = listC[li];
+        const int o = off[x], L = off[x + 1] - o;
+        if (L <= SegCta<K>::CAP) continue;   // handled by k_segsort_cta
+        K *src = seg + o;
+        K *dst = gkeys + 2 * (size_t)o;
+        for (int sbit = 0; sbit < col_bits; sbit += 8) {
+            const int shift = shift0 + sbit;
+            hist[tid] = 0;
+            __syncthreads();
+            for (int i = tid; i < L; i += 256) atomicAdd(&hist[(int)((src[i] >> shift) & 255)], 1);
+            __syncthreads();
+            {
+                int tot;
+                const int h = hist[tid];
+                int x2 = h;
+#pragma unroll
+                for (int q = 1; q < 32; q <<= 1) {
+                    const int t = __shfl_up_sync(FULL, x2, q);
+                    if (lane >= q) x2 += t;
+                }
+                if (lane == 31) sh[w] = x2;
+                __syncthreads();
+                int wb = 0;
+                tot = 0;
+                for (int q = 0; q < 8; ++q) {
+                    if (q < w) wb += sh[q];
+                    tot += sh[q];
+                }
+                base[tid] = wb + x2 - h;
+                __syncthreads();
+            }
+            for (int t0 = 0; t0 < L; t0 += 256) {
+                const int i = t0 + tid;
+                const bool valid = i < L;
+                const K k = valid ? src[i] : (K)0;
+                const int d = valid ? (int)((k >> shift) & 255) : 256;
+#pragma unroll
+                for (int q = 0; q < 8; ++q) wcnt[q][tid] = 0;
+                __syncthreads();
+                const unsigned peers = __match_any_sync(FULL, d);
+                const int rank = __popc(peers & lt);
+                if (valid && lane == __ffs(peers) - 1) wcnt[w][d] = __popc(peers);
+                __syncthreads();
+                // per digit (thread tid = digit): prefix over warps, then advance the base
+                {
+                    int run = 0;
+                    for (int q = 0; q < 8; ++q) {
+                        const int c = wcnt[q][tid];
+                        wcnt[q][tid] = run;
+                        run += c;
+                    }
+                    hist[tid] = run;   // this tile's count of digit tid
+                }
+                __syncthreads();
+                if (valid) dst[base[d] + wcnt[w][d] + rank] = k;
+                __syncthreads();
+                base[tid] += hist[tid];
+                __syncthreads();
+            }
+            K *t = src;
+            src = dst;
+            dst = t;
+            __syncthreads();
+        }
+        const int u = rle_runs<K, 256>(src, L, ghp + 2 * (size_t)o, tcol + o, tcnt + o, tid, sh);
+        if (tid == 0) nnz[x] = u;
+        __syncthreads();
+    }
+}
+
+// 5. compact line x's runs from its segment to ptr[x]: idx, cnt, cum, line id,
+// and the line's total weight (dout or din)
+__global__ void k_line_copy(int B, const int *__restrict__ off, const int *__restrict__ nnz,
+                            const int *__restrict__ ptr, const int *__restrict__ tcol, const int *__restrict__ tcnt,
+                            int *__restrict__ idx, int *__restrict__ cnt, int *__restrict__ cum,
+                            int *__restrict__ lineid, int *__restrict__ deg) {
+    const int lane = threadIdx.x & 31;
+    for (int x = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < B; x += (gridDim.x * blockDim.x) >> 5) {
+        const int o = off[x], n = nnz[x], p = ptr[x];
+        int run = 0;
+        for (int k0 = 0; k0 < n; k0 += 32) {
+            const int k = k0 + lane;
+            const int c = k < n ? tcnt[o + k] : 0;
+            const int sc = warp_incl_scan(c) + run;
+            if (k < n) {
+                idx[p + k] = tcol[o + k];
+                cnt[p + k] = c;
+                cum[p + k] = sc;
+                lineid[p + k] = x;
+            }
+            run = __shfl_sync(FULL, sc, 31);
+        }
+        if (lane == 0) deg[x] = run;
+    }
+}
+
+}  // namespace gsap

@@ -67,8 +67,11 @@ def test_rebuild_bit_exact(G, oracle_mod, gname, B):
 def test_rebuild_20k_all_regimes(G, oracle_mod):
     rowptr, col, truth, cfg = dcsbm.make("20k")
     ctx, orc = make_pair(G, oracle_mod, rowptr, col)
-    for B in (32, 1000, 1375, 1376, 5000, 20000):
-        b = dcsbm.random_partition(cfg.V, B, B)
+    skew = dcsbm.random_partition(cfg.V, 20000, 7)
+    skew[: cfg.V // 2] = 0                        # one giant block: lines of > 2^17 entries
+    skew = np.unique(skew, return_inverse=True)[1].astype(np.int32)
+    for B, b in [(B, dcsbm.random_partition(cfg.V, B, B)) for B in (32, 1000, 1375, 1376, 5000, 20000)] + \
+            [(int(skew.max()) + 1, skew)]:
         set_both(ctx, orc, b, B)
         assert_same_blockmodel(ctx, orc)
         m_g, S_g = ctx.gsap_mdl()
@@ -291,3 +294,17 @@ def test_cuda_graph_path_matches_stream_path(G, oracle_mod):
     b = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED, cuda_graphs=0)).gsap_run()
     assert np.array_equal(a["b"], b["b"]) and a["B"] == b["B"] and a["mdl"] == b["mdl"]
     assert np.array_equal(a["trace"][:, :4], b["trace"][:, :4])
+
+
+def test_rebuild_weighted_long_lines(G, oracle_mod):
+    """Weighted graph, sparse regime, with lines in every segment class (warp, CTA, global)."""
+    rowptr, col, truth, cfg = dcsbm.make("20k")
+    w = np.random.default_rng(3).integers(1, 6, len(col)).astype(np.int32)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w)
+    b = dcsbm.random_partition(cfg.V, 8000, 11)
+    b[: cfg.V // 3] = 0
+    b = np.unique(b, return_inverse=True)[1].astype(np.int32)
+    set_both(ctx, orc, b, int(b.max()) + 1)
+    assert_same_blockmodel(ctx, orc)
+    s = ctx.gsap_propose(G.GSAP_MOVE, 1, 2, 0, 2000)
+    assert np.array_equal(s, orc.propose(1, SEED, 1, 2, 0, 2000))
