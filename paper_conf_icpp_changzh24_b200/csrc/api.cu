@@ -185,7 +185,7 @@ static void check_sm100() {
 static void free_ctx(Ctx &c) {
     void *ptrs[] = {c.rowptr, c.col, c.wgt, c.cscptr, c.cscsrc, c.cscwgt, c.esrc, c.kout, c.kin, c.selfw,
                     c.big, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
-                    c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT, c.rtab, c.ctab,
+                    c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT,
                     c.rcp, c.fh, c.fl, c.keys0,
                     c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
                     c.rowid, c.counts, c.scan_tmp, c.rownnz, c.seg_len, c.seg_off, c.seg_cur, c.seg_nnz,
@@ -312,8 +312,6 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, 65536), (size_t)1 << 28);
     c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
     c.dense = dalloc<int>(c.dense_cap);
-    c.rtab = dalloc<int2>(2 * Es);
-    c.ctab = dalloc<int2>(2 * Es);
     c.rcp = dalloc<double>(Vs);
     {   // f-table: f(m) = m ln m in long double, split into double hi + float lo
         std::vector<double> fh(FT_N);

@@ -140,9 +140,6 @@ GSAP_DEV int warp_incl_scan(int v) {
 struct BM {
     int B;
     const int *__restrict__ dense;   // nullptr in the sparse regime
-    const int2 *__restrict__ rtab;   // sparse regime: per-row open-addressing tables {col, cnt},
-                                     // row x owns slots [2 rowptr[x], 2 rowptr[x+1])
-    const int2 *__restrict__ ctab;   // the same per column of the CSC: {row, cnt}
     const double *__restrict__ fh;   // f(m) = m ln m for m < FT_N, double-double (hi, lo)
     const float *__restrict__ fl;
     const double *__restrict__ rcp;  // 1 / (d_x + B) per block
@@ -168,37 +165,36 @@ GSAP_DEV int upper_bound(const int *__restrict__ a, int lo, int hi, long long p)
     return lo;
 }
 
-// ---- per-row hash tables (sparse regime): row x has 2 len(x) slots {col, cnt},
-// col = -1 empty, home slot = multiply-shift of the column, linear probing.
-GSAP_DEV unsigned col_mix(int y) { return (unsigned)y * 0x9E3779B1u; }
-
-// one row's (or column's) table, resolved once and probed many times
+// one row (or column) of M, resolved once and searched many times: the
+// lookups of a move all land in rows r, s and columns r, s, so the lines stay
+// hot in L1 and a binary search costs a few cache hits
 struct Line {
-    const int2 *__restrict__ t;
-    int cap;
+    const int *__restrict__ idx;
+    const int *__restrict__ cnt;
+    int len;
 };
 
-GSAP_DEV Line line_of(const int2 *__restrict__ tab, const int *__restrict__ ptr, int x) {
+GSAP_DEV Line line_of(const int *__restrict__ idx, const int *__restrict__ cnt, const int *__restrict__ ptr, int x) {
     const int lo = __ldg(ptr + x);
     Line L;
-    L.t = tab + 2 * (size_t)lo;
-    L.cap = 2 * (__ldg(ptr + x + 1) - lo);
+    L.idx = idx + lo;
+    L.cnt = cnt + lo;
+    L.len = __ldg(ptr + x + 1) - lo;
     return L;
 }
 
 GSAP_DEV int line_get(const Line &L, int y) {
-    if (L.cap == 0) return 0;
-    int sl = (int)pick(col_mix(y), (uint32_t)L.cap);
-    while (true) {
-        const int2 e = __ldg(L.t + sl);
-        if (e.x == y) return e.y;
-        if (e.x == -1) return 0;
-        if (++sl == L.cap) sl = 0;
+    int a = 0, b = L.len;
+    while (a < b) {
+        const int mid = (a + b) >> 1;
+        if (__ldg(L.idx + mid) < y) a = mid + 1;
+        else b = mid;
     }
+    return (a < L.len && __ldg(L.idx + a) == y) ? __ldg(L.cnt + a) : 0;
 }
 
-GSAP_DEV Line row_line(const BM &m, int x) { return line_of(m.rtab, m.rowptr, x); }
-GSAP_DEV Line col_line(const BM &m, int y) { return line_of(m.ctab, m.colptr, y); }
+GSAP_DEV Line row_line(const BM &m, int x) { return line_of(m.col, m.cnt, m.rowptr, x); }
+GSAP_DEV Line col_line(const BM &m, int y) { return line_of(m.row, m.ccnt, m.colptr, y); }
 
 GSAP_DEV int bm_at(const BM &m, int x, int y) {
     if (m.dense) return __ldg(m.dense + (size_t)x * m.B + y);

@@ -59,8 +59,6 @@ struct Ctx {
     int *bm_colptr = nullptr, *bm_row = nullptr, *bm_ccnt = nullptr, *bm_ccum = nullptr;
     int *dout = nullptr, *din = nullptr, *d_nnz = nullptr;
     int *dense = nullptr, *denseT = nullptr;
-    int2 *rtab = nullptr;          // sparse-regime per-row hash tables (2 slots per entry)
-    int2 *ctab = nullptr;          // ... and per-column (CSC) hash tables
     double *fh = nullptr;          // f-table hi / lo (FT_N entries)
     float *fl = nullptr;
     double *rcp = nullptr;         // 1 / (d_x + B), refreshed by every rebuild
@@ -114,8 +112,6 @@ struct Ctx {
         BM m;
         m.B = B;
         m.dense = dense_mode ? dense : nullptr;
-        m.rtab = rtab;
-        m.ctab = ctab;
         m.fh = fh;
         m.fl = fl;
         m.rcp = rcp;

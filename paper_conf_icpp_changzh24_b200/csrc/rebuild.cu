@@ -342,27 +342,6 @@ __global__ void k_csc_unpack(const int *__restrict__ d_n, const unsigned *__rest
     }
 }
 
-// per-row hash tables of M used for O(1) lookups in the sparse regime
-__global__ void k_rtab_clear(const int *__restrict__ d_n, int2 *__restrict__ tab) {
-    const long long n = 2LL * *d_n;
-    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
-        tab[i] = make_int2(-1, 0);
-}
-
-__global__ void k_rtab_insert(const int *__restrict__ d_n, const int *__restrict__ rowid, const int *__restrict__ col,
-                              const int *__restrict__ cnt, const int *__restrict__ rowptr, int2 *__restrict__ tab) {
-    const int n = *d_n;
-    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-        const int x = rowid[i], y = col[i];
-        const int lo = rowptr[x], cap = 2 * (rowptr[x + 1] - lo);
-        int2 *t = tab + 2 * (size_t)lo;
-        int sl = (int)pick(col_mix(y), (uint32_t)cap);
-        while (atomicCAS(&t[sl].x, -1, y) != -1)
-            if (++sl == cap) sl = 0;
-        t[sl].y = cnt[i];
-    }
-}
-
 __global__ void k_rcp(int B, const int *__restrict__ dout, const int *__restrict__ din, double *__restrict__ rcp) {
     for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < B; x += gridDim.x * blockDim.x)
         rcp[x] = 1.0 / ((double)dout[x] + (double)din[x] + (double)B);
@@ -413,7 +392,6 @@ static void rebuild_sparse(Ctx &c) {
         GSAP_CUDA(cudaMemsetAsync(c.d_nnz, 0, sizeof(int), c.stream));
         return;
     }
-    const int g = grid_for(E, 256);
     if (c.weighted) {
         build_lines<u64>(c, c.rowptr, c.col, c.wgt, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.rowid, c.dout,
                          c.d_nnz);
@@ -425,12 +403,6 @@ static void rebuild_sparse(Ctx &c) {
         build_lines<unsigned>(c, c.cscptr, c.cscsrc, nullptr, c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum,
                               c.flags, c.din, nullptr);
     }
-    // per-row and per-column hash tables for O(1) lookups
-    k_rtab_clear<<<grid_for(2LL * E, 256), 256, 0, c.stream>>>(c.d_nnz, c.rtab);
-    k_rtab_clear<<<grid_for(2LL * E, 256), 256, 0, c.stream>>>(c.d_nnz, c.ctab);
-    k_rtab_insert<<<g, 256, 0, c.stream>>>(c.d_nnz, c.rowid, c.bm_col, c.bm_cnt, c.bm_rowptr, c.rtab);
-    k_rtab_insert<<<g, 256, 0, c.stream>>>(c.d_nnz, c.flags, c.bm_row, c.bm_ccnt, c.bm_colptr, c.ctab);
-    c.launches += 4;
     GSAP_CHECK_LAUNCH();
 }
 
