@@ -63,7 +63,7 @@ typedef struct {
     int32_t cuda_graphs;      /* 1: capture each MCMC iteration as one CUDA graph (default) */
 } gsap_params;
 
-/* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU */
+/* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */
 typedef struct {
     int32_t nranks, rank, device;
     uint8_t nccl_id[128];     /* ncclUniqueId from rank 0, broadcast by the caller */
@@ -211,6 +211,26 @@ gsap_status gsap_sync(gsap_ctx *ctx);
  */
 gsap_status gsap_run(gsap_ctx *ctx, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
                      double *trace, int32_t trace_cap, int32_t *rounds_out);
+
+/*
+ * Multi-GPU: one process per GPU, every rank passes the same
+ * graph and a gsap_dist {nranks, rank, device, nccl_id}; each MOVE batch and
+ * each merge phase is split into contiguous slices (whole 1024-vertex chunks
+ * / block ranges), whose results are exchanged with ncclAllGather; every rank
+ * then applies them identically.  Results are bit-identical for any nranks.
+ * gsap_nccl_unique_id: rank 0 creates the id (host, 128 bytes) and the caller
+ * broadcasts it (e.g. with torch.distributed).  NCCL is loaded at run time.
+ */
+gsap_status gsap_nccl_unique_id(uint8_t *id_out);
+
+/*
+ * The slice of [0, n) rank `rank` of `nranks` owns: ceil(ceil(n/chunk)/nranks)
+ * whole chunks per rank, contiguous, in rank order (the last ranks may own
+ * fewer or none).  Host outputs: *first, *count, *per_rank (= the padded
+ * all-gather block, in elements).  Pure host function (no device needed).
+ */
+gsap_status gsap_shard_slice(int32_t n, int32_t chunk, int32_t nranks, int32_t rank, int32_t *first,
+                             int32_t *count, int32_t *per_rank);
 
 #ifdef __cplusplus
 }

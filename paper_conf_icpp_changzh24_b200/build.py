@@ -8,9 +8,9 @@ import subprocess
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libgsap.so")
-SOURCES = ["api.cu", "rebuild.cu", "move.cu", "merge.cu", "mdl.cu"]
+SOURCES = ["api.cu", "rebuild.cu", "move.cu", "merge.cu", "mdl.cu", "comm.cu"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
-              "-Xcompiler", "-fPIC", "-shared", "-cudart", "static"]
+              "-Xcompiler", "-fPIC", "-shared", "-cudart", "static", "-ldl"]
 
 
 def _stale() -> bool:

@@ -190,7 +190,7 @@ static void free_ctx(Ctx &c) {
                     c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
                     c.rowid, c.counts, c.scan_tmp, c.rownnz, c.seg_len, c.seg_off, c.seg_cur, c.seg_nnz,
                     c.seg_listW, c.seg_listC, c.seg_ctr, c.xl_hp, c.xl_keys, c.s, c.dS, c.H, c.acc, c.best, c.dSbest,
-                    c.partials, c.scal, c.scal_i, c.Dh, c.d_itr, c.skey0, c.skey1, c.sval0, c.sval1, c.rank,
+                    c.partials, c.scal, c.scal_i, c.Dh, c.d_itr, c.skey0, c.skey1, c.sval0, c.sval1, c.sel_rank,
                     c.nxt0, c.nxt1, c.mx0, c.mx1, c.oncyc, c.label, c.present, c.slot_b[0], c.slot_b[1],
                     c.slot_b[2]};
     for (void *p : ptrs)
@@ -203,6 +203,10 @@ static void free_ctx(Ctx &c) {
             cudaEventDestroy(p.second);
         }
         for (auto e : k->pool) cudaEventDestroy(e);
+    }
+    try {
+        comm_destroy(c);
+    } catch (...) {
     }
     if (c.own_stream && c.stream) cudaStreamDestroy(c.stream);
 }
@@ -218,8 +222,6 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
                         const gsap_params *params, const gsap_dist *dist, void *stream) {
     REQUIRE(V >= 1, GSAP_EINVAL, "V must be >= 1");
     REQUIRE(rowptr && (col || true), GSAP_EINVAL, "rowptr is NULL");
-    REQUIRE(!dist || dist->nranks <= 1, GSAP_EUNSUPPORTED,
-            "multi-GPU contexts are not built in this version (use one context per GPU)");
     check_sm100();
     if (params) c.prm = *params;
     else gsap_default_params(&c.prm);
@@ -259,6 +261,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.own_stream = true;
     }
     GSAP_CUDA(cudaGetDevice(&c.dev));
+    comm_init(c, dist);
+    if (c.nranks > 1) c.prm.cuda_graphs = 0;
     // host-side static info
     c.h_rowptr.resize((size_t)V + 1);
     for (int v = 0; v <= V; ++v) c.h_rowptr[v] = (int)rp[v];
@@ -354,13 +358,15 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.counts = dalloc<int>(c.counts_cap);
     c.scan_tmp_cap = std::max(c.counts_cap, VE) / 4096 + 16;
     c.scan_tmp = dalloc<int>(c.scan_tmp_cap);
-    c.s = dalloc<int>(Vs * (size_t)P);
-    c.dS = dalloc<double>(Vs * (size_t)P);
-    c.H = dalloc<double>(Vs);
-    c.acc = dalloc<unsigned char>(Vs);
-    c.best = dalloc<int>(Vs);
-    c.dSbest = dalloc<double>(Vs);
-    c.partials = dalloc<double>(VE / 512 + 64);   // >= max(E, B) / MDL_CHUNK, V / APPLY_CHUNK
+    // per-batch / per-phase buffers, padded for the rank-blocked all-gathers
+    const size_t pad = 65536;
+    c.s = dalloc<int>(std::max(Vs * (size_t)P, Vs + pad));
+    c.dS = dalloc<double>(std::max(Vs * (size_t)P, Vs + pad));
+    c.H = dalloc<double>(Vs + pad);
+    c.acc = dalloc<unsigned char>(Vs + pad);
+    c.best = dalloc<int>(Vs + pad);
+    c.dSbest = dalloc<double>(Vs + pad);
+    c.partials = dalloc<double>(VE / 512 + 1024);   // >= max(E, B) / MDL_CHUNK, V / APPLY_CHUNK + ranks
     c.scal = dalloc<double>(8);
     c.scal_i = dalloc<int>(8);
     c.Dh = dalloc<double>((size_t)c.prm.max_nodal_itr + 1);
@@ -369,7 +375,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.skey1 = dalloc<unsigned long long>(Vs);
     c.sval0 = dalloc<int>(Vs);
     c.sval1 = dalloc<int>(Vs);
-    c.rank = dalloc<int>(Vs);
+    c.sel_rank = dalloc<int>(Vs);
     c.nxt0 = dalloc<int>(Vs);
     c.nxt1 = dalloc<int>(Vs);
     c.mx0 = dalloc<int>(Vs);
@@ -416,19 +422,49 @@ static void merge_phase(Ctx &c, uint32_t outer, int K, int *best_out, double *dS
     REQUIRE(c.B >= 2, GSAP_ESTATE, "a merge phase needs B >= 2");
     REQUIRE(K >= 0 && K <= c.B / 2, GSAP_EINVAL, "K must be in [0, B/2]");
     const int B = c.B;
-    launch_merge_props(c, outer, 0, B, true, nullptr, nullptr, c.best, c.dSbest);
+    if (c.nranks == 1) {
+        launch_merge_props(c, outer, 0, B, true, nullptr, nullptr, c.best, c.dSbest);
+        c.st.n_merge_prop += (long long)B * c.prm.num_proposals;
+    } else {
+        // each rank proposes for its slice of blocks; winners all-gathered
+        int f, n, per;
+        shard_slice(B, 1, c.nranks, c.rank, &f, &n, &per);
+        launch_merge_props(c, outer, f, n, true, nullptr, nullptr, c.best + f, c.dSbest + f);
+        comm_allgather(c, c.best, (size_t)per, 1);
+        comm_allgather(c, c.dSbest, (size_t)per, 2);
+        c.st.n_merge_prop += (long long)n * c.prm.num_proposals;
+    }
     copy_out(c, best_out, c.best, sizeof(int) * (size_t)B);
     copy_out(c, dSbest_out, c.dSbest, sizeof(double) * (size_t)B);
     select_merges(c, c.best, c.dSbest, K, nullptr);
     rebuild(c);
-    c.st.n_merge_prop += (long long)B * c.prm.num_proposals;
 }
 
 static void move_batch(Ctx &c, uint32_t outer, uint32_t itr, int first, int count, double *dsum) {
-    launch_move(c, MOVE_FUSED, outer, itr, first, count, c.s, c.dS, nullptr, c.acc);
-    launch_apply(c, first, count, c.s, c.acc, c.dS, dsum, c.scal_i + 1);
+    if (c.nranks == 1) {
+        launch_move(c, MOVE_FUSED, outer, itr, first, count, c.s, c.dS, nullptr, c.acc);
+        launch_apply(c, first, count, c.s, c.acc, c.dS, dsum, c.scal_i + 1);
+        rebuild(c);
+        c.st.n_move_prop += count;
+        return;
+    }
+    // this rank's slice of the batch (whole APPLY_CHUNK_V chunks), results and
+    // fixed-chunk dS partials all-gathered, then applied and rebuilt everywhere
+    int f, n, per;
+    shard_slice(count, APPLY_CHUNK_V, c.nranks, c.rank, &f, &n, &per);
+    const int pc = per / APPLY_CHUNK_V;
+    const size_t boff = (size_t)c.rank * per, poff = (size_t)c.rank * pc;
+    if (n > 0) {
+        launch_move(c, MOVE_FUSED, outer, itr, first + f, n, c.s + boff, c.dS + boff, nullptr, c.acc + boff);
+        launch_partials(c, first + f, n, c.s + boff, c.acc + boff, c.dS + boff, c.partials + poff);
+    }
+    comm_allgather(c, c.s, (size_t)per, 1);
+    comm_allgather(c, c.acc, (size_t)per, 0);
+    comm_allgather(c, c.partials, (size_t)pc, 2);
+    const int chunks = (count + APPLY_CHUNK_V - 1) / APPLY_CHUNK_V;
+    launch_apply_gathered(c, first, count, c.s, c.acc, c.partials, chunks, dsum, c.scal_i + 1);
     rebuild(c);
-    c.st.n_move_prop += count;
+    c.st.n_move_prop += n;
 }
 
 static bool converged(Ctx &c, const std::vector<double> &D, int itr, double S, double thresh) {
@@ -931,6 +967,22 @@ gsap_status gsap_run(gsap_ctx *ctx, int32_t *bmap_out, int32_t *B_out, double *m
     API_TRY
     REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
     run_impl(ctx->c, bmap_out, B_out, mdl_out, trace, trace_cap, rounds_out);
+    API_CATCH
+}
+
+gsap_status gsap_nccl_unique_id(uint8_t *id_out) {
+    API_TRY
+    REQUIRE(id_out, GSAP_EINVAL, "NULL argument");
+    comm_unique_id(id_out);
+    API_CATCH
+}
+
+gsap_status gsap_shard_slice(int32_t n, int32_t chunk, int32_t nranks, int32_t rank, int32_t *first,
+                             int32_t *count, int32_t *per_rank) {
+    API_TRY
+    REQUIRE(n >= 0 && chunk >= 1 && nranks >= 1 && rank >= 0 && rank < nranks && first && count && per_rank,
+            GSAP_EINVAL, "bad argument");
+    shard_slice(n, chunk, nranks, rank, first, count, per_rank);
     API_CATCH
 }
 

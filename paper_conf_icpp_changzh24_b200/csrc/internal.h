@@ -90,12 +90,16 @@ struct Ctx {
     int *slot_b[3] = {nullptr, nullptr, nullptr};   // golden-section bracket partitions
     // merge selection scratch
     unsigned long long *skey0 = nullptr, *skey1 = nullptr;
-    int *sval0 = nullptr, *sval1 = nullptr, *rank = nullptr, *nxt0 = nullptr, *nxt1 = nullptr,
+    int *sval0 = nullptr, *sval1 = nullptr, *sel_rank = nullptr, *nxt0 = nullptr, *nxt1 = nullptr,
         *mx0 = nullptr, *mx1 = nullptr, *oncyc = nullptr, *label = nullptr, *present = nullptr;
 
     // pinned host scalars
     double *h_scal = nullptr;
     int *h_int = nullptr;
+
+    // multi-GPU
+    int nranks = 1, rank = 0;
+    void *nccl_comm = nullptr;
 
     // CUDA-graph capture of an MCMC iteration (N1: launch overhead, §5)
     unsigned *d_itr = nullptr;     // MCMC iteration read by k_move (device scalar)
@@ -153,6 +157,21 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
                  int *s, double *dS, double *H, unsigned char *acc, const unsigned *d_itr = nullptr);
 void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned char *acc,
                   const double *dS, double *dsum, int *nacc);
+
+void launch_partials(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
+                     double *partials);
+void launch_apply_gathered(Ctx &c, int first, int count, const int *s, const unsigned char *acc,
+                           const double *partials, int n, double *dsum, int *nacc);
+constexpr int APPLY_CHUNK_V = 1024;   // fixed reduction chunk of the accepted-dS sums (move.cu)
+
+// comm.cu: multi-GPU (one process per GPU, NCCL over NVLink, loaded at run time)
+void comm_init(Ctx &c, const gsap_dist *d);
+void comm_destroy(Ctx &c);
+void comm_allgather(Ctx &c, void *recv, size_t count_per_rank, int dtype);   // dtype: 0 int8, 1 int32, 2 f64
+void comm_unique_id(uint8_t out[128]);
+// the slice of [0, n) that rank g of G owns: whole chunks of `chunk`, contiguous,
+// ceil(ceil(n/chunk)/G) chunks per rank (the last ranks may own less or none)
+void shard_slice(int n, int chunk, int G, int g, int *first, int *count, int *per_rank);
 
 // merge.cu
 void launch_merge_props(Ctx &c, uint32_t outer, int first, int count, bool propose, int *s,

@@ -247,8 +247,8 @@ void select_merges(Ctx &c, const int *best, const double *dS, int K, int *label_
     const int w = radix_sort<u64, int, true>(c.skey0, c.skey1, c.sval0, c.sval1, nullptr, B, 64, c.counts,
                                              c.scan_tmp, L);
     const int *sorted = w ? c.sval1 : c.sval0;
-    k_sel_rank<<<g256(B), 256, 0, c.stream>>>(B, sorted, c.rank);
-    k_sel_init<<<g256(B), 256, 0, c.stream>>>(B, best, c.rank, c.nxt0, c.mx0, c.oncyc);
+    k_sel_rank<<<g256(B), 256, 0, c.stream>>>(B, sorted, c.sel_rank);
+    k_sel_init<<<g256(B), 256, 0, c.stream>>>(B, best, c.sel_rank, c.nxt0, c.mx0, c.oncyc);
     c.launches += 2;
     int *n0 = c.nxt0, *n1 = c.nxt1, *m0 = c.mx0, *m1 = c.mx1;
     for (int k = 0; k < rounds; ++k) {
@@ -257,7 +257,7 @@ void select_merges(Ctx &c, const int *best, const double *dS, int K, int *label_
         std::swap(m0, m1);
     }
     k_sel_mark<<<g256(B), 256, 0, c.stream>>>(B, n0, c.oncyc);
-    k_sel_accepted<<<g256(B), 256, 0, c.stream>>>(B, sorted, c.rank, m0, c.oncyc, c.flags);
+    k_sel_accepted<<<g256(B), 256, 0, c.stream>>>(B, sorted, c.sel_rank, m0, c.oncyc, c.flags);
     c.launches += rounds + 2;
     device_scan<int>(c.flags, c.pos, nullptr, B, true, c.scan_tmp, nullptr, L);
     k_sel_applied<<<g256(B), 256, 0, c.stream>>>(B, K, sorted, c.flags, c.pos, best, c.nxt0);

@@ -525,7 +525,7 @@ __global__ void __launch_bounds__(256) k_apply(int first, int count, const int *
     for (int k = threadIdx.x; k < APPLY_CHUNK; k += 256) {
         const int i = base + k;
         if (i < count && acc[i]) {
-            b[first + i] = s[i];
+            if (b) b[first + i] = s[i];
             sum += dS ? dS[i] : 0.0;
             ++na;
         }
@@ -535,7 +535,7 @@ __global__ void __launch_bounds__(256) k_apply(int first, int count, const int *
     sum = warp_sum(sum);
     if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = sum;
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (threadIdx.x == 0 && partials) {
         double t = 0.0;
         for (int w = 0; w < 8; ++w) t += sh[w];
         partials[blockIdx.x] = t;
@@ -564,6 +564,28 @@ void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned cha
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
     k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, c.b, c.partials, nacc);
     k_sum_partials<<<1, 256, 0, c.stream>>>(c.partials, nb, dsum, 1);
+    c.launches += 2;
+    GSAP_CHECK_LAUNCH();
+}
+
+// sharded batches: the fixed-chunk sums of accepted dS over [first, first+count)
+// (first aligned to APPLY_CHUNK from the batch start) into partials[0, ...)
+void launch_partials(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
+                     double *partials) {
+    if (count <= 0) return;
+    const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
+    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, nullptr, partials, nullptr);
+    ++c.launches;
+    GSAP_CHECK_LAUNCH();
+}
+
+// sharded batches: apply all gathered moves, then the ordered sum of n partials
+void launch_apply_gathered(Ctx &c, int first, int count, const int *s, const unsigned char *acc,
+                           const double *partials, int n, double *dsum, int *nacc) {
+    if (count <= 0) return;
+    const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
+    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, nullptr, c.b, nullptr, nacc);
+    k_sum_partials<<<1, 256, 0, c.stream>>>(partials, n, dsum, 1);
     c.launches += 2;
     GSAP_CHECK_LAUNCH();
 }

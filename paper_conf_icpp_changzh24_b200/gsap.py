@@ -26,7 +26,7 @@ EXPORTED = ["gsap_default_params", "gsap_last_error", "gsap_partition", "gsap_cr
             "gsap_set_partition", "gsap_get_partition", "gsap_update_blockmodel", "gsap_propose",
             "gsap_delta_mdl", "gsap_select_merges", "gsap_apply_moves", "gsap_move_batch",
             "gsap_merge_phase", "gsap_mdl", "gsap_get_blockmodel", "gsap_get_stats", "gsap_reset_stats",
-            "gsap_sync", "gsap_run"]
+            "gsap_sync", "gsap_run", "gsap_nccl_unique_id", "gsap_shard_slice"]
 
 
 class gsap_params(C.Structure):
@@ -99,6 +99,8 @@ def lib():
         L.gsap_reset_stats.argtypes = [vp]
         L.gsap_sync.argtypes = [vp]
         L.gsap_run.argtypes = [vp, vp, C.POINTER(i32), C.POINTER(C.c_double), vp, i32, C.POINTER(i32)]
+        L.gsap_nccl_unique_id.argtypes = [vp]
+        L.gsap_shard_slice.argtypes = [i32, i32, i32, i32, C.POINTER(i32), C.POINTER(i32), C.POINTER(i32)]
         for name in EXPORTED:
             if name not in ("gsap_default_params", "gsap_last_error", "gsap_destroy"):
                 getattr(L, name).restype = C.c_int
@@ -150,7 +152,38 @@ def gsap_default_params(**overrides) -> gsap_params:
     return p
 
 
-def gsap_partition(rowptr, col, wgt=None, params=None, device=False):
+def gsap_nccl_unique_id() -> bytes:
+    """A fresh ncclUniqueId (128 bytes) for gsap_dist; rank 0 creates, the caller broadcasts."""
+    buf = (C.c_uint8 * 128)()
+    _check(lib().gsap_nccl_unique_id(C.cast(buf, C.c_void_p)))
+    return bytes(buf)
+
+
+def gsap_shard_slice(n, chunk, nranks, rank):
+    """(first, count, per_rank) of the slice of [0, n) a rank owns (host only)."""
+    f, c, p = C.c_int32(0), C.c_int32(0), C.c_int32(0)
+    _check(lib().gsap_shard_slice(n, chunk, nranks, rank, C.byref(f), C.byref(c), C.byref(p)))
+    return f.value, c.value, p.value
+
+
+def make_dist(nranks, rank, device, nccl_id: bytes) -> gsap_dist:
+    d = gsap_dist(nranks=nranks, rank=rank, device=device)
+    C.memmove(d.nccl_id, nccl_id, 128)
+    return d
+
+
+def dist_from_torch(group=None):
+    """gsap_dist for this process from an initialised torch.distributed group."""
+    import torch
+    import torch.distributed as tdist
+    rank, world = tdist.get_rank(group), tdist.get_world_size(group)
+    obj = [gsap_nccl_unique_id() if rank == 0 else None]
+    tdist.broadcast_object_list(obj, src=0, group=group)
+    dev = torch.cuda.current_device() if torch.cuda.is_available() else 0
+    return make_dist(world, rank, dev, obj[0])
+
+
+def gsap_partition(rowptr, col, wgt=None, params=None, device=False, dist=None):
     """One-shot SBP on a CSR digraph; returns dict(b, B, mdl, stats)."""
     rowptr = np.ascontiguousarray(rowptr, np.int64) if isinstance(rowptr, (list, np.ndarray)) else rowptr
     V = int(rowptr.shape[0]) - 1
@@ -160,20 +193,22 @@ def gsap_partition(rowptr, col, wgt=None, params=None, device=False):
     mdl = C.c_double(0)
     st = gsap_stats()
     _check(lib().gsap_partition(V, _ptr(rowptr, np.int64), _ptr(col, np.int32), _ptr(wgt, np.int32),
-                                C.byref(params), None, _ptr(b), C.byref(B), C.byref(mdl), C.byref(st)))
+                                C.byref(params), C.byref(dist) if dist is not None else None, _ptr(b),
+                                C.byref(B), C.byref(mdl), C.byref(st)))
     return dict(b=b, B=B.value, mdl=mdl.value, stats=st.as_dict())
 
 
 class Context:
     """A gsap_ctx: device-resident graph, partition and blockmodel (stepwise API)."""
 
-    def __init__(self, rowptr, col, wgt=None, params=None, stream=None):
+    def __init__(self, rowptr, col, wgt=None, params=None, stream=None, dist=None):
         self.params = params or gsap_default_params()
         self.V = int(rowptr.shape[0]) - 1
         self._keep = (rowptr, col, wgt)
         h = C.c_void_p()
         _check(lib().gsap_create(self.V, _ptr(rowptr, np.int64), _ptr(col, np.int32),
-                                 _ptr(wgt, np.int32), C.byref(self.params), None, stream, C.byref(h)))
+                                 _ptr(wgt, np.int32), C.byref(self.params),
+                                 C.byref(dist) if dist is not None else None, stream, C.byref(h)))
         self.h = h
 
     def close(self):
