@@ -220,6 +220,51 @@ __global__ void __launch_bounds__(PT_THREADS) k_rs_downsweep(const K *__restrict
     }
 }
 
+// one CTA scans everything (small arrays: one launch instead of three)
+constexpr int SS_THREADS = 1024, SS_ITEMS = 8;
+template <typename T, bool INCLUSIVE>
+__global__ void __launch_bounds__(SS_THREADS) k_scan_single(const T *in, T *out, const int *d_n, int n_static,
+                                                             T *total) {
+    __shared__ T sh[SS_THREADS / 32];
+    const int n = read_n(d_n, n_static);
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    T carry = 0;
+    for (int base = 0; base < n; base += SS_THREADS * SS_ITEMS) {
+        T v[SS_ITEMS], s = 0;
+#pragma unroll
+        for (int i = 0; i < SS_ITEMS; ++i) {
+            const int idx = base + threadIdx.x * SS_ITEMS + i;
+            v[i] = idx < n ? in[idx] : T(0);
+            s += v[i];
+        }
+        T x = s;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const T t = __shfl_up_sync(FULL, x, o);
+            if (lane >= o) x += t;
+        }
+        if (lane == 31) sh[w] = x;
+        __syncthreads();
+        T wb = 0, tot = 0;
+        for (int i = 0; i < SS_THREADS / 32; ++i) {
+            const T q = sh[i];
+            if (i < w) wb += q;
+            tot += q;
+        }
+        __syncthreads();
+        T ex = carry + wb + x - s;
+#pragma unroll
+        for (int i = 0; i < SS_ITEMS; ++i) {
+            const int idx = base + threadIdx.x * SS_ITEMS + i;
+            if (INCLUSIVE) ex += v[i];
+            if (idx < n) out[idx] = ex;
+            if (!INCLUSIVE) ex += v[i];
+        }
+        carry += tot;
+    }
+    if (total && threadIdx.x == 0) *total = carry;
+}
+
 // host side -----------------------------------------------------------------
 struct Launcher {
     cudaStream_t stream;
@@ -234,6 +279,12 @@ void device_scan(const T *in, T *out, const int *d_n, int n_max, bool inclusive,
                  T *total, const Launcher &L) {
     const int nt = tiles_for(n_max);
     if (nt == 0) return;
+    if (n_max <= 4 * SS_THREADS * SS_ITEMS) {
+        if (inclusive) k_scan_single<T, true><<<1, SS_THREADS, 0, L.stream>>>(in, out, d_n, n_max, total);
+        else k_scan_single<T, false><<<1, SS_THREADS, 0, L.stream>>>(in, out, d_n, n_max, total);
+        *L.launches += 1;
+        return;
+    }
     k_tile_sums<T><<<nt, PT_THREADS, 0, L.stream>>>(in, d_n, n_max, tmp);
     k_scan_small<T><<<1, PT_THREADS, 0, L.stream>>>(tmp, nt, total);
     if (inclusive)

@@ -153,7 +153,127 @@ __global__ void k_line_classify(int B, const int *__restrict__ off, int *__restr
     }
 }
 
-// 4b. short segments: one warp each, sorted in shared memory
+// bitonic sort of 32*E keys held in registers, blocked layout (lane l holds
+// elements l*E .. l*E+E-1): partners inside a lane swap registers, partners
+// in other lanes come over __shfl_xor_sync.  Fully unrolled.
+template <typename K, int E>
+GSAP_DEV void warp_bitonic(K (&v)[E]) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int k = 2; k <= 32 * E; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            if (j >= E) {
+#pragma unroll
+                for (int e = 0; e < E; ++e) {
+                    const int i = lane * E + e;
+                    const K o = __shfl_xor_sync(FULL, v[e], j / E);
+                    const bool up = (i & k) == 0, lower = (i & j) == 0;
+                    v[e] = (lower == up) ? (v[e] < o ? v[e] : o) : (v[e] < o ? o : v[e]);
+                }
+            } else {
+#pragma unroll
+                for (int e = 0; e < E; ++e) {
+                    if ((e & j) == 0) {
+                        const int i = lane * E + e;
+                        const bool up = (i & k) == 0;
+                        const K a = v[e], b = v[e + j];
+                        if ((a > b) == up) {
+                            v[e] = b;
+                            v[e + j] = a;
+                        }
+                    }
+                }
+            }
+        }
+    }
+}
+
+// sort + RLE of one segment of L <= 32*E keys by one warp, in registers;
+// runs written to ocol / ocnt, returns the run count (warp-uniform)
+template <typename K, int E>
+GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict__ ocol, int *__restrict__ ocnt) {
+    const int lane = threadIdx.x & 31;
+    K v[E];
+#pragma unroll
+    for (int e = 0; e < E; ++e) {   // coalesced (striped) load: the sort permutes anyway
+        const int i = e * 32 + lane;
+        v[e] = i < L ? src[i] : key_max<K>();
+    }
+    warp_bitonic<K, E>(v);
+    // run heads and their ranks
+    const K prev_last = __shfl_up_sync(FULL, v[E - 1], 1);
+    int heads = 0;
+    bool head[E];
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+        const int i = lane * E + e;
+        const K p = e == 0 ? prev_last : v[e - 1];
+        head[e] = i < L && (i == 0 || key_col(v[e]) != key_col(p));
+        heads += head[e] ? 1 : 0;
+    }
+    int x = heads;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(FULL, x, o);
+        if (lane >= o) x += t;
+    }
+    const int total = __shfl_sync(FULL, x, 31);
+    int q = x - heads;
+    // weight of each run: inclusive prefix of weights, differenced at heads
+    int wsum[E], run = 0;
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+        const int i = lane * E + e;
+        run += i < L ? key_w(v[e]) : 0;
+        wsum[e] = run;
+    }
+    int y = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(FULL, y, o);
+        if (lane >= o) y += t;
+    }
+    const int lane_base = y - run;   // weight before this lane's first element
+    // a run's weight = (prefix at its last element) - (prefix before its head):
+    // the head's lane writes the negative start prefix, then (after a
+    // __syncwarp) the lane holding the run's last element adds its prefix
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+        if (head[e]) {
+            ocol[q] = key_col(v[e]);
+            ocnt[q] = -(lane_base + (e == 0 ? 0 : wsum[e - 1]));
+            ++q;
+        }
+    }
+    __syncwarp();
+    const bool nb_head0 = __shfl_down_sync(FULL, head[0] ? 1 : 0, 1) != 0;   // lane+1's first flag
+    const int qbase = x - heads;
+    int seen = 0;
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+        const int i = lane * E + e;
+        seen += head[e] ? 1 : 0;
+        if (i < L && (i == L - 1 || (e + 1 < E ? head[e + 1] : nb_head0)))
+            ocnt[qbase + seen - 1] += lane_base + wsum[e];
+    }
+    __syncwarp();
+    return total;
+}
+
+// 4b. short segments: one warp each, sorted in registers
+template <typename K, int E>
+GSAP_DEV void seg_warp_one(const int *__restrict__ off, const K *__restrict__ seg, int x, int *tcol, int *tcnt,
+                           int *nnz) {
+    const int o = off[x], L = off[x + 1] - o;
+    const int u = warp_segsort_rle<K, E>(seg + o, L, tcol + o, tcnt + o);
+    if ((threadIdx.x & 31) == 0) nnz[x] = u;
+}
+
+#ifndef GSAP_SEG_REG
+#define GSAP_SEG_REG 0   // 1: register bitonic (slower for 256 < L <= 512 on B200, kept for reference)
+#endif
+#if !GSAP_SEG_REG
 template <typename K>
 __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__restrict__ off, K *__restrict__ seg,
                                                                  const int *__restrict__ listW,
@@ -176,6 +296,26 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__re
         if (lane == 0) nnz[x] = u;
     }
 }
+#else
+template <typename K>
+__global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__restrict__ off, K *__restrict__ seg,
+                                                                 const int *__restrict__ listW,
+                                                                 const int *__restrict__ counters,
+                                                                 int *__restrict__ tcol, int *__restrict__ tcnt,
+                                                                 int *__restrict__ nnz) {
+    const int w = threadIdx.x >> 5;
+    const int n_lines = counters[0];
+    for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
+        const int x = listW[li];
+        const int L = off[x + 1] - off[x];
+        if (L <= 32) seg_warp_one<K, 1>(off, seg, x, tcol, tcnt, nnz);
+        else if (L <= 64) seg_warp_one<K, 2>(off, seg, x, tcol, tcnt, nnz);
+        else if (L <= 128) seg_warp_one<K, 4>(off, seg, x, tcol, tcnt, nnz);
+        else if (L <= 256) seg_warp_one<K, 8>(off, seg, x, tcol, tcnt, nnz);
+        else seg_warp_one<K, 16>(off, seg, x, tcol, tcnt, nnz);
+    }
+}
+#endif
 
 // 4c. long segments: one CTA each, in shared memory (<= 4096) or in a global
 // scratch region at 2 * off (Sum of regions <= 2E)
