@@ -61,6 +61,7 @@ typedef struct {
     int32_t max_rounds;       /* guard on merge+MCMC rounds; default 500 */
     int32_t profile;          /* 1: time kernels with CUDA events (gsap_stats k_*) */
     int32_t cuda_graphs;      /* 1: capture each MCMC iteration as one CUDA graph (default) */
+    int32_t dense_max_B;      /* dense blockmodel iff B <= this; 0 = auto (B^2 <= max(4E, 2^24)) */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */

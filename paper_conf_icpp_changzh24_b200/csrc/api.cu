@@ -313,8 +313,10 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.dout = dalloc<int>(Vs);
     c.din = dalloc<int>(Vs);
     c.d_nnz = dalloc<int>(1);
-    c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, 65536), (size_t)1 << 28);
+    c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, (size_t)1 << 24), (size_t)1 << 28);
     c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
+    if (c.prm.dense_max_B > 0)
+        c.dense_cap = std::min<size_t>(c.dense_cap, (size_t)c.prm.dense_max_B * (size_t)c.prm.dense_max_B);
     c.dense = dalloc<int>(c.dense_cap);
     c.rcp = dalloc<double>(Vs);
     {   // f-table: f(m) = m ln m in long double, split into double hi + float lo
@@ -724,6 +726,7 @@ void gsap_default_params(gsap_params *p) {
     p->max_rounds = 500;
     p->profile = 0;
     p->cuda_graphs = 1;
+    p->dense_max_B = 0;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }

@@ -5,12 +5,12 @@
 // as CSR (rows ascending column) + CSC (columns ascending row) with the
 // in-row / in-column inclusive prefix `cum` used by the proposal walks, and the
 // out / in block degrees.  Two regimes:
-//   dense  (B^2 <= 4E): shared-memory-privatised (B <= 221) or L2-atomic
+//   dense  (B^2 <= max(4E, 2^24)): shared-memory-privatised (B <= 221) or L2-atomic
 //          histogram into a dense B x B matrix, tiled transpose, warp-per-row
 //          compaction into CSR / CSC;
-//   sparse (B^2 > 4E): 64-bit keys (b_src << sh | b_dst), stable LSD radix sort
-//          (prims.cuh), run-length encode, row pointers by lower bound, cum by
-//          one global scan; CSC by a second stable radix sort on the column.
+//   sparse (otherwise): counting sort of the edges by line + per-line segment
+//          sort and run-length encoding (segsort.cuh), for rows (out-CSR) and
+//          columns (in-CSC) alike.
 #include <algorithm>
 
 #include "internal.h"
@@ -223,8 +223,107 @@ __global__ void k_row_compact(const int *__restrict__ M, int B, const int *__res
     }
 }
 
+// both dense matrices (M: lines x < B, its transpose: lines x >= B) in one launch
+__global__ void k_row_stats2(const int *__restrict__ M, const int *__restrict__ Mt, int B, int *__restrict__ nnzA,
+                             int *__restrict__ sumA, int *__restrict__ nnzB, int *__restrict__ sumB) {
+    const int lane = threadIdx.x & 31;
+    for (int x2 = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x2 < 2 * B; x2 += (gridDim.x * blockDim.x) >> 5) {
+        const bool t = x2 >= B;
+        const int x = t ? x2 - B : x2;
+        const int *__restrict__ R = (t ? Mt : M) + (size_t)x * B;
+        int c = 0, s = 0;
+        for (int y = lane; y < B; y += 32) {
+            const int v = R[y];
+            c += v != 0;
+            s += v;
+        }
+        c = warp_sum(c);
+        s = warp_sum(s);
+        if (lane == 0) {
+            (t ? nnzB : nnzA)[x] = c;
+            (t ? sumB : sumA)[x] = s;
+        }
+    }
+}
+
+// two exclusive scans of n <= 32K ints, one CTA each (dense regime: B <= 16384)
+__global__ void __launch_bounds__(1024) k_scan2(const int *a0, int *o0, const int *a1, int *o1, int n) {
+    __shared__ int sh[32];
+    const int *in = blockIdx.x ? a1 : a0;
+    int *out = blockIdx.x ? o1 : o0;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int carry = 0;
+    for (int base = 0; base < n; base += 1024 * 8) {
+        int v[8], sm = 0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int idx = base + threadIdx.x * 8 + i;
+            v[i] = idx < n ? in[idx] : 0;
+            sm += v[i];
+        }
+        int x = sm;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(FULL, x, o);
+            if (lane >= o) x += t;
+        }
+        if (lane == 31) sh[w] = x;
+        __syncthreads();
+        int wb = 0, tot = 0;
+        for (int i = 0; i < 32; ++i) {
+            const int q = sh[i];
+            if (i < w) wb += q;
+            tot += q;
+        }
+        __syncthreads();
+        int ex = carry + wb + x - sm;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int idx = base + threadIdx.x * 8 + i;
+            if (idx < n) out[idx] = ex;
+            ex += v[i];
+        }
+        carry += tot;
+    }
+    if (threadIdx.x == 0) out[n] = carry;
+}
+
+// compaction of both matrices + nnz + rcp = 1 / (d_x + B)
+__global__ void k_row_compact2(const int *__restrict__ M, const int *__restrict__ Mt, int B,
+                               const int *__restrict__ ptrA, int *__restrict__ idxA, int *__restrict__ cntA,
+                               int *__restrict__ cumA, const int *__restrict__ ptrB, int *__restrict__ idxB,
+                               int *__restrict__ cntB, int *__restrict__ cumB, const int *__restrict__ dout,
+                               const int *__restrict__ din, double *__restrict__ rcp, int *__restrict__ d_nnz) {
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *d_nnz = ptrA[B];
+    for (int x2 = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x2 < 2 * B; x2 += (gridDim.x * blockDim.x) >> 5) {
+        const bool t = x2 >= B;
+        const int x = t ? x2 - B : x2;
+        const int *__restrict__ R = (t ? Mt : M) + (size_t)x * B;
+        int *__restrict__ idx = t ? idxB : idxA;
+        int *__restrict__ cnt = t ? cntB : cntA;
+        int *__restrict__ cum = t ? cumB : cumA;
+        int base = (t ? ptrB : ptrA)[x], run = 0;
+        if (!t && lane == 0) rcp[x] = 1.0 / ((double)dout[x] + (double)din[x] + (double)B);
+        for (int y0 = 0; y0 < B; y0 += 32) {
+            const int y = y0 + lane;
+            const int v = y < B ? R[y] : 0;
+            const unsigned bal = __ballot_sync(FULL, v != 0);
+            const int sc = warp_incl_scan(v) + run;
+            if (v != 0) {
+                const int p = base + __popc(bal & lt);
+                idx[p] = y;
+                cnt[p] = v;
+                cum[p] = sc;
+            }
+            base += __popc(bal);
+            run = __shfl_sync(FULL, sc, 31);
+        }
+    }
+}
+
 static void rebuild_dense(Ctx &c) {
-    Launcher L{c.stream, &c.launches};
     const int B = c.B, E = c.E;
     const size_t BB = (size_t)B * B;
     GSAP_CUDA(cudaMemsetAsync(c.dense, 0, sizeof(int) * BB, c.stream));
@@ -249,16 +348,13 @@ static void rebuild_dense(Ctx &c) {
     }
     dim3 tg((B + 31) / 32, (B + 31) / 32), tb(32, 8);
     k_transpose<<<tg, tb, 0, c.stream>>>(c.dense, B, c.denseT);
-    const int rg = grid_for((long long)B * 32, 256);
-    k_row_stats<<<rg, 256, 0, c.stream>>>(c.dense, B, c.rownnz, c.dout);
-    k_row_stats<<<rg, 256, 0, c.stream>>>(c.denseT, B, c.tmpi, c.din);
-    c.launches += 3;
-    device_scan<int>(c.rownnz, c.bm_rowptr, nullptr, B, false, c.scan_tmp, c.bm_rowptr + B, L);
-    device_scan<int>(c.tmpi, c.bm_colptr, nullptr, B, false, c.scan_tmp, c.bm_colptr + B, L);
-    k_row_compact<<<rg, 256, 0, c.stream>>>(c.dense, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum);
-    k_row_compact<<<rg, 256, 0, c.stream>>>(c.denseT, B, c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum);
-    c.launches += 2;
-    GSAP_CUDA(cudaMemcpyAsync(c.d_nnz, c.bm_rowptr + B, sizeof(int), cudaMemcpyDeviceToDevice, c.stream));
+    const int rg = grid_for(2LL * B * 32, 256);
+    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.rownnz, c.dout, c.tmpi, c.din);
+    k_scan2<<<2, 1024, 0, c.stream>>>(c.rownnz, c.bm_rowptr, c.tmpi, c.bm_colptr, B);
+    k_row_compact2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum,
+                                             c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp,
+                                             c.d_nnz);
+    c.launches += 4;
     GSAP_CHECK_LAUNCH();
 }
 
@@ -410,10 +506,13 @@ void rebuild(Ctx &c) {
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_rebuild, &ev);
     c.dense_mode = dense_ok(c, c.B);
-    if (c.dense_mode) rebuild_dense(c);
-    else rebuild_sparse(c);
-    k_rcp<<<grid_for(c.B, 256), 256, 0, c.stream>>>(c.B, c.dout, c.din, c.rcp);
-    ++c.launches;
+    if (c.dense_mode) {
+        rebuild_dense(c);   // rcp written by the compaction
+    } else {
+        rebuild_sparse(c);
+        k_rcp<<<grid_for(c.B, 256), 256, 0, c.stream>>>(c.B, c.dout, c.din, c.rcp);
+        ++c.launches;
+    }
     // algorithmic bytes: the compulsory inputs (dst ids,
     // row pointers, b) and the fixed-size outputs (row / column pointers,
     // degrees); the nnz-sized outputs are left out (nnz stays on the device)

@@ -25,6 +25,9 @@ def G():
     return gsap
 
 
+SPARSE = {"dense_max_B": 1}     # force the sparse (CSR-line) blockmodel regime
+
+
 def make_pair(G, oracle_mod, rowptr, col, wgt=None, **params):
     p = G.gsap_default_params(seed=SEED, **params)
     ctx = G.Context(rowptr, col, wgt, params=p)
@@ -51,13 +54,14 @@ GRAPHS = {
 }
 
 
+@pytest.mark.parametrize("regime", ["auto", "sparse"])
 @pytest.mark.parametrize("gname", list(GRAPHS))
 @pytest.mark.parametrize("B", [1, 2, 7, 11, 150, 222, 299, 300])
-def test_rebuild_bit_exact(G, oracle_mod, gname, B):
+def test_rebuild_bit_exact(G, oracle_mod, gname, B, regime):
     rowptr, col, w = GRAPHS[gname]()
     V = len(rowptr) - 1
     B = min(B, V)
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **(SPARSE if regime == "sparse" else {}))
     assert_same_blockmodel(ctx, orc)      # singleton partition at create
     b = dcsbm.random_partition(V, B, B)
     set_both(ctx, orc, b, B)
@@ -86,11 +90,12 @@ def _states(V, rng_seed):
         yield B, dcsbm.random_partition(V, B, int(rng.integers(1 << 30)))
 
 
+@pytest.mark.parametrize("regime", ["auto", "sparse"])
 @pytest.mark.parametrize("gname", list(GRAPHS))
-def test_move_proposals_dS_accept(G, oracle_mod, gname):
+def test_move_proposals_dS_accept(G, oracle_mod, gname, regime):
     rowptr, col, w = GRAPHS[gname]()
     V = len(rowptr) - 1
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **(SPARSE if regime == "sparse" else {}))
     nties = 0
     for B, b in _states(V, 5):
         set_both(ctx, orc, b, B)
@@ -108,11 +113,12 @@ def test_move_proposals_dS_accept(G, oracle_mod, gname):
     print("MH ties:", nties)
 
 
+@pytest.mark.parametrize("regime", ["auto", "sparse"])
 @pytest.mark.parametrize("gname", list(GRAPHS))
-def test_merge_proposals_dS_best(G, oracle_mod, gname):
+def test_merge_proposals_dS_best(G, oracle_mod, gname, regime):
     rowptr, col, w = GRAPHS[gname]()
     V = len(rowptr) - 1
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **(SPARSE if regime == "sparse" else {}))
     for B, b in _states(V, 9):
         if B < 2:
             continue
@@ -150,9 +156,10 @@ def test_select_merges_bit_exact(G, oracle_mod, seed):
     assert_same_blockmodel(ctx, orc)
 
 
-def test_merge_phase_lockstep(G, oracle_mod):
+@pytest.mark.parametrize("regime", ["auto", "sparse"])
+def test_merge_phase_lockstep(G, oracle_mod, regime):
     rowptr, col, truth, cfg = dcsbm.make("1k")
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **(SPARSE if regime == "sparse" else {}))
     for outer in range(4):
         B = ctx.B
         K = int(0.4 * B)
@@ -173,11 +180,12 @@ def test_merge_phase_lockstep(G, oracle_mod):
         assert_same_blockmodel(ctx, orc)
 
 
+@pytest.mark.parametrize("regime", ["auto", "sparse"])
 @pytest.mark.parametrize("name", ["1k", "20k"])
-def test_mcmc_lockstep(G, oracle_mod, name):
+def test_mcmc_lockstep(G, oracle_mod, name, regime):
     """Batches of the fused hot loop vs the oracle, state compared after every batch."""
     rowptr, col, truth, cfg = dcsbm.make(name)
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **(SPARSE if regime == "sparse" else {}))
     # start from a merged state (as after the first merge phases)
     V = cfg.V
     B = max(2, int(V ** 0.5))
@@ -208,7 +216,8 @@ def test_mcmc_lockstep(G, oracle_mod, name):
     print("MH ties:", nties)
 
 
-def test_big_vertices_and_global_tables(G, oracle_mod):
+@pytest.mark.parametrize("regime", ["auto", "sparse"])
+def test_big_vertices_and_global_tables(G, oracle_mod, regime):
     """Hubs with > 128 and > 2048 distinct neighbour blocks (CTA path, global table)."""
     rng = np.random.default_rng(0)
     V = 6000
@@ -226,7 +235,7 @@ def test_big_vertices_and_global_tables(G, oracle_mod):
     np.add.at(rowptr, src[order] + 1, 1)
     rowptr = np.cumsum(rowptr)
     col = dst[order].astype(np.int32)
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **(SPARSE if regime == "sparse" else {}))
     for B in (100, 3000, V):
         b = dcsbm.random_partition(V, B, B)
         set_both(ctx, orc, b, B)
@@ -263,9 +272,10 @@ def test_edge_cases(G, oracle_mod):
         G.Context(np.array([0, 2], np.int64), np.array([0, 5], np.int32))
 
 
-def test_end_to_end_1k(G, oracle_mod):
+@pytest.mark.parametrize("regime", ["auto", "sparse"])
+def test_end_to_end_1k(G, oracle_mod, regime):
     rowptr, col, truth, cfg = dcsbm.make("1k")
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **(SPARSE if regime == "sparse" else {}))
     res = ctx.gsap_run()
     ref = orc.partition_run()
     assert abs(res["mdl"] - ref["mdl"]) <= 0.01 * ref["mdl"]
@@ -300,7 +310,7 @@ def test_rebuild_weighted_long_lines(G, oracle_mod):
     """Weighted graph, sparse regime, with lines in every segment class (warp, CTA, global)."""
     rowptr, col, truth, cfg = dcsbm.make("20k")
     w = np.random.default_rng(3).integers(1, 6, len(col)).astype(np.int32)
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **SPARSE)
     b = dcsbm.random_partition(cfg.V, 8000, 11)
     b[: cfg.V // 3] = 0
     b = np.unique(b, return_inverse=True)[1].astype(np.int32)
