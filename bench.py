@@ -232,12 +232,16 @@ def main():
     classes = {"move": (st["k_move_ms"], st["k_move_bytes"], st["k_move_launches"]),
                "rebuild": (st["k_rebuild_ms"], st["k_rebuild_bytes"], st["k_rebuild_launches"]),
                "merge": (st["k_merge_ms"], st["k_merge_bytes"], st["k_merge_launches"])}
-    dom = max(classes, key=lambda k: classes[k][0])
+    # the dominant single kernel of the step is k_move (fused proposal + dS + MH,
+    # timed with its k_propose half): see profiles/r01_bench20k_launches.txt;
+    # the rebuild "class" is ~15 different small kernels
+    dom = "move"
     ms, byts, launches = classes[dom]
     hbm = pk.get("hbm_gbs", 6650.0)
     achieved = (byts / launches) / (ms / launches / 1e3) / 1e9 if ms > 0 and launches else 0.0
     roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                "frac": achieved / hbm, "traffic": traffic_for(dom), "kernel": dom,
+                "frac": achieved / hbm, "traffic": traffic_for(dom),
+                "kernel": "k_propose + k_move (fused proposal, dS, Hastings, MH accept; one MOVE batch)",
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in pk else "fallback 6650",
                 "share_of_step": (ms / total_ms) if total_ms else None,
                 "launches": launches, "ms_per_launch": ms / max(launches, 1),

@@ -186,7 +186,7 @@ static void free_ctx(Ctx &c) {
     void *ptrs[] = {c.rowptr, c.col, c.wgt, c.cscptr, c.cscsrc, c.cscwgt, c.esrc, c.kout, c.kin, c.selfw,
                     c.big, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
                     c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT,
-                    c.rcp, c.fh, c.fl, c.keys0,
+                    c.rcp, c.ft, c.keys0,
                     c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
                     c.rowid, c.counts, c.scan_tmp, c.rownnz, c.seg_len, c.seg_off, c.seg_cur, c.seg_nnz,
                     c.seg_listW, c.seg_listC, c.seg_ctr, c.xl_hp, c.xl_keys, c.s, c.dS, c.H, c.acc, c.best, c.dSbest,
@@ -319,18 +319,15 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.dense_cap = std::min<size_t>(c.dense_cap, (size_t)c.prm.dense_max_B * (size_t)c.prm.dense_max_B);
     c.dense = dalloc<int>(c.dense_cap);
     c.rcp = dalloc<double>(Vs);
-    {   // f-table: f(m) = m ln m in long double, split into double hi + float lo
-        std::vector<double> fh(FT_N);
-        std::vector<float> fl(FT_N);
+    {   // f-table: f(m) = m ln m in long double, split into double hi + double lo
+        std::vector<double2> ft(FT_N);
         for (int m = 0; m < FT_N; ++m) {
             const long double f = m > 0 ? (long double)m * logl((long double)m) : 0.0L;
-            fh[m] = (double)f;
-            fl[m] = (float)(f - (long double)fh[m]);
+            ft[m].x = (double)f;
+            ft[m].y = (double)(f - (long double)ft[m].x);
         }
-        c.fh = dalloc<double>(FT_N);
-        c.fl = dalloc<float>(FT_N);
-        GSAP_CUDA(cudaMemcpy(c.fh, fh.data(), sizeof(double) * FT_N, cudaMemcpyHostToDevice));
-        GSAP_CUDA(cudaMemcpy(c.fl, fl.data(), sizeof(float) * FT_N, cudaMemcpyHostToDevice));
+        c.ft = dalloc<double2>(FT_N);
+        GSAP_CUDA(cudaMemcpy(c.ft, ft.data(), sizeof(double2) * FT_N, cudaMemcpyHostToDevice));
     }
     c.denseT = dalloc<int>(c.dense_cap);
     c.keys0 = dalloc<unsigned long long>(Es);

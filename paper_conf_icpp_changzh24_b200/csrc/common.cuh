@@ -56,8 +56,9 @@ constexpr int FT_N = 1 << 16;
 
 GSAP_DEV double fx(double m) { return m > 0.0 ? m * log(m) : 0.0; }
 
-GSAP_DEV double ftab(const double *__restrict__ fh, const float *__restrict__ fl, long long n) {
-    return __ldg(fh + n) + (double)__ldg(fl + n);
+GSAP_DEV double ftab(const double2 *__restrict__ ft, long long n) {
+    const double2 e = __ldg(ft + n);
+    return e.x + e.y;
 }
 
 GSAP_DEV double df_big(long long m, long long d) {
@@ -82,11 +83,13 @@ GSAP_DEV double df_big(long long m, long long d) {
     return fma((double)d, log((double)n), tail);
 }
 
-GSAP_DEV double df_t(const double *__restrict__ fh, const float *__restrict__ fl, long long m, long long d) {
+GSAP_DEV double df_t(const double2 *__restrict__ ft, long long m, long long d) {
     if (d == 0) return 0.0;
     const long long n = m + d;
-    if (m < FT_N && n < FT_N)
-        return (__ldg(fh + n) - __ldg(fh + m)) + (double)(__ldg(fl + n) - __ldg(fl + m));
+    if (m < FT_N && n < FT_N) {
+        const double2 a = __ldg(ft + n), b = __ldg(ft + m);
+        return (a.x - b.x) + (a.y - b.y);
+    }
     return df_big(m, d);
 }
 
@@ -96,11 +99,12 @@ GSAP_DEV double g2(long long a, long long c) {
     return (double)a * log1p((double)c / (double)a) + (double)c * log1p((double)a / (double)c);
 }
 
-GSAP_DEV double g2_t(const double *__restrict__ fh, const float *__restrict__ fl, long long a, long long c) {
+GSAP_DEV double g2_t(const double2 *__restrict__ ft, long long a, long long c) {
     if (a == 0 || c == 0) return 0.0;
-    if (a + c < FT_N)
-        return ((__ldg(fh + a + c) - __ldg(fh + a)) - __ldg(fh + c)) +
-               (double)((__ldg(fl + a + c) - __ldg(fl + a)) - __ldg(fl + c));
+    if (a + c < FT_N) {
+        const double2 x = __ldg(ft + a + c), y = __ldg(ft + a), z = __ldg(ft + c);
+        return ((x.x - y.x) - z.x) + ((x.y - y.y) - z.y);
+    }
     return g2(a, c);
 }
 
@@ -140,8 +144,7 @@ GSAP_DEV int warp_incl_scan(int v) {
 struct BM {
     int B;
     const int *__restrict__ dense;   // nullptr in the sparse regime
-    const double *__restrict__ fh;   // f(m) = m ln m for m < FT_N, double-double (hi, lo)
-    const float *__restrict__ fl;
+    const double2 *__restrict__ ft;  // f(m) = m ln m for m < FT_N, double-double {hi, lo}
     const double *__restrict__ rcp;  // 1 / (d_x + B) per block
     const int *__restrict__ rowptr;  // [B+1]
     const int *__restrict__ col;

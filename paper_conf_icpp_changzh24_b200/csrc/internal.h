@@ -59,8 +59,7 @@ struct Ctx {
     int *bm_colptr = nullptr, *bm_row = nullptr, *bm_ccnt = nullptr, *bm_ccum = nullptr;
     int *dout = nullptr, *din = nullptr, *d_nnz = nullptr;
     int *dense = nullptr, *denseT = nullptr;
-    double *fh = nullptr;          // f-table hi / lo (FT_N entries)
-    float *fl = nullptr;
+    double2 *ft = nullptr;         // f-table {hi, lo} (FT_N entries)
     double *rcp = nullptr;         // 1 / (d_x + B), refreshed by every rebuild
     size_t dense_cap = 0;   // elements
     bool dense_mode = false;
@@ -116,8 +115,7 @@ struct Ctx {
         BM m;
         m.B = B;
         m.dense = dense_mode ? dense : nullptr;
-        m.fh = fh;
-        m.fl = fl;
+        m.ft = ft;
         m.rcp = rcp;
         m.rowptr = bm_rowptr; m.col = bm_col; m.cnt = bm_cnt; m.cum = bm_cum;
         m.colptr = bm_colptr; m.row = bm_row; m.ccnt = bm_ccnt; m.ccum = bm_ccum;

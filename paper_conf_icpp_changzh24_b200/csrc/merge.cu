@@ -63,7 +63,7 @@ GSAP_DEV double inter_sum(const BM &m, bool cols, int a, int b, int r, int s) {
         if (t == r || t == s) continue;
         const int m1 = __ldg(cnt + i);
         const int m2 = cols ? col_at(m, L, other, t) : row_at(m, L, other, t);
-        acc += g2_t(m.fh, m.fl, m1, m2);
+        acc += g2_t(m.ft, m1, m2);
     }
     return acc;
 }
@@ -74,10 +74,10 @@ GSAP_DEV double merge_delta(const BM &m, int r, int s) {
     acc = warp_sum(acc);
     const long long Mss = bm_at(m, s, s), Msr = bm_at(m, s, r), Mrs = bm_at(m, r, s), Mrr = bm_at(m, r, r);
     // f(a+b+c+d) - f(a) - f(b) - f(c) - f(d), telescoped into g's
-    const double core = g2_t(m.fh, m.fl, Mss, Msr) + g2_t(m.fh, m.fl, Mss + Msr, Mrs) +
-                        g2_t(m.fh, m.fl, Mss + Msr + Mrs, Mrr);
-    const double deg = g2_t(m.fh, m.fl, __ldg(m.dout + s), __ldg(m.dout + r)) +
-                       g2_t(m.fh, m.fl, __ldg(m.din + s), __ldg(m.din + r));
+    const double core = g2_t(m.ft, Mss, Msr) + g2_t(m.ft, Mss + Msr, Mrs) +
+                        g2_t(m.ft, Mss + Msr + Mrs, Mrr);
+    const double deg = g2_t(m.ft, __ldg(m.dout + s), __ldg(m.dout + r)) +
+                       g2_t(m.ft, __ldg(m.din + s), __ldg(m.din + r));
     return -acc - core + deg;
 }
 

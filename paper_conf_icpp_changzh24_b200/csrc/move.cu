@@ -126,8 +126,7 @@ struct MoveCtx {
 // dS / Hastings terms of one unique neighbour block t (out weight ot, in weight it)
 GSAP_DEV void t_terms(const MoveArgs &a, const MoveCtx &q, int t, long long ot, long long it, double &accS,
                       double &pf, double &pb) {
-    const double *__restrict__ fh = a.m.fh;
-    const float *__restrict__ fl = a.m.fl;
+    const double2 *__restrict__ ft = a.m.ft;
     const double *__restrict__ rcp = a.m.rcp;
     const double c = (double)(ot + it);
     if (t == q.r) {
@@ -140,7 +139,7 @@ GSAP_DEV void t_terms(const MoveArgs &a, const MoveCtx &q, int t, long long ot, 
         const long long Mrt = row_at(a.m, q.Rr, q.r, t), Mst = row_at(a.m, q.Rs, q.s, t);
         const long long Mtr = col_at(a.m, q.Cr, q.r, t), Mts = col_at(a.m, q.Cs, q.s, t);
         const double rt = __ldg(rcp + t);
-        accS -= df_t(fh, fl, Mrt, -ot) + df_t(fh, fl, Mst, ot) + df_t(fh, fl, Mtr, -it) + df_t(fh, fl, Mts, it);
+        accS -= df_t(ft, Mrt, -ot) + df_t(ft, Mst, ot) + df_t(ft, Mtr, -it) + df_t(ft, Mts, it);
         pf += c * (double)(Mts + Mst + 1) * rt;
         pb += c * (double)(Mtr - it + Mrt - ot + 1) * rt;
     }
@@ -148,17 +147,16 @@ GSAP_DEV void t_terms(const MoveArgs &a, const MoveCtx &q, int t, long long ot, 
 
 // the 2x2 core, the four degree terms and the two self-loop terms: term k of 10
 GSAP_DEV void core_term(const MoveArgs &a, const MoveCtx &q, int k, double &accS, double &pf, double &pb) {
-    const double *__restrict__ fh = a.m.fh;
-    const float *__restrict__ fl = a.m.fl;
+    const double2 *__restrict__ ft = a.m.ft;
     switch (k) {
-        case 0: accS -= df_t(fh, fl, q.Mrr, -(q.o_r + q.i_r + q.l)); break;
-        case 1: accS -= df_t(fh, fl, q.Mrs, q.i_r - q.o_s); break;
-        case 2: accS -= df_t(fh, fl, q.Msr, q.o_r - q.i_s); break;
-        case 3: accS -= df_t(fh, fl, q.Mss, q.o_s + q.i_s + q.l); break;
-        case 4: accS += df_t(fh, fl, __ldg(a.m.dout + q.r), -q.kout); break;
-        case 5: accS += df_t(fh, fl, __ldg(a.m.dout + q.s), q.kout); break;
-        case 6: accS += df_t(fh, fl, __ldg(a.m.din + q.r), -q.kin); break;
-        case 7: accS += df_t(fh, fl, __ldg(a.m.din + q.s), q.kin); break;
+        case 0: accS -= df_t(ft, q.Mrr, -(q.o_r + q.i_r + q.l)); break;
+        case 1: accS -= df_t(ft, q.Mrs, q.i_r - q.o_s); break;
+        case 2: accS -= df_t(ft, q.Msr, q.o_r - q.i_s); break;
+        case 3: accS -= df_t(ft, q.Mss, q.o_s + q.i_s + q.l); break;
+        case 4: accS += df_t(ft, __ldg(a.m.dout + q.r), -q.kout); break;
+        case 5: accS += df_t(ft, __ldg(a.m.dout + q.s), q.kout); break;
+        case 6: accS += df_t(ft, __ldg(a.m.din + q.r), -q.kin); break;
+        case 7: accS += df_t(ft, __ldg(a.m.din + q.s), q.kin); break;
         case 8:
             if (q.l > 0) pf += 2.0 * (double)q.l * (double)(q.Mrs + q.Msr + 1) * __ldg(a.m.rcp + q.r);
             break;
@@ -463,9 +461,9 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     a.gtab = nullptr;
     a.gtab_log2 = 0;
     if (mode != MOVE_DELTA) {   // (a1): thread per vertex
-        const int pg = (int)std::min<long long>(((long long)count + 255) / 256, 148LL * 16);
-        if (c.weighted) k_propose<true><<<pg, 256, 0, c.stream>>>(a);
-        else k_propose<false><<<pg, 256, 0, c.stream>>>(a);
+        const int pg = (int)std::min<long long>(((long long)count + 63) / 64, 148LL * 64);
+        if (c.weighted) k_propose<true><<<pg, 64, 0, c.stream>>>(a);
+        else k_propose<false><<<pg, 64, 0, c.stream>>>(a);
         ++c.launches;
         GSAP_CHECK_LAUNCH();
         if (mode == MOVE_PROPOSE) {

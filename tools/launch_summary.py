@@ -14,7 +14,8 @@ def load(path):
         if len(r) <= vi:
             continue
         v = float(r[vi].replace(",", ""))
-        v *= {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3, "second": 1e6}.get(r[ui], 1.0)
+        v *= {"ns": 1e-3, "nsecond": 1e-3, "us": 1.0, "usecond": 1.0, "ms": 1e3, "msecond": 1e3,
+              "s": 1e6, "second": 1e6}.get(r[ui], 1.0)   # -> microseconds
         name = r[ki].split("(")[0].replace("void ", "")[:58]
         agg[name][0] += 1
         agg[name][1] += v
