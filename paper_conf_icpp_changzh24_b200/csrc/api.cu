@@ -184,7 +184,7 @@ static void check_sm100() {
 
 static void free_ctx(Ctx &c) {
     void *ptrs[] = {c.rowptr, c.col, c.wgt, c.cscptr, c.cscsrc, c.cscwgt, c.esrc, c.kout, c.kin, c.selfw,
-                    c.big, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
+                    c.big, c.huge, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
                     c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT,
                     c.rcp, c.ft, c.keys0,
                     c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
@@ -272,9 +272,11 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     int kmax_big = 0;
     for (int v = 0; v < V; ++v) {
         const int k = (c.h_rowptr[v + 1] - c.h_rowptr[v]) + (c.h_cscptr[v + 1] - c.h_cscptr[v]);
-        if (k > 128) {
-            c.h_big.push_back(v);
+        if (k > 1024) {          // move.cu HUGE_THR
+            c.h_huge.push_back(v);
             kmax_big = std::max(kmax_big, k);
+        } else if (k > 128) {    // move.cu BIG_THR
+            c.h_big.push_back(v);
         }
     }
     // allocation ---------------------------------------------------------
@@ -293,8 +295,9 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.kout = dalloc<int>(Vs);
     c.kin = dalloc<int>(Vs);
     c.selfw = dalloc<int>(Vs);
-    if (!c.h_big.empty()) {
-        c.big = dalloc<int>(c.h_big.size());
+    if (!c.h_big.empty()) c.big = dalloc<int>(c.h_big.size());
+    if (!c.h_huge.empty()) {
+        c.huge = dalloc<int>(c.h_huge.size());
         const int log2cap = std::max(log2_ceil_h(2LL * std::min(kmax_big, V)), 5);
         if ((1 << log2cap) > 2048) {
             c.big_table_slots = (size_t)296 << log2cap;
@@ -392,6 +395,9 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     if (!c.h_big.empty())
         GSAP_CUDA(cudaMemcpyAsync(c.big, c.h_big.data(), sizeof(int) * c.h_big.size(), cudaMemcpyHostToDevice,
                                   c.stream));
+    if (!c.h_huge.empty())
+        GSAP_CUDA(cudaMemcpyAsync(c.huge, c.h_huge.data(), sizeof(int) * c.h_huge.size(),
+                                  cudaMemcpyHostToDevice, c.stream));
     GSAP_CUDA(cudaMemsetAsync(c.scal, 0, 8 * sizeof(double), c.stream));
     GSAP_CUDA(cudaMemsetAsync(c.scal_i, 0, 8 * sizeof(int), c.stream));
     build_graph_device(c);

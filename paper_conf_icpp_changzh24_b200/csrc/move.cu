@@ -29,7 +29,7 @@ constexpr int BIG_THR = 128;           // warp path iff min(k_v, B) <= BIG_THR
 constexpr int MOVE_WARPS = 8;          // warps per CTA, warp kernel
 constexpr int CTA_THREADS = 256;       // big-vertex role: one CTA per vertex
 constexpr int CTA_SMEM_SLOTS = MOVE_WARPS * WARP_TAB;   // big-vertex shared table (<= 1024 keys)
-constexpr int BIG_CTAS_MAX = 296;
+// vertices with > 1024 adjacency entries take the huge role (global tables when B > 1024)
 #ifndef GSAP_MOVE_MINB
 #define GSAP_MOVE_MINB 3               // CTAs per SM the register budget is sized for
 #endif      // CTAs of the big-vertex role (grid-stride)
@@ -51,9 +51,13 @@ struct MoveArgs {
     int *s_out;
     double *dS, *H;
     unsigned char *acc;
-    int4 *gtab;                     // global tables (big-vertex role), per CTA, or nullptr
-    int gtab_log2;
+    int big_log2;                   // big role: shared table of 2^big_log2 slots
     int nbig_ctas;                  // CTAs [0, nbig_ctas) take the big-vertex role
+    const int *__restrict__ hlist;  // huge vertices (> 1024 adjacency entries), sorted ids
+    int hlist_count;
+    int4 *gtab;                     // huge role: global tables per CTA, or nullptr (shared)
+    int gtab_log2;
+    int nhuge_ctas;                 // CTAs [nbig_ctas, nbig_ctas + nhuge_ctas): huge role
 };
 
 GSAP_DEV unsigned hash_slot(int t, int log2cap) {
@@ -402,12 +406,21 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
     __shared__ double sh[3 * MOVE_WARPS];
     const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if ((int)blockIdx.x < a.nbig_ctas) {
-        int4 *tab = a.gtab ? a.gtab + ((size_t)blockIdx.x << a.gtab_log2) : tabs;
-        const int log2cap = a.gtab_log2;
         for (int li = blockIdx.x; li < a.list_count; li += a.nbig_ctas) {
-            tab_clear<CTA_THREADS>(tab, 1 << log2cap, threadIdx.x);
+            tab_clear<CTA_THREADS>(tabs, 1 << a.big_log2, threadIdx.x);
             __syncthreads();
-            do_vertex<CTA_THREADS, WEIGHTED>(a, a.list[li], tab, log2cap, nullptr, sh);
+            do_vertex<CTA_THREADS, WEIGHTED>(a, a.list[li], tabs, a.big_log2, nullptr, sh);
+            __syncthreads();
+        }
+        return;
+    }
+    if ((int)blockIdx.x < a.nbig_ctas + a.nhuge_ctas) {
+        const int hb = blockIdx.x - a.nbig_ctas;
+        int4 *tab = a.gtab ? a.gtab + ((size_t)hb << a.gtab_log2) : tabs;
+        for (int li = hb; li < a.hlist_count; li += a.nhuge_ctas) {
+            tab_clear<CTA_THREADS>(tab, 1 << a.gtab_log2, threadIdx.x);
+            __syncthreads();
+            do_vertex<CTA_THREADS, WEIGHTED>(a, a.hlist[li], tab, a.gtab_log2, nullptr, sh);
             __syncthreads();
         }
         return;
@@ -416,9 +429,10 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
     int *list = lists + wl * (WARP_TAB / 2);
     tab_clear<32>(tab, WARP_TAB, lane);
     __syncwarp();
-    const int nwarps = (gridDim.x - a.nbig_ctas) * MOVE_WARPS;
+    const int role0 = a.nbig_ctas + a.nhuge_ctas;
+    const int nwarps = (gridDim.x - role0) * MOVE_WARPS;
     const bool skip_big = a.B > BIG_THR;
-    for (int i = (blockIdx.x - a.nbig_ctas) * MOVE_WARPS + wl; i < a.count; i += nwarps) {
+    for (int i = (blockIdx.x - role0) * MOVE_WARPS + wl; i < a.count; i += nwarps) {
         const int v = a.first + i;
         // adjacency entries bound the number of unique neighbour blocks
         if (skip_big &&
@@ -472,31 +486,47 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         }
     }
     a.nbig_ctas = 0;
-    if (c.B > BIG_THR && !c.h_big.empty()) {
-        // the big vertices inside [first, first + count)
-        const auto lo = std::lower_bound(c.h_big.begin(), c.h_big.end(), first);
-        const auto hi = std::lower_bound(c.h_big.begin(), c.h_big.end(), first + count);
-        const int nbig = (int)(hi - lo);
-        if (nbig > 0) {
-            a.list = c.big + (lo - c.h_big.begin());
-            a.list_count = nbig;
-            int kmax = 0;
+    a.nhuge_ctas = 0;
+    a.hlist = nullptr;
+    a.hlist_count = 0;
+    a.big_log2 = 5;
+    if (c.B > BIG_THR) {
+        // the big (128 < k <= 1024) and huge (k > 1024) vertices inside [first, first + count)
+        auto range = [&](const std::vector<int> &h, int &n, int &kmax) {
+            const auto lo = std::lower_bound(h.begin(), h.end(), first);
+            const auto hi = std::lower_bound(h.begin(), h.end(), first + count);
+            n = (int)(hi - lo);
+            kmax = 0;
             for (auto it = lo; it != hi; ++it) {
                 const int v = *it;
                 kmax = std::max(kmax, (c.h_rowptr[v + 1] - c.h_rowptr[v]) + (c.h_cscptr[v + 1] - c.h_cscptr[v]));
             }
-            const int log2cap = std::max(log2_ceil(2LL * std::min(kmax, c.B)), 5);
-            a.gtab_log2 = log2cap;
-            a.nbig_ctas = std::min(nbig, BIG_CTAS_MAX);
-            if ((1 << log2cap) > CTA_SMEM_SLOTS) {
-                if (((size_t)a.nbig_ctas << log2cap) > c.big_table_slots)
-                    throw Error{GSAP_ENOMEM, "big-vertex table too small"};
+            return (int)(lo - h.begin());
+        };
+        int nbig = 0, kbig = 0, nhuge = 0, khuge = 0;
+        const int obig = range(c.h_big, nbig, kbig);
+        const int ohuge = range(c.h_huge, nhuge, khuge);
+        if (nbig > 0) {
+            a.list = c.big + obig;
+            a.list_count = nbig;
+            a.big_log2 = std::max(log2_ceil(2LL * std::min(kbig, c.B)), 5);   // <= 11: shared
+            a.nbig_ctas = std::min(nbig, 148 * 16);
+        }
+        if (nhuge > 0) {
+            a.hlist = c.huge + ohuge;
+            a.hlist_count = nhuge;
+            a.gtab_log2 = std::max(log2_ceil(2LL * std::min(khuge, c.B)), 5);
+            if ((1 << a.gtab_log2) > CTA_SMEM_SLOTS) {
+                a.nhuge_ctas = (int)std::min<long long>(nhuge, (long long)(c.big_table_slots >> a.gtab_log2));
+                if (a.nhuge_ctas < 1) throw Error{GSAP_ENOMEM, "huge-vertex table too small"};
                 a.gtab = reinterpret_cast<int4 *>(c.big_tables);
+            } else {
+                a.nhuge_ctas = std::min(nhuge, 148 * 16);
             }
         }
     }
     const long long need = ((long long)count + MOVE_WARPS - 1) / MOVE_WARPS;
-    const int grid = a.nbig_ctas + (int)std::max<long long>(1, std::min<long long>(need, 148LL * 8));
+    const int grid = a.nbig_ctas + a.nhuge_ctas + (int)std::max<long long>(1, std::min<long long>(need, 148LL * 8));
     if (c.weighted) k_move<true><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a);
     else k_move<false><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a);
     ++c.launches;
