@@ -274,11 +274,16 @@ def test_edge_cases(G, oracle_mod):
 
 @pytest.mark.parametrize("regime", ["auto", "sparse"])
 def test_end_to_end_1k(G, oracle_mod, regime):
+    from gen import metrics
     rowptr, col, truth, cfg = dcsbm.make("1k")
     ctx, orc = make_pair(G, oracle_mod, rowptr, col, **(SPARSE if regime == "sparse" else {}))
     res = ctx.gsap_run()
     ref = orc.partition_run()
+    # layer 3 (north_star): final MDL within 1%, pairwise P/R within 0.02 of the oracle's
     assert abs(res["mdl"] - ref["mdl"]) <= 0.01 * ref["mdl"]
+    pg, rg = metrics.pairwise_precision_recall(truth, res["b"])
+    po, ro = metrics.pairwise_precision_recall(truth, ref["b"])
+    assert abs(pg - po) <= 0.02 and abs(rg - ro) <= 0.02
     from sklearn.metrics import normalized_mutual_info_score as nmi
     print("GPU", res["B"], res["mdl"], nmi(truth, res["b"]), "oracle", ref["B"], ref["mdl"],
           nmi(truth, ref["b"]))
@@ -318,3 +323,18 @@ def test_rebuild_weighted_long_lines(G, oracle_mod):
     assert_same_blockmodel(ctx, orc)
     s = ctx.gsap_propose(G.GSAP_MOVE, 1, 2, 0, 2000)
     assert np.array_equal(s, orc.propose(1, SEED, 1, 2, 0, 2000))
+
+
+def test_end_to_end_5k_layer3(G, oracle_mod):
+    """5K-LL (Table 1 shape: 50 850 edges, 19 blocks): layer-3 parity."""
+    from gen import metrics
+    rowptr, col, truth = dcsbm.generate(5000, 50850, 10.0, 5.0, seed=5000)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    res = ctx.gsap_run()
+    ref = orc.partition_run()
+    assert abs(res["mdl"] - ref["mdl"]) <= 0.01 * ref["mdl"]
+    pg, rg = metrics.pairwise_precision_recall(truth, res["b"])
+    po, ro = metrics.pairwise_precision_recall(truth, ref["b"])
+    assert abs(pg - po) <= 0.02 and abs(rg - ro) <= 0.02
+    print("5K: GPU B", res["B"], "NMI", metrics.nmi(truth, res["b"]), "oracle B", ref["B"],
+          "NMI", metrics.nmi(truth, ref["b"]))

@@ -468,3 +468,22 @@ def test_generator_shapes():
         # determinism
         r2, c2, t2, _ = dcsbm.make(name)
         assert np.array_equal(col, c2) and np.array_equal(truth, t2)
+
+
+def test_metrics_against_sklearn_and_hand_cases(tmp_path):
+    """NMI vs scikit-learn; pairwise precision/recall on hand-counted cases; TSV ingest."""
+    from sklearn.metrics import normalized_mutual_info_score as sk_nmi
+    from gen import metrics
+    rng = np.random.default_rng(0)
+    for _ in range(5):
+        a = rng.integers(0, 5, 200)
+        b = rng.integers(0, 7, 200)
+        assert abs(metrics.nmi(a, b) - sk_nmi(a, b)) < 1e-12
+    # truth {0,1,2},{3,4}; pred {0,1},{2,3,4}: same-pred pairs 1+3=4, same-truth 3+1=4, both 1+1=2
+    p, r = metrics.pairwise_precision_recall([0, 0, 0, 1, 1], [0, 0, 1, 1, 1])
+    assert (p, r) == (0.5, 0.5)
+    assert metrics.pairwise_precision_recall([0, 0, 1], [5, 5, 7]) == (1.0, 1.0)
+    f = tmp_path / "g.tsv"
+    f.write_text("1\t2\n2\t3\n3\t1\n1\t3\n")
+    rowptr, col, w = metrics.load_tsv(str(f))
+    assert rowptr.tolist() == [0, 2, 3, 4] and col.tolist() == [1, 2, 2, 0] and w is None
