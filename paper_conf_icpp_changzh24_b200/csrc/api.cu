@@ -184,7 +184,7 @@ static void check_sm100() {
 
 static void free_ctx(Ctx &c) {
     void *ptrs[] = {c.rowptr, c.col, c.wgt, c.cscptr, c.cscsrc, c.cscwgt, c.esrc, c.kout, c.kin, c.selfw,
-                    c.big, c.huge, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
+                    c.big, c.huge, c.mid, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
                     c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT,
                     c.rcp, c.ft, c.keys0,
                     c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
@@ -275,8 +275,10 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         if (k > 1024) {          // move.cu HUGE_THR
             c.h_huge.push_back(v);
             kmax_big = std::max(kmax_big, k);
-        } else if (k > 128) {    // move.cu BIG_THR
+        } else if (k > 256) {    // move.cu: 64-thread groups up to 256 entries
             c.h_big.push_back(v);
+        } else if (k > 128) {    // move.cu BIG_THR
+            c.h_mid.push_back(v);
         }
     }
     // allocation ---------------------------------------------------------
@@ -296,6 +298,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.kin = dalloc<int>(Vs);
     c.selfw = dalloc<int>(Vs);
     if (!c.h_big.empty()) c.big = dalloc<int>(c.h_big.size());
+    if (!c.h_mid.empty()) c.mid = dalloc<int>(c.h_mid.size());
     if (!c.h_huge.empty()) {
         c.huge = dalloc<int>(c.h_huge.size());
         const int log2cap = std::max(log2_ceil_h(2LL * std::min(kmax_big, V)), 5);
@@ -394,6 +397,9 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         GSAP_CUDA(cudaMemcpyAsync(c.wgt, hw.data(), sizeof(int) * (size_t)E, cudaMemcpyHostToDevice, c.stream));
     if (!c.h_big.empty())
         GSAP_CUDA(cudaMemcpyAsync(c.big, c.h_big.data(), sizeof(int) * c.h_big.size(), cudaMemcpyHostToDevice,
+                                  c.stream));
+    if (!c.h_mid.empty())
+        GSAP_CUDA(cudaMemcpyAsync(c.mid, c.h_mid.data(), sizeof(int) * c.h_mid.size(), cudaMemcpyHostToDevice,
                                   c.stream));
     if (!c.h_huge.empty())
         GSAP_CUDA(cudaMemcpyAsync(c.huge, c.h_huge.data(), sizeof(int) * c.h_huge.size(),

@@ -28,6 +28,8 @@ constexpr int WARP_TAB_LOG2 = 8;
 constexpr int BIG_THR = 128;           // warp path iff min(k_v, B) <= BIG_THR
 constexpr int MOVE_WARPS = 8;          // warps per CTA, warp kernel
 constexpr int CTA_THREADS = 256;       // big-vertex role: one CTA per vertex
+constexpr int MID_TAB = 512;           // mid role: 64-thread group tables (<= 256 keys)
+constexpr int MID_TAB_LOG2 = 9;
 constexpr int CTA_SMEM_SLOTS = MOVE_WARPS * WARP_TAB;   // big-vertex shared table (<= 1024 keys)
 // vertices with > 1024 adjacency entries take the huge role (global tables when B > 1024)
 #ifndef GSAP_MOVE_MINB
@@ -51,6 +53,9 @@ struct MoveArgs {
     int *s_out;
     double *dS, *H;
     unsigned char *acc;
+    const int *__restrict__ mlist;  // mid vertices (128 < entries <= 256): 64-thread groups
+    int mlist_count;
+    int nmid_ctas;                  // CTAs [0, nmid_ctas): mid role (4 groups each)
     int big_log2;                   // big role: shared table of 2^big_log2 slots
     int nbig_ctas;                  // CTAs [0, nbig_ctas) take the big-vertex role
     const int *__restrict__ hlist;  // huge vertices (> 1024 adjacency entries), sorted ids
@@ -87,19 +92,30 @@ GSAP_DEV int tab_find(const int4 *tab, int log2cap, int t) {
 }
 
 // group-wide sums of three values (deterministic fixed trees)
+// barrier of a G-thread group (G = 32: the warp; 256: the CTA; 64: one of
+// four named-barrier groups of the CTA)
+template <int G>
+GSAP_DEV void gsync() {
+    if (G == 32) __syncwarp();
+    else if (G == 256) __syncthreads();
+    else asm volatile("bar.sync %0, %1;" ::"r"(1 + (int)(threadIdx.x / G)), "r"(G) : "memory");
+}
+
+// group-wide sums of three values (deterministic fixed trees); sh: 3 G/32
+// doubles owned by this group
 template <int G>
 GSAP_DEV void group_sum3(double &x, double &y, double &z, double *sh) {
     x = warp_sum(x);
     y = warp_sum(y);
     z = warp_sum(z);
     if (G == 32) return;
-    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int w = (threadIdx.x % G) >> 5, lane = threadIdx.x & 31;
     if (lane == 0) {
         sh[w] = x;
         sh[G / 32 + w] = y;
         sh[2 * (G / 32) + w] = z;
     }
-    __syncthreads();
+    gsync<G>();
     double a = 0.0, b = 0.0, c = 0.0;
 #pragma unroll
     for (int i = 0; i < G / 32; ++i) {
@@ -107,17 +123,12 @@ GSAP_DEV void group_sum3(double &x, double &y, double &z, double *sh) {
         b += sh[G / 32 + i];
         c += sh[2 * (G / 32) + i];
     }
-    __syncthreads();
+    gsync<G>();
     x = a;
     y = b;
     z = c;
 }
 
-template <int G>
-GSAP_DEV void group_sync() {
-    if (G == 32) __syncwarp();
-    else __syncthreads();
-}
 
 // the state of one move r -> s that every term needs
 struct MoveCtx {
@@ -292,16 +303,17 @@ GSAP_DEV void eval_move_warp(const MoveArgs &a, int v, int r, int s, uint4 w, in
     mh_decide(a, q, w, accS, pf, pb, dS_out, H_out, acc_out);
 }
 
-// (a2), one CTA per (big) vertex: every unique block owned by its first
-// adjacency position; threads sum their owned terms in position order.
-template <bool WEIGHTED>
-GSAP_DEV void eval_move_cta(const MoveArgs &a, int v, int r, int s, uint4 w, int4 *tab, int log2cap,
-                            double *sh, double &dS_out, double &H_out, bool &acc_out) {
-    const int gt = threadIdx.x;
+// (a2), one G-thread group (64: a quarter CTA, 256: a CTA) per big vertex:
+// every unique block owned by its first adjacency position; threads sum their
+// owned terms in position order.
+template <int G, bool WEIGHTED>
+GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, int4 *tab, int log2cap,
+                              double *sh, double &dS_out, double &H_out, bool &acc_out) {
+    const int gt = threadIdx.x % G;
     const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
     const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
     const int deg = nout + nin;
-    for (int j = gt; j < deg; j += CTA_THREADS) {
+    for (int j = gt; j < deg; j += G) {
         const bool out = j < nout;
         const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
         if (nb == v) continue;   // the self-loop is carried by selfw
@@ -311,11 +323,11 @@ GSAP_DEV void eval_move_cta(const MoveArgs &a, int v, int r, int s, uint4 w, int
         atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
         atomicMin(&tab[sl].w, j);
     }
-    __syncthreads();
+    gsync<G>();
     MoveCtx q;
     move_ctx(a, v, r, s, tab, log2cap, q);
     double accS = 0.0, pf = 0.0, pb = 0.0;
-    for (int j = gt; j < deg; j += CTA_THREADS) {
+    for (int j = gt; j < deg; j += G) {
         const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
         if (nb == v) continue;
         const int4 e = tab[tab_find(tab, log2cap, __ldg(a.b + nb))];
@@ -323,7 +335,7 @@ GSAP_DEV void eval_move_cta(const MoveArgs &a, int v, int r, int s, uint4 w, int
         t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
     }
     if (gt < 10) core_term(a, q, gt, accS, pf, pb);
-    group_sum3<CTA_THREADS>(accS, pf, pb, sh);
+    group_sum3<G>(accS, pf, pb, sh);
     mh_decide(a, q, w, accS, pf, pb, dS_out, H_out, acc_out);
 }
 
@@ -344,7 +356,7 @@ GSAP_DEV void do_vertex(const MoveArgs &a, int v, int4 *tab, int log2cap, int *l
     bool acc = false;
     if (s != r) {
         if (G == 32) eval_move_warp<WEIGHTED>(a, v, r, s, w, tab, list, dS, H, acc);
-        else eval_move_cta<WEIGHTED>(a, v, r, s, w, tab, log2cap, sh, dS, H, acc);
+        else eval_move_group<G, WEIGHTED>(a, v, r, s, w, tab, log2cap, sh, dS, H, acc);
     }
     if ((threadIdx.x & (G - 1)) == 0) {
         if (a.dS) a.dS[i] = dS;
@@ -405,8 +417,20 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
     __shared__ int lists[MOVE_WARPS * (WARP_TAB / 2)];
     __shared__ double sh[3 * MOVE_WARPS];
     const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    if ((int)blockIdx.x < a.nbig_ctas) {
-        for (int li = blockIdx.x; li < a.list_count; li += a.nbig_ctas) {
+    if ((int)blockIdx.x < a.nmid_ctas) {
+        // four 64-thread groups per CTA, one mid vertex each
+        const int gid = threadIdx.x >> 6, gt = threadIdx.x & 63;
+        int4 *tab = tabs + gid * MID_TAB;
+        for (int li = blockIdx.x * 4 + gid; li < a.mlist_count; li += a.nmid_ctas * 4) {
+            tab_clear<64>(tab, MID_TAB, gt);
+            gsync<64>();
+            do_vertex<64, WEIGHTED>(a, a.mlist[li], tab, MID_TAB_LOG2, nullptr, sh + gid * 6);
+            gsync<64>();
+        }
+        return;
+    }
+    if ((int)blockIdx.x < a.nmid_ctas + a.nbig_ctas) {
+        for (int li = blockIdx.x - a.nmid_ctas; li < a.list_count; li += a.nbig_ctas) {
             tab_clear<CTA_THREADS>(tabs, 1 << a.big_log2, threadIdx.x);
             __syncthreads();
             do_vertex<CTA_THREADS, WEIGHTED>(a, a.list[li], tabs, a.big_log2, nullptr, sh);
@@ -414,8 +438,8 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
         }
         return;
     }
-    if ((int)blockIdx.x < a.nbig_ctas + a.nhuge_ctas) {
-        const int hb = blockIdx.x - a.nbig_ctas;
+    if ((int)blockIdx.x < a.nmid_ctas + a.nbig_ctas + a.nhuge_ctas) {
+        const int hb = blockIdx.x - a.nmid_ctas - a.nbig_ctas;
         int4 *tab = a.gtab ? a.gtab + ((size_t)hb << a.gtab_log2) : tabs;
         for (int li = hb; li < a.hlist_count; li += a.nhuge_ctas) {
             tab_clear<CTA_THREADS>(tab, 1 << a.gtab_log2, threadIdx.x);
@@ -429,7 +453,7 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
     int *list = lists + wl * (WARP_TAB / 2);
     tab_clear<32>(tab, WARP_TAB, lane);
     __syncwarp();
-    const int role0 = a.nbig_ctas + a.nhuge_ctas;
+    const int role0 = a.nmid_ctas + a.nbig_ctas + a.nhuge_ctas;
     const int nwarps = (gridDim.x - role0) * MOVE_WARPS;
     const bool skip_big = a.B > BIG_THR;
     for (int i = (blockIdx.x - role0) * MOVE_WARPS + wl; i < a.count; i += nwarps) {
@@ -487,6 +511,9 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     }
     a.nbig_ctas = 0;
     a.nhuge_ctas = 0;
+    a.nmid_ctas = 0;
+    a.mlist = nullptr;
+    a.mlist_count = 0;
     a.hlist = nullptr;
     a.hlist_count = 0;
     a.big_log2 = 5;
@@ -503,7 +530,13 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
             }
             return (int)(lo - h.begin());
         };
-        int nbig = 0, kbig = 0, nhuge = 0, khuge = 0;
+        int nmid = 0, kmid = 0, nbig = 0, kbig = 0, nhuge = 0, khuge = 0;
+        const int omid = range(c.h_mid, nmid, kmid);
+        if (nmid > 0) {
+            a.mlist = c.mid + omid;
+            a.mlist_count = nmid;
+            a.nmid_ctas = std::min((nmid + 3) / 4, 148 * 16);
+        }
         const int obig = range(c.h_big, nbig, kbig);
         const int ohuge = range(c.h_huge, nhuge, khuge);
         if (nbig > 0) {
@@ -526,7 +559,8 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         }
     }
     const long long need = ((long long)count + MOVE_WARPS - 1) / MOVE_WARPS;
-    const int grid = a.nbig_ctas + a.nhuge_ctas + (int)std::max<long long>(1, std::min<long long>(need, 148LL * 8));
+    const int grid = a.nmid_ctas + a.nbig_ctas + a.nhuge_ctas +
+                     (int)std::max<long long>(1, std::min<long long>(need, 148LL * 8));
     if (c.weighted) k_move<true><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a);
     else k_move<false><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a);
     ++c.launches;
