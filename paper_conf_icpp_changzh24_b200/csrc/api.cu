@@ -7,6 +7,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <mutex>
 #include <new>
 #include <vector>
 
@@ -130,18 +131,6 @@ void kc_resolve(Ctx &c, KClass &k) {
 
 }  // namespace gsap
 
-template <typename T>
-static T *dalloc(size_t n) {
-    void *p = nullptr;
-    const cudaError_t e = cudaMalloc(&p, std::max<size_t>(n, 1) * sizeof(T));
-    if (e == cudaErrorMemoryAllocation) {
-        cudaGetLastError();
-        throw Error{GSAP_ENOMEM, "cudaMalloc failed"};
-    }
-    GSAP_CUDA(e);
-    return static_cast<T *>(p);
-}
-
 static bool is_dev(const void *p) {
     if (!p) return false;
     cudaPointerAttributes a;
@@ -183,18 +172,8 @@ static void check_sm100() {
 }
 
 static void free_ctx(Ctx &c) {
-    void *ptrs[] = {c.rowptr, c.col, c.wgt, c.cscptr, c.cscsrc, c.cscwgt, c.esrc, c.kout, c.kin, c.selfw,
-                    c.big, c.huge, c.mid, c.big_tables, c.b, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr,
-                    c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.d_nnz, c.dense, c.denseT,
-                    c.rcp, c.ft, c.keys0,
-                    c.keys1, c.vals64a, c.vals64b, c.ukeys0, c.ukeys1, c.wa, c.wb, c.flags, c.pos, c.tmpi,
-                    c.rowid, c.counts, c.scan_tmp, c.rownnz, c.seg_len, c.seg_off, c.seg_cur, c.seg_nnz,
-                    c.seg_listW, c.seg_listC, c.seg_ctr, c.xl_hp, c.xl_keys, c.s, c.dS, c.H, c.acc, c.best, c.dSbest,
-                    c.partials, c.scal, c.scal_i, c.Dh, c.d_itr, c.skey0, c.skey1, c.sval0, c.sval1, c.sel_rank,
-                    c.nxt0, c.nxt1, c.mx0, c.mx1, c.oncyc, c.label, c.present, c.slot_b[0], c.slot_b[1],
-                    c.slot_b[2]};
-    for (void *p : ptrs)
-        if (p) cudaFree(p);
+    if (c.arena) cudaFree(c.arena);
+    c.arena = nullptr;
     if (c.h_scal) cudaFreeHost(c.h_scal);
     if (c.h_int) cudaFreeHost(c.h_int);
     for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl}) {
@@ -210,6 +189,19 @@ static void free_ctx(Ctx &c) {
     }
     if (c.own_stream && c.stream) cudaStreamDestroy(c.stream);
 }
+
+// one device allocation per context, carved into aligned sub-buffers
+struct Arena {
+    char *base = nullptr;   // nullptr: measuring pass
+    size_t off = 0;
+    template <typename T>
+    T *take(size_t n) {
+        off = (off + 255) & ~(size_t)255;
+        T *p = base ? reinterpret_cast<T *>(base + off) : nullptr;
+        off += std::max<size_t>(n, 1) * sizeof(T);
+        return p;
+    }
+};
 
 static int log2_ceil_h(long long x) {
     int l = 0;
@@ -281,113 +273,137 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
             c.h_mid.push_back(v);
         }
     }
-    // allocation ---------------------------------------------------------
+    // allocation: one device arena (one cudaMalloc / cudaFree per context),
+    // planned in a measuring pass and then carved ---------------------------
     const size_t Vs = (size_t)V, Es = (size_t)std::max(E, 1);
     const size_t VE = std::max(Vs, Es) + 1;
     const int P = c.prm.num_proposals;
-    c.rowptr = dalloc<int>(Vs + 1);
-    c.col = dalloc<int>(Es);
-    if (c.weighted) {
-        c.wgt = dalloc<int>(Es);
-        c.cscwgt = dalloc<int>(Es);
-    }
-    c.cscptr = dalloc<int>(Vs + 1);
-    c.cscsrc = dalloc<int>(Es);
-    c.esrc = dalloc<int>(Es);
-    c.kout = dalloc<int>(Vs);
-    c.kin = dalloc<int>(Vs);
-    c.selfw = dalloc<int>(Vs);
-    if (!c.h_big.empty()) c.big = dalloc<int>(c.h_big.size());
-    if (!c.h_mid.empty()) c.mid = dalloc<int>(c.h_mid.size());
-    if (!c.h_huge.empty()) {
-        c.huge = dalloc<int>(c.h_huge.size());
-        const int log2cap = std::max(log2_ceil_h(2LL * std::min(kmax_big, V)), 5);
-        if ((1 << log2cap) > 2048) {
-            c.big_table_slots = (size_t)296 << log2cap;
-            c.big_tables = dalloc<int>(c.big_table_slots * 4);
+    auto carve = [&](Arena &A) {
+        c.rowptr = A.take<int>(Vs + 1);
+        c.col = A.take<int>(Es);
+        if (c.weighted) {
+            c.wgt = A.take<int>(Es);
+            c.cscwgt = A.take<int>(Es);
         }
-    }
-    c.b = dalloc<int>(Vs);
-    c.bm_rowptr = dalloc<int>(Vs + 1);
-    c.bm_colptr = dalloc<int>(Vs + 1);
-    c.bm_col = dalloc<int>(Es);
-    c.bm_cnt = dalloc<int>(Es);
-    c.bm_cum = dalloc<int>(Es);
-    c.bm_row = dalloc<int>(Es);
-    c.bm_ccnt = dalloc<int>(Es);
-    c.bm_ccum = dalloc<int>(Es);
-    c.dout = dalloc<int>(Vs);
-    c.din = dalloc<int>(Vs);
-    c.d_nnz = dalloc<int>(1);
-    c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, (size_t)1 << 24), (size_t)1 << 28);
-    c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
-    if (c.prm.dense_max_B > 0)
-        c.dense_cap = std::min<size_t>(c.dense_cap, (size_t)c.prm.dense_max_B * (size_t)c.prm.dense_max_B);
-    c.dense = dalloc<int>(c.dense_cap);
-    c.rcp = dalloc<double>(Vs);
-    {   // f-table: f(m) = m ln m in long double, split into double hi + double lo
-        std::vector<double2> ft(FT_N);
-        for (int m = 0; m < FT_N; ++m) {
-            const long double f = m > 0 ? (long double)m * logl((long double)m) : 0.0L;
-            ft[m].x = (double)f;
-            ft[m].y = (double)(f - (long double)ft[m].x);
+        c.cscptr = A.take<int>(Vs + 1);
+        c.cscsrc = A.take<int>(Es);
+        c.esrc = A.take<int>(Es);
+        c.kout = A.take<int>(Vs);
+        c.kin = A.take<int>(Vs);
+        c.selfw = A.take<int>(Vs);
+        if (!c.h_big.empty()) c.big = A.take<int>(c.h_big.size());
+        if (!c.h_mid.empty()) c.mid = A.take<int>(c.h_mid.size());
+        if (!c.h_huge.empty()) {
+            c.huge = A.take<int>(c.h_huge.size());
+            const int log2cap = std::max(log2_ceil_h(2LL * std::min(kmax_big, V)), 5);
+            if ((1 << log2cap) > 2048) {
+                c.big_table_slots = (size_t)296 << log2cap;
+                c.big_tables = A.take<int>(c.big_table_slots * 4);
+            }
         }
-        c.ft = dalloc<double2>(FT_N);
-        GSAP_CUDA(cudaMemcpy(c.ft, ft.data(), sizeof(double2) * FT_N, cudaMemcpyHostToDevice));
+        c.b = A.take<int>(Vs);
+        c.bm_rowptr = A.take<int>(Vs + 1);
+        c.bm_colptr = A.take<int>(Vs + 1);
+        c.bm_col = A.take<int>(Es);
+        c.bm_cnt = A.take<int>(Es);
+        c.bm_cum = A.take<int>(Es);
+        c.bm_row = A.take<int>(Es);
+        c.bm_ccnt = A.take<int>(Es);
+        c.bm_ccum = A.take<int>(Es);
+        c.dout = A.take<int>(Vs);
+        c.din = A.take<int>(Vs);
+        c.d_nnz = A.take<int>(1);
+        c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, (size_t)1 << 24), (size_t)1 << 28);
+        c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
+        if (c.prm.dense_max_B > 0)
+            c.dense_cap = std::min<size_t>(c.dense_cap, (size_t)c.prm.dense_max_B * (size_t)c.prm.dense_max_B);
+        c.dense = A.take<int>(c.dense_cap);
+        c.rcp = A.take<double>(Vs);
+        c.ft = A.take<double2>(FT_N);
+        c.denseT = A.take<int>(c.dense_cap);
+        c.keys0 = A.take<unsigned long long>(Es);
+        c.keys1 = A.take<unsigned long long>(Es);
+        c.vals64a = A.take<unsigned long long>(Es);
+        c.vals64b = A.take<unsigned long long>(Es);
+        c.ukeys0 = A.take<unsigned>(Es);
+        c.ukeys1 = A.take<unsigned>(Es);
+        c.wa = A.take<int>(VE);
+        c.wb = A.take<int>(VE);
+        c.flags = A.take<int>(VE);
+        c.pos = A.take<int>(VE);
+        c.tmpi = A.take<int>(VE);
+        c.rowid = A.take<int>(VE);
+        c.rownnz = A.take<int>(Vs + 1);
+        c.seg_len = A.take<int>(Vs + 1);
+        c.seg_off = A.take<int>(Vs + 1);
+        c.seg_cur = A.take<int>(Vs + 1);
+        c.seg_nnz = A.take<int>(Vs + 1);
+        c.seg_listW = A.take<int>(Vs + 1);
+        c.seg_listC = A.take<int>(Vs + 1);
+        c.seg_ctr = A.take<int>(4);
+        c.xl_keys = A.take<unsigned long long>(2 * Es);
+        c.xl_hp = A.take<int>(2 * Es);
+        const size_t tiles = (VE + 4095) / 4096 + 1;
+        c.counts_cap = 256 * tiles;
+        c.counts = A.take<int>(c.counts_cap);
+        c.scan_tmp_cap = std::max(c.counts_cap, VE) / 4096 + 16;
+        c.scan_tmp = A.take<int>(c.scan_tmp_cap);
+        // per-batch / per-phase buffers, padded for the rank-blocked all-gathers
+        const size_t pad = 65536;
+        c.s = A.take<int>(std::max(Vs * (size_t)P, Vs + pad));
+        c.dS = A.take<double>(std::max(Vs * (size_t)P, Vs + pad));
+        c.H = A.take<double>(Vs + pad);
+        c.acc = A.take<unsigned char>(Vs + pad);
+        c.best = A.take<int>(Vs + pad);
+        c.dSbest = A.take<double>(Vs + pad);
+        c.partials = A.take<double>(VE / 512 + 1024);   // >= max(E, B) / MDL_CHUNK, V / APPLY_CHUNK + ranks
+        c.scal = A.take<double>(8);
+        c.scal_i = A.take<int>(8);
+        c.Dh = A.take<double>((size_t)c.prm.max_nodal_itr + 1);
+        c.d_itr = A.take<unsigned>(1);
+        c.skey0 = A.take<unsigned long long>(Vs);
+        c.skey1 = A.take<unsigned long long>(Vs);
+        c.sval0 = A.take<int>(Vs);
+        c.sval1 = A.take<int>(Vs);
+        c.sel_rank = A.take<int>(Vs);
+        c.nxt0 = A.take<int>(Vs);
+        c.nxt1 = A.take<int>(Vs);
+        c.mx0 = A.take<int>(Vs);
+        c.mx1 = A.take<int>(Vs);
+        c.oncyc = A.take<int>(Vs);
+        c.label = A.take<int>(Vs);
+        c.present = A.take<int>(Vs + 1);
+        for (int i = 0; i < 3; ++i) c.slot_b[i] = A.take<int>(Vs);
+    };
+    {
+        Arena measure;
+        carve(measure);
+        void *base = nullptr;
+        const cudaError_t e = cudaMalloc(&base, measure.off);
+        if (e == cudaErrorMemoryAllocation) {
+            cudaGetLastError();
+            throw Error{GSAP_ENOMEM, "cudaMalloc of the context arena failed"};
+        }
+        GSAP_CUDA(e);
+        c.arena = base;
+        c.arena_bytes = measure.off;
+        Arena cut;
+        cut.base = (char *)base;
+        carve(cut);
     }
-    c.denseT = dalloc<int>(c.dense_cap);
-    c.keys0 = dalloc<unsigned long long>(Es);
-    c.keys1 = dalloc<unsigned long long>(Es);
-    c.vals64a = dalloc<unsigned long long>(Es);
-    c.vals64b = dalloc<unsigned long long>(Es);
-    c.ukeys0 = dalloc<unsigned>(Es);
-    c.ukeys1 = dalloc<unsigned>(Es);
-    c.wa = dalloc<int>(VE);
-    c.wb = dalloc<int>(VE);
-    c.flags = dalloc<int>(VE);
-    c.pos = dalloc<int>(VE);
-    c.tmpi = dalloc<int>(VE);
-    c.rowid = dalloc<int>(VE);
-    c.rownnz = dalloc<int>(Vs + 1);
-    c.seg_len = dalloc<int>(Vs + 1);
-    c.seg_off = dalloc<int>(Vs + 1);
-    c.seg_cur = dalloc<int>(Vs + 1);
-    c.seg_nnz = dalloc<int>(Vs + 1);
-    c.seg_listW = dalloc<int>(Vs + 1);
-    c.seg_listC = dalloc<int>(Vs + 1);
-    c.seg_ctr = dalloc<int>(4);
-    c.xl_keys = dalloc<unsigned long long>(2 * Es);
-    c.xl_hp = dalloc<int>(2 * Es);
-    const size_t tiles = (VE + 4095) / 4096 + 1;
-    c.counts_cap = 256 * tiles;
-    c.counts = dalloc<int>(c.counts_cap);
-    c.scan_tmp_cap = std::max(c.counts_cap, VE) / 4096 + 16;
-    c.scan_tmp = dalloc<int>(c.scan_tmp_cap);
-    // per-batch / per-phase buffers, padded for the rank-blocked all-gathers
-    const size_t pad = 65536;
-    c.s = dalloc<int>(std::max(Vs * (size_t)P, Vs + pad));
-    c.dS = dalloc<double>(std::max(Vs * (size_t)P, Vs + pad));
-    c.H = dalloc<double>(Vs + pad);
-    c.acc = dalloc<unsigned char>(Vs + pad);
-    c.best = dalloc<int>(Vs + pad);
-    c.dSbest = dalloc<double>(Vs + pad);
-    c.partials = dalloc<double>(VE / 512 + 1024);   // >= max(E, B) / MDL_CHUNK, V / APPLY_CHUNK + ranks
-    c.scal = dalloc<double>(8);
-    c.scal_i = dalloc<int>(8);
-    c.Dh = dalloc<double>((size_t)c.prm.max_nodal_itr + 1);
-    c.d_itr = dalloc<unsigned>(1);
-    c.skey0 = dalloc<unsigned long long>(Vs);
-    c.skey1 = dalloc<unsigned long long>(Vs);
-    c.sval0 = dalloc<int>(Vs);
-    c.sval1 = dalloc<int>(Vs);
-    c.sel_rank = dalloc<int>(Vs);
-    c.nxt0 = dalloc<int>(Vs);
-    c.nxt1 = dalloc<int>(Vs);
-    c.mx0 = dalloc<int>(Vs);
-    c.mx1 = dalloc<int>(Vs);
-    c.oncyc = dalloc<int>(Vs);
-    c.label = dalloc<int>(Vs);
-    c.present = dalloc<int>(Vs + 1);
+    {   // f-table: f(m) = m ln m in long double, split into double hi + double lo (once per process)
+        static std::vector<double2> ft;
+        static std::once_flag once;
+        std::call_once(once, [] {
+            ft.resize(FT_N);
+            for (int m = 0; m < FT_N; ++m) {
+                const long double f = m > 0 ? (long double)m * logl((long double)m) : 0.0L;
+                ft[m].x = (double)f;
+                ft[m].y = (double)(f - (long double)ft[m].x);
+            }
+        });
+        GSAP_CUDA(cudaMemcpyAsync(c.ft, ft.data(), sizeof(double2) * FT_N, cudaMemcpyHostToDevice, c.stream));
+    }
     GSAP_CUDA(cudaMallocHost(&c.h_scal, 8 * sizeof(double)));
     GSAP_CUDA(cudaMallocHost(&c.h_int, 8 * sizeof(int)));
     // upload ---------------------------------------------------------------
@@ -623,8 +639,6 @@ bool bracket_update(Ctx &c, Bracket &br, int B, double S, int *K, int *restart) 
 static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out, double *trace, int trace_cap,
                      int32_t *rounds_out) {
     const auto t0 = std::chrono::steady_clock::now();
-    for (int i = 0; i < 3; ++i)
-        if (!c.slot_b[i]) c.slot_b[i] = dalloc<int>((size_t)c.V);
     GSAP_CUDA(cudaMemsetAsync(c.scal_i + 1, 0, sizeof(int), c.stream));
     set_iota(c);
     rebuild(c);

@@ -31,6 +31,8 @@ struct KClass {
 
 struct Ctx {
     int dev = 0;
+    void *arena = nullptr;         // the single device allocation all buffers live in
+    size_t arena_bytes = 0;
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     gsap_params prm{};
