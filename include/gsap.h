@@ -206,10 +206,12 @@ gsap_status gsap_sync(gsap_ctx *ctx);
 /*
  * Full SBP on an existing context (gsap_partition without the copy-in):
  * restarts from b = iota.  bmap_out: host or device, nullable.
- * trace (host, nullable): rows of [outer, B after merge, MCMC iterations, MDL,
- * round seconds, accepted moves] per round, at most trace_cap rows;
- * *rounds_out (host, nullable).
+ * trace (host, nullable): GSAP_TRACE_COLS doubles per round, at most
+ * trace_cap rows: [outer, B after merge, MCMC iterations, MDL, round seconds,
+ * accepted moves, device ms of the move / rebuild / merge kernels (profile = 1,
+ * else 0)]; *rounds_out (host, nullable).
  */
+#define GSAP_TRACE_COLS 9
 gsap_status gsap_run(gsap_ctx *ctx, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
                      double *trace, int32_t trace_cap, int32_t *rounds_out);
 

@@ -657,7 +657,14 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
     while (!done && rounds < c.prm.max_rounds) {
         const bool bracket = br.S[2] != INFINITY;
         int acc_before = 0;
+        double ms0[3] = {0.0, 0.0, 0.0};
         if (trace && rounds < trace_cap) {
+            kc_resolve(c, c.k_move);
+            kc_resolve(c, c.k_rebuild);
+            kc_resolve(c, c.k_merge);
+            ms0[0] = c.k_move.ms;
+            ms0[1] = c.k_rebuild.ms;
+            ms0[2] = c.k_merge.ms;
             GSAP_CUDA(cudaMemcpyAsync(c.h_int + 3, c.scal_i + 1, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
             GSAP_CUDA(cudaStreamSynchronize(c.stream));
             acc_before = c.h_int[3];
@@ -676,12 +683,20 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
         if (trace && rounds < trace_cap) {
             GSAP_CUDA(cudaMemcpyAsync(c.h_int + 3, c.scal_i + 1, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
             GSAP_CUDA(cudaStreamSynchronize(c.stream));
-            trace[6 * rounds + 0] = (double)outer;
-            trace[6 * rounds + 1] = (double)B;
-            trace[6 * rounds + 2] = (double)itrs;
-            trace[6 * rounds + 3] = S;
-            trace[6 * rounds + 4] = std::chrono::duration<double>(td - ta).count();
-            trace[6 * rounds + 5] = (double)(c.h_int[3] - acc_before);
+            double *row = trace + (size_t)GSAP_TRACE_COLS * rounds;
+            row[0] = (double)outer;
+            row[1] = (double)B;
+            row[2] = (double)itrs;
+            row[3] = S;
+            row[4] = std::chrono::duration<double>(td - ta).count();
+            row[5] = (double)(c.h_int[3] - acc_before);
+            // device ms of the kernel classes in this round (profile = 1)
+            kc_resolve(c, c.k_move);
+            kc_resolve(c, c.k_rebuild);
+            kc_resolve(c, c.k_merge);
+            row[6] = c.k_move.ms - ms0[0];
+            row[7] = c.k_rebuild.ms - ms0[1];
+            row[8] = c.k_merge.ms - ms0[2];
         }
         c.st.mcmc_itr_total += itrs;
         ++rounds;

@@ -19,6 +19,7 @@ LIB_PATH = os.environ.get("GSAP_LIB", os.path.join(HERE, "libgsap.so"))
 
 GSAP_OK, GSAP_EINVAL, GSAP_ENOMEM, GSAP_ECUDA, GSAP_ENCCL, GSAP_ESTATE, GSAP_EUNSUPPORTED = range(7)
 GSAP_MERGE, GSAP_MOVE = 0, 1
+TRACE_COLS = 9                  # GSAP_TRACE_COLS (gsap.h)
 STATUS_NAMES = ["GSAP_OK", "GSAP_EINVAL", "GSAP_ENOMEM", "GSAP_ECUDA", "GSAP_ENCCL", "GSAP_ESTATE",
                 "GSAP_EUNSUPPORTED"]
 
@@ -331,8 +332,8 @@ class Context:
         B = C.c_int32(0)
         mdl = C.c_double(0)
         rounds = C.c_int32(0)
-        trace = np.zeros(6 * trace_cap)
+        trace = np.zeros(TRACE_COLS * trace_cap)
         _check(lib().gsap_run(self.h, _ptr(b), C.byref(B), C.byref(mdl), trace.ctypes.data, trace_cap,
                               C.byref(rounds)))
-        tr = trace[:6 * min(rounds.value, trace_cap)].reshape(-1, 6)
+        tr = trace[:TRACE_COLS * min(rounds.value, trace_cap)].reshape(-1, TRACE_COLS)
         return dict(b=b, B=B.value, mdl=mdl.value, trace=tr, rounds=rounds.value)

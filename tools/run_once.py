@@ -29,5 +29,6 @@ for i in range(a.runs):
           f"itrs={st['mcmc_itr_total']}", flush=True)
     if i == 0:
         for row in res["trace"]:
-            print(f"   outer={int(row[0]):3d} B={int(row[1]):8d} itrs={int(row[2]):3d} MDL={row[3]:.6e} sec={row[4]:.4f} acc={int(row[5])}")
+            print(f"   outer={int(row[0]):3d} B={int(row[1]):8d} itrs={int(row[2]):3d} MDL={row[3]:.6e} sec={row[4]:.4f} acc={int(row[5])} "
+                  f"move={row[6]:.2f}ms rebuild={row[7]:.2f}ms merge={row[8]:.2f}ms")
     ctx.gsap_reset_stats()
