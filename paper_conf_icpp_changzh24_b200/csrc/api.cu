@@ -188,6 +188,9 @@ static void free_ctx(Ctx &c) {
     } catch (...) {
     }
     if (c.own_stream && c.stream) cudaStreamDestroy(c.stream);
+    if (c.side) cudaStreamDestroy(c.side);
+    if (c.ev_fork) cudaEventDestroy(c.ev_fork);
+    if (c.ev_join) cudaEventDestroy(c.ev_join);
 }
 
 // one device allocation per context, carved into aligned sub-buffers
@@ -252,6 +255,9 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         GSAP_CUDA(cudaStreamCreateWithFlags(&c.stream, cudaStreamNonBlocking));
         c.own_stream = true;
     }
+    GSAP_CUDA(cudaStreamCreateWithFlags(&c.side, cudaStreamNonBlocking));
+    GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_fork, cudaEventDisableTiming));
+    GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_join, cudaEventDisableTiming));
     GSAP_CUDA(cudaGetDevice(&c.dev));
     comm_init(c, dist);
     if (c.nranks > 1) c.prm.cuda_graphs = 0;

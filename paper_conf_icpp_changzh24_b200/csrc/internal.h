@@ -35,6 +35,8 @@ struct Ctx {
     size_t arena_bytes = 0;
     cudaStream_t stream = nullptr;
     bool own_stream = false;
+    cudaStream_t side = nullptr;                 // second stream (group roles of k_move run beside the warp role)
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     gsap_params prm{};
 
     // graph (device): out CSR in the caller's order, in CSC (by source id, then

@@ -18,6 +18,7 @@
 // owns in adjacency order, followed by a fixed shuffle tree: the result is
 // deterministic and independent of the launch shape.
 #include <algorithm>
+#include <cstdlib>
 
 #include "internal.h"
 
@@ -31,6 +32,7 @@ constexpr int CTA_THREADS = 256;       // big-vertex role: one CTA per vertex
 constexpr int MID_TAB = 512;           // mid role: 64-thread group tables (<= 256 keys)
 constexpr int MID_TAB_LOG2 = 9;
 constexpr int CTA_SMEM_SLOTS = MOVE_WARPS * WARP_TAB;   // big-vertex shared table (<= 1024 keys)
+constexpr size_t MOVE_SMEM = sizeof(int4) * MOVE_WARPS * WARP_TAB + sizeof(int) * MOVE_WARPS * (WARP_TAB / 2);
 // vertices with > 1024 adjacency entries take the huge role (global tables when B > 1024)
 #ifndef GSAP_MOVE_MINB
 #define GSAP_MOVE_MINB 3               // CTAs per SM the register budget is sized for
@@ -49,6 +51,7 @@ struct MoveArgs {
     int first, count;
     const int *__restrict__ list;   // big-vertex kernel: sorted vertex ids
     int list_count;
+    int propose;                    // 1: k_move draws the proposal itself (MOVE_FUSED), else reads s_in
     const int *s_in;                // MOVE_DELTA
     int *s_out;
     double *dS, *H;
@@ -130,6 +133,35 @@ GSAP_DEV void group_sum3(double &x, double &y, double &z, double *sh) {
 }
 
 
+// sparse regime: four lookups (line k, key y_k) as interleaved branchless
+// binary searches -- each step issues four independent loads, so a lane's
+// dependent-load depth is log2(max len) + 1 instead of four times that
+// (the lines of M live in HBM once the blockmodel outgrows L2)
+GSAP_DEV void lookup4(const Line (&L)[4], const int (&y)[4], int (&out)[4]) {
+    int p[4] = {0, 0, 0, 0}, n[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) n[k] = L[k].len;
+    while (n[0] > 1 || n[1] > 1 || n[2] > 1 || n[3] > 1) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            if (n[k] > 1) {
+                const int h = n[k] >> 1;
+                p[k] = __ldg(L[k].idx + p[k] + h) <= y[k] ? p[k] + h : p[k];
+                n[k] -= h;
+            }
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        int v = 0;
+        if (L[k].len > 0) {
+            const int id = __ldg(L[k].idx + p[k]), cn = __ldg(L[k].cnt + p[k]);
+            v = id == y[k] ? cn : 0;
+        }
+        out[k] = v;
+    }
+}
+
 // the state of one move r -> s that every term needs
 struct MoveCtx {
     int v, r, s;
@@ -151,8 +183,22 @@ GSAP_DEV void t_terms(const MoveArgs &a, const MoveCtx &q, int t, long long ot, 
         pf += c * (double)(2 * q.Mss + 1) * __ldg(rcp + q.s);
         pb += c * (double)(q.Msr2 + q.Mrs2 + 1) / ((double)q.ds2 + q.Bd);
     } else {
-        const long long Mrt = row_at(a.m, q.Rr, q.r, t), Mst = row_at(a.m, q.Rs, q.s, t);
-        const long long Mtr = col_at(a.m, q.Cr, q.r, t), Mts = col_at(a.m, q.Cs, q.s, t);
+        long long Mrt, Mst, Mtr, Mts;
+        if (a.m.dense) {
+            Mrt = row_at(a.m, q.Rr, q.r, t);
+            Mst = row_at(a.m, q.Rs, q.s, t);
+            Mtr = col_at(a.m, q.Cr, q.r, t);
+            Mts = col_at(a.m, q.Cs, q.s, t);
+        } else {
+            const Line Ln[4] = {q.Rr, q.Rs, q.Cr, q.Cs};
+            const int yt[4] = {t, t, t, t};
+            int o4[4];
+            lookup4(Ln, yt, o4);
+            Mrt = o4[0];
+            Mst = o4[1];
+            Mtr = o4[2];
+            Mts = o4[3];
+        }
         const double rt = __ldg(rcp + t);
         accS -= df_t(ft, Mrt, -ot) + df_t(ft, Mst, ot) + df_t(ft, Mtr, -it) + df_t(ft, Mts, it);
         pf += c * (double)(Mts + Mst + 1) * rt;
@@ -224,83 +270,238 @@ GSAP_DEV void mh_decide(const MoveArgs &a, const MoveCtx &q, uint4 w, double dS,
     acc_out = u <= p;
 }
 
-// (a2), one warp per vertex: phase A builds the neighbour-block table and
-// compacts the unique blocks into `list` in first-occurrence order; phase B
-// gives each lane whole unique blocks (all lanes busy).  Table left empty.
+// (a1) one thread per vertex: the proposal chain is a handful of dependent
+// loads, so 32 vertices per warp keep them in flight (R:O.4).
 template <bool WEIGHTED>
-GSAP_DEV void eval_move_warp(const MoveArgs &a, int v, int r, int s, uint4 w, int4 *tab, int *list,
-                             double &dS_out, double &H_out, bool &acc_out) {
+GSAP_DEV int propose_move_thread(const MoveArgs &a, int v, uint4 w) {
+    const uint32_t B = (uint32_t)a.B;
+    const uint32_t K = (uint32_t)(__ldg(a.kout + v) + __ldg(a.kin + v));
+    if (K == 0) return (int)pick(w.z, B);
+    const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
+    const int ci = __ldg(a.cscptr + v);
+    const uint32_t p = pick(w.x, K);
+    int n;
+    if (!WEIGHTED) {
+        n = (int)p < nout ? __ldg(a.col + ro + p) : __ldg(a.cscsrc + ci + (p - nout));
+    } else {
+        long long acc = 0;
+        n = -1;
+        for (int e = 0; e < nout && n < 0; ++e) {
+            acc += __ldg(a.wgt + ro + e);
+            if ((long long)p < acc) n = __ldg(a.col + ro + e);
+        }
+        const int nin = __ldg(a.cscptr + v + 1) - ci;
+        for (int e = 0; e < nin && n < 0; ++e) {
+            acc += __ldg(a.cscwgt + ci + e);
+            if ((long long)p < acc) n = __ldg(a.cscsrc + ci + e);
+        }
+    }
+    const int u = __ldg(a.b + n);
+    const uint32_t du = (uint32_t)bm_deg(a.m, u);
+    if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
+    return bm_walk(a.m, u, (long long)pick(w.z, du), -1);
+}
+
+// the proposal of a warp-path vertex (R:O.4, Alg. 1): the neighbour at
+// position p and its block come from the adjacency registers (nb, tb: entry
+// 32 c + lane in nb[c]) when p < 128 in an unweighted graph; the walk over
+// row / column u is a 32-ary warp search.  Same integer result as
+// propose_move_thread.
+template <bool WEIGHTED>
+GSAP_DEV int propose_warp(const MoveArgs &a, int v, uint4 w, int deg, const int (&tb)[4]) {
+    const uint32_t B = (uint32_t)a.B;
+    if (WEIGHTED || deg > 128) return propose_move_thread<WEIGHTED>(a, v, w);   // warp-uniform
+    if (deg == 0) return (int)pick(w.z, B);
+    const uint32_t p = pick(w.x, (uint32_t)deg);
+    const int c = (int)(p >> 5);
+    const int x = c == 0 ? tb[0] : c == 1 ? tb[1] : c == 2 ? tb[2] : tb[3];
+    const int u = __shfl_sync(FULL, x, (int)(p & 31u));
+    const uint32_t du = (uint32_t)bm_deg(a.m, u);
+    if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
+    return bm_walk_warp(a.m, u, (long long)pick(w.z, du));
+}
+
+// (a1 + a2), one warp per vertex (at most 128 adjacency entries, or B <= 128):
+// adjacency ids and their blocks are loaded once into registers and serve
+// both the proposal and the neighbour-block histogram; phase A builds the
+// shared-memory table and compacts the unique blocks into `list` in
+// first-occurrence order; phase B gives each lane whole unique blocks.  The
+// 2x2 core and the four degree terms take lanes 0..7 with one df each.
+// int32 throughout (weights and counts < 2^30, gsap.h).  Table left empty.
+template <bool WEIGHTED, bool DENSE>
+GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
     const int lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
+    const int v = a.first + i;
     const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
     const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
     const int deg = nout + nin;
-    int keep[4];
+    int nb[4], tb[4];
 #pragma unroll
     for (int c = 0; c < 4; ++c) {
-        keep[c] = -1;
         const int j = c * 32 + lane;
-        if (j < deg) {
-            const bool out = j < nout;
-            const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-            if (nb != v) {
-                const int t = __ldg(a.b + nb);
+        nb[c] = j < deg ? (j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout)) : -1;
+    }
+#pragma unroll
+    for (int c = 0; c < 4; ++c) tb[c] = nb[c] >= 0 ? __ldg(a.b + nb[c]) : -1;
+    const int r = __ldg(a.b + v);
+    const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
+    const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
+    int s;
+    if (a.propose) {
+        s = propose_warp<WEIGHTED>(a, v, w, deg, tb);
+        if (lane == 0) a.s_out[i] = s;
+    } else {
+        s = a.s_in[i];
+    }
+    double dS = 0.0, H = 1.0;
+    bool acc = false;
+    if (s != r) {
+        // ---- phase A: histogram of v's neighbour blocks (self-loop excluded)
+        int keep[4];
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            keep[c] = -1;
+            const int j = c * 32 + lane;
+            if (nb[c] >= 0 && nb[c] != v) {
+                const bool out = j < nout;
                 const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
-                const int sl = tab_insert(tab, WARP_TAB_LOG2, t);
+                const int sl = tab_insert(tab, WARP_TAB_LOG2, tb[c]);
                 atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
                 atomicMin(&tab[sl].w, j);
                 keep[c] = sl;
             }
         }
-    }
-    for (int j = 128 + lane; j < deg; j += 32) {   // only when B <= 128 (<= B keys)
-        const bool out = j < nout;
-        const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-        if (nb == v) continue;
-        const int t = __ldg(a.b + nb);
-        const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
-        const int sl = tab_insert(tab, WARP_TAB_LOG2, t);
-        atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
-        atomicMin(&tab[sl].w, j);
-    }
-    __syncwarp();
-    int nuniq = 0;
-#pragma unroll
-    for (int c = 0; c < 4; ++c) {
-        const int sl = keep[c];
-        const bool own = sl >= 0 && tab[sl].w == c * 32 + lane;
-        const unsigned bal = __ballot_sync(FULL, own);
-        if (own) list[nuniq + __popc(bal & lt)] = sl;
-        nuniq += __popc(bal);
-    }
-    for (int base = 128; base < deg; base += 32) {
-        const int j = base + lane;
-        int sl = -1;
-        if (j < deg) {
-            const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-            if (nb != v) sl = tab_find(tab, WARP_TAB_LOG2, __ldg(a.b + nb));
+        for (int j = 128 + lane; j < deg; j += 32) {   // only when B <= 128 (<= B keys)
+            const bool out = j < nout;
+            const int n = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+            if (n == v) continue;
+            const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
+            const int sl = tab_insert(tab, WARP_TAB_LOG2, __ldg(a.b + n));
+            atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
+            atomicMin(&tab[sl].w, j);
         }
-        const bool own = sl >= 0 && tab[sl].w == j;
-        const unsigned bal = __ballot_sync(FULL, own);
-        if (own) list[nuniq + __popc(bal & lt)] = sl;
-        nuniq += __popc(bal);
+        __syncwarp();
+        int nuniq = 0;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            const int sl = keep[c];
+            const bool own = sl >= 0 && tab[sl].w == c * 32 + lane;
+            const unsigned bal = __ballot_sync(FULL, own);
+            if (own) list[nuniq + __popc(bal & lt)] = sl;
+            nuniq += __popc(bal);
+        }
+        for (int base = 128; base < deg; base += 32) {
+            const int j = base + lane;
+            int sl = -1;
+            if (j < deg) {
+                const int n = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+                if (n != v) sl = tab_find(tab, WARP_TAB_LOG2, __ldg(a.b + n));
+            }
+            const bool own = sl >= 0 && tab[sl].w == j;
+            const unsigned bal = __ballot_sync(FULL, own);
+            if (own) list[nuniq + __popc(bal & lt)] = sl;
+            nuniq += __popc(bal);
+        }
+        __syncwarp();
+        // ---- core state
+        const int slr = tab_find(tab, WARP_TAB_LOG2, r), sls = tab_find(tab, WARP_TAB_LOG2, s);
+        const int o_r = slr >= 0 ? tab[slr].y : 0, i_r = slr >= 0 ? tab[slr].z : 0;
+        const int o_s = sls >= 0 ? tab[sls].y : 0, i_s = sls >= 0 ? tab[sls].z : 0;
+        const int kout = __ldg(a.kout + v), kin = __ldg(a.kin + v), l = __ldg(a.selfw + v);
+        const int dout_r = __ldg(a.m.dout + r), dout_s = __ldg(a.m.dout + s);
+        const int din_r = __ldg(a.m.din + r), din_s = __ldg(a.m.din + s);
+        const int *__restrict__ D = a.m.dense;   // non-null iff DENSE
+        const int B = a.m.B;
+        int Mrr, Mrs, Msr, Mss;
+        Line Ln[4];   // sparse: row r, row s, column r, column s of M
+        if (DENSE) {
+            Mrr = __ldg(D + (size_t)r * B + r);
+            Mrs = __ldg(D + (size_t)r * B + s);
+            Msr = __ldg(D + (size_t)s * B + r);
+            Mss = __ldg(D + (size_t)s * B + s);
+        } else {
+            Ln[0] = row_line(a.m, r);
+            Ln[1] = row_line(a.m, s);
+            Ln[2] = col_line(a.m, r);
+            Ln[3] = col_line(a.m, s);
+            const Line Lc[4] = {Ln[0], Ln[0], Ln[1], Ln[1]};
+            const int yc[4] = {r, s, r, s};
+            int oc[4];
+            lookup4(Lc, yc, oc);
+            Mrr = oc[0];
+            Mrs = oc[1];
+            Msr = oc[2];
+            Mss = oc[3];
+        }
+        const double Bd = (double)B;
+        const int Mrr2 = Mrr - o_r - i_r - l, Mrs2 = Mrs + i_r - o_s, Msr2 = Msr + o_r - i_s;
+        const int dr2 = dout_r + din_r - kout - kin, ds2 = dout_s + din_s + kout + kin;
+        const double2 *__restrict__ ft = a.m.ft;
+        const double *__restrict__ rcp = a.m.rcp;
+        // ---- phase B: one unique neighbour block per lane
+        double accS = 0.0, pf = 0.0, pb = 0.0;
+        for (int k = lane; k < nuniq; k += 32) {
+            const int4 e = tab[list[k]];
+            const int t = e.x, ot = e.y, it = e.z;
+            const double cw = (double)(ot + it);
+            if (t == r) {
+                pf += cw * (double)(Mrs + Msr + 1) * __ldg(rcp + r);
+                pb += cw * (double)(2 * Mrr2 + 1) / ((double)dr2 + Bd);
+            } else if (t == s) {
+                pf += cw * (double)(2 * Mss + 1) * __ldg(rcp + s);
+                pb += cw * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd);
+            } else {
+                int Mrt, Mst, Mtr, Mts;
+                if (DENSE) {
+                    Mrt = __ldg(D + (size_t)r * B + t);
+                    Mst = __ldg(D + (size_t)s * B + t);
+                    Mtr = __ldg(D + (size_t)t * B + r);
+                    Mts = __ldg(D + (size_t)t * B + s);
+                } else {
+                    const int yt[4] = {t, t, t, t};
+                    int o4[4];
+                    lookup4(Ln, yt, o4);
+                    Mrt = o4[0];
+                    Mst = o4[1];
+                    Mtr = o4[2];
+                    Mts = o4[3];
+                }
+                const double rt = __ldg(rcp + t);
+                accS -= df_t(ft, Mrt, -ot) + df_t(ft, Mst, ot) + df_t(ft, Mtr, -it) + df_t(ft, Mts, it);
+                pf += cw * (double)(Mts + Mst + 1) * rt;
+                pb += cw * (double)(Mtr - it + Mrt - ot + 1) * rt;
+            }
+        }
+        // the 2x2 core (lanes 0..3) and the degree terms (lanes 4..7), one df each
+        if (lane < 8) {
+            const int m = lane == 0 ? Mrr : lane == 1 ? Mrs : lane == 2 ? Msr : lane == 3 ? Mss
+                        : lane == 4 ? dout_r : lane == 5 ? dout_s : lane == 6 ? din_r : din_s;
+            const int d = lane == 0 ? -(o_r + i_r + l) : lane == 1 ? i_r - o_s : lane == 2 ? o_r - i_s
+                        : lane == 3 ? o_s + i_s + l : lane == 4 ? -kout : lane == 5 ? kout : lane == 6 ? -kin : kin;
+            const double x = df_t(ft, m, d);
+            accS += lane < 4 ? -x : x;
+        }
+        if (lane == 0 && l > 0) {   // v's self-loop in the forward / backward proposal laws (R:Z26)
+            pf += 2.0 * (double)l * (double)(Mrs + Msr + 1) * __ldg(rcp + r);
+            pb += 2.0 * (double)l * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd);
+        }
+        accS = warp_sum(accS);
+        pf = warp_sum(pf);
+        pb = warp_sum(pb);
+        // leave the table empty: exactly the listed slots were used
+        for (int k = lane; k < nuniq; k += 32) tab[list[k]] = make_int4(-1, 0, 0, 0x7fffffff);
+        __syncwarp();
+        dS = accS;
+        H = (kout + kin == 0) ? 1.0 : pb / pf;
+        const double p = exp(-a.beta * dS) * H;
+        acc = ((double)w.w + 0.5) * (1.0 / 4294967296.0) <= p;
     }
-    __syncwarp();
-    MoveCtx q;
-    move_ctx(a, v, r, s, tab, WARP_TAB_LOG2, q);
-    double accS = 0.0, pf = 0.0, pb = 0.0;
-    for (int k = lane; k < nuniq; k += 32) {
-        const int4 e = tab[list[k]];
-        t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
+    if (lane == 0) {
+        if (a.dS) a.dS[i] = dS;
+        if (a.H) a.H[i] = H;
+        if (a.acc) a.acc[i] = acc ? 1 : 0;
     }
-    if (lane < 10) core_term(a, q, lane, accS, pf, pb);
-    accS = warp_sum(accS);
-    pf = warp_sum(pf);
-    pb = warp_sum(pb);
-    // leave the table empty: exactly the listed slots were used
-    for (int k = lane; k < nuniq; k += 32) tab[list[k]] = make_int4(-1, 0, 0, 0x7fffffff);
-    __syncwarp();
-    mh_decide(a, q, w, accS, pf, pb, dS_out, H_out, acc_out);
 }
 
 // (a2), one G-thread group (64: a quarter CTA, 256: a CTA) per big vertex:
@@ -350,51 +551,31 @@ GSAP_DEV void do_vertex(const MoveArgs &a, int v, int4 *tab, int log2cap, int *l
     const int i = v - a.first;
     const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
     const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
-    const int s = a.s_in[i];
+    int s;
+    if (a.propose) {   // one thread draws, the group reads it back (sh[3 G/32] is this group's slot)
+        int *sp = reinterpret_cast<int *>(sh + 3 * (G / 32));
+        if ((threadIdx.x & (G - 1)) == 0) {
+            s = propose_move_thread<WEIGHTED>(a, v, w);
+            *sp = s;
+            a.s_out[i] = s;
+        }
+        gsync<G>();
+        s = *sp;
+        gsync<G>();
+    } else {
+        s = a.s_in[i];
+    }
     const int r = __ldg(a.b + v);
     double dS = 0.0, H = 1.0;
     bool acc = false;
     if (s != r) {
-        if (G == 32) eval_move_warp<WEIGHTED>(a, v, r, s, w, tab, list, dS, H, acc);
-        else eval_move_group<G, WEIGHTED>(a, v, r, s, w, tab, log2cap, sh, dS, H, acc);
+        eval_move_group<G, WEIGHTED>(a, v, r, s, w, tab, log2cap, sh, dS, H, acc);
     }
     if ((threadIdx.x & (G - 1)) == 0) {
         if (a.dS) a.dS[i] = dS;
         if (a.H) a.H[i] = H;
         if (a.acc) a.acc[i] = acc ? 1 : 0;
     }
-}
-
-// (a1) one thread per vertex: the proposal chain is a handful of dependent
-// loads, so 32 vertices per warp keep them in flight (R:O.4).
-template <bool WEIGHTED>
-GSAP_DEV int propose_move_thread(const MoveArgs &a, int v, uint4 w) {
-    const uint32_t B = (uint32_t)a.B;
-    const uint32_t K = (uint32_t)(__ldg(a.kout + v) + __ldg(a.kin + v));
-    if (K == 0) return (int)pick(w.z, B);
-    const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
-    const int ci = __ldg(a.cscptr + v);
-    const uint32_t p = pick(w.x, K);
-    int n;
-    if (!WEIGHTED) {
-        n = (int)p < nout ? __ldg(a.col + ro + p) : __ldg(a.cscsrc + ci + (p - nout));
-    } else {
-        long long acc = 0;
-        n = -1;
-        for (int e = 0; e < nout && n < 0; ++e) {
-            acc += __ldg(a.wgt + ro + e);
-            if ((long long)p < acc) n = __ldg(a.col + ro + e);
-        }
-        const int nin = __ldg(a.cscptr + v + 1) - ci;
-        for (int e = 0; e < nin && n < 0; ++e) {
-            acc += __ldg(a.cscwgt + ci + e);
-            if ((long long)p < acc) n = __ldg(a.cscsrc + ci + e);
-        }
-    }
-    const int u = __ldg(a.b + n);
-    const uint32_t du = (uint32_t)bm_deg(a.m, u);
-    if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
-    return bm_walk(a.m, u, (long long)pick(w.z, du), -1);
 }
 
 template <bool WEIGHTED>
@@ -412,11 +593,9 @@ __global__ void __launch_bounds__(256) k_propose(MoveArgs a) {
 // CTAs take every other vertex of [first, first + count) one warp per vertex.
 // The shared memory is the 8 warp tables, or one CTA table over the same bytes.
 template <bool WEIGHTED>
-__global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveArgs a) {
-    __shared__ int4 tabs[MOVE_WARPS * WARP_TAB];
-    __shared__ int lists[MOVE_WARPS * (WARP_TAB / 2)];
-    __shared__ double sh[3 * MOVE_WARPS];
-    const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
+__global__ void __launch_bounds__(MOVE_WARPS * 32) k_move_groups(MoveArgs a) {
+    __shared__ int4 tabs[CTA_SMEM_SLOTS];
+    __shared__ double sh[3 * MOVE_WARPS + 8];   // group sums + the broadcast proposal
     if ((int)blockIdx.x < a.nmid_ctas) {
         // four 64-thread groups per CTA, one mid vertex each
         const int gid = threadIdx.x >> 6, gt = threadIdx.x & 63;
@@ -424,7 +603,7 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
         for (int li = blockIdx.x * 4 + gid; li < a.mlist_count; li += a.nmid_ctas * 4) {
             tab_clear<64>(tab, MID_TAB, gt);
             gsync<64>();
-            do_vertex<64, WEIGHTED>(a, a.mlist[li], tab, MID_TAB_LOG2, nullptr, sh + gid * 6);
+            do_vertex<64, WEIGHTED>(a, a.mlist[li], tab, MID_TAB_LOG2, nullptr, sh + gid * 8);
             gsync<64>();
         }
         return;
@@ -447,22 +626,30 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
             do_vertex<CTA_THREADS, WEIGHTED>(a, a.hlist[li], tab, a.gtab_log2, nullptr, sh);
             __syncthreads();
         }
-        return;
-    }
+        }
+}
+
+// (a1 + a2) warp role: every vertex of [first, first + count) that is not in
+// a group list, one warp per vertex (launched beside k_move_groups)
+template <bool WEIGHTED, bool DENSE>
+__global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveArgs a) {
+    extern __shared__ int4 move_smem[];   // MOVE_SMEM bytes
+    int4 *tabs = move_smem;                                         // MOVE_WARPS * WARP_TAB
+    int *lists = reinterpret_cast<int *>(tabs + MOVE_WARPS * WARP_TAB);   // MOVE_WARPS * WARP_TAB / 2
+    const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
     int4 *tab = tabs + wl * WARP_TAB;
     int *list = lists + wl * (WARP_TAB / 2);
     tab_clear<32>(tab, WARP_TAB, lane);
     __syncwarp();
-    const int role0 = a.nmid_ctas + a.nbig_ctas + a.nhuge_ctas;
-    const int nwarps = (gridDim.x - role0) * MOVE_WARPS;
+    const int nwarps = gridDim.x * MOVE_WARPS;
     const bool skip_big = a.B > BIG_THR;
-    for (int i = (blockIdx.x - role0) * MOVE_WARPS + wl; i < a.count; i += nwarps) {
+    for (int i = blockIdx.x * MOVE_WARPS + wl; i < a.count; i += nwarps) {
         const int v = a.first + i;
         // adjacency entries bound the number of unique neighbour blocks
         if (skip_big &&
             (__ldg(a.rowptr + v + 1) - __ldg(a.rowptr + v)) + (__ldg(a.cscptr + v + 1) - __ldg(a.cscptr + v)) > BIG_THR)
             continue;
-        do_vertex<32, WEIGHTED>(a, v, tab, WARP_TAB_LOG2, list, nullptr);
+        move_vertex_warp<WEIGHTED, DENSE>(a, i, tab, list);
     }
 }
 
@@ -498,16 +685,15 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     a.dS = dS; a.H = H; a.acc = acc;
     a.gtab = nullptr;
     a.gtab_log2 = 0;
-    if (mode != MOVE_DELTA) {   // (a1): thread per vertex
+    a.propose = mode == MOVE_FUSED ? 1 : 0;
+    if (mode == MOVE_PROPOSE) {   // (a1) alone: thread per vertex
         const int pg = (int)std::min<long long>(((long long)count + 63) / 64, 148LL * 64);
         if (c.weighted) k_propose<true><<<pg, 64, 0, c.stream>>>(a);
         else k_propose<false><<<pg, 64, 0, c.stream>>>(a);
         ++c.launches;
         GSAP_CHECK_LAUNCH();
-        if (mode == MOVE_PROPOSE) {
-            kc_end(c, c.k_move, ev, 0.0);
-            return;
-        }
+        kc_end(c, c.k_move, ev, 0.0);
+        return;
     }
     a.nbig_ctas = 0;
     a.nhuge_ctas = 0;
@@ -559,12 +745,37 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         }
     }
     const long long need = ((long long)count + MOVE_WARPS - 1) / MOVE_WARPS;
-    const int grid = a.nmid_ctas + a.nbig_ctas + a.nhuge_ctas +
-                     (int)std::max<long long>(1, std::min<long long>(need, 148LL * 8));
-    if (c.weighted) k_move<true><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a);
-    else k_move<false><<<grid, MOVE_WARPS * 32, 0, c.stream>>>(a);
+    const int grid = (int)std::max<long long>(1, std::min<long long>(need, 148LL * 8));
+    const int ggrid = a.nmid_ctas + a.nbig_ctas + a.nhuge_ctas;
+    if (ggrid > 0) {   // the group roles run beside the warp role (fork / join on the side stream)
+        GSAP_CUDA(cudaEventRecord(c.ev_fork, c.stream));
+        GSAP_CUDA(cudaStreamWaitEvent(c.side, c.ev_fork, 0));
+        if (c.weighted) k_move_groups<true><<<ggrid, MOVE_WARPS * 32, 0, c.side>>>(a);
+        else k_move_groups<false><<<ggrid, MOVE_WARPS * 32, 0, c.side>>>(a);
+        ++c.launches;
+        GSAP_CHECK_LAUNCH();
+        GSAP_CUDA(cudaEventRecord(c.ev_join, c.side));
+    }
+    static bool attr = false;
+    if (!attr) {
+        const int sm = (int)MOVE_SMEM;
+        GSAP_CUDA(cudaFuncSetAttribute(k_move<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+        GSAP_CUDA(cudaFuncSetAttribute(k_move<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+        GSAP_CUDA(cudaFuncSetAttribute(k_move<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+        GSAP_CUDA(cudaFuncSetAttribute(k_move<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+        attr = true;
+    }
+    const bool dense = a.m.dense != nullptr;
+    if (c.weighted) {
+        if (dense) k_move<true, true><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);
+        else k_move<true, false><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);
+    } else {
+        if (dense) k_move<false, true><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);
+        else k_move<false, false><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);
+    }
     ++c.launches;
     GSAP_CHECK_LAUNCH();
+    if (ggrid > 0) GSAP_CUDA(cudaStreamWaitEvent(c.stream, c.ev_join, 0));
     // algorithmic bytes: adjacency ids (+ weights),
     // row / column pointers, b[v], the outputs (s, dS, acc)
     const long long adj = (long long)(c.h_rowptr[first + count] - c.h_rowptr[first]) +
