@@ -465,8 +465,8 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     k_segsort_warp<K><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(c.seg_off, seg, c.seg_listW, c.seg_ctr, c.wa, c.wb,
                                                            c.seg_nnz);
     const int gc = (int)std::min<long long>(std::max(1, B / 4), 148LL * 4);
-    k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(c.seg_off, seg, c.seg_listC, c.seg_ctr, c.wa, c.wb, c.seg_nnz,
-                                               reinterpret_cast<K *>(c.xl_keys), c.xl_hp);
+    k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(c.seg_off, seg, c.seg_listC, c.seg_ctr, bits_for(B), c.wa, c.wb,
+                                               c.seg_nnz);
     k_segsort_xl<K><<<gc, 256, 0, c.stream>>>(c.seg_off, seg, c.seg_listC, c.seg_ctr, bits_for(B), c.wa, c.wb,
                                               c.seg_nnz, reinterpret_cast<K *>(c.xl_keys), c.xl_hp);
     c.launches += 5;

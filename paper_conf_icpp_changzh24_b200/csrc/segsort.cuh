@@ -317,30 +317,105 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__re
 }
 #endif
 
+// stable LSD radix sort of a[0, L) by the block bits of the key (key_col),
+// 4-bit digits, NT threads.  Each thread owns a contiguous chunk of an odd
+// number of keys (conflict-free shared-memory strides); its 16 digit
+// counters are packed two per word (16-bit fields, L <= 4096) in its own
+// column of cntp[8][NT], so counting needs no atomics, and one block-wide
+// scan of the packed 8-word vectors gives every (digit, thread) offset.
+// Ping-pongs between a and b; returns the buffer holding the result.
+// O(L * passes) instead of bitonic's O(L log^2 L).
+template <typename K, int NT>
+GSAP_DEV K *cta_radix_sort(K *a, K *b, int L, int col_bits, unsigned *cntp, unsigned *wsum) {
+    const int tid = threadIdx.x % NT, lane = tid & 31, w = tid >> 5;
+    const int C = ((L + NT - 1) / NT) | 1;
+    const int lo = min(L, tid * C), hi = min(L, lo + C);
+    for (int sh = 0; sh < col_bits; sh += 4) {
+#pragma unroll
+        for (int k = 0; k < 8; ++k) cntp[k * NT + tid] = 0u;
+        for (int i = lo; i < hi; ++i) {
+            const int d = (key_col(a[i]) >> sh) & 15;
+            cntp[(d >> 1) * NT + tid] += 1u << ((d & 1) * 16);
+        }
+        unsigned c[8], x[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) x[k] = c[k] = cntp[k * NT + tid];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                const unsigned t = __shfl_up_sync(FULL, x[k], o);
+                if (lane >= o) x[k] += t;
+            }
+        }
+        if (NT > 32) {
+            if (lane == 31) {
+#pragma unroll
+                for (int k = 0; k < 8; ++k) wsum[w * 8 + k] = x[k];
+            }
+            __syncthreads();
+        }
+        unsigned wp[8], tot[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            wp[k] = 0u;
+            tot[k] = NT > 32 ? 0u : __shfl_sync(FULL, x[k], 31);
+        }
+        if (NT > 32) {
+            for (int q = 0; q < NT / 32; ++q) {
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const unsigned v = wsum[q * 8 + k];
+                    wp[k] += q < w ? v : 0u;
+                    tot[k] += v;
+                }
+            }
+        }
+        unsigned run = 0u;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const unsigned t0 = tot[k] & 0xffffu, t1 = tot[k] >> 16;
+            const unsigned base = run | ((run + t0) << 16);   // bases of digits 2k, 2k + 1
+            run += t0 + t1;
+            cntp[k * NT + tid] = x[k] - c[k] + wp[k] + base;
+        }
+        for (int i = lo; i < hi; ++i) {
+            const K key = a[i];
+            const int d = (key_col(key) >> sh) & 15;
+            const unsigned f = (d & 1) * 16;
+            const unsigned p = cntp[(d >> 1) * NT + tid];
+            cntp[(d >> 1) * NT + tid] = p + (1u << f);
+            b[(p >> f) & 0xffffu] = key;
+        }
+        nt_sync<NT>();
+        K *t = a;
+        a = b;
+        b = t;
+    }
+    return a;
+}
+
 // 4c. long segments: one CTA each, in shared memory (<= 4096) or in a global
 // scratch region at 2 * off (Sum of regions <= 2E)
 template <typename K>
 __global__ void __launch_bounds__(256) k_segsort_cta(const int *__restrict__ off, K *__restrict__ seg,
                                                      const int *__restrict__ listC, const int *__restrict__ counters,
-                                                     int *__restrict__ tcol, int *__restrict__ tcnt,
-                                                     int *__restrict__ nnz, K *__restrict__ gkeys,
-                                                     int *__restrict__ ghp) {
+                                                     int col_bits, int *__restrict__ tcol, int *__restrict__ tcnt,
+                                                     int *__restrict__ nnz) {
     constexpr int CAP = SegCta<K>::CAP;
-    __shared__ K skeys[CAP];
-    __shared__ int shp[CAP];
+    __shared__ K skeys[2][CAP];
+    __shared__ unsigned cntp[8 * 256];
+    __shared__ unsigned wsum[8 * 8];
     __shared__ int sh[8];
     const int n_lines = counters[1];
     for (int li = blockIdx.x; li < n_lines; li += gridDim.x) {
         const int x = listC[li];
         const int o = off[x], L = off[x + 1] - o;
         if (L > CAP) continue;   // k_segsort_xl
-        int n = 1;
-        while (n < L) n <<= 1;
-        K *keys = skeys;
-        int *hp = shp;
-        for (int i = threadIdx.x; i < n; i += 256) keys[i] = i < L ? seg[o + i] : key_max<K>();
+        for (int i = threadIdx.x; i < L; i += 256) skeys[0][i] = seg[o + i];
         __syncthreads();
-        bitonic<K, 256>(keys, n, threadIdx.x);
+        K *keys = cta_radix_sort<K, 256>(skeys[0], skeys[1], L, col_bits, cntp, wsum);
+        int *hp = reinterpret_cast<int *>(keys == skeys[0] ? skeys[1] : skeys[0]);
         const int u = rle_runs<K, 256>(keys, L, hp, tcol + o, tcnt + o, threadIdx.x, sh);
         if (threadIdx.x == 0) nnz[x] = u;
         __syncthreads();
