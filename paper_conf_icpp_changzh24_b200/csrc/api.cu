@@ -319,7 +319,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.dout = A.take<int>(Vs);
         c.din = A.take<int>(Vs);
         c.d_nnz = A.take<int>(1);
-        c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, (size_t)1 << 24), (size_t)1 << 28);
+        c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, (size_t)1 << 24), (size_t)1 << 29);
         c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
         if (c.prm.dense_max_B > 0)
             c.dense_cap = std::min<size_t>(c.dense_cap, (size_t)c.prm.dense_max_B * (size_t)c.prm.dense_max_B);
@@ -713,6 +713,11 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
         c.B = br.B[restart];
         rebuild(c);
         ++outer;
+    }
+    if (br.B[1] == 0) {   // no round ran (max_rounds = 0): the answer is the current partition
+        br.B[1] = c.B;
+        br.S[1] = mdl_now(c);
+        GSAP_CUDA(cudaMemcpyAsync(c.slot_b[1], c.b, sizeof(int) * (size_t)c.V, cudaMemcpyDeviceToDevice, c.stream));
     }
     // the answer: slot 1
     GSAP_CUDA(cudaMemcpyAsync(c.b, c.slot_b[1], sizeof(int) * (size_t)c.V, cudaMemcpyDeviceToDevice, c.stream));
