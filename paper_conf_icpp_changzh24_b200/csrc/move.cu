@@ -238,10 +238,21 @@ GSAP_DEV void move_ctx(const MoveArgs &a, int v, int r, int s, const int4 *tab, 
         q.Cr = col_line(a.m, r);
         q.Cs = col_line(a.m, s);
     }
-    q.Mrr = row_at(a.m, q.Rr, r, r);
-    q.Mrs = row_at(a.m, q.Rr, r, s);
-    q.Msr = row_at(a.m, q.Rs, s, r);
-    q.Mss = row_at(a.m, q.Rs, s, s);
+    if (a.m.dense) {
+        q.Mrr = row_at(a.m, q.Rr, r, r);
+        q.Mrs = row_at(a.m, q.Rr, r, s);
+        q.Msr = row_at(a.m, q.Rs, s, r);
+        q.Mss = row_at(a.m, q.Rs, s, s);
+    } else {
+        const Line Lc[4] = {q.Rr, q.Rr, q.Rs, q.Rs};
+        const int yc[4] = {r, s, r, s};
+        int oc[4];
+        lookup4(Lc, yc, oc);
+        q.Mrr = oc[0];
+        q.Mrs = oc[1];
+        q.Msr = oc[2];
+        q.Mss = oc[3];
+    }
     const int slr = tab_find(tab, log2cap, r), sls = tab_find(tab, log2cap, s);
     q.o_r = slr >= 0 ? tab[slr].y : 0;
     q.i_r = slr >= 0 ? tab[slr].z : 0;
@@ -507,14 +518,13 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
 // (a2), one G-thread group (64: a quarter CTA, 256: a CTA) per big vertex:
 // every unique block owned by its first adjacency position; threads sum their
 // owned terms in position order.
+// phase A of a group vertex: its neighbour-block table, built by group
+// threads [t0, G) (t0 = 32 when warp 0 of the group is drawing the proposal)
 template <int G, bool WEIGHTED>
-GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, int4 *tab, int log2cap,
-                              double *sh, double &dS_out, double &H_out, bool &acc_out) {
-    const int gt = threadIdx.x % G;
-    const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
-    const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
-    const int deg = nout + nin;
-    for (int j = gt; j < deg; j += G) {
+GSAP_DEV void group_table(const MoveArgs &a, int v, int ro, int nout, int ci, int deg, int4 *tab, int log2cap,
+                          int t0) {
+    for (int j = (int)(threadIdx.x % G) - t0; j < deg; j += G - t0) {
+        if (j < 0) break;
         const bool out = j < nout;
         const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
         if (nb == v) continue;   // the self-loop is carried by selfw
@@ -524,7 +534,14 @@ GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, i
         atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
         atomicMin(&tab[sl].w, j);
     }
-    gsync<G>();
+}
+
+// phase B of a group vertex (table complete): every unique block owned by its
+// first adjacency position; threads sum their owned terms in position order.
+template <int G, bool WEIGHTED>
+GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, int ro, int nout, int ci, int deg,
+                              int4 *tab, int log2cap, double *sh, double &dS_out, double &H_out, bool &acc_out) {
+    const int gt = threadIdx.x % G;
     MoveCtx q;
     move_ctx(a, v, r, s, tab, log2cap, q);
     double accS = 0.0, pf = 0.0, pb = 0.0;
@@ -540,6 +557,46 @@ GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, i
     mh_decide(a, q, w, accS, pf, pb, dS_out, H_out, acc_out);
 }
 
+// the proposal of a group vertex, by one whole warp (R:O.4; same integer
+// result as propose_move_thread): the weighted neighbour by a warp prefix
+// scan of the weights (unweighted: direct index), the walk over row /
+// column u by the 32-ary warp search
+template <bool WEIGHTED>
+GSAP_DEV int propose_vertex_warp(const MoveArgs &a, int v, uint4 w, int ro, int nout, int ci, int deg) {
+    const uint32_t B = (uint32_t)a.B;
+    const uint32_t K = (uint32_t)(__ldg(a.kout + v) + __ldg(a.kin + v));
+    if (K == 0) return (int)pick(w.z, B);
+    const uint32_t p = pick(w.x, K);
+    int n;
+    if (!WEIGHTED) {
+        n = (int)p < nout ? __ldg(a.col + ro + p) : __ldg(a.cscsrc + ci + (p - nout));
+    } else {
+        const int lane = threadIdx.x & 31;
+        long long base = 0;
+        n = -1;
+        for (int j0 = 0; j0 < deg && n < 0; j0 += 32) {
+            const int j = j0 + lane;
+            const int wt = j < deg ? (j < nout ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 0;
+            int incl = wt;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int t = __shfl_up_sync(FULL, incl, o);
+                if (lane >= o) incl += t;
+            }
+            const unsigned bal = __ballot_sync(FULL, j < deg && base + incl > (long long)p);
+            if (bal) {
+                const int jj = j0 + __ffs(bal) - 1;
+                n = jj < nout ? __ldg(a.col + ro + jj) : __ldg(a.cscsrc + ci + jj - nout);
+            }
+            base += __shfl_sync(FULL, incl, 31);
+        }
+    }
+    const int u = __ldg(a.b + n);
+    const uint32_t du = (uint32_t)bm_deg(a.m, u);
+    if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
+    return bm_walk_warp(a.m, u, (long long)pick(w.z, du));
+}
+
 template <int G>
 GSAP_DEV void tab_clear(int4 *tab, int slots, int gt) {
     for (int i = gt; i < slots; i += G) tab[i] = make_int4(-1, 0, 0, 0x7fffffff);
@@ -551,26 +608,28 @@ GSAP_DEV void do_vertex(const MoveArgs &a, int v, int4 *tab, int log2cap, int *l
     const int i = v - a.first;
     const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
     const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
-    int s;
-    if (a.propose) {   // one thread draws, the group reads it back (sh[3 G/32] is this group's slot)
-        int *sp = reinterpret_cast<int *>(sh + 3 * (G / 32));
-        if ((threadIdx.x & (G - 1)) == 0) {
-            s = propose_move_thread<WEIGHTED>(a, v, w);
-            *sp = s;
-            a.s_out[i] = s;
-        }
-        gsync<G>();
-        s = *sp;
-        gsync<G>();
-    } else {
-        s = a.s_in[i];
-    }
+    const int gt = threadIdx.x % G;
+    const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
+    const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
+    const int deg = nout + nin;
     const int r = __ldg(a.b + v);
+    // phase A beside the proposal: warp 0 of the group draws s (fused mode),
+    // the other threads build the neighbour-block table (it does not depend on s)
+    int *sp = reinterpret_cast<int *>(sh + 3 * (G / 32));
+    if (a.propose && gt < 32) {
+        const int s0 = propose_vertex_warp<WEIGHTED>(a, v, w, ro, nout, ci, deg);
+        if (gt == 0) {
+            *sp = s0;
+            a.s_out[i] = s0;
+        }
+    } else {
+        group_table<G, WEIGHTED>(a, v, ro, nout, ci, deg, tab, log2cap, a.propose ? 32 : 0);
+    }
+    gsync<G>();
+    const int s = a.propose ? *sp : a.s_in[i];
     double dS = 0.0, H = 1.0;
     bool acc = false;
-    if (s != r) {
-        eval_move_group<G, WEIGHTED>(a, v, r, s, w, tab, log2cap, sh, dS, H, acc);
-    }
+    if (s != r) eval_move_group<G, WEIGHTED>(a, v, r, s, w, ro, nout, ci, deg, tab, log2cap, sh, dS, H, acc);
     if ((threadIdx.x & (G - 1)) == 0) {
         if (a.dS) a.dS[i] = dS;
         if (a.H) a.H[i] = H;
