@@ -47,6 +47,8 @@ typedef enum {
 typedef enum { GSAP_MERGE = 0, GSAP_MOVE = 1 } gsap_phase;
 
 /* SBP parameters: Table 2 (P:295-305 4.1) + readings Z3-Z5, Z10 */
+#define GSAP_COOP_MAX_E (1 << 23)
+
 typedef struct {
     uint64_t seed;            /* Philox key (R:O.3); default 0x5B9D2024 */
     double beta;              /* MH inverse temperature (R:Z5); default 3 */
@@ -62,6 +64,8 @@ typedef struct {
     int32_t profile;          /* 1: time kernels with CUDA events (gsap_stats k_*) */
     int32_t cuda_graphs;      /* 1: capture each MCMC iteration as one CUDA graph (default) */
     int32_t dense_max_B;      /* dense blockmodel iff B <= this; 0 = auto (B^2 <= max(4E, 2^24)) */
+    int32_t sparse_coop;      /* 1 (default): sparse-regime rebuild as one persistent kernel when
+                                 E <= GSAP_COOP_MAX_E; 0: the multi-kernel rebuild (same result) */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */

@@ -6,6 +6,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <chrono>
 #include <mutex>
 #include <new>
@@ -281,6 +282,9 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     }
     // allocation: one device arena (one cudaMalloc / cudaFree per context),
     // planned in a measuring pass and then carved ---------------------------
+    // persistent single-kernel sparse rebuild for graphs whose multi-kernel
+    // rebuild is launch-bound (params.sparse_coop)
+    c.coop_ok = c.prm.sparse_coop != 0 && (long long)E <= GSAP_COOP_MAX_E;
     const size_t Vs = (size_t)V, Es = (size_t)std::max(E, 1);
     const size_t VE = std::max(Vs, Es) + 1;
     const int P = c.prm.num_proposals;
@@ -349,6 +353,16 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.seg_ctr = A.take<int>(4);
         c.xl_keys = A.take<unsigned long long>(2 * Es);
         c.xl_hp = A.take<int>(2 * Es);
+        if (c.coop_ok) {
+            c.seg2_len = A.take<int>(Vs + 1);
+            c.seg2_off = A.take<int>(Vs + 1);
+            c.seg2_cur = A.take<int>(Vs + 1);
+            c.seg2_nnz = A.take<int>(Vs + 1);
+            c.seg2_listC = A.take<int>(Vs + 1);
+            c.xl2_keys = A.take<unsigned long long>(2 * Es);
+            c.xl2_hp = A.take<int>(2 * Es);
+        }
+        c.coop_bar = A.take<unsigned>(2);
         const size_t tiles = (VE + 4095) / 4096 + 1;
         c.counts_cap = 256 * tiles;
         c.counts = A.take<int>(c.counts_cap);
@@ -410,6 +424,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         });
         GSAP_CUDA(cudaMemcpyAsync(c.ft, ft.data(), sizeof(double2) * FT_N, cudaMemcpyHostToDevice, c.stream));
     }
+    GSAP_CUDA(cudaMemsetAsync(c.coop_bar, 0, 2 * sizeof(unsigned), c.stream));
     GSAP_CUDA(cudaMallocHost(&c.h_scal, 8 * sizeof(double)));
     GSAP_CUDA(cudaMallocHost(&c.h_int, 8 * sizeof(int)));
     // upload ---------------------------------------------------------------
@@ -776,6 +791,7 @@ void gsap_default_params(gsap_params *p) {
     p->profile = 0;
     p->cuda_graphs = 1;
     p->dense_max_B = 0;
+    p->sparse_coop = 1;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }

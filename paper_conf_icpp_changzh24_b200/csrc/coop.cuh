@@ -1,0 +1,254 @@
+// coop.cuh -- the sparse-regime blockmodel rebuild (Alg. 2, P:268-283 3.4) as
+// ONE persistent kernel with grid-wide barriers, for graphs small enough that
+// the multi-kernel path of segsort.cuh is bound by launch latency and per-
+// kernel ramp/tail rather than by work (e.g. 20K vertices, 0.5M edges:
+// ~20 launches of a few microseconds of work each).
+//
+// Same algorithm and the same bits as rebuild_sparse (both sides -- rows of
+// M from the out-CSR, columns of M from the in-CSC -- in the same phases):
+//   P0 zero line lengths / cursors / degrees          | barrier
+//   P1 line lengths (counting sort pass 1), dout, din  | barrier
+//   P2 CTA 0 / 1 scan the row / column lengths into segment offsets and list
+//      the long lines; the other CTAs write rcp = 1 / (d + B)  | barrier
+//   P3 scatter the neighbour blocks into their line's segment  | barrier
+//   P4 per-line sort + run-length encoding: warps take the short lines,
+//      CTAs the long ones (shared-memory radix <= CAP, global radix beyond) | barrier
+//   P5 CTA 0 / 1 scan the run counts into the CSR / CSC pointers  | barrier
+//   P6 compact the runs to the pointers with the in-line prefix `cum`.
+// The grid is sized to be co-resident (occupancy x SMs) and launched
+// cooperatively; the barrier is the usual arrive-counter + generation flag.
+#pragma once
+
+#include "segsort.cuh"
+
+namespace gsap {
+
+struct CoopSide {
+    const int *__restrict__ gptr;   // graph lines: out-CSR rowptr / in-CSC cscptr
+    const int *__restrict__ gidx;   // neighbour ids
+    const int *__restrict__ gw;     // weights or nullptr
+    int *len, *off, *cur, *nnz, *listC;   // [B + 1] line scratch
+    void *seg;                      // K[E] segment keys
+    int *tcol, *tcnt;               // [E] runs at segment offsets
+    void *xl_keys;                  // K[2E] global radix scratch
+    int *xl_hp;                     // [2E]
+    int *ptr, *idx, *cnt, *cum, *deg;   // outputs: pointers [B + 1], entries, line sums
+};
+
+struct CoopArgs {
+    int V, B, col_bits;
+    const int *__restrict__ b;
+    const int *__restrict__ kout;
+    const int *__restrict__ kin;
+    CoopSide sd[2];
+    double *rcp;
+    int *d_nnz;
+    int *nlong;       // [2] long lines per side
+    unsigned *bar;    // [2] barrier: arrivals, generation
+};
+
+GSAP_DEV void grid_sync(unsigned *bar) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        volatile unsigned *gen = bar + 1;
+        const unsigned g = *gen;
+        __threadfence();
+        if (atomicAdd(bar, 1u) == gridDim.x - 1) {
+            atomicExch(bar, 0u);
+            __threadfence();
+            atomicAdd(bar + 1, 1u);
+        } else {
+            while (*gen == g) __nanosleep(32);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+// exclusive scan of in[0, n) into out[0, n], out[n] = total, by one 256-thread
+// CTA; lines longer than SEG_WARP_MAX are appended to list (count in *nlist)
+GSAP_DEV void cta_scan_lines(const int *in, int *out, int n, int *list, int *nlist, int *sh) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int carry = 0;
+    for (int base = 0; base < n; base += 256 * 8) {
+        int v[8], sm = 0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int idx = base + threadIdx.x * 8 + i;
+            v[i] = idx < n ? in[idx] : 0;
+            sm += v[i];
+            if (list && v[i] > SEG_WARP_MAX) list[atomicAdd(nlist, 1)] = idx;
+        }
+        const int x = warp_incl_scan(sm);
+        if (lane == 31) sh[w] = x;
+        __syncthreads();
+        int wb = 0, tot = 0;
+        for (int i = 0; i < 8; ++i) {
+            const int q = sh[i];
+            if (i < w) wb += q;
+            tot += q;
+        }
+        __syncthreads();
+        int ex = carry + wb + x - sm;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int idx = base + threadIdx.x * 8 + i;
+            if (idx < n) out[idx] = ex;
+            ex += v[i];
+        }
+        carry += tot;
+    }
+    if (threadIdx.x == 0) out[n] = carry;
+}
+
+// shared memory of the persistent rebuild: the union of its phases
+template <typename K>
+union CoopSmem {
+    struct {
+        K keys[SEG_WARPS][SEG_WARP_MAX];
+        int hp[SEG_WARPS][SEG_WARP_MAX];
+    } warp;
+    struct {
+        K keys[2][SegCta<K>::CAP];
+        unsigned cntp[8 * 256];
+        unsigned wsum[8 * 8];
+        int sh[8];
+    } cta;
+    XlSmem xl;
+    int scan[8];
+};
+
+template <typename K>
+__global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
+    extern __shared__ __align__(16) unsigned char coop_raw[];
+    CoopSmem<K> &S = *reinterpret_cast<CoopSmem<K> *>(coop_raw);
+    const int B = a.B, V = a.V;
+    const int gtid = blockIdx.x * blockDim.x + threadIdx.x, gthreads = gridDim.x * blockDim.x;
+    const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+    const int gwarp = gtid >> 5, gwarps = gthreads >> 5;
+    // P0
+    for (int x = gtid; x <= B; x += gthreads) {
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            a.sd[q].len[x] = 0;
+            a.sd[q].cur[x] = 0;
+            if (x < B) a.sd[q].deg[x] = 0;
+        }
+    }
+    if (gtid < 2) a.nlong[gtid] = 0;
+    grid_sync(a.bar);
+    // P1
+    for (int v = gtid; v < V; v += gthreads) {
+        const int x = __ldg(a.b + v);
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            const int d = __ldg(a.sd[q].gptr + v + 1) - __ldg(a.sd[q].gptr + v);
+            if (d) atomicAdd(a.sd[q].len + x, d);
+        }
+        const int ko = __ldg(a.kout + v), ki = __ldg(a.kin + v);
+        if (ko) atomicAdd(a.sd[0].deg + x, ko);
+        if (ki) atomicAdd(a.sd[1].deg + x, ki);
+    }
+    grid_sync(a.bar);
+    // P2
+    if (blockIdx.x < 2) {
+        CoopSide &sd = a.sd[blockIdx.x];
+        cta_scan_lines(sd.len, sd.off, B, sd.listC, a.nlong + blockIdx.x, S.scan);
+    } else {
+        for (int x = gtid - 2 * (int)blockDim.x; x < B; x += gthreads - 2 * (int)blockDim.x)
+            a.rcp[x] = 1.0 / ((double)a.sd[0].deg[x] + (double)a.sd[1].deg[x] + (double)B);
+    }
+    grid_sync(a.bar);
+    // P3: scatter (warp per (side, vertex))
+    for (int task = gwarp; task < 2 * V; task += gwarps) {
+        const int q = task >= V, v = q ? task - V : task;
+        const CoopSide &sd = a.sd[q];
+        K *seg = reinterpret_cast<K *>(sd.seg);
+        const int lo = __ldg(sd.gptr + v), n = __ldg(sd.gptr + v + 1) - lo;
+        if (n == 0) continue;
+        const int x = __ldg(a.b + v);
+        int base = 0;
+        if (lane == 0) base = sd.off[x] + atomicAdd(sd.cur + x, n);
+        base = __shfl_sync(FULL, base, 0);
+        for (int j = lane; j < n; j += 32) {
+            const int t = __ldg(a.b + __ldg(sd.gidx + lo + j));
+            if (sizeof(K) == 8)
+                seg[base + j] = (K)(((unsigned long long)(unsigned)t << 32) | (unsigned)__ldg(sd.gw + lo + j));
+            else
+                seg[base + j] = (K)(unsigned)t;
+        }
+    }
+    grid_sync(a.bar);
+    // P4a: short lines, one warp each (bitonic in shared memory + RLE)
+    for (int task = gwarp; task < 2 * B; task += gwarps) {
+        const int q = task >= B, x = q ? task - B : task;
+        const CoopSide &sd = a.sd[q];
+        const int o = sd.off[x], L = sd.off[x + 1] - o;
+        if (L > SEG_WARP_MAX) continue;
+        if (L == 0) {
+            if (lane == 0) sd.nnz[x] = 0;
+            continue;
+        }
+        const K *seg = reinterpret_cast<const K *>(sd.seg);
+        int n = 1;
+        while (n < L) n <<= 1;
+        for (int i = lane; i < n; i += 32) S.warp.keys[wl][i] = i < L ? seg[o + i] : key_max<K>();
+        __syncwarp();
+        bitonic<K, 32>(S.warp.keys[wl], n, lane);
+        const int u = rle_runs<K, 32>(S.warp.keys[wl], L, S.warp.hp[wl], sd.tcol + o, sd.tcnt + o, lane, nullptr);
+        if (lane == 0) sd.nnz[x] = u;
+    }
+    __syncthreads();   // the shared memory changes role
+    // P4b: long lines, one CTA each
+    {
+        const int n0 = a.nlong[0], n1 = a.nlong[1];
+        for (int li = blockIdx.x; li < n0 + n1; li += gridDim.x) {
+            const int q = li >= n0;
+            const CoopSide &sd = a.sd[q];
+            const int x = sd.listC[q ? li - n0 : li];
+            const int o = sd.off[x], L = sd.off[x + 1] - o;
+            K *seg = reinterpret_cast<K *>(sd.seg);
+            int u;
+            if (L <= SegCta<K>::CAP) {
+                for (int i = threadIdx.x; i < L; i += 256) S.cta.keys[0][i] = seg[o + i];
+                __syncthreads();
+                K *keys = cta_radix_sort<K, 256>(S.cta.keys[0], S.cta.keys[1], L, a.col_bits, S.cta.cntp, S.cta.wsum);
+                int *hp = reinterpret_cast<int *>(keys == S.cta.keys[0] ? S.cta.keys[1] : S.cta.keys[0]);
+                u = rle_runs<K, 256>(keys, L, hp, sd.tcol + o, sd.tcnt + o, threadIdx.x, S.cta.sh);
+            } else {
+                u = xl_sort_line<K>(seg, o, L, a.col_bits, sd.tcol, sd.tcnt, reinterpret_cast<K *>(sd.xl_keys),
+                                    sd.xl_hp, S.xl);
+            }
+            if (threadIdx.x == 0) sd.nnz[x] = u;
+            __syncthreads();
+        }
+    }
+    grid_sync(a.bar);
+    // P5
+    if (blockIdx.x < 2) {
+        CoopSide &sd = a.sd[blockIdx.x];
+        cta_scan_lines(sd.nnz, sd.ptr, B, nullptr, nullptr, S.scan);
+        if (blockIdx.x == 0 && threadIdx.x == 0) *a.d_nnz = sd.ptr[B];
+    }
+    grid_sync(a.bar);
+    // P6: compact the runs (warp per (side, line))
+    for (int task = gwarp; task < 2 * B; task += gwarps) {
+        const int q = task >= B, x = q ? task - B : task;
+        const CoopSide &sd = a.sd[q];
+        const int o = sd.off[x], n = sd.nnz[x], p = sd.ptr[x];
+        int run = 0;
+        for (int k0 = 0; k0 < n; k0 += 32) {
+            const int k = k0 + lane;
+            const int c = k < n ? sd.tcnt[o + k] : 0;
+            const int sc = warp_incl_scan(c) + run;
+            if (k < n) {
+                sd.idx[p + k] = sd.tcol[o + k];
+                sd.cnt[p + k] = c;
+                sd.cum[p + k] = sc;
+            }
+            run = __shfl_sync(FULL, sc, 31);
+        }
+    }
+}
+
+}  // namespace gsap

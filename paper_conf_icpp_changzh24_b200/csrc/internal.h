@@ -78,6 +78,13 @@ struct Ctx {
     int *seg_len = nullptr, *seg_off = nullptr, *seg_cur = nullptr, *seg_nnz = nullptr, *seg_listW = nullptr,
         *seg_listC = nullptr, *seg_ctr = nullptr, *xl_hp = nullptr;
     unsigned long long *xl_keys = nullptr;   // 2E: long-segment sort scratch
+    // persistent sparse rebuild (coop.cuh; small graphs): the column side's
+    // line scratch, its long-segment scratch, the grid barrier
+    bool coop_ok = false;
+    int *seg2_len = nullptr, *seg2_off = nullptr, *seg2_cur = nullptr, *seg2_nnz = nullptr, *seg2_listC = nullptr;
+    unsigned long long *xl2_keys = nullptr;
+    int *xl2_hp = nullptr;
+    unsigned *coop_bar = nullptr;
 
     // per-phase buffers
     int *s = nullptr;            // proposals: V (MOVE) or B * P (MERGE)

@@ -16,6 +16,7 @@
 #include "internal.h"
 #include "prims.cuh"
 #include "segsort.cuh"
+#include "coop.cuh"
 
 namespace gsap {
 
@@ -478,8 +479,61 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     GSAP_CHECK_LAUNCH();
 }
 
+// the persistent single-kernel sparse rebuild (coop.cuh)
+template <typename K>
+static void rebuild_sparse_coop(Ctx &c) {
+    const int B = c.B;
+    CoopArgs a;
+    a.V = c.V;
+    a.B = B;
+    a.col_bits = bits_for(B);
+    a.b = c.b;
+    a.kout = c.kout;
+    a.kin = c.kin;
+    CoopSide &r = a.sd[0], &q = a.sd[1];
+    r.gptr = c.rowptr; r.gidx = c.col; r.gw = c.wgt;
+    r.len = c.seg_len; r.off = c.seg_off; r.cur = c.seg_cur; r.nnz = c.seg_nnz; r.listC = c.seg_listC;
+    r.seg = c.keys0; r.tcol = c.wa; r.tcnt = c.wb; r.xl_keys = c.xl_keys; r.xl_hp = c.xl_hp;
+    r.ptr = c.bm_rowptr; r.idx = c.bm_col; r.cnt = c.bm_cnt; r.cum = c.bm_cum; r.deg = c.dout;
+    q.gptr = c.cscptr; q.gidx = c.cscsrc; q.gw = c.cscwgt;
+    q.len = c.seg2_len; q.off = c.seg2_off; q.cur = c.seg2_cur; q.nnz = c.seg2_nnz; q.listC = c.seg2_listC;
+    q.seg = c.keys1; q.tcol = c.flags; q.tcnt = c.pos; q.xl_keys = c.xl2_keys; q.xl_hp = c.xl2_hp;
+    q.ptr = c.bm_colptr; q.idx = c.bm_row; q.cnt = c.bm_ccnt; q.cum = c.bm_ccum; q.deg = c.din;
+    a.rcp = c.rcp;
+    a.d_nnz = c.d_nnz;
+    a.nlong = c.seg_ctr;
+    a.bar = c.coop_bar;
+    const size_t smem = sizeof(CoopSmem<K>);
+    static int grid = 0;
+    if (grid == 0) {
+        GSAP_CUDA(cudaFuncSetAttribute(k_rebuild_coop<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        int per_sm = 0, sms = 0, dev = 0;
+        GSAP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rebuild_coop<K>, 256, smem));
+        GSAP_CUDA(cudaGetDevice(&dev));
+        GSAP_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        grid = std::max(3, per_sm * sms);
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(256);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = c.stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    GSAP_CUDA(cudaLaunchKernelEx(&cfg, k_rebuild_coop<K>, a));
+    ++c.launches;
+}
+
 static void rebuild_sparse(Ctx &c) {
     const int B = c.B, E = c.E;
+    if (E > 0 && c.coop_ok) {
+        if (c.weighted) rebuild_sparse_coop<u64>(c);
+        else rebuild_sparse_coop<unsigned>(c);
+        return;
+    }
     if (E == 0) {
         GSAP_CUDA(cudaMemsetAsync(c.bm_rowptr, 0, sizeof(int) * ((size_t)B + 1), c.stream));
         GSAP_CUDA(cudaMemsetAsync(c.bm_colptr, 0, sizeof(int) * ((size_t)B + 1), c.stream));
@@ -510,8 +564,10 @@ void rebuild(Ctx &c) {
         rebuild_dense(c);   // rcp written by the compaction
     } else {
         rebuild_sparse(c);
-        k_rcp<<<grid_for(c.B, 256), 256, 0, c.stream>>>(c.B, c.dout, c.din, c.rcp);
-        ++c.launches;
+        if (!(c.coop_ok && c.E > 0)) {
+            k_rcp<<<grid_for(c.B, 256), 256, 0, c.stream>>>(c.B, c.dout, c.din, c.rcp);
+            ++c.launches;
+        }
     }
     // algorithmic bytes: the compulsory inputs (dst ids,
     // row pointers, b) and the fixed-size outputs (row / column pointers,

@@ -422,6 +422,83 @@ __global__ void __launch_bounds__(256) k_segsort_cta(const int *__restrict__ off
     }
 }
 
+// shared memory of one xl line sort
+struct XlSmem {
+    int hist[256];
+    int base[256];
+    int wcnt[8][256];
+    int sh[8];
+};
+
+// LSD radix sort (8-bit digits over col_bits) + RLE of one very long segment
+// seg[o, o + L) by a 256-thread CTA, ping-ponging with gkeys[2 o, ...);
+// returns the run count (runs in tcol / tcnt at o)
+template <typename K>
+GSAP_DEV int xl_sort_line(K *__restrict__ seg, int o, int L, int col_bits, int *__restrict__ tcol,
+                          int *__restrict__ tcnt, K *__restrict__ gkeys, int *__restrict__ ghp, XlSmem &S) {
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+    const int shift0 = sizeof(K) == 8 ? 32 : 0;
+    K *src = seg + o;
+    K *dst = gkeys + 2 * (size_t)o;
+    for (int sbit = 0; sbit < col_bits; sbit += 8) {
+        const int shift = shift0 + sbit;
+        S.hist[tid] = 0;
+        __syncthreads();
+        for (int i = tid; i < L; i += 256) atomicAdd(&S.hist[(int)((src[i] >> shift) & 255)], 1);
+        __syncthreads();
+        {
+            const int h = S.hist[tid];
+            int x2 = h;
+#pragma unroll
+            for (int q = 1; q < 32; q <<= 1) {
+                const int t = __shfl_up_sync(FULL, x2, q);
+                if (lane >= q) x2 += t;
+            }
+            if (lane == 31) S.sh[w] = x2;
+            __syncthreads();
+            int wb = 0;
+            for (int q = 0; q < 8; ++q)
+                if (q < w) wb += S.sh[q];
+            S.base[tid] = wb + x2 - h;
+            __syncthreads();
+        }
+        for (int t0 = 0; t0 < L; t0 += 256) {
+            const int i = t0 + tid;
+            const bool valid = i < L;
+            const K k = valid ? src[i] : (K)0;
+            const int d = valid ? (int)((k >> shift) & 255) : 256;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) S.wcnt[q][tid] = 0;
+            __syncthreads();
+            const unsigned peers = __match_any_sync(FULL, d);
+            const int rank = __popc(peers & lt);
+            if (valid && lane == __ffs(peers) - 1) S.wcnt[w][d] = __popc(peers);
+            __syncthreads();
+            // per digit (thread tid = digit): prefix over warps, then advance the base
+            {
+                int run = 0;
+                for (int q = 0; q < 8; ++q) {
+                    const int c = S.wcnt[q][tid];
+                    S.wcnt[q][tid] = run;
+                    run += c;
+                }
+                S.hist[tid] = run;   // this tile's count of digit tid
+            }
+            __syncthreads();
+            if (valid) dst[S.base[d] + S.wcnt[w][d] + rank] = k;
+            __syncthreads();
+            S.base[tid] += S.hist[tid];
+            __syncthreads();
+        }
+        K *t = src;
+        src = dst;
+        dst = t;
+        __syncthreads();
+    }
+    return rle_runs<K, 256>(src, L, ghp + 2 * (size_t)o, tcol + o, tcnt + o, tid, S.sh);
+}
+
 // 4d. very long segments (> SegCta::CAP): one CTA each, LSD radix sort of the
 // segment over the key's block bits in global memory (8-bit digits; a tile of
 // 256 keys ranked stably with __match_any_sync per warp + per-warp digit
@@ -431,81 +508,14 @@ __global__ void __launch_bounds__(256) k_segsort_xl(const int *__restrict__ off,
                                                     const int *__restrict__ listC, const int *__restrict__ counters,
                                                     int col_bits, int *__restrict__ tcol, int *__restrict__ tcnt,
                                                     int *__restrict__ nnz, K *__restrict__ gkeys, int *__restrict__ ghp) {
-    __shared__ int hist[256];
-    __shared__ int base[256];
-    __shared__ int wcnt[8][256];
-    __shared__ int sh[8];
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    const unsigned lt = (1u << lane) - 1u;
+    __shared__ XlSmem S;
     const int n_lines = counters[1];
-    const int shift0 = sizeof(K) == 8 ? 32 : 0;
     for (int li = blockIdx.x; li < n_lines; li += gridDim.x) {
         const int x = listC[li];
         const int o = off[x], L = off[x + 1] - o;
         if (L <= SegCta<K>::CAP) continue;   // handled by k_segsort_cta
-        K *src = seg + o;
-        K *dst = gkeys + 2 * (size_t)o;
-        for (int sbit = 0; sbit < col_bits; sbit += 8) {
-            const int shift = shift0 + sbit;
-            hist[tid] = 0;
-            __syncthreads();
-            for (int i = tid; i < L; i += 256) atomicAdd(&hist[(int)((src[i] >> shift) & 255)], 1);
-            __syncthreads();
-            {
-                int tot;
-                const int h = hist[tid];
-                int x2 = h;
-#pragma unroll
-                for (int q = 1; q < 32; q <<= 1) {
-                    const int t = __shfl_up_sync(FULL, x2, q);
-                    if (lane >= q) x2 += t;
-                }
-                if (lane == 31) sh[w] = x2;
-                __syncthreads();
-                int wb = 0;
-                tot = 0;
-                for (int q = 0; q < 8; ++q) {
-                    if (q < w) wb += sh[q];
-                    tot += sh[q];
-                }
-                base[tid] = wb + x2 - h;
-                __syncthreads();
-            }
-            for (int t0 = 0; t0 < L; t0 += 256) {
-                const int i = t0 + tid;
-                const bool valid = i < L;
-                const K k = valid ? src[i] : (K)0;
-                const int d = valid ? (int)((k >> shift) & 255) : 256;
-#pragma unroll
-                for (int q = 0; q < 8; ++q) wcnt[q][tid] = 0;
-                __syncthreads();
-                const unsigned peers = __match_any_sync(FULL, d);
-                const int rank = __popc(peers & lt);
-                if (valid && lane == __ffs(peers) - 1) wcnt[w][d] = __popc(peers);
-                __syncthreads();
-                // per digit (thread tid = digit): prefix over warps, then advance the base
-                {
-                    int run = 0;
-                    for (int q = 0; q < 8; ++q) {
-                        const int c = wcnt[q][tid];
-                        wcnt[q][tid] = run;
-                        run += c;
-                    }
-                    hist[tid] = run;   // this tile's count of digit tid
-                }
-                __syncthreads();
-                if (valid) dst[base[d] + wcnt[w][d] + rank] = k;
-                __syncthreads();
-                base[tid] += hist[tid];
-                __syncthreads();
-            }
-            K *t = src;
-            src = dst;
-            dst = t;
-            __syncthreads();
-        }
-        const int u = rle_runs<K, 256>(src, L, ghp + 2 * (size_t)o, tcol + o, tcnt + o, tid, sh);
-        if (tid == 0) nnz[x] = u;
+        const int u = xl_sort_line<K>(seg, o, L, col_bits, tcol, tcnt, gkeys, ghp, S);
+        if (threadIdx.x == 0) nnz[x] = u;
         __syncthreads();
     }
 }

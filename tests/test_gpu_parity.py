@@ -26,6 +26,9 @@ def G():
 
 
 SPARSE = {"dense_max_B": 1}     # force the sparse (CSR-line) blockmodel regime
+# the sparse regime through the multi-kernel rebuild instead of the persistent one
+SPARSE_MK = {"dense_max_B": 1, "sparse_coop": 0}
+REGIMES = {"auto": {}, "sparse": SPARSE, "sparse_mk": SPARSE_MK}
 
 
 def make_pair(G, oracle_mod, rowptr, col, wgt=None, **params):
@@ -54,23 +57,24 @@ GRAPHS = {
 }
 
 
-@pytest.mark.parametrize("regime", ["auto", "sparse"])
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk"])
 @pytest.mark.parametrize("gname", list(GRAPHS))
 @pytest.mark.parametrize("B", [1, 2, 7, 11, 150, 222, 299, 300])
 def test_rebuild_bit_exact(G, oracle_mod, gname, B, regime):
     rowptr, col, w = GRAPHS[gname]()
     V = len(rowptr) - 1
     B = min(B, V)
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **(SPARSE if regime == "sparse" else {}))
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **REGIMES[regime])
     assert_same_blockmodel(ctx, orc)      # singleton partition at create
     b = dcsbm.random_partition(V, B, B)
     set_both(ctx, orc, b, B)
     assert_same_blockmodel(ctx, orc)
 
 
-def test_rebuild_20k_all_regimes(G, oracle_mod):
+@pytest.mark.parametrize("coop", [1, 0])
+def test_rebuild_20k_all_regimes(G, oracle_mod, coop):
     rowptr, col, truth, cfg = dcsbm.make("20k")
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, sparse_coop=coop)
     skew = dcsbm.random_partition(cfg.V, 20000, 7)
     skew[: cfg.V // 2] = 0                        # one giant block: lines of > 2^17 entries
     skew = np.unique(skew, return_inverse=True)[1].astype(np.int32)
@@ -95,7 +99,7 @@ def _states(V, rng_seed):
 def test_move_proposals_dS_accept(G, oracle_mod, gname, regime):
     rowptr, col, w = GRAPHS[gname]()
     V = len(rowptr) - 1
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **(SPARSE if regime == "sparse" else {}))
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **REGIMES[regime])
     nties = 0
     for B, b in _states(V, 5):
         set_both(ctx, orc, b, B)
@@ -118,7 +122,7 @@ def test_move_proposals_dS_accept(G, oracle_mod, gname, regime):
 def test_merge_proposals_dS_best(G, oracle_mod, gname, regime):
     rowptr, col, w = GRAPHS[gname]()
     V = len(rowptr) - 1
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **(SPARSE if regime == "sparse" else {}))
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **REGIMES[regime])
     for B, b in _states(V, 9):
         if B < 2:
             continue
@@ -159,7 +163,7 @@ def test_select_merges_bit_exact(G, oracle_mod, seed):
 @pytest.mark.parametrize("regime", ["auto", "sparse"])
 def test_merge_phase_lockstep(G, oracle_mod, regime):
     rowptr, col, truth, cfg = dcsbm.make("1k")
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **(SPARSE if regime == "sparse" else {}))
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **REGIMES[regime])
     for outer in range(4):
         B = ctx.B
         K = int(0.4 * B)
@@ -180,12 +184,12 @@ def test_merge_phase_lockstep(G, oracle_mod, regime):
         assert_same_blockmodel(ctx, orc)
 
 
-@pytest.mark.parametrize("regime", ["auto", "sparse"])
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk"])
 @pytest.mark.parametrize("name", ["1k", "20k"])
 def test_mcmc_lockstep(G, oracle_mod, name, regime):
     """Batches of the fused hot loop vs the oracle, state compared after every batch."""
     rowptr, col, truth, cfg = dcsbm.make(name)
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **(SPARSE if regime == "sparse" else {}))
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **REGIMES[regime])
     # start from a merged state (as after the first merge phases)
     V = cfg.V
     B = max(2, int(V ** 0.5))
@@ -235,7 +239,7 @@ def test_big_vertices_and_global_tables(G, oracle_mod, regime):
     np.add.at(rowptr, src[order] + 1, 1)
     rowptr = np.cumsum(rowptr)
     col = dst[order].astype(np.int32)
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **(SPARSE if regime == "sparse" else {}))
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **REGIMES[regime])
     for B in (100, 3000, V):
         b = dcsbm.random_partition(V, B, B)
         set_both(ctx, orc, b, B)
@@ -276,7 +280,7 @@ def test_edge_cases(G, oracle_mod):
 def test_end_to_end_1k(G, oracle_mod, regime):
     from gen import metrics
     rowptr, col, truth, cfg = dcsbm.make("1k")
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **(SPARSE if regime == "sparse" else {}))
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **REGIMES[regime])
     res = ctx.gsap_run()
     ref = orc.partition_run()
     # layer 3 (north_star): final MDL within 1%, pairwise P/R within 0.02 of the oracle's
@@ -311,11 +315,12 @@ def test_cuda_graph_path_matches_stream_path(G, oracle_mod):
     assert np.array_equal(a["trace"][:, :4], b["trace"][:, :4])
 
 
-def test_rebuild_weighted_long_lines(G, oracle_mod):
+@pytest.mark.parametrize("regime", ["sparse", "sparse_mk"])
+def test_rebuild_weighted_long_lines(G, oracle_mod, regime):
     """Weighted graph, sparse regime, with lines in every segment class (warp, CTA, global)."""
     rowptr, col, truth, cfg = dcsbm.make("20k")
     w = np.random.default_rng(3).integers(1, 6, len(col)).astype(np.int32)
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **SPARSE)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **REGIMES[regime])
     b = dcsbm.random_partition(cfg.V, 8000, 11)
     b[: cfg.V // 3] = 0
     b = np.unique(b, return_inverse=True)[1].astype(np.int32)
