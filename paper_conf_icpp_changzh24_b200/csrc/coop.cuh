@@ -190,6 +190,14 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             continue;
         }
         const K *seg = reinterpret_cast<const K *>(sd.seg);
+        if (L <= 128) {   // short lines: bitonic in registers, RLE in registers
+            int u;
+            if (L <= 32) u = warp_segsort_rle<K, 1>(seg + o, L, sd.tcol + o, sd.tcnt + o);
+            else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, sd.tcol + o, sd.tcnt + o);
+            else u = warp_segsort_rle<K, 4>(seg + o, L, sd.tcol + o, sd.tcnt + o);
+            if (lane == 0) sd.nnz[x] = u;
+            continue;
+        }
         int n = 1;
         while (n < L) n <<= 1;
         for (int i = lane; i < n; i += 32) S.warp.keys[wl][i] = i < L ? seg[o + i] : key_max<K>();
