@@ -890,13 +890,62 @@ __global__ void __launch_bounds__(256) k_sum_partials(const double *__restrict__
     }
 }
 
+// k_apply + the ordered sum of its partials in one launch: the last CTA to
+// finish (arrival counter, reset by that CTA) adds partials[0, nb) in index
+// order to *dsum -- the same fixed-order sum as k_sum_partials
+__global__ void __launch_bounds__(256) k_apply_sum(int first, int count, const int *__restrict__ s,
+                                                   const unsigned char *__restrict__ acc,
+                                                   const double *__restrict__ dS, int *__restrict__ b,
+                                                   double *__restrict__ partials, int *__restrict__ nacc,
+                                                   unsigned *__restrict__ arrivals, double *__restrict__ dsum) {
+    __shared__ double sh[8];
+    __shared__ bool last;
+    const int base = blockIdx.x * APPLY_CHUNK;
+    double sum = 0.0;
+    int na = 0;
+    for (int k = threadIdx.x; k < APPLY_CHUNK; k += 256) {
+        const int i = base + k;
+        if (i < count && acc[i]) {
+            b[first + i] = s[i];
+            sum += dS ? dS[i] : 0.0;
+            ++na;
+        }
+    }
+    na = warp_sum(na);
+    if (nacc && (threadIdx.x & 31) == 0 && na) atomicAdd(nacc, na);
+    sum = warp_sum(sum);
+    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = sum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < 8; ++w) t += sh[w];
+        partials[blockIdx.x] = t;
+        __threadfence();
+        last = atomicAdd(arrivals, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    double v = 0.0;
+    for (int i = threadIdx.x; i < (int)gridDim.x; i += 256) v += *((volatile double *)(partials + i));
+    v = warp_sum(v);
+    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = v;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < 8; ++w) t += sh[w];
+        *dsum += t;
+        *arrivals = 0u;
+    }
+}
+
 void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
                   double *dsum, int *nacc) {
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
-    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, c.b, c.partials, nacc);
-    k_sum_partials<<<1, 256, 0, c.stream>>>(c.partials, nb, dsum, 1);
-    c.launches += 2;
+    k_apply_sum<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, c.b, c.partials, nacc,
+                                          reinterpret_cast<unsigned *>(c.scal_i + 4), dsum);
+    c.launches += 1;
     GSAP_CHECK_LAUNCH();
 }
 

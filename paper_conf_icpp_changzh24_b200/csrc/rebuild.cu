@@ -181,50 +181,11 @@ __global__ void k_transpose(const int *__restrict__ M, int B, int *__restrict__ 
     }
 }
 
-// per row of a dense B x B matrix: number of non-zeros and the row sum
-__global__ void k_row_stats(const int *__restrict__ M, int B, int *__restrict__ nnz, int *__restrict__ sum) {
-    const int lane = threadIdx.x & 31;
-    for (int x = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < B; x += (gridDim.x * blockDim.x) >> 5) {
-        int c = 0, s = 0;
-        for (int y = lane; y < B; y += 32) {
-            const int v = M[(size_t)x * B + y];
-            c += v != 0;
-            s += v;
-        }
-        c = warp_sum(c);
-        s = warp_sum(s);
-        if (lane == 0) {
-            nnz[x] = c;
-            sum[x] = s;
-        }
-    }
-}
 
-// compact the non-zeros of each row into (idx, cnt, cum) at ptr[row]
-__global__ void k_row_compact(const int *__restrict__ M, int B, const int *__restrict__ ptr,
-                              int *__restrict__ idx, int *__restrict__ cnt, int *__restrict__ cum) {
-    const int lane = threadIdx.x & 31;
-    const unsigned lt = (1u << lane) - 1u;
-    for (int x = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < B; x += (gridDim.x * blockDim.x) >> 5) {
-        int base = ptr[x], run = 0;
-        for (int y0 = 0; y0 < B; y0 += 32) {
-            const int y = y0 + lane;
-            const int v = y < B ? M[(size_t)x * B + y] : 0;
-            const unsigned bal = __ballot_sync(FULL, v != 0);
-            const int sc = warp_incl_scan(v) + run;
-            if (v != 0) {
-                const int p = base + __popc(bal & lt);
-                idx[p] = y;
-                cnt[p] = v;
-                cum[p] = sc;
-            }
-            base += __popc(bal);
-            run = __shfl_sync(FULL, sc, 31);
-        }
-    }
-}
 
-// both dense matrices (M: lines x < B, its transpose: lines x >= B) in one launch
+// both dense matrices (M: lines x < B, its transpose: lines x >= B) in one
+// launch: non-zeros and sum per line; four consecutive entries per lane per
+// step (128 per warp step, independent loads)
 __global__ void k_row_stats2(const int *__restrict__ M, const int *__restrict__ Mt, int B, int *__restrict__ nnzA,
                              int *__restrict__ sumA, int *__restrict__ nnzB, int *__restrict__ sumB) {
     const int lane = threadIdx.x & 31;
@@ -233,13 +194,16 @@ __global__ void k_row_stats2(const int *__restrict__ M, const int *__restrict__ 
         const int x = t ? x2 - B : x2;
         const int *__restrict__ R = (t ? Mt : M) + (size_t)x * B;
         int c = 0, s = 0;
-        for (int y = lane; y < B; y += 32) {
-            const int v = R[y];
-            c += v != 0;
-            s += v;
+        for (int y0 = 4 * lane; y0 < B; y0 += 128) {
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const int v = y0 + k < B ? __ldg(R + y0 + k) : 0;
+                c += v != 0;
+                s += v;
+            }
         }
-        c = warp_sum(c);
-        s = warp_sum(s);
+        c = __reduce_add_sync(FULL, c);
+        s = __reduce_add_sync(FULL, s);
         if (lane == 0) {
             (t ? nnzB : nnzA)[x] = c;
             (t ? sumB : sumA)[x] = s;
@@ -289,14 +253,15 @@ __global__ void __launch_bounds__(1024) k_scan2(const int *a0, int *o0, const in
     if (threadIdx.x == 0) out[n] = carry;
 }
 
-// compaction of both matrices + nnz + rcp = 1 / (d_x + B)
+// compaction of both matrices + nnz + rcp = 1 / (d_x + B): a warp step
+// covers 128 consecutive entries, four per lane (one warp scan of the lane's
+// count and one of its sum per step instead of one per 32 entries)
 __global__ void k_row_compact2(const int *__restrict__ M, const int *__restrict__ Mt, int B,
                                const int *__restrict__ ptrA, int *__restrict__ idxA, int *__restrict__ cntA,
                                int *__restrict__ cumA, const int *__restrict__ ptrB, int *__restrict__ idxB,
                                int *__restrict__ cntB, int *__restrict__ cumB, const int *__restrict__ dout,
                                const int *__restrict__ din, double *__restrict__ rcp, int *__restrict__ d_nnz) {
     const int lane = threadIdx.x & 31;
-    const unsigned lt = (1u << lane) - 1u;
     if (blockIdx.x == 0 && threadIdx.x == 0) *d_nnz = ptrA[B];
     for (int x2 = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x2 < 2 * B; x2 += (gridDim.x * blockDim.x) >> 5) {
         const bool t = x2 >= B;
@@ -307,19 +272,29 @@ __global__ void k_row_compact2(const int *__restrict__ M, const int *__restrict_
         int *__restrict__ cum = t ? cumB : cumA;
         int base = (t ? ptrB : ptrA)[x], run = 0;
         if (!t && lane == 0) rcp[x] = 1.0 / ((double)dout[x] + (double)din[x] + (double)B);
-        for (int y0 = 0; y0 < B; y0 += 32) {
-            const int y = y0 + lane;
-            const int v = y < B ? R[y] : 0;
-            const unsigned bal = __ballot_sync(FULL, v != 0);
-            const int sc = warp_incl_scan(v) + run;
-            if (v != 0) {
-                const int p = base + __popc(bal & lt);
-                idx[p] = y;
-                cnt[p] = v;
-                cum[p] = sc;
+        for (int y0 = 0; y0 < B; y0 += 128) {
+            const int y = y0 + 4 * lane;
+            int v[4], nz = 0, sm = 0;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                v[k] = y + k < B ? __ldg(R + y + k) : 0;
+                nz += v[k] != 0;
+                sm += v[k];
             }
-            base += __popc(bal);
-            run = __shfl_sync(FULL, sc, 31);
+            const int nzi = warp_incl_scan(nz), smi = warp_incl_scan(sm);
+            int p = base + nzi - nz, sc = run + smi - sm;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                sc += v[k];
+                if (v[k] != 0) {
+                    idx[p] = y + k;
+                    cnt[p] = v[k];
+                    cum[p] = sc;
+                    ++p;
+                }
+            }
+            base += __shfl_sync(FULL, nzi, 31);
+            run += __shfl_sync(FULL, smi, 31);
         }
     }
 }
@@ -360,85 +335,6 @@ static void rebuild_dense(Ctx &c) {
 }
 
 // ---------------------------------------------------------------- sparse --
-__global__ void k_keys(int E, const int *__restrict__ esrc, const int *__restrict__ col,
-                       const int *__restrict__ wgt, const int *__restrict__ b, int sh,
-                       u64 *__restrict__ keys, int *__restrict__ w) {
-    for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < E; e += (long long)gridDim.x * blockDim.x) {
-        keys[e] = ((u64)(unsigned)__ldg(b + __ldg(esrc + e)) << sh) | (u64)(unsigned)__ldg(b + __ldg(col + e));
-        if (wgt) w[e] = wgt[e];
-    }
-}
-
-__global__ void k_heads(int n, const u64 *__restrict__ keys, int *__restrict__ flags) {
-    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
-        flags[i] = (i == 0 || keys[i] != keys[i - 1]) ? 1 : 0;
-}
-
-__global__ void k_unique(int n, const u64 *__restrict__ keys, const int *__restrict__ flags,
-                         const int *__restrict__ pos, int sh, int *__restrict__ rowid, int *__restrict__ colv,
-                         int *__restrict__ headidx) {
-    const u64 mask = (1ULL << sh) - 1ULL;
-    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
-        if (flags[i]) {
-            const int u = pos[i];
-            const u64 k = keys[i];
-            rowid[u] = (int)(k >> sh);
-            colv[u] = (int)(k & mask);
-            headidx[u] = (int)i;
-        }
-    }
-}
-
-__global__ void k_cnt_runs(int n, const int *__restrict__ headidx, const int *__restrict__ d_nnz, int *__restrict__ cnt) {
-    const int nnz = *d_nnz;
-    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < nnz; u += gridDim.x * blockDim.x)
-        cnt[u] = (u + 1 < nnz ? headidx[u + 1] : n) - headidx[u];
-}
-
-__global__ void k_cnt_weighted(int n, const int *__restrict__ flags, const int *__restrict__ pos,
-                               const int *__restrict__ w, int *__restrict__ cnt) {
-    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
-        atomicAdd(cnt + pos[i] + flags[i] - 1, w[i]);
-}
-
-// cum[u] = P[u] - P[start of u's segment - 1]; P = inclusive scan of cnt
-__global__ void k_seg_cum(const int *__restrict__ ids, const int *__restrict__ ptr, const int *__restrict__ P,
-                          const int *__restrict__ d_n, int *__restrict__ cum) {
-    const int n = *d_n;
-    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < n; u += gridDim.x * blockDim.x) {
-        const int s = ptr[ids[u]];
-        cum[u] = P[u] - (s > 0 ? P[s - 1] : 0);
-    }
-}
-
-__global__ void k_seg_deg(int B, const int *__restrict__ ptr, const int *__restrict__ P, int *__restrict__ deg) {
-    for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < B; x += gridDim.x * blockDim.x) {
-        const int lo = ptr[x], hi = ptr[x + 1];
-        deg[x] = hi > lo ? P[hi - 1] - (lo > 0 ? P[lo - 1] : 0) : 0;
-    }
-}
-
-__global__ void k_csc_keys(const int *__restrict__ d_n, const int *__restrict__ colv, const int *__restrict__ rowid,
-                           const int *__restrict__ cnt, unsigned *__restrict__ keys, u64 *__restrict__ vals) {
-    const int n = *d_n;
-    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < n; u += gridDim.x * blockDim.x) {
-        keys[u] = (unsigned)colv[u];
-        vals[u] = ((u64)(unsigned)rowid[u] << 32) | (u64)(unsigned)cnt[u];
-    }
-}
-
-__global__ void k_csc_unpack(const int *__restrict__ d_n, const unsigned *__restrict__ keys,
-                             const u64 *__restrict__ vals, int *__restrict__ colid, int *__restrict__ row,
-                             int *__restrict__ ccnt) {
-    const int n = *d_n;
-    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < n; u += gridDim.x * blockDim.x) {
-        colid[u] = (int)keys[u];
-        const u64 v = vals[u];
-        row[u] = (int)(v >> 32);
-        ccnt[u] = (int)(unsigned)(v & 0xffffffffULL);
-    }
-}
-
 __global__ void k_rcp(int B, const int *__restrict__ dout, const int *__restrict__ din, double *__restrict__ rcp) {
     for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < B; x += gridDim.x * blockDim.x)
         rcp[x] = 1.0 / ((double)dout[x] + (double)din[x] + (double)B);
