@@ -66,6 +66,9 @@ typedef struct {
     int32_t dense_max_B;      /* dense blockmodel iff B <= this; 0 = auto (B^2 <= max(4E, 2^24)) */
     int32_t sparse_coop;      /* 1 (default): sparse-regime rebuild as one persistent kernel when
                                  E <= GSAP_COOP_MAX_E; 0: the multi-kernel rebuild (same result) */
+    int32_t dense_coop;       /* 1 (default): dense-regime rebuild as one persistent kernel when
+                                 B <= 221 (B x B histogram in shared memory); 0: the multi-kernel
+                                 dense rebuild (same result) */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */

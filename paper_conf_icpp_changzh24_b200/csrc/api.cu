@@ -363,6 +363,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
             c.xl2_hp = A.take<int>(2 * Es);
         }
         c.coop_bar = A.take<unsigned>(2);
+        if (c.prm.dense_coop) c.small_acc = A.take<int>((size_t)SMALL_MAX_B * SMALL_MAX_B);
         const size_t tiles = (VE + 4095) / 4096 + 1;
         c.counts_cap = 256 * tiles;
         c.counts = A.take<int>(c.counts_cap);
@@ -425,6 +426,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         GSAP_CUDA(cudaMemcpyAsync(c.ft, ft.data(), sizeof(double2) * FT_N, cudaMemcpyHostToDevice, c.stream));
     }
     GSAP_CUDA(cudaMemsetAsync(c.coop_bar, 0, 2 * sizeof(unsigned), c.stream));
+    if (c.small_acc)
+        GSAP_CUDA(cudaMemsetAsync(c.small_acc, 0, sizeof(int) * SMALL_MAX_B * SMALL_MAX_B, c.stream));
     GSAP_CUDA(cudaMallocHost(&c.h_scal, 8 * sizeof(double)));
     GSAP_CUDA(cudaMallocHost(&c.h_int, 8 * sizeof(int)));
     // upload ---------------------------------------------------------------
@@ -792,6 +795,7 @@ void gsap_default_params(gsap_params *p) {
     p->cuda_graphs = 1;
     p->dense_max_B = 0;
     p->sparse_coop = 1;
+    p->dense_coop = 1;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }

@@ -85,6 +85,8 @@ struct Ctx {
     unsigned long long *xl2_keys = nullptr;
     int *xl2_hp = nullptr;
     unsigned *coop_bar = nullptr;
+    // persistent dense rebuild for B <= SMALL_MAX_B (params.dense_coop): B^2 accumulator, zero between calls
+    int *small_acc = nullptr;
 
     // per-phase buffers
     int *s = nullptr;            // proposals: V (MOVE) or B * P (MERGE)
@@ -159,6 +161,7 @@ void kc_resolve(Ctx &c, KClass &k);
 void build_graph_device(Ctx &c);                 // CSC, esrc, degrees (create time)
 void rebuild(Ctx &c);                            // Alg. 2 from c.b, c.B
 bool dense_ok(const Ctx &c, int B);
+constexpr int SMALL_MAX_B = 221;               // B^2 ints in one CTA's shared memory (195 KB)
 
 // move.cu
 enum MoveMode { MOVE_FUSED = 0, MOVE_PROPOSE = 1, MOVE_DELTA = 2 };

@@ -299,6 +299,201 @@ __global__ void k_row_compact2(const int *__restrict__ M, const int *__restrict_
     }
 }
 
+// ---------------------------------------------------- dense, small B --
+// The whole dense rebuild as ONE persistent cooperative kernel when B <= 221
+// (the B x B histogram fits one CTA's shared memory).  At such B the multi-
+// kernel path (memset, histogram, transpose, stats, scan, compaction) is six
+// launches of a few microseconds of work each; here they are three phases
+// separated by two grid barriers:
+//   P1 every CTA histograms a contiguous edge chunk (four edges per thread
+//      per step, 16-byte loads) in shared memory and adds its non-zeros into
+//      `acc` (zero on entry); din / column counts zeroed      | barrier
+//   P2 one warp per row x: M[x][.] = acc[x][.] (acc row re-zeroed for the
+//      next call), Mt[.][x], row non-zeros and dout; column non-zeros and din
+//      by integer atomics                                     | barrier
+//   P3 one warp per line (rows of M, then rows of Mt = columns of M): its
+//      offset = sum of the preceding lines' non-zeros, then the compaction of
+//      k_row_compact2 (idx, cnt, in-line prefix cum) and rcp = 1 / (d + B).
+// Integer arithmetic throughout: the same bits as rebuild_dense.
+constexpr int SMALL_THREADS = 512;
+
+struct SmallArgs {
+    int E, B;
+    const int *__restrict__ esrc;
+    const int *__restrict__ col;
+    const int *__restrict__ wgt;
+    const int *__restrict__ b;
+    int *acc, *M, *Mt, *rownnz, *colnnz, *dout, *din;
+    int *ptrA, *idxA, *cntA, *cumA, *ptrB, *idxB, *cntB, *cumB;
+    double *rcp;
+    int *d_nnz;
+    unsigned *bar;
+};
+
+__global__ void __launch_bounds__(SMALL_THREADS) k_rebuild_small(SmallArgs a) {
+    extern __shared__ int h[];
+    const int B = a.B, BB = B * B, E = a.E;
+    const int gtid = blockIdx.x * blockDim.x + threadIdx.x, gthreads = gridDim.x * blockDim.x;
+    const int lane = threadIdx.x & 31, gwarp = gtid >> 5, gwarps = gthreads >> 5;
+    // P1
+    for (int i = gtid; i < B; i += gthreads) {
+        a.din[i] = 0;
+        a.colnnz[i] = 0;
+    }
+    for (int i = threadIdx.x; i < BB; i += blockDim.x) h[i] = 0;
+    __syncthreads();
+    const long long chunk = ((((long long)E + gridDim.x - 1) / gridDim.x) + 3) & ~3LL;
+    const long long lo = (long long)blockIdx.x * chunk;
+    const long long hi = min((long long)E, lo + chunk);
+    for (long long base = lo; base < hi; base += 4LL * blockDim.x) {   // uniform trip count per CTA
+        const long long e0 = base + 4LL * threadIdx.x;
+        int src[4], dst[4], w[4] = {1, 1, 1, 1};
+        if (e0 + 3 < hi) {
+            const int4 s4 = __ldg(reinterpret_cast<const int4 *>(a.esrc + e0));
+            const int4 d4 = __ldg(reinterpret_cast<const int4 *>(a.col + e0));
+            src[0] = s4.x; src[1] = s4.y; src[2] = s4.z; src[3] = s4.w;
+            dst[0] = d4.x; dst[1] = d4.y; dst[2] = d4.z; dst[3] = d4.w;
+            if (a.wgt) {
+                const int4 w4 = __ldg(reinterpret_cast<const int4 *>(a.wgt + e0));
+                w[0] = w4.x; w[1] = w4.y; w[2] = w4.z; w[3] = w4.w;
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const bool ok = e0 + k < hi;
+                src[k] = ok ? __ldg(a.esrc + e0 + k) : -1;
+                dst[k] = ok ? __ldg(a.col + e0 + k) : -1;
+                if (a.wgt) w[k] = ok ? __ldg(a.wgt + e0 + k) : 0;
+            }
+        }
+        int key[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) key[k] = src[k] >= 0 ? __ldg(a.b + src[k]) * B + __ldg(a.b + dst[k]) : -1;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            if (a.wgt) {
+                if (key[k] >= 0) atomicAdd(h + key[k], w[k]);
+            } else {
+                const unsigned peers = __match_any_sync(FULL, key[k]);
+                if (key[k] >= 0 && lane == __ffs(peers) - 1) atomicAdd(h + key[k], __popc(peers));
+            }
+        }
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < BB; i += blockDim.x) {
+        const int v = h[i];
+        if (v) atomicAdd(a.acc + i, v);
+    }
+    grid_sync(a.bar);
+    // P2
+    for (int x = gwarp; x < B; x += gwarps) {
+        int c = 0, sm = 0;
+        for (int y = lane; y < B; y += 32) {
+            const int v = __ldcg(a.acc + (size_t)x * B + y);
+            a.acc[(size_t)x * B + y] = 0;
+            a.M[(size_t)x * B + y] = v;
+            a.Mt[(size_t)y * B + x] = v;
+            if (v) {
+                ++c;
+                sm += v;
+                atomicAdd(a.colnnz + y, 1);
+                atomicAdd(a.din + y, v);
+            }
+        }
+        c = __reduce_add_sync(FULL, c);
+        sm = __reduce_add_sync(FULL, sm);
+        if (lane == 0) {
+            a.rownnz[x] = c;
+            a.dout[x] = sm;
+        }
+    }
+    grid_sync(a.bar);
+    // P3
+    for (int x2 = gwarp; x2 < 2 * B; x2 += gwarps) {
+        const bool t = x2 >= B;
+        const int x = t ? x2 - B : x2;
+        const int *nz = t ? a.colnnz : a.rownnz;
+        int off = 0;
+        for (int y = lane; y < x; y += 32) off += __ldcg(nz + y);
+        off = __reduce_add_sync(FULL, off);
+        int *__restrict__ ptr = t ? a.ptrB : a.ptrA;
+        if (lane == 0) {
+            ptr[x] = off;
+            if (x == B - 1) {
+                const int tot = off + __ldcg(nz + x);
+                ptr[B] = tot;
+                if (!t) *a.d_nnz = tot;
+            }
+            if (!t) a.rcp[x] = 1.0 / ((double)__ldcg(a.dout + x) + (double)__ldcg(a.din + x) + (double)B);
+        }
+        const int *R = (t ? a.Mt : a.M) + (size_t)x * B;
+        int *__restrict__ idx = t ? a.idxB : a.idxA;
+        int *__restrict__ cnt = t ? a.cntB : a.cntA;
+        int *__restrict__ cum = t ? a.cumB : a.cumA;
+        int base = off, run = 0;
+        for (int y0 = 0; y0 < B; y0 += 128) {
+            const int y = y0 + 4 * lane;
+            int v[4], nzc = 0, s4 = 0;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                v[k] = y + k < B ? __ldcg(R + y + k) : 0;
+                nzc += v[k] != 0;
+                s4 += v[k];
+            }
+            const int nzi = warp_incl_scan(nzc), smi = warp_incl_scan(s4);
+            int p = base + nzi - nzc, sc = run + smi - s4;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                sc += v[k];
+                if (v[k] != 0) {
+                    idx[p] = y + k;
+                    cnt[p] = v[k];
+                    cum[p] = sc;
+                    ++p;
+                }
+            }
+            base += __shfl_sync(FULL, nzi, 31);
+            run += __shfl_sync(FULL, smi, 31);
+        }
+    }
+}
+
+static void rebuild_dense_small(Ctx &c) {
+    SmallArgs a;
+    a.E = c.E;
+    a.B = c.B;
+    a.esrc = c.esrc; a.col = c.col; a.wgt = c.wgt; a.b = c.b;
+    a.acc = c.small_acc; a.M = c.dense; a.Mt = c.denseT;
+    a.rownnz = c.rownnz; a.colnnz = c.tmpi; a.dout = c.dout; a.din = c.din;
+    a.ptrA = c.bm_rowptr; a.idxA = c.bm_col; a.cntA = c.bm_cnt; a.cumA = c.bm_cum;
+    a.ptrB = c.bm_colptr; a.idxB = c.bm_row; a.cntB = c.bm_ccnt; a.cumB = c.bm_ccum;
+    a.rcp = c.rcp;
+    a.d_nnz = c.d_nnz;
+    a.bar = c.coop_bar;
+    static int grid = 0;
+    if (grid == 0) {
+        const int smem_max = SMALL_MAX_B * SMALL_MAX_B * 4;
+        GSAP_CUDA(cudaFuncSetAttribute(k_rebuild_small, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max));
+        int per_sm = 0, sms = 0, dev = 0;
+        GSAP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rebuild_small, SMALL_THREADS, smem_max));
+        GSAP_CUDA(cudaGetDevice(&dev));
+        GSAP_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        grid = std::max(1, std::min(per_sm, 1) * sms);
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(SMALL_THREADS);
+    cfg.dynamicSmemBytes = sizeof(int) * (size_t)c.B * c.B;
+    cfg.stream = c.stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    GSAP_CUDA(cudaLaunchKernelEx(&cfg, k_rebuild_small, a));
+    ++c.launches;
+}
+
 static void rebuild_dense(Ctx &c) {
     const int B = c.B, E = c.E;
     const size_t BB = (size_t)B * B;
@@ -456,7 +651,9 @@ void rebuild(Ctx &c) {
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_rebuild, &ev);
     c.dense_mode = dense_ok(c, c.B);
-    if (c.dense_mode) {
+    if (c.dense_mode && c.small_acc && c.B <= SMALL_MAX_B) {
+        rebuild_dense_small(c);
+    } else if (c.dense_mode) {
         rebuild_dense(c);   // rcp written by the compaction
     } else {
         rebuild_sparse(c);

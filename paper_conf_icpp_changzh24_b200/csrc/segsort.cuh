@@ -287,6 +287,14 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__re
     for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
         const int x = listW[li];
         const int o = off[x], L = off[x + 1] - o;
+        if (L <= 128) {   // short lines: bitonic + RLE in registers (fewer instructions than shared memory)
+            int u;
+            if (L <= 32) u = warp_segsort_rle<K, 1>(seg + o, L, tcol + o, tcnt + o);
+            else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, tcol + o, tcnt + o);
+            else u = warp_segsort_rle<K, 4>(seg + o, L, tcol + o, tcnt + o);
+            if (lane == 0) nnz[x] = u;
+            continue;
+        }
         int n = 1;
         while (n < L) n <<= 1;
         for (int i = lane; i < n; i += 32) keys[w][i] = i < L ? seg[o + i] : key_max<K>();

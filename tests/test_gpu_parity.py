@@ -28,7 +28,9 @@ def G():
 SPARSE = {"dense_max_B": 1}     # force the sparse (CSR-line) blockmodel regime
 # the sparse regime through the multi-kernel rebuild instead of the persistent one
 SPARSE_MK = {"dense_max_B": 1, "sparse_coop": 0}
-REGIMES = {"auto": {}, "sparse": SPARSE, "sparse_mk": SPARSE_MK}
+# the dense regime (B <= 221) through the multi-kernel rebuild instead of the persistent one
+DENSE_MK = {"dense_coop": 0}
+REGIMES = {"auto": {}, "sparse": SPARSE, "sparse_mk": SPARSE_MK, "dense_mk": DENSE_MK}
 
 
 def make_pair(G, oracle_mod, rowptr, col, wgt=None, **params):
@@ -57,9 +59,9 @@ GRAPHS = {
 }
 
 
-@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk"])
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk", "dense_mk"])
 @pytest.mark.parametrize("gname", list(GRAPHS))
-@pytest.mark.parametrize("B", [1, 2, 7, 11, 150, 222, 299, 300])
+@pytest.mark.parametrize("B", [1, 2, 7, 11, 150, 221, 222, 299, 300])
 def test_rebuild_bit_exact(G, oracle_mod, gname, B, regime):
     rowptr, col, w = GRAPHS[gname]()
     V = len(rowptr) - 1
