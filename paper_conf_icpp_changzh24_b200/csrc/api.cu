@@ -8,6 +8,8 @@
 #include <algorithm>
 #include <cstdlib>
 #include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <mutex>
 #include <new>
 #include <vector>
@@ -322,6 +324,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.bm_ccum = A.take<int>(Es);
         c.dout = A.take<int>(Vs);
         c.din = A.take<int>(Vs);
+        c.bm_rowend = A.take<int>(Vs);
+        c.bm_colend = A.take<int>(Vs);
         c.d_nnz = A.take<int>(1);
         c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, (size_t)1 << 24), (size_t)1 << 29);
         c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
@@ -541,6 +545,7 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh) {
     cudaGraph_t graph = nullptr;
     cudaGraphExec_t exec = nullptr;
     const long long l0 = c.launches;
+    const auto tcs = std::chrono::steady_clock::now();
     GSAP_CUDA(cudaStreamBeginCapture(c.stream, cudaStreamCaptureModeThreadLocal));
     c.capturing = true;
     try {
@@ -564,7 +569,9 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh) {
     GSAP_CUDA(cudaStreamEndCapture(c.stream, &graph));
     const long long kernels = c.launches - l0;
     c.launches = l0;
+    const auto tc0 = std::chrono::steady_clock::now();
     GSAP_CUDA(cudaGraphInstantiate(&exec, graph, 0));
+    const auto tc1 = std::chrono::steady_clock::now();
     std::vector<double> D((size_t)c.prm.max_nodal_itr + 1, 0.0);
     int ran = 0;
     try {
@@ -590,6 +597,13 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh) {
     GSAP_CUDA(cudaGraphExecDestroy(exec));
     GSAP_CUDA(cudaGraphDestroy(graph));
     graph_release_events(c);
+    if (getenv("GSAP_TIMING")) {
+        const auto tc2 = std::chrono::steady_clock::now();
+        fprintf(stderr, "[gsap] mcmc B=%d kernels/itr=%lld capture %.3f ms instantiate %.3f ms %d itrs %.3f ms\n", c.B,
+                kernels, std::chrono::duration<double, std::milli>(tc0 - tcs).count(),
+                std::chrono::duration<double, std::milli>(tc1 - tc0).count(), ran,
+                std::chrono::duration<double, std::milli>(tc2 - tc1).count());
+    }
     return ran;
 }
 
@@ -701,6 +715,11 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
         auto tc = std::chrono::steady_clock::now();
         const double S = mdl_now(c);
         auto td = std::chrono::steady_clock::now();
+        if (getenv("GSAP_TIMING"))
+            fprintf(stderr, "[gsap] round %d B=%d merge %.3f ms mcmc %.3f ms mdl %.3f ms\n", rounds, B,
+                    std::chrono::duration<double, std::milli>(tb - ta).count(),
+                    std::chrono::duration<double, std::milli>(tc - tb).count(),
+                    std::chrono::duration<double, std::milli>(td - tc).count());
         t_merge += std::chrono::duration<double>(tb - ta).count();
         t_move += std::chrono::duration<double>(tc - tb).count();
         t_mdl += std::chrono::duration<double>(td - tc).count();
@@ -971,12 +990,57 @@ gsap_status gsap_mdl(gsap_ctx *ctx, double *mdl_out, double *data_term_out) {
     API_CATCH
 }
 
+// export of a padded CSR / CSC (multi-kernel sparse rebuild): compacted on the host
+static gsap_status get_blockmodel_padded(Ctx &c, int64_t *nnz_io, int64_t *rowptr, int32_t *col, int32_t *cnt,
+                                         int32_t *cum, int64_t *colptr, int32_t *row, int32_t *ccnt, int32_t *ccum,
+                                         int32_t *dout, int32_t *din) {
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    const size_t B = (size_t)c.B, E = (size_t)c.E;
+    const std::vector<int> rp = to_host(c.bm_rowptr, B), re = to_host(c.bm_rowend, B);
+    const std::vector<int> cp = to_host(c.bm_colptr, B), ce = to_host(c.bm_colend, B);
+    int64_t nnz = 0, nnzc = 0;
+    for (size_t x = 0; x < B; ++x) {
+        nnz += re[x] - rp[x];
+        nnzc += ce[x] - cp[x];
+    }
+    REQUIRE(nnz == nnzc, GSAP_ECUDA, "row / column entry counts differ");
+    const bool any = col || cnt || cum || row || ccnt || ccum;
+    REQUIRE(!any || *nnz_io >= nnz, GSAP_EINVAL, "entry arrays too small (see *nnz_io)");
+    *nnz_io = nnz;
+    auto ptr_out = [&](int64_t *dst, const std::vector<int> &p, const std::vector<int> &e) {
+        if (!dst) return;
+        std::vector<int64_t> w(B + 1, 0);
+        for (size_t x = 0; x < B; ++x) w[x + 1] = w[x] + (e[x] - p[x]);
+        GSAP_CUDA(cudaMemcpy(dst, w.data(), sizeof(int64_t) * (B + 1), cudaMemcpyDefault));
+    };
+    auto ent_out = [&](int32_t *dst, const int *src, const std::vector<int> &p, const std::vector<int> &e) {
+        if (!dst) return;
+        const std::vector<int> h = to_host(src, E);
+        std::vector<int> w;
+        w.reserve((size_t)nnz);
+        for (size_t x = 0; x < B; ++x) w.insert(w.end(), h.begin() + p[x], h.begin() + e[x]);
+        if (!w.empty()) GSAP_CUDA(cudaMemcpy(dst, w.data(), sizeof(int) * w.size(), cudaMemcpyDefault));
+    };
+    ptr_out(rowptr, rp, re);
+    ptr_out(colptr, cp, ce);
+    ent_out(col, c.bm_col, rp, re);
+    ent_out(cnt, c.bm_cnt, rp, re);
+    ent_out(cum, c.bm_cum, rp, re);
+    ent_out(row, c.bm_row, cp, ce);
+    ent_out(ccnt, c.bm_ccnt, cp, ce);
+    ent_out(ccum, c.bm_ccum, cp, ce);
+    if (dout) GSAP_CUDA(cudaMemcpy(dout, c.dout, sizeof(int) * B, cudaMemcpyDefault));
+    if (din) GSAP_CUDA(cudaMemcpy(din, c.din, sizeof(int) * B, cudaMemcpyDefault));
+    return GSAP_OK;
+}
+
 gsap_status gsap_get_blockmodel(gsap_ctx *ctx, int64_t *nnz_io, int64_t *rowptr, int32_t *col, int32_t *cnt,
                                 int32_t *cum, int64_t *colptr, int32_t *row, int32_t *ccnt, int32_t *ccum,
                                 int32_t *dout, int32_t *din) {
     API_TRY
     REQUIRE(ctx && nnz_io, GSAP_EINVAL, "NULL argument");
     Ctx &c = ctx->c;
+    if (c.padded) return get_blockmodel_padded(c, nnz_io, rowptr, col, cnt, cum, colptr, row, ccnt, ccum, dout, din);
     GSAP_CUDA(cudaMemcpyAsync(c.h_int, c.d_nnz, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
     GSAP_CUDA(cudaStreamSynchronize(c.stream));
     const int64_t nnz = c.h_int[0];

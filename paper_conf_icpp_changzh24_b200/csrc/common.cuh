@@ -141,16 +141,21 @@ GSAP_DEV int warp_incl_scan(int v) {
 // CSR (rows ascending column) + CSC (columns ascending row), cum = inclusive
 // prefix of cnt within a row / column, out/in degrees (P:143-162 3.1), and a
 // dense row-major copy M[x*B+y] when B is small.
+// Line x occupies [rowptr[x], rowend[x]): compact producers pass rowend =
+// rowptr + 1; the multi-kernel sparse rebuild leaves each line in its
+// counting-sort segment (padded CSR, cnt = 0 in the padding).
 struct BM {
     int B;
     const int *__restrict__ dense;   // nullptr in the sparse regime
     const double2 *__restrict__ ft;  // f(m) = m ln m for m < FT_N, double-double {hi, lo}
     const double *__restrict__ rcp;  // 1 / (d_x + B) per block
     const int *__restrict__ rowptr;  // [B+1]
+    const int *__restrict__ rowend;  // [B]: end of line x
     const int *__restrict__ col;
     const int *__restrict__ cnt;
     const int *__restrict__ cum;
     const int *__restrict__ colptr;  // [B+1]
+    const int *__restrict__ colend;  // [B]
     const int *__restrict__ row;
     const int *__restrict__ ccnt;
     const int *__restrict__ ccum;
@@ -177,12 +182,13 @@ struct Line {
     int len;
 };
 
-GSAP_DEV Line line_of(const int *__restrict__ idx, const int *__restrict__ cnt, const int *__restrict__ ptr, int x) {
+GSAP_DEV Line line_of(const int *__restrict__ idx, const int *__restrict__ cnt, const int *__restrict__ ptr,
+                      const int *__restrict__ end, int x) {
     const int lo = __ldg(ptr + x);
     Line L;
     L.idx = idx + lo;
     L.cnt = cnt + lo;
-    L.len = __ldg(ptr + x + 1) - lo;
+    L.len = __ldg(end + x) - lo;
     return L;
 }
 
@@ -196,8 +202,8 @@ GSAP_DEV int line_get(const Line &L, int y) {
     return (a < L.len && __ldg(L.idx + a) == y) ? __ldg(L.cnt + a) : 0;
 }
 
-GSAP_DEV Line row_line(const BM &m, int x) { return line_of(m.col, m.cnt, m.rowptr, x); }
-GSAP_DEV Line col_line(const BM &m, int y) { return line_of(m.row, m.ccnt, m.colptr, y); }
+GSAP_DEV Line row_line(const BM &m, int x) { return line_of(m.col, m.cnt, m.rowptr, m.rowend, x); }
+GSAP_DEV Line col_line(const BM &m, int y) { return line_of(m.row, m.ccnt, m.colptr, m.colend, y); }
 
 GSAP_DEV int bm_at(const BM &m, int x, int y) {
     if (m.dense) return __ldg(m.dense + (size_t)x * m.B + y);
@@ -241,7 +247,7 @@ GSAP_DEV int bm_deg(const BM &m, int x) { return __ldg(m.dout + x) + __ldg(m.din
 // the weighted neighbour block of u at offset p of (out-row u ++ in-col u),
 // skipping id `skip` (-1: none) -- binary search on cum (R:O.4 step 4)
 GSAP_DEV int bm_walk(const BM &m, int u, long long p, int skip) {
-    const int rlo = __ldg(m.rowptr + u), rhi = __ldg(m.rowptr + u + 1);
+    const int rlo = __ldg(m.rowptr + u), rhi = __ldg(m.rowend + u);
     const int dout_u = __ldg(m.dout + u);
     int wskip = 0;
     if (skip >= 0) {
@@ -259,7 +265,7 @@ GSAP_DEV int bm_walk(const BM &m, int u, long long p, int skip) {
     }
     if (p < dout_u) return __ldg(m.col + upper_bound(m.cum, rlo, rhi, p));
     long long q = p - dout_u;
-    const int clo = __ldg(m.colptr + u), chi = __ldg(m.colptr + u + 1);
+    const int clo = __ldg(m.colptr + u), chi = __ldg(m.colend + u);
     if (skip >= 0) {
         int a = clo, b = chi;
         while (a < b) {
@@ -280,10 +286,10 @@ GSAP_DEV int bm_walk(const BM &m, int u, long long p, int skip) {
 GSAP_DEV int bm_walk_warp(const BM &m, int u, long long p) {
     const int dout_u = __ldg(m.dout + u);
     if (p < dout_u) {
-        const int i = warp_upper_bound(m.cum, __ldg(m.rowptr + u), __ldg(m.rowptr + u + 1), p);
+        const int i = warp_upper_bound(m.cum, __ldg(m.rowptr + u), __ldg(m.rowend + u), p);
         return __ldg(m.col + i);
     }
-    const int i = warp_upper_bound(m.ccum, __ldg(m.colptr + u), __ldg(m.colptr + u + 1), p - dout_u);
+    const int i = warp_upper_bound(m.ccum, __ldg(m.colptr + u), __ldg(m.colend + u), p - dout_u);
     return __ldg(m.row + i);
 }
 

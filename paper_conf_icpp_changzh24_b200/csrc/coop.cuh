@@ -12,9 +12,9 @@
 //      the long lines; the other CTAs write rcp = 1 / (d + B)  | barrier
 //   P3 scatter the neighbour blocks into their line's segment  | barrier
 //   P4 per-line sort + run-length encoding: warps take the short lines,
-//      CTAs the long ones (shared-memory radix <= CAP, global radix beyond) | barrier
-//   P5 CTA 0 / 1 scan the run counts into the CSR / CSC pointers  | barrier
-//   P6 compact the runs to the pointers with the in-line prefix `cum`.
+//      CTAs the long ones (shared-memory radix <= CAP, global radix beyond);
+//      the runs stay at the line's segment offset (padded CSR / CSC: the
+//      same warp / CTA writes cum, end[x] and zero counts in the padding).
 // The grid is sized to be co-resident (occupancy x SMs) and launched
 // cooperatively; the barrier is the usual arrive-counter + generation flag.
 #pragma once
@@ -27,12 +27,13 @@ struct CoopSide {
     const int *__restrict__ gptr;   // graph lines: out-CSR rowptr / in-CSC cscptr
     const int *__restrict__ gidx;   // neighbour ids
     const int *__restrict__ gw;     // weights or nullptr
-    int *len, *off, *cur, *nnz, *listC;   // [B + 1] line scratch
+    int *len, *cur, *nnz, *listC;   // [B + 1] line scratch
+    int *off;                       // out: [B + 1] segment offsets = line pointers (padded)
     void *seg;                      // K[E] segment keys
-    int *tcol, *tcnt;               // [E] runs at segment offsets
+    int *tcol, *tcnt;               // out: [E] runs (block, count) at the segment offsets
     void *xl_keys;                  // K[2E] global radix scratch
     int *xl_hp;                     // [2E]
-    int *ptr, *idx, *cnt, *cum, *deg;   // outputs: pointers [B + 1], entries, line sums
+    int *cum, *end, *deg;           // out: in-line prefix [E], line ends [B], line sums [B]
 };
 
 struct CoopArgs {
@@ -186,9 +187,13 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
         const int o = sd.off[x], L = sd.off[x + 1] - o;
         if (L > SEG_WARP_MAX) continue;
         if (L == 0) {
-            if (lane == 0) sd.nnz[x] = 0;
+            if (lane == 0) {
+                sd.nnz[x] = 0;
+                sd.end[x] = o;
+            }
             continue;
         }
+        const LineOut out{sd.cum, sd.end, sd.deg};
         const K *seg = reinterpret_cast<const K *>(sd.seg);
         if (L <= 128) {   // short lines: bitonic in registers, RLE in registers
             int u;
@@ -196,6 +201,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, sd.tcol + o, sd.tcnt + o);
             else u = warp_segsort_rle<K, 4>(seg + o, L, sd.tcol + o, sd.tcnt + o);
             if (lane == 0) sd.nnz[x] = u;
+            line_epilogue<32>(out, sd.tcnt, o, u, L, x, lane, nullptr);
             continue;
         }
         int n = 1;
@@ -205,6 +211,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
         bitonic<K, 32>(S.warp.keys[wl], n, lane);
         const int u = rle_runs<K, 32>(S.warp.keys[wl], L, S.warp.hp[wl], sd.tcol + o, sd.tcnt + o, lane, nullptr);
         if (lane == 0) sd.nnz[x] = u;
+        line_epilogue<32>(out, sd.tcnt, o, u, L, x, lane, nullptr);
     }
     __syncthreads();   // the shared memory changes role
     // P4b: long lines, one CTA each
@@ -216,6 +223,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             const int x = sd.listC[q ? li - n0 : li];
             const int o = sd.off[x], L = sd.off[x + 1] - o;
             K *seg = reinterpret_cast<K *>(sd.seg);
+            const LineOut out{sd.cum, sd.end, sd.deg};
             int u;
             if (L <= SegCta<K>::CAP) {
                 for (int i = threadIdx.x; i < L; i += 256) S.cta.keys[0][i] = seg[o + i];
@@ -223,40 +231,17 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
                 K *keys = cta_radix_sort<K, 256>(S.cta.keys[0], S.cta.keys[1], L, a.col_bits, S.cta.cntp, S.cta.wsum);
                 int *hp = reinterpret_cast<int *>(keys == S.cta.keys[0] ? S.cta.keys[1] : S.cta.keys[0]);
                 u = rle_runs<K, 256>(keys, L, hp, sd.tcol + o, sd.tcnt + o, threadIdx.x, S.cta.sh);
+                line_epilogue<256>(out, sd.tcnt, o, u, L, x, threadIdx.x, S.cta.sh);
             } else {
                 u = xl_sort_line<K>(seg, o, L, a.col_bits, sd.tcol, sd.tcnt, reinterpret_cast<K *>(sd.xl_keys),
                                     sd.xl_hp, S.xl);
+                line_epilogue<256>(out, sd.tcnt, o, u, L, x, threadIdx.x, S.xl.sh);
             }
             if (threadIdx.x == 0) sd.nnz[x] = u;
             __syncthreads();
         }
     }
-    grid_sync(a.bar);
-    // P5
-    if (blockIdx.x < 2) {
-        CoopSide &sd = a.sd[blockIdx.x];
-        cta_scan_lines(sd.nnz, sd.ptr, B, nullptr, nullptr, S.scan);
-        if (blockIdx.x == 0 && threadIdx.x == 0) *a.d_nnz = sd.ptr[B];
-    }
-    grid_sync(a.bar);
-    // P6: compact the runs (warp per (side, line))
-    for (int task = gwarp; task < 2 * B; task += gwarps) {
-        const int q = task >= B, x = q ? task - B : task;
-        const CoopSide &sd = a.sd[q];
-        const int o = sd.off[x], n = sd.nnz[x], p = sd.ptr[x];
-        int run = 0;
-        for (int k0 = 0; k0 < n; k0 += 32) {
-            const int k = k0 + lane;
-            const int c = k < n ? sd.tcnt[o + k] : 0;
-            const int sc = warp_incl_scan(c) + run;
-            if (k < n) {
-                sd.idx[p + k] = sd.tcol[o + k];
-                sd.cnt[p + k] = c;
-                sd.cum[p + k] = sc;
-            }
-            run = __shfl_sync(FULL, sc, 31);
-        }
-    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) *a.d_nnz = a.sd[0].off[B];   // the extent E (padding has cnt 0)
 }
 
 }  // namespace gsap

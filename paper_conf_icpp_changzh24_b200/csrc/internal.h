@@ -62,6 +62,11 @@ struct Ctx {
     int *bm_rowptr = nullptr, *bm_col = nullptr, *bm_cnt = nullptr, *bm_cum = nullptr;
     int *bm_colptr = nullptr, *bm_row = nullptr, *bm_ccnt = nullptr, *bm_ccum = nullptr;
     int *dout = nullptr, *din = nullptr, *d_nnz = nullptr;
+    // padded CSR/CSC (multi-kernel sparse rebuild): line x = [ptr[x], end[x]) inside
+    // its counting-sort segment [ptr[x], ptr[x + 1]), cnt = 0 in the padding and
+    // d_nnz = E (the extent the MDL sums over); otherwise compact (end = ptr + 1)
+    bool padded = false;
+    int *bm_rowend = nullptr, *bm_colend = nullptr;
     int *dense = nullptr, *denseT = nullptr;
     double2 *ft = nullptr;         // f-table {hi, lo} (FT_N entries)
     double *rcp = nullptr;         // 1 / (d_x + B), refreshed by every rebuild
@@ -132,6 +137,8 @@ struct Ctx {
         m.rcp = rcp;
         m.rowptr = bm_rowptr; m.col = bm_col; m.cnt = bm_cnt; m.cum = bm_cum;
         m.colptr = bm_colptr; m.row = bm_row; m.ccnt = bm_ccnt; m.ccum = bm_ccum;
+        m.rowend = padded ? bm_rowend : bm_rowptr + 1;
+        m.colend = padded ? bm_colend : bm_colptr + 1;
         m.dout = dout; m.din = din;
         return m;
     }

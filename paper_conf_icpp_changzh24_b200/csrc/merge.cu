@@ -49,10 +49,11 @@ GSAP_DEV int propose_merge(const BM &m, int r, uint32_t j, uint64_t seed, uint32
 // look the other one up in its hash table (or the dense copy)
 GSAP_DEV double inter_sum(const BM &m, bool cols, int a, int b, int r, int s) {
     const int *__restrict__ ptr = cols ? m.colptr : m.rowptr;
+    const int *__restrict__ end = cols ? m.colend : m.rowend;
     const int *__restrict__ idx = cols ? m.row : m.col;
     const int *__restrict__ cnt = cols ? m.ccnt : m.cnt;
-    const int alo = __ldg(ptr + a), ahi = __ldg(ptr + a + 1);
-    const int blo = __ldg(ptr + b), bhi = __ldg(ptr + b + 1);
+    const int alo = __ldg(ptr + a), ahi = __ldg(end + a);
+    const int blo = __ldg(ptr + b), bhi = __ldg(end + b);
     const bool walk_a = (ahi - alo) <= (bhi - blo);
     const int lo = walk_a ? alo : blo, hi = walk_a ? ahi : bhi, other = walk_a ? b : a;
     Line L{};

@@ -536,10 +536,13 @@ __global__ void k_rcp(int B, const int *__restrict__ dout, const int *__restrict
 }
 
 // one side of the sparse blockmodel: lines (rows of M from the out-CSR, or
-// columns of M from the in-CSC) by counting sort + per-line segment sort
+// columns of M from the in-CSC) by counting sort + per-line segment sort,
+// written as a padded CSR: line x's runs stay at its segment offset ptr[x]
+// (= the exclusive scan of the line lengths), end[x] marks their end, cnt is
+// zero in the rest of the segment.  No second scan and no compaction pass.
 template <typename K>
-static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw, int *ptr, int *idx, int *cnt,
-                        int *cum, int *lineid, int *deg, int *total) {
+static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw, int *ptr, int *end, int *idx,
+                        int *cnt, int *cum, int *deg, int *extent) {
     Launcher L{c.stream, &c.launches};
     const int B = c.B, V = c.V;
     K *seg = reinterpret_cast<K *>(c.keys0);
@@ -548,25 +551,21 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     GSAP_CUDA(cudaMemsetAsync(c.seg_ctr, 0, 2 * sizeof(int), c.stream));
     k_line_len<<<grid_for(V, 256), 256, 0, c.stream>>>(V, gptr, c.b, c.seg_len);
     ++c.launches;
-    device_scan<int>(c.seg_len, c.seg_off, nullptr, B, false, c.scan_tmp, c.seg_off + B, L);
-    k_line_scatter<K><<<grid_for((long long)V * 32, 256), 256, 0, c.stream>>>(V, gptr, gidx, gw, c.b, c.seg_off,
+    device_scan<int>(c.seg_len, ptr, nullptr, B, false, c.scan_tmp, ptr + B, L);
+    k_line_scatter<K><<<grid_for((long long)V * 32, 256), 256, 0, c.stream>>>(V, gptr, gidx, gw, c.b, ptr,
                                                                              c.seg_cur, seg);
-    k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, c.seg_off, c.seg_nnz, c.seg_listW, c.seg_listC,
-                                                           c.seg_ctr);
+    const LineOut out{cum, end, deg};
+    k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, ptr, c.seg_nnz, c.seg_listW, c.seg_listC,
+                                                           c.seg_ctr, out, extent);
     const int gw_ = (int)std::min<long long>(((long long)B + SEG_WARPS - 1) / SEG_WARPS, 148LL * 16);
-    k_segsort_warp<K><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(c.seg_off, seg, c.seg_listW, c.seg_ctr, c.wa, c.wb,
-                                                           c.seg_nnz);
+    k_segsort_warp<K><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(ptr, seg, c.seg_listW, c.seg_ctr, idx, cnt,
+                                                           c.seg_nnz, out);
     const int gc = (int)std::min<long long>(std::max(1, B / 4), 148LL * 4);
-    k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(c.seg_off, seg, c.seg_listC, c.seg_ctr, bits_for(B), c.wa, c.wb,
-                                               c.seg_nnz);
-    k_segsort_xl<K><<<gc, 256, 0, c.stream>>>(c.seg_off, seg, c.seg_listC, c.seg_ctr, bits_for(B), c.wa, c.wb,
-                                              c.seg_nnz, reinterpret_cast<K *>(c.xl_keys), c.xl_hp);
+    k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(ptr, seg, c.seg_listC, c.seg_ctr, bits_for(B), idx, cnt,
+                                               c.seg_nnz, out);
+    k_segsort_xl<K><<<gc, 256, 0, c.stream>>>(ptr, seg, c.seg_listC, c.seg_ctr, bits_for(B), idx, cnt,
+                                              c.seg_nnz, reinterpret_cast<K *>(c.xl_keys), c.xl_hp, out);
     c.launches += 5;
-    device_scan<int>(c.seg_nnz, ptr, nullptr, B, false, c.scan_tmp, ptr + B, L);
-    k_line_copy<<<grid_for((long long)B * 32, 256), 256, 0, c.stream>>>(B, c.seg_off, c.seg_nnz, ptr, c.wa, c.wb,
-                                                                       idx, cnt, cum, lineid, deg);
-    ++c.launches;
-    if (total) GSAP_CUDA(cudaMemcpyAsync(total, ptr + B, sizeof(int), cudaMemcpyDeviceToDevice, c.stream));
     GSAP_CHECK_LAUNCH();
 }
 
@@ -583,13 +582,13 @@ static void rebuild_sparse_coop(Ctx &c) {
     a.kin = c.kin;
     CoopSide &r = a.sd[0], &q = a.sd[1];
     r.gptr = c.rowptr; r.gidx = c.col; r.gw = c.wgt;
-    r.len = c.seg_len; r.off = c.seg_off; r.cur = c.seg_cur; r.nnz = c.seg_nnz; r.listC = c.seg_listC;
-    r.seg = c.keys0; r.tcol = c.wa; r.tcnt = c.wb; r.xl_keys = c.xl_keys; r.xl_hp = c.xl_hp;
-    r.ptr = c.bm_rowptr; r.idx = c.bm_col; r.cnt = c.bm_cnt; r.cum = c.bm_cum; r.deg = c.dout;
+    r.len = c.seg_len; r.off = c.bm_rowptr; r.cur = c.seg_cur; r.nnz = c.seg_nnz; r.listC = c.seg_listC;
+    r.seg = c.keys0; r.tcol = c.bm_col; r.tcnt = c.bm_cnt; r.xl_keys = c.xl_keys; r.xl_hp = c.xl_hp;
+    r.cum = c.bm_cum; r.end = c.bm_rowend; r.deg = c.dout;
     q.gptr = c.cscptr; q.gidx = c.cscsrc; q.gw = c.cscwgt;
-    q.len = c.seg2_len; q.off = c.seg2_off; q.cur = c.seg2_cur; q.nnz = c.seg2_nnz; q.listC = c.seg2_listC;
-    q.seg = c.keys1; q.tcol = c.flags; q.tcnt = c.pos; q.xl_keys = c.xl2_keys; q.xl_hp = c.xl2_hp;
-    q.ptr = c.bm_colptr; q.idx = c.bm_row; q.cnt = c.bm_ccnt; q.cum = c.bm_ccum; q.deg = c.din;
+    q.len = c.seg2_len; q.off = c.bm_colptr; q.cur = c.seg2_cur; q.nnz = c.seg2_nnz; q.listC = c.seg2_listC;
+    q.seg = c.keys1; q.tcol = c.bm_row; q.tcnt = c.bm_ccnt; q.xl_keys = c.xl2_keys; q.xl_hp = c.xl2_hp;
+    q.cum = c.bm_ccum; q.end = c.bm_colend; q.deg = c.din;
     a.rcp = c.rcp;
     a.d_nnz = c.d_nnz;
     a.nlong = c.seg_ctr;
@@ -616,6 +615,7 @@ static void rebuild_sparse_coop(Ctx &c) {
     cfg.numAttrs = 1;
     GSAP_CUDA(cudaLaunchKernelEx(&cfg, k_rebuild_coop<K>, a));
     ++c.launches;
+    c.padded = true;
 }
 
 static void rebuild_sparse(Ctx &c) {
@@ -633,17 +633,19 @@ static void rebuild_sparse(Ctx &c) {
         GSAP_CUDA(cudaMemsetAsync(c.d_nnz, 0, sizeof(int), c.stream));
         return;
     }
+    // padded CSR / CSC; d_nnz = the extent E the MDL sums cnt over (zeros in the padding)
     if (c.weighted) {
-        build_lines<u64>(c, c.rowptr, c.col, c.wgt, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.rowid, c.dout,
+        build_lines<u64>(c, c.rowptr, c.col, c.wgt, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt, c.bm_cum, c.dout,
                          c.d_nnz);
-        build_lines<u64>(c, c.cscptr, c.cscsrc, c.cscwgt, c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.flags,
+        build_lines<u64>(c, c.cscptr, c.cscsrc, c.cscwgt, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt, c.bm_ccum,
                          c.din, nullptr);
     } else {
-        build_lines<unsigned>(c, c.rowptr, c.col, nullptr, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum, c.rowid,
+        build_lines<unsigned>(c, c.rowptr, c.col, nullptr, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt, c.bm_cum,
                               c.dout, c.d_nnz);
-        build_lines<unsigned>(c, c.cscptr, c.cscsrc, nullptr, c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum,
-                              c.flags, c.din, nullptr);
+        build_lines<unsigned>(c, c.cscptr, c.cscsrc, nullptr, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt,
+                              c.bm_ccum, c.din, nullptr);
     }
+    c.padded = true;
     GSAP_CHECK_LAUNCH();
 }
 
@@ -651,6 +653,7 @@ void rebuild(Ctx &c) {
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_rebuild, &ev);
     c.dense_mode = dense_ok(c, c.B);
+    c.padded = false;   // set by the multi-kernel sparse path
     if (c.dense_mode && c.small_acc && c.B <= SMALL_MAX_B) {
         rebuild_dense_small(c);
     } else if (c.dense_mode) {

@@ -8,8 +8,10 @@
 //      segment (one atomic per vertex, coalesced writes; the order inside a
 //      segment is arbitrary, the sort below makes it canonical)
 //   4. per segment: sort + run-length encode (a warp for <= 512 entries, a CTA
-//      in shared memory for <= 4096, a CTA in global scratch beyond)
-//   5. compact: line pointers by scan, copy with cum and line sums.
+//      in shared memory for <= 4096, a CTA in global scratch beyond); the runs
+//      stay at the segment offset (padded CSR: end[x], cum, line sums and
+//      zero counts in the padding written by the same warp / CTA), or go to
+//      scratch for the persistent kernel's compaction (coop.cuh).
 //
 // Keys are the neighbour block (unweighted, u32) or (block << 32 | weight)
 // (weighted, u64): equal blocks become adjacent and their weights are summed.
@@ -113,6 +115,48 @@ GSAP_DEV int rle_runs(const K *a, int L, int *hp, int *ocol, int *ocnt, int tid,
     return total;
 }
 
+// padded output (rebuild_sparse, multi-kernel): the runs of line x stay at
+// its segment offset o in the final idx / cnt arrays; the epilogue writes the
+// in-line prefix cum, zeroes cnt in the padding [o + u, o + L), and records
+// end[x] = o + u and the line's total weight deg[x].  cum == nullptr: off.
+struct LineOut {
+    int *cum, *end, *deg;
+};
+
+template <int NT>
+GSAP_DEV void line_epilogue(const LineOut &out, int *__restrict__ cnt, int o, int u, int L, int x, int tid,
+                            int *sh) {
+    nt_sync<NT>();   // the runs written by the other threads are visible
+    const int lane = tid & 31, w = tid >> 5;
+    int carry = 0;
+    for (int base = 0; base < u; base += NT) {
+        const int i = base + tid;
+        const int c = i < u ? cnt[o + i] : 0;
+        const int xi = warp_incl_scan(c);
+        int before = 0, total;
+        if (NT == 32) {
+            total = __shfl_sync(FULL, xi, 31);
+        } else {
+            if (lane == 31) sh[w] = xi;
+            __syncthreads();
+            total = 0;
+            for (int q = 0; q < NT / 32; ++q) {
+                const int t = sh[q];
+                if (q < w) before += t;
+                total += t;
+            }
+            __syncthreads();
+        }
+        if (i < u) out.cum[o + i] = carry + before + xi;
+        carry += total;
+    }
+    for (int i = u + tid; i < L; i += NT) cnt[o + i] = 0;
+    if (tid == 0) {
+        out.end[x] = o + u;
+        out.deg[x] = carry;
+    }
+}
+
 // 1. len[b[v]] += deg(v)
 __global__ void k_line_len(int V, const int *__restrict__ gptr, const int *__restrict__ b, int *__restrict__ len) {
     for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
@@ -144,10 +188,18 @@ __global__ void k_line_scatter(int V, const int *__restrict__ gptr, const int *_
 
 // 4a. classify lines by segment length
 __global__ void k_line_classify(int B, const int *__restrict__ off, int *__restrict__ nnz, int *__restrict__ listW,
-                                int *__restrict__ listC, int *__restrict__ counters) {
+                                int *__restrict__ listC, int *__restrict__ counters, LineOut out,
+                                int *__restrict__ extent) {
+    if (extent && blockIdx.x == 0 && threadIdx.x == 0) *extent = off[B];
     for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < B; x += gridDim.x * blockDim.x) {
         const int L = off[x + 1] - off[x];
-        if (L == 0) nnz[x] = 0;
+        if (L == 0) {
+            nnz[x] = 0;
+            if (out.cum) {
+                out.end[x] = off[x];
+                out.deg[x] = 0;
+            }
+        }
         else if (L <= SEG_WARP_MAX) listW[atomicAdd(counters, 1)] = x;
         else listC[atomicAdd(counters + 1, 1)] = x;
     }
@@ -261,25 +313,14 @@ GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict_
     return total;
 }
 
-// 4b. short segments: one warp each, sorted in registers
-template <typename K, int E>
-GSAP_DEV void seg_warp_one(const int *__restrict__ off, const K *__restrict__ seg, int x, int *tcol, int *tcnt,
-                           int *nnz) {
-    const int o = off[x], L = off[x + 1] - o;
-    const int u = warp_segsort_rle<K, E>(seg + o, L, tcol + o, tcnt + o);
-    if ((threadIdx.x & 31) == 0) nnz[x] = u;
-}
-
-#ifndef GSAP_SEG_REG
-#define GSAP_SEG_REG 0   // 1: register bitonic (slower for 256 < L <= 512 on B200, kept for reference)
-#endif
-#if !GSAP_SEG_REG
+// 4b. short segments (<= SEG_WARP_MAX): one warp each -- <= 128 entries
+// bitonic + RLE in registers, longer ones bitonic in shared memory
 template <typename K>
 __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__restrict__ off, K *__restrict__ seg,
                                                                  const int *__restrict__ listW,
                                                                  const int *__restrict__ counters,
                                                                  int *__restrict__ tcol, int *__restrict__ tcnt,
-                                                                 int *__restrict__ nnz) {
+                                                                 int *__restrict__ nnz, LineOut out) {
     __shared__ K keys[SEG_WARPS][SEG_WARP_MAX];
     __shared__ int hp[SEG_WARPS][SEG_WARP_MAX];
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -293,6 +334,7 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__re
             else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, tcol + o, tcnt + o);
             else u = warp_segsort_rle<K, 4>(seg + o, L, tcol + o, tcnt + o);
             if (lane == 0) nnz[x] = u;
+            if (out.cum) line_epilogue<32>(out, tcnt, o, u, L, x, lane, nullptr);
             continue;
         }
         int n = 1;
@@ -302,28 +344,9 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__re
         bitonic<K, 32>(keys[w], n, lane);
         const int u = rle_runs<K, 32>(keys[w], L, hp[w], tcol + o, tcnt + o, lane, nullptr);
         if (lane == 0) nnz[x] = u;
+        if (out.cum) line_epilogue<32>(out, tcnt, o, u, L, x, lane, nullptr);
     }
 }
-#else
-template <typename K>
-__global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__restrict__ off, K *__restrict__ seg,
-                                                                 const int *__restrict__ listW,
-                                                                 const int *__restrict__ counters,
-                                                                 int *__restrict__ tcol, int *__restrict__ tcnt,
-                                                                 int *__restrict__ nnz) {
-    const int w = threadIdx.x >> 5;
-    const int n_lines = counters[0];
-    for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
-        const int x = listW[li];
-        const int L = off[x + 1] - off[x];
-        if (L <= 32) seg_warp_one<K, 1>(off, seg, x, tcol, tcnt, nnz);
-        else if (L <= 64) seg_warp_one<K, 2>(off, seg, x, tcol, tcnt, nnz);
-        else if (L <= 128) seg_warp_one<K, 4>(off, seg, x, tcol, tcnt, nnz);
-        else if (L <= 256) seg_warp_one<K, 8>(off, seg, x, tcol, tcnt, nnz);
-        else seg_warp_one<K, 16>(off, seg, x, tcol, tcnt, nnz);
-    }
-}
-#endif
 
 // stable LSD radix sort of a[0, L) by the block bits of the key (key_col),
 // 4-bit digits, NT threads.  Each thread owns a contiguous chunk of an odd
@@ -409,7 +432,7 @@ template <typename K>
 __global__ void __launch_bounds__(256) k_segsort_cta(const int *__restrict__ off, K *__restrict__ seg,
                                                      const int *__restrict__ listC, const int *__restrict__ counters,
                                                      int col_bits, int *__restrict__ tcol, int *__restrict__ tcnt,
-                                                     int *__restrict__ nnz) {
+                                                     int *__restrict__ nnz, LineOut out) {
     constexpr int CAP = SegCta<K>::CAP;
     __shared__ K skeys[2][CAP];
     __shared__ unsigned cntp[8 * 256];
@@ -426,6 +449,7 @@ __global__ void __launch_bounds__(256) k_segsort_cta(const int *__restrict__ off
         int *hp = reinterpret_cast<int *>(keys == skeys[0] ? skeys[1] : skeys[0]);
         const int u = rle_runs<K, 256>(keys, L, hp, tcol + o, tcnt + o, threadIdx.x, sh);
         if (threadIdx.x == 0) nnz[x] = u;
+        if (out.cum) line_epilogue<256>(out, tcnt, o, u, L, x, threadIdx.x, sh);
         __syncthreads();
     }
 }
@@ -515,7 +539,8 @@ template <typename K>
 __global__ void __launch_bounds__(256) k_segsort_xl(const int *__restrict__ off, K *__restrict__ seg,
                                                     const int *__restrict__ listC, const int *__restrict__ counters,
                                                     int col_bits, int *__restrict__ tcol, int *__restrict__ tcnt,
-                                                    int *__restrict__ nnz, K *__restrict__ gkeys, int *__restrict__ ghp) {
+                                                    int *__restrict__ nnz, K *__restrict__ gkeys, int *__restrict__ ghp,
+                                                    LineOut out) {
     __shared__ XlSmem S;
     const int n_lines = counters[1];
     for (int li = blockIdx.x; li < n_lines; li += gridDim.x) {
@@ -524,33 +549,8 @@ __global__ void __launch_bounds__(256) k_segsort_xl(const int *__restrict__ off,
         if (L <= SegCta<K>::CAP) continue;   // handled by k_segsort_cta
         const int u = xl_sort_line<K>(seg, o, L, col_bits, tcol, tcnt, gkeys, ghp, S);
         if (threadIdx.x == 0) nnz[x] = u;
+        if (out.cum) line_epilogue<256>(out, tcnt, o, u, L, x, threadIdx.x, S.sh);
         __syncthreads();
-    }
-}
-
-// 5. compact line x's runs from its segment to ptr[x]: idx, cnt, cum, line id,
-// and the line's total weight (dout or din)
-__global__ void k_line_copy(int B, const int *__restrict__ off, const int *__restrict__ nnz,
-                            const int *__restrict__ ptr, const int *__restrict__ tcol, const int *__restrict__ tcnt,
-                            int *__restrict__ idx, int *__restrict__ cnt, int *__restrict__ cum,
-                            int *__restrict__ lineid, int *__restrict__ deg) {
-    const int lane = threadIdx.x & 31;
-    for (int x = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < B; x += (gridDim.x * blockDim.x) >> 5) {
-        const int o = off[x], n = nnz[x], p = ptr[x];
-        int run = 0;
-        for (int k0 = 0; k0 < n; k0 += 32) {
-            const int k = k0 + lane;
-            const int c = k < n ? tcnt[o + k] : 0;
-            const int sc = warp_incl_scan(c) + run;
-            if (k < n) {
-                idx[p + k] = tcol[o + k];
-                cnt[p + k] = c;
-                cum[p + k] = sc;
-                lineid[p + k] = x;
-            }
-            run = __shfl_sync(FULL, sc, 31);
-        }
-        if (lane == 0) deg[x] = run;
     }
 }
 

@@ -86,3 +86,12 @@ def test_product_never_imports_the_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h")):
                 txt = open(os.path.join(dp, f)).read()
                 assert "oracle" not in re.sub(r"(#|//).*", "", txt).lower() or f == "__init__.py", f
+
+
+def test_bench_and_entry_compile():
+    """bench.py / __graft_entry__.py are valid Python (the driver runs them on the GPU box)."""
+    import py_compile
+    import os
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    for f in ("bench.py", "__graft_entry__.py"):
+        py_compile.compile(os.path.join(root, f), doraise=True)

@@ -96,7 +96,7 @@ def _states(V, rng_seed):
         yield B, dcsbm.random_partition(V, B, int(rng.integers(1 << 30)))
 
 
-@pytest.mark.parametrize("regime", ["auto", "sparse"])
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk"])
 @pytest.mark.parametrize("gname", list(GRAPHS))
 def test_move_proposals_dS_accept(G, oracle_mod, gname, regime):
     rowptr, col, w = GRAPHS[gname]()
@@ -119,7 +119,7 @@ def test_move_proposals_dS_accept(G, oracle_mod, gname, regime):
     print("MH ties:", nties)
 
 
-@pytest.mark.parametrize("regime", ["auto", "sparse"])
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk"])
 @pytest.mark.parametrize("gname", list(GRAPHS))
 def test_merge_proposals_dS_best(G, oracle_mod, gname, regime):
     rowptr, col, w = GRAPHS[gname]()
@@ -162,7 +162,7 @@ def test_select_merges_bit_exact(G, oracle_mod, seed):
     assert_same_blockmodel(ctx, orc)
 
 
-@pytest.mark.parametrize("regime", ["auto", "sparse"])
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk"])
 def test_merge_phase_lockstep(G, oracle_mod, regime):
     rowptr, col, truth, cfg = dcsbm.make("1k")
     ctx, orc = make_pair(G, oracle_mod, rowptr, col, **REGIMES[regime])
@@ -222,7 +222,7 @@ def test_mcmc_lockstep(G, oracle_mod, name, regime):
     print("MH ties:", nties)
 
 
-@pytest.mark.parametrize("regime", ["auto", "sparse"])
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk"])
 def test_big_vertices_and_global_tables(G, oracle_mod, regime):
     """Hubs with > 128 and > 2048 distinct neighbour blocks (CTA path, global table)."""
     rng = np.random.default_rng(0)
@@ -278,7 +278,7 @@ def test_edge_cases(G, oracle_mod):
         G.Context(np.array([0, 2], np.int64), np.array([0, 5], np.int32))
 
 
-@pytest.mark.parametrize("regime", ["auto", "sparse"])
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk"])
 def test_end_to_end_1k(G, oracle_mod, regime):
     from gen import metrics
     rowptr, col, truth, cfg = dcsbm.make("1k")
