@@ -62,13 +62,16 @@ typedef struct {
     int32_t model_term;       /* 0: E h(B^2/E) (Eq. 2); 1: GraphChallenge variant (R:Z3) */
     int32_t max_rounds;       /* guard on merge+MCMC rounds; default 500 */
     int32_t profile;          /* 1: time kernels with CUDA events (gsap_stats k_*) */
-    int32_t cuda_graphs;      /* 1: capture each MCMC iteration as one CUDA graph (default) */
+    int32_t cuda_graphs;      /* 0: plain launches; 1: each MCMC iteration one CUDA graph launch
+                                 (default); 2: the whole MCMC phase one graph launch, a device-side
+                                 while loop (conditional node) with the convergence test on the GPU */
     int32_t dense_max_B;      /* dense blockmodel iff B <= this; 0 = auto (B^2 <= max(4E, 2^24)) */
     int32_t sparse_coop;      /* 1 (default): sparse-regime rebuild as one persistent kernel when
                                  E <= GSAP_COOP_MAX_E; 0: the multi-kernel rebuild (same result) */
-    int32_t dense_coop;       /* 1 (default): dense-regime rebuild as one persistent kernel when
-                                 B <= 221 (B x B histogram in shared memory); 0: the multi-kernel
-                                 dense rebuild (same result) */
+    int32_t dense_coop;       /* dense-regime rebuild: 1 (default) one persistent kernel when
+                                 B <= 221 (shared-memory histogram), the multi-kernel path above;
+                                 2: the persistent kernel for every dense B (L2 atomics above 221;
+                                 slower there on B200); 0: always multi-kernel.  Same result. */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */

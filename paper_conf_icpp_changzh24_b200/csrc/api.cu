@@ -607,8 +607,114 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh) {
     return ran;
 }
 
+// End of one MCMC iteration inside the device-side loop (R:O.8, R:Z19): D[itr]
+// = the iteration's sum of accepted dS, the GraphChallenge convergence test on
+// the device -- the same double operations in the same order as converged()
+// on the host -- and the while-condition of the enclosing conditional node.
+__global__ void k_mcmc_step(cudaGraphConditionalHandle h, unsigned *d_itr, double *scal, double *Dh, int max_itr,
+                            int w, double model, double thresh) {
+    const int itr = (int)*d_itr;
+    Dh[itr] = scal[0];
+    scal[0] = 0.0;
+    bool stop = itr + 1 >= max_itr;
+    if (!stop && itr >= w - 1) {
+        double sum = 0.0;
+        int n = 0;
+        for (int j = itr - w + 1; j < itr; ++j) {
+            sum += Dh[j];
+            ++n;
+        }
+        const double mean = n ? sum / n : 0.0;
+        const double mdl = model + scal[1];
+        stop = -mean < thresh * mdl;
+    }
+    *d_itr = (unsigned)(itr + 1);
+    cudaGraphSetConditional(h, stop ? 0u : 1u);
+}
+
+// The whole MCMC phase as ONE graph launch: a conditional WHILE node whose
+// body is one iteration (num_batches x (move + apply + rebuild), the MDL
+// reduction, k_mcmc_step); the loop runs on the device until the
+// convergence test or max_nodal_itr stops it -- no host round trip per
+// iteration (N1, P:385 5).  Event nodes are not allowed in conditional
+// bodies, so profile = 1 uses mcmc_phase_graph.
+static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh) {
+    const int V = c.V, nb = c.prm.num_batches;
+    const int bs = (V + nb - 1) / nb;
+    const long long l0 = c.launches;
+    const auto tcs = std::chrono::steady_clock::now();
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t exec = nullptr;
+    GSAP_CUDA(cudaGraphCreate(&graph, 0));
+    try {
+        cudaGraphConditionalHandle h;
+        GSAP_CUDA(cudaGraphConditionalHandleCreate(&h, graph, 1u, cudaGraphCondAssignDefault));
+        cudaGraphNodeParams np = {};
+        np.type = cudaGraphNodeTypeConditional;
+        np.conditional.handle = h;
+        np.conditional.type = cudaGraphCondTypeWhile;
+        np.conditional.size = 1;
+        cudaGraphNode_t node;
+        GSAP_CUDA(cudaGraphAddNode(&node, graph, nullptr, 0, &np));
+        cudaGraph_t body = np.conditional.phGraph_out[0];
+        GSAP_CUDA(cudaStreamBeginCaptureToGraph(c.stream, body, nullptr, nullptr, 0,
+                                                cudaStreamCaptureModeThreadLocal));
+        c.capturing = true;
+        try {
+            for (int k = 0; k < nb; ++k) {
+                const int first = k * bs, last = std::min(V, first + bs);
+                if (first >= last) continue;
+                launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
+                launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1);
+                rebuild(c);
+            }
+            launch_data_term(c);
+            const double model = model_term(c.W, c.V, c.B, c.prm.model_term);
+            k_mcmc_step<<<1, 1, 0, c.stream>>>(h, c.d_itr, c.scal, c.Dh, c.prm.max_nodal_itr, c.prm.window, model,
+                                              thresh);
+            GSAP_CHECK_LAUNCH();
+            ++c.launches;
+        } catch (...) {
+            c.capturing = false;
+            cudaGraph_t g2 = nullptr;
+            cudaStreamEndCapture(c.stream, &g2);
+            throw;
+        }
+        c.capturing = false;
+        GSAP_CUDA(cudaStreamEndCapture(c.stream, &body));
+        const long long kernels = c.launches - l0;
+        c.launches = l0;
+        const auto tc0 = std::chrono::steady_clock::now();
+        GSAP_CUDA(cudaGraphInstantiate(&exec, graph, 0));
+        const auto tc1 = std::chrono::steady_clock::now();
+        GSAP_CUDA(cudaMemsetAsync(c.scal, 0, sizeof(double), c.stream));
+        GSAP_CUDA(cudaMemsetAsync(c.d_itr, 0, sizeof(unsigned), c.stream));
+        GSAP_CUDA(cudaGraphLaunch(exec, c.stream));
+        GSAP_CUDA(cudaMemcpyAsync(c.h_int + 2, c.d_itr, sizeof(unsigned), cudaMemcpyDeviceToHost, c.stream));
+        GSAP_CUDA(cudaStreamSynchronize(c.stream));
+        const int ran = c.h_int[2];
+        c.launches += kernels * ran;
+        c.st.n_move_prop += (long long)V * ran;
+        GSAP_CUDA(cudaGraphExecDestroy(exec));
+        GSAP_CUDA(cudaGraphDestroy(graph));
+        if (getenv("GSAP_TIMING")) {
+            const auto tc2 = std::chrono::steady_clock::now();
+            fprintf(stderr, "[gsap] mcmc(device loop) B=%d kernels/itr=%lld capture %.3f ms instantiate %.3f ms "
+                    "%d itrs %.3f ms\n", c.B, kernels, std::chrono::duration<double, std::milli>(tc0 - tcs).count(),
+                    std::chrono::duration<double, std::milli>(tc1 - tc0).count(), ran,
+                    std::chrono::duration<double, std::milli>(tc2 - tc1).count());
+        }
+        return ran;
+    } catch (...) {
+        if (exec) cudaGraphExecDestroy(exec);
+        cudaGraphDestroy(graph);
+        throw;
+    }
+}
+
 // returns the number of MCMC iterations run (O.8)
 static int mcmc_phase(Ctx &c, uint32_t outer, double thresh) {
+    if (c.prm.cuda_graphs == 2 && !c.prm.profile && c.nranks == 1) return mcmc_phase_device_loop(c, outer, thresh);
     if (c.prm.cuda_graphs) return mcmc_phase_graph(c, outer, thresh);
     const int V = c.V, nb = c.prm.num_batches, w = c.prm.window;
     const int bs = (V + nb - 1) / nb;

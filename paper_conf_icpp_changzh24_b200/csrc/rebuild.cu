@@ -299,25 +299,34 @@ __global__ void k_row_compact2(const int *__restrict__ M, const int *__restrict_
     }
 }
 
-// ---------------------------------------------------- dense, small B --
-// The whole dense rebuild as ONE persistent cooperative kernel when B <= 221
-// (the B x B histogram fits one CTA's shared memory).  At such B the multi-
-// kernel path (memset, histogram, transpose, stats, scan, compaction) is six
-// launches of a few microseconds of work each; here they are three phases
-// separated by two grid barriers:
-//   P1 every CTA histograms a contiguous edge chunk (four edges per thread
-//      per step, 16-byte loads) in shared memory and adds its non-zeros into
-//      `acc` (zero on entry); din / column counts zeroed      | barrier
-//   P2 one warp per row x: M[x][.] = acc[x][.] (acc row re-zeroed for the
-//      next call), Mt[.][x], row non-zeros and dout; column non-zeros and din
-//      by integer atomics                                     | barrier
-//   P3 one warp per line (rows of M, then rows of Mt = columns of M): its
-//      offset = sum of the preceding lines' non-zeros, then the compaction of
-//      k_row_compact2 (idx, cnt, in-line prefix cum) and rcp = 1 / (d + B).
+// ------------------------------------------------ dense, one kernel --
+// The whole dense rebuild as ONE persistent cooperative kernel (params.dense_coop).
+// The multi-kernel path (memset, histogram, transpose, stats, scan,
+// compaction) is six launches of a few microseconds of work each at the B of
+// the late rounds; here they are phases separated by grid barriers:
+//   SMEM (B <= 221: the B x B histogram fits one CTA's shared memory)
+//     P1 every CTA histograms a contiguous edge chunk (four edges per thread
+//        per step, 16-byte loads, match_any aggregation) in shared memory and
+//        adds its non-zeros into `acc` (zero on entry); line stats zeroed | barrier
+//     P2 one warp per row x: M[x][.] = acc[x][.] (acc row re-zeroed for the
+//        next call), Mt[.][x], row non-zeros and dout; column non-zeros and
+//        din by integer atomics                                           | barrier
+//     P3 one warp per line (rows of M, then rows of Mt = columns of M): its
+//        offset = sum of the preceding lines' non-zeros, then the compaction
+//        (idx, cnt, in-line prefix cum) and rcp = 1 / (d + B).
+//   global (221 < B, B^2 <= dense_cap)
+//     P0 zero M and the line stats                                        | barrier
+//     P1 the same edge loop with L2 atomics straight into M                | barrier
+//     P2 one warp per 32 x 32 tile of M: 32 independent loads, Mt through a
+//        shared-memory tile, line non-zeros and sums by atomics            | barrier
+//     P2b CTA 0 / 1 scan the row / column non-zeros into the pointers      | barrier
+//     P3 compaction at the scanned offsets.
 // Integer arithmetic throughout: the same bits as rebuild_dense.
-constexpr int SMALL_THREADS = 512;
+constexpr int DC_THREADS = 512;
+constexpr int DC_WARPS = DC_THREADS / 32;
+constexpr size_t DC_TILE_SMEM = sizeof(int) * DC_WARPS * 32 * 33;
 
-struct SmallArgs {
+struct DenseArgs {
     int E, B;
     const int *__restrict__ esrc;
     const int *__restrict__ col;
@@ -330,18 +339,66 @@ struct SmallArgs {
     unsigned *bar;
 };
 
-__global__ void __launch_bounds__(SMALL_THREADS) k_rebuild_small(SmallArgs a) {
-    extern __shared__ int h[];
-    const int B = a.B, BB = B * B, E = a.E;
-    const int gtid = blockIdx.x * blockDim.x + threadIdx.x, gthreads = gridDim.x * blockDim.x;
-    const int lane = threadIdx.x & 31, gwarp = gtid >> 5, gwarps = gthreads >> 5;
-    // P1
-    for (int i = gtid; i < B; i += gthreads) {
-        a.din[i] = 0;
-        a.colnnz[i] = 0;
+// exclusive scan of in[0, n) into out[0, n], out[n] = total, by one CTA of DC_THREADS
+GSAP_DEV void dc_cta_scan(const int *in, int *out, int n, int *sh) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int carry = 0;
+    for (int base = 0; base < n; base += DC_THREADS * 8) {
+        int v[8], sm = 0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int idx = base + threadIdx.x * 8 + i;
+            v[i] = idx < n ? __ldcg(in + idx) : 0;
+            sm += v[i];
+        }
+        const int x = warp_incl_scan(sm);
+        if (lane == 31) sh[w] = x;
+        __syncthreads();
+        int wb = 0, tot = 0;
+        for (int i = 0; i < DC_WARPS; ++i) {
+            const int q = sh[i];
+            if (i < w) wb += q;
+            tot += q;
+        }
+        __syncthreads();
+        int ex = carry + wb + x - sm;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int idx = base + threadIdx.x * 8 + i;
+            if (idx < n) out[idx] = ex;
+            ex += v[i];
+        }
+        carry += tot;
     }
-    for (int i = threadIdx.x; i < BB; i += blockDim.x) h[i] = 0;
-    __syncthreads();
+    if (threadIdx.x == 0) out[n] = carry;
+}
+
+template <bool SMEM>
+__global__ void __launch_bounds__(DC_THREADS) k_rebuild_dense(DenseArgs a) {
+    extern __shared__ int h[];
+    const int B = a.B, E = a.E;
+    const size_t BB = (size_t)B * B;
+    const int gtid = blockIdx.x * blockDim.x + threadIdx.x, gthreads = gridDim.x * blockDim.x;
+    const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5, gwarp = gtid >> 5, gwarps = gthreads >> 5;
+    int *hist = SMEM ? h : a.M;
+    // P0 / P1: line stats zeroed (read again after the next barrier)
+    for (int i = gtid; i < B; i += gthreads) {
+        a.rownnz[i] = 0;
+        a.colnnz[i] = 0;
+        a.dout[i] = 0;
+        a.din[i] = 0;
+    }
+    if (SMEM) {
+        for (int i = threadIdx.x; i < (int)BB; i += blockDim.x) h[i] = 0;
+        __syncthreads();
+    } else {
+        int4 *M4 = reinterpret_cast<int4 *>(a.M);
+        const size_t n4 = BB >> 2;
+        for (size_t i = gtid; i < n4; i += gthreads) M4[i] = make_int4(0, 0, 0, 0);
+        for (size_t i = (n4 << 2) + gtid; i < BB; i += gthreads) a.M[i] = 0;
+        grid_sync(a.bar);
+    }
+    // P1: histogram of (b[src], b[dst]) over a contiguous edge chunk per CTA
     const long long chunk = ((((long long)E + gridDim.x - 1) / gridDim.x) + 3) & ~3LL;
     const long long lo = (long long)blockIdx.x * chunk;
     const long long hi = min((long long)E, lo + chunk);
@@ -372,71 +429,134 @@ __global__ void __launch_bounds__(SMALL_THREADS) k_rebuild_small(SmallArgs a) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
             if (a.wgt) {
-                if (key[k] >= 0) atomicAdd(h + key[k], w[k]);
+                if (key[k] >= 0) atomicAdd(hist + key[k], w[k]);
             } else {
                 const unsigned peers = __match_any_sync(FULL, key[k]);
-                if (key[k] >= 0 && lane == __ffs(peers) - 1) atomicAdd(h + key[k], __popc(peers));
+                if (key[k] >= 0 && lane == __ffs(peers) - 1) atomicAdd(hist + key[k], __popc(peers));
             }
         }
     }
-    __syncthreads();
-    for (int i = threadIdx.x; i < BB; i += blockDim.x) {
-        const int v = h[i];
-        if (v) atomicAdd(a.acc + i, v);
+    if (SMEM) {
+        __syncthreads();
+        for (int i = threadIdx.x; i < (int)BB; i += blockDim.x) {
+            const int v = h[i];
+            if (v) atomicAdd(a.acc + i, v);
+        }
     }
     grid_sync(a.bar);
-    // P2
-    for (int x = gwarp; x < B; x += gwarps) {
-        int c = 0, sm = 0;
-        for (int y = lane; y < B; y += 32) {
-            const int v = __ldcg(a.acc + (size_t)x * B + y);
-            a.acc[(size_t)x * B + y] = 0;
-            a.M[(size_t)x * B + y] = v;
-            a.Mt[(size_t)y * B + x] = v;
-            if (v) {
-                ++c;
-                sm += v;
-                atomicAdd(a.colnnz + y, 1);
-                atomicAdd(a.din + y, v);
+    // P2 (SMEM, small B): one warp per row x -- M[x][.] = acc[x][.] (acc row
+    // re-zeroed), Mt[.][x], row non-zeros / dout; columns by atomics
+    if (SMEM) {
+        for (int x = gwarp; x < B; x += gwarps) {
+            int c = 0, sm = 0;
+            for (int y = lane; y < B; y += 32) {
+                const int v = __ldcg(a.acc + (size_t)x * B + y);
+                a.acc[(size_t)x * B + y] = 0;
+                a.M[(size_t)x * B + y] = v;
+                a.Mt[(size_t)y * B + x] = v;
+                if (v) {
+                    ++c;
+                    sm += v;
+                    atomicAdd(a.colnnz + y, 1);
+                    atomicAdd(a.din + y, v);
+                }
+            }
+            c = __reduce_add_sync(FULL, c);
+            sm = __reduce_add_sync(FULL, sm);
+            if (lane == 0) {
+                a.rownnz[x] = c;
+                a.dout[x] = sm;
             }
         }
-        c = __reduce_add_sync(FULL, c);
-        sm = __reduce_add_sync(FULL, sm);
-        if (lane == 0) {
-            a.rownnz[x] = c;
-            a.dout[x] = sm;
+    }
+    // P2 (global, larger B): 32 x 32 tiles, one warp each
+    if (!SMEM) {
+        const int nt = (B + 31) >> 5;
+        int *tile = h + wl * (32 * 33);   // the histogram's shared memory is free again
+        const int *src = SMEM ? a.acc : a.M;
+        for (int t = gwarp; t < nt * nt; t += gwarps) {
+            const int x0 = (t / nt) << 5, y0 = (t % nt) << 5, y = y0 + lane;
+            const int rows = min(32, B - x0);
+            int v[32];
+#pragma unroll
+            for (int i = 0; i < 32; ++i)   // 32 independent loads in flight
+                v[i] = (i < rows && y < B) ? __ldcg(src + (size_t)(x0 + i) * B + y) : 0;
+            int cn = 0, cs = 0;
+#pragma unroll
+            for (int i = 0; i < 32; ++i) {
+                if (SMEM && i < rows && y < B) {
+                    const size_t at = (size_t)(x0 + i) * B + y;
+                    a.M[at] = v[i];
+                    a.acc[at] = 0;
+                }
+                tile[i * 33 + lane] = v[i];
+                const int rn = __reduce_add_sync(FULL, v[i] != 0 ? 1 : 0);
+                const int rs = __reduce_add_sync(FULL, v[i]);
+                if (lane == i && rn) {   // row i's sums, one lane each
+                    atomicAdd(a.rownnz + x0 + i, rn);
+                    atomicAdd(a.dout + x0 + i, rs);
+                }
+                cn += v[i] != 0;
+                cs += v[i];
+            }
+            if (y < B && cn) {
+                atomicAdd(a.colnnz + y, cn);
+                atomicAdd(a.din + y, cs);
+            }
+            __syncwarp();
+            const int xx = x0 + lane;
+            for (int i = 0; i < 32 && y0 + i < B; ++i)
+                if (xx < B) a.Mt[(size_t)(y0 + i) * B + xx] = tile[lane * 33 + i];
+            __syncwarp();
         }
     }
     grid_sync(a.bar);
+    if (!SMEM) {   // P2b
+        if (blockIdx.x < 2) {
+            dc_cta_scan(blockIdx.x ? a.colnnz : a.rownnz, blockIdx.x ? a.ptrB : a.ptrA, B, h);
+            if (blockIdx.x == 0 && threadIdx.x == 0) *a.d_nnz = a.ptrA[B];
+        }
+        grid_sync(a.bar);
+    }
     // P3
     for (int x2 = gwarp; x2 < 2 * B; x2 += gwarps) {
         const bool t = x2 >= B;
         const int x = t ? x2 - B : x2;
-        const int *nz = t ? a.colnnz : a.rownnz;
-        int off = 0;
-        for (int y = lane; y < x; y += 32) off += __ldcg(nz + y);
-        off = __reduce_add_sync(FULL, off);
         int *__restrict__ ptr = t ? a.ptrB : a.ptrA;
-        if (lane == 0) {
-            ptr[x] = off;
-            if (x == B - 1) {
-                const int tot = off + __ldcg(nz + x);
-                ptr[B] = tot;
-                if (!t) *a.d_nnz = tot;
+        int off;
+        if (SMEM) {
+            const int *nz = t ? a.colnnz : a.rownnz;
+            off = 0;
+            for (int y = lane; y < x; y += 32) off += __ldcg(nz + y);
+            off = __reduce_add_sync(FULL, off);
+            if (lane == 0) {
+                ptr[x] = off;
+                if (x == B - 1) {
+                    const int tot = off + __ldcg(nz + x);
+                    ptr[B] = tot;
+                    if (!t) *a.d_nnz = tot;
+                }
             }
-            if (!t) a.rcp[x] = 1.0 / ((double)__ldcg(a.dout + x) + (double)__ldcg(a.din + x) + (double)B);
+        } else {
+            off = __ldcg(ptr + x);
         }
+        if (!t && lane == 0)
+            a.rcp[x] = 1.0 / ((double)__ldcg(a.dout + x) + (double)__ldcg(a.din + x) + (double)B);
         const int *R = (t ? a.Mt : a.M) + (size_t)x * B;
         int *__restrict__ idx = t ? a.idxB : a.idxA;
         int *__restrict__ cnt = t ? a.cntB : a.cntA;
         int *__restrict__ cum = t ? a.cumB : a.cumA;
         int base = off, run = 0;
+        int nxt[4];   // the next step's entries, loaded one step ahead
+#pragma unroll
+        for (int k = 0; k < 4; ++k) nxt[k] = 4 * lane + k < B ? __ldcg(R + 4 * lane + k) : 0;
         for (int y0 = 0; y0 < B; y0 += 128) {
             const int y = y0 + 4 * lane;
             int v[4], nzc = 0, s4 = 0;
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
-                v[k] = y + k < B ? __ldcg(R + y + k) : 0;
+                v[k] = nxt[k];
+                nxt[k] = y + 128 + k < B ? __ldcg(R + y + 128 + k) : 0;
                 nzc += v[k] != 0;
                 s4 += v[k];
             }
@@ -458,8 +578,9 @@ __global__ void __launch_bounds__(SMALL_THREADS) k_rebuild_small(SmallArgs a) {
     }
 }
 
-static void rebuild_dense_small(Ctx &c) {
-    SmallArgs a;
+template <bool SMEM>
+static void launch_rebuild_dense_coop(Ctx &c) {
+    DenseArgs a;
     a.E = c.E;
     a.B = c.B;
     a.esrc = c.esrc; a.col = c.col; a.wgt = c.wgt; a.b = c.b;
@@ -470,27 +591,29 @@ static void rebuild_dense_small(Ctx &c) {
     a.rcp = c.rcp;
     a.d_nnz = c.d_nnz;
     a.bar = c.coop_bar;
+    const size_t smem_max = SMEM ? std::max(DC_TILE_SMEM, sizeof(int) * SMALL_MAX_B * SMALL_MAX_B) : DC_TILE_SMEM;
     static int grid = 0;
     if (grid == 0) {
-        const int smem_max = SMALL_MAX_B * SMALL_MAX_B * 4;
-        GSAP_CUDA(cudaFuncSetAttribute(k_rebuild_small, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max));
+        GSAP_CUDA(cudaFuncSetAttribute(k_rebuild_dense<SMEM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)smem_max));
         int per_sm = 0, sms = 0, dev = 0;
-        GSAP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rebuild_small, SMALL_THREADS, smem_max));
+        GSAP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rebuild_dense<SMEM>, DC_THREADS,
+                                                                smem_max));
         GSAP_CUDA(cudaGetDevice(&dev));
         GSAP_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-        grid = std::max(1, std::min(per_sm, 1) * sms);
+        grid = std::max(1, std::min(per_sm, SMEM ? 1 : 2) * sms);
     }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
-    cfg.blockDim = dim3(SMALL_THREADS);
-    cfg.dynamicSmemBytes = sizeof(int) * (size_t)c.B * c.B;
+    cfg.blockDim = dim3(DC_THREADS);
+    cfg.dynamicSmemBytes = SMEM ? std::max(DC_TILE_SMEM, sizeof(int) * (size_t)c.B * c.B) : DC_TILE_SMEM;
     cfg.stream = c.stream;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeCooperative;
     attr[0].val.cooperative = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    GSAP_CUDA(cudaLaunchKernelEx(&cfg, k_rebuild_small, a));
+    GSAP_CUDA(cudaLaunchKernelEx(&cfg, k_rebuild_dense<SMEM>, a));
     ++c.launches;
 }
 
@@ -654,8 +777,10 @@ void rebuild(Ctx &c) {
     kc_begin(c, c.k_rebuild, &ev);
     c.dense_mode = dense_ok(c, c.B);
     c.padded = false;   // set by the multi-kernel sparse path
-    if (c.dense_mode && c.small_acc && c.B <= SMALL_MAX_B) {
-        rebuild_dense_small(c);
+    if (c.dense_mode && c.prm.dense_coop && c.E > 0 && c.B <= SMALL_MAX_B) {
+        launch_rebuild_dense_coop<true>(c);
+    } else if (c.dense_mode && c.prm.dense_coop == 2 && c.E > 0) {
+        launch_rebuild_dense_coop<false>(c);   // measured slower than the multi-kernel path above B = 221
     } else if (c.dense_mode) {
         rebuild_dense(c);   // rcp written by the compaction
     } else {

@@ -30,7 +30,9 @@ SPARSE = {"dense_max_B": 1}     # force the sparse (CSR-line) blockmodel regime
 SPARSE_MK = {"dense_max_B": 1, "sparse_coop": 0}
 # the dense regime (B <= 221) through the multi-kernel rebuild instead of the persistent one
 DENSE_MK = {"dense_coop": 0}
-REGIMES = {"auto": {}, "sparse": SPARSE, "sparse_mk": SPARSE_MK, "dense_mk": DENSE_MK}
+# the persistent dense rebuild for every dense B (L2-atomic variant above B = 221)
+DENSE_COOP2 = {"dense_coop": 2}
+REGIMES = {"auto": {}, "sparse": SPARSE, "sparse_mk": SPARSE_MK, "dense_mk": DENSE_MK, "dense_coop2": DENSE_COOP2}
 
 
 def make_pair(G, oracle_mod, rowptr, col, wgt=None, **params):
@@ -59,7 +61,7 @@ GRAPHS = {
 }
 
 
-@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk", "dense_mk"])
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sparse_mk", "dense_mk", "dense_coop2"])
 @pytest.mark.parametrize("gname", list(GRAPHS))
 @pytest.mark.parametrize("B", [1, 2, 7, 11, 150, 221, 222, 299, 300])
 def test_rebuild_bit_exact(G, oracle_mod, gname, B, regime):
@@ -345,3 +347,17 @@ def test_end_to_end_5k_layer3(G, oracle_mod):
     assert abs(pg - po) <= 0.02 and abs(rg - ro) <= 0.02
     print("5K: GPU B", res["B"], "NMI", metrics.nmi(truth, res["b"]), "oracle B", ref["B"],
           "NMI", metrics.nmi(truth, ref["b"]))
+
+
+def test_device_loop_graph_matches_host_loop(G):
+    """cuda_graphs = 2 (whole MCMC phase one graph launch, convergence test on the
+    device) takes exactly the decisions of the host-driven loop (cuda_graphs = 1)."""
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    out = []
+    for g in (1, 2, 0):
+        ctx = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED, cuda_graphs=g))
+        r = ctx.gsap_run()
+        st = ctx.gsap_get_stats()
+        out.append((r["B"], r["mdl"], st["mcmc_itr_total"], r["rounds"], r["b"].tobytes()))
+        ctx.close()
+    assert out[0] == out[1] == out[2]

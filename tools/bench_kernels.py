@@ -21,6 +21,7 @@ ap.add_argument("--rounds", type=int, nargs="+", default=[1, 3, 5, 8, 19])
 ap.add_argument("--batches", type=int, default=16)
 ap.add_argument("--json", default=None)
 ap.add_argument("--dense-max-B", type=int, default=0)
+ap.add_argument("--param", action="append", default=[], help="extra gsap_params field=value (repeatable)")
 ap.add_argument("--profile-range", action="store_true",
                 help="cudaProfilerStart/Stop around the timed batches (ncu --profile-from-start off)")
 a = ap.parse_args()
@@ -33,7 +34,8 @@ from paper_conf_icpp_changzh24_b200 import gsap  # noqa: E402
 rowptr, col, truth, cfg = dcsbm.make(a.config)
 out = []
 for R in a.rounds:
-    prm = gsap.gsap_default_params(seed=dcsbm.RUN_SEED, profile=1, max_rounds=R, dense_max_B=a.dense_max_B)
+    extra = {k: int(v) for k, v in (p.split("=") for p in a.param)}
+    prm = gsap.gsap_default_params(seed=dcsbm.RUN_SEED, profile=1, max_rounds=R, dense_max_B=a.dense_max_B, **extra)
     ctx = gsap.Context(rowptr, col, params=prm)
     ctx.gsap_run()
     B = ctx.B
