@@ -44,7 +44,7 @@ struct CoopArgs {
     CoopSide sd[2];
     double *rcp;
     int *d_nnz;
-    int *nlong;       // [2] long lines per side
+    int *nlong;       // [3] long lines per side, short-line work counter
     unsigned *bar;    // [2] barrier: arrivals, generation
 };
 
@@ -136,7 +136,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             if (x < B) a.sd[q].deg[x] = 0;
         }
     }
-    if (gtid < 2) a.nlong[gtid] = 0;
+    if (gtid < 3) a.nlong[gtid] = 0;   // [0, 1] long lines per side, [2] P4a work counter
     grid_sync(a.bar);
     // P1
     for (int v = gtid; v < V; v += gthreads) {
@@ -160,61 +160,16 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             a.rcp[x] = 1.0 / ((double)a.sd[0].deg[x] + (double)a.sd[1].deg[x] + (double)B);
     }
     grid_sync(a.bar);
-    // P3: scatter (warp per (side, vertex))
-    for (int task = gwarp; task < 2 * V; task += gwarps) {
-        const int q = task >= V, v = q ? task - V : task;
-        const CoopSide &sd = a.sd[q];
-        K *seg = reinterpret_cast<K *>(sd.seg);
-        const int lo = __ldg(sd.gptr + v), n = __ldg(sd.gptr + v + 1) - lo;
-        if (n == 0) continue;
-        const int x = __ldg(a.b + v);
-        int base = 0;
-        if (lane == 0) base = sd.off[x] + atomicAdd(sd.cur + x, n);
-        base = __shfl_sync(FULL, base, 0);
-        for (int j = lane; j < n; j += 32) {
-            const int t = __ldg(a.b + __ldg(sd.gidx + lo + j));
-            if (sizeof(K) == 8)
-                seg[base + j] = (K)(((unsigned long long)(unsigned)t << 32) | (unsigned)__ldg(sd.gw + lo + j));
-            else
-                seg[base + j] = (K)(unsigned)t;
-        }
+    // P3: scatter, 32 (side, vertex) tasks per warp step (segsort.cuh scatter_batched)
+    {
+        const ScatterSide<K> s0{a.sd[0].gptr, a.sd[0].gidx, a.sd[0].gw, a.sd[0].off, a.sd[0].cur,
+                                reinterpret_cast<K *>(a.sd[0].seg)};
+        const ScatterSide<K> s1{a.sd[1].gptr, a.sd[1].gidx, a.sd[1].gw, a.sd[1].off, a.sd[1].cur,
+                                reinterpret_cast<K *>(a.sd[1].seg)};
+        scatter_batched<K>(s0, s1, 2, V, a.b, gwarp, gwarps);
     }
     grid_sync(a.bar);
-    // P4a: short lines, one warp each (bitonic in shared memory + RLE)
-    for (int task = gwarp; task < 2 * B; task += gwarps) {
-        const int q = task >= B, x = q ? task - B : task;
-        const CoopSide &sd = a.sd[q];
-        const int o = sd.off[x], L = sd.off[x + 1] - o;
-        if (L > SEG_WARP_MAX) continue;
-        if (L == 0) {
-            if (lane == 0) {
-                sd.nnz[x] = 0;
-                sd.end[x] = o;
-            }
-            continue;
-        }
-        const LineOut out{sd.cum, sd.end, sd.deg};
-        const K *seg = reinterpret_cast<const K *>(sd.seg);
-        if (L <= 128) {   // short lines: bitonic in registers, RLE in registers
-            int u;
-            if (L <= 32) u = warp_segsort_rle<K, 1>(seg + o, L, sd.tcol + o, sd.tcnt + o);
-            else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, sd.tcol + o, sd.tcnt + o);
-            else u = warp_segsort_rle<K, 4>(seg + o, L, sd.tcol + o, sd.tcnt + o);
-            if (lane == 0) sd.nnz[x] = u;
-            line_epilogue<32>(out, sd.tcnt, o, u, L, x, lane, nullptr);
-            continue;
-        }
-        int n = 1;
-        while (n < L) n <<= 1;
-        for (int i = lane; i < n; i += 32) S.warp.keys[wl][i] = i < L ? seg[o + i] : key_max<K>();
-        __syncwarp();
-        bitonic<K, 32>(S.warp.keys[wl], n, lane);
-        const int u = rle_runs<K, 32>(S.warp.keys[wl], L, S.warp.hp[wl], sd.tcol + o, sd.tcnt + o, lane, nullptr);
-        if (lane == 0) sd.nnz[x] = u;
-        line_epilogue<32>(out, sd.tcnt, o, u, L, x, lane, nullptr);
-    }
-    __syncthreads();   // the shared memory changes role
-    // P4b: long lines, one CTA each
+    // P4b: long lines first, one CTA each (static: CTA i takes long lines i, i + grid, ...)
     {
         const int n0 = a.nlong[0], n1 = a.nlong[1];
         for (int li = blockIdx.x; li < n0 + n1; li += gridDim.x) {
@@ -239,6 +194,49 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             }
             if (threadIdx.x == 0) sd.nnz[x] = u;
             __syncthreads();
+        }
+    }
+    __syncthreads();   // the shared memory changes role
+    // P4a: short lines, one warp each (bitonic + RLE in registers / shared
+    // memory), fetched two at a time from a work counter: warps of CTAs that
+    // sorted a long line first join late, the others keep going -- the phase
+    // ends within ~one line of the slowest warp
+    for (;;) {
+        int t0 = 0;
+        if (lane == 0) t0 = atomicAdd(a.nlong + 2, 2);
+        t0 = __shfl_sync(FULL, t0, 0);
+        if (t0 >= 2 * B) break;
+        for (int task = t0; task < min(t0 + 2, 2 * B); ++task) {
+            const int q = task >= B, x = q ? task - B : task;
+            const CoopSide &sd = a.sd[q];
+            const int o = sd.off[x], L = sd.off[x + 1] - o;
+            if (L > SEG_WARP_MAX) continue;
+            if (L == 0) {
+                if (lane == 0) {
+                    sd.nnz[x] = 0;
+                    sd.end[x] = o;
+                }
+                continue;
+            }
+            const LineOut out{sd.cum, sd.end, sd.deg};
+            const K *seg = reinterpret_cast<const K *>(sd.seg);
+            if (L <= 128) {   // short lines: bitonic in registers, RLE in registers
+                int u;
+                if (L <= 32) u = warp_segsort_rle<K, 1>(seg + o, L, sd.tcol + o, sd.tcnt + o);
+                else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, sd.tcol + o, sd.tcnt + o);
+                else u = warp_segsort_rle<K, 4>(seg + o, L, sd.tcol + o, sd.tcnt + o);
+                if (lane == 0) sd.nnz[x] = u;
+                line_epilogue<32>(out, sd.tcnt, o, u, L, x, lane, nullptr);
+                continue;
+            }
+            int n = 1;
+            while (n < L) n <<= 1;
+            for (int i = lane; i < n; i += 32) S.warp.keys[wl][i] = i < L ? seg[o + i] : key_max<K>();
+            __syncwarp();
+            bitonic<K, 32>(S.warp.keys[wl], n, lane);
+            const int u = rle_runs<K, 32>(S.warp.keys[wl], L, S.warp.hp[wl], sd.tcol + o, sd.tcnt + o, lane, nullptr);
+            if (lane == 0) sd.nnz[x] = u;
+            line_epilogue<32>(out, sd.tcnt, o, u, L, x, lane, nullptr);
         }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *a.d_nnz = a.sd[0].off[B];   // the extent E (padding has cnt 0)

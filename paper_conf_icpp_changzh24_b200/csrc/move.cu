@@ -358,63 +358,106 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
     const int r = __ldg(a.b + v);
     const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
     const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
-    int s;
-    if (a.propose) {
-        s = propose_warp<WEIGHTED>(a, v, w, deg, tb);
-        if (lane == 0) a.s_out[i] = s;
-    } else {
-        s = a.s_in[i];
+    const int B = a.m.B;
+    // ---- (a1) first half of the proposal (R:O.4): the neighbour's block u
+    // comes from the adjacency registers; every load the walk over row /
+    // column u needs is issued now, so it overlaps the histogram below
+    const bool fast = a.propose && !WEIGHTED && deg <= 128 && deg > 0;
+    int u = 0, dout_u = 0, din_u = 0, rlo = 0, rhi = 0, clo = 0, chi = 0;
+    if (fast) {
+        const uint32_t p = pick(w.x, (uint32_t)deg);
+        const int c = (int)(p >> 5);
+        const int x = c == 0 ? tb[0] : c == 1 ? tb[1] : c == 2 ? tb[2] : tb[3];
+        u = __shfl_sync(FULL, x, (int)(p & 31u));
+        dout_u = __ldg(a.m.dout + u);
+        din_u = __ldg(a.m.din + u);
+        rlo = __ldg(a.m.rowptr + u);
+        rhi = __ldg(a.m.rowend + u);
+        clo = __ldg(a.m.colptr + u);
+        chi = __ldg(a.m.colend + u);
     }
+    // ---- phase A: histogram of v's neighbour blocks (self-loop excluded),
+    // independent of the proposal; unique blocks compacted into `list`
+    int keep[4];
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+        keep[c] = -1;
+        const int j = c * 32 + lane;
+        if (nb[c] >= 0 && nb[c] != v) {
+            const bool out = j < nout;
+            const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
+            const int sl = tab_insert(tab, WARP_TAB_LOG2, tb[c]);
+            atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
+            atomicMin(&tab[sl].w, j);
+            keep[c] = sl;
+        }
+    }
+    for (int j = 128 + lane; j < deg; j += 32) {   // only when B <= 128 (<= B keys)
+        const bool out = j < nout;
+        const int n = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+        if (n == v) continue;
+        const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
+        const int sl = tab_insert(tab, WARP_TAB_LOG2, __ldg(a.b + n));
+        atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
+        atomicMin(&tab[sl].w, j);
+    }
+    __syncwarp();
+    int nuniq = 0;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+        const int sl = keep[c];
+        const bool own = sl >= 0 && tab[sl].w == c * 32 + lane;
+        const unsigned bal = __ballot_sync(FULL, own);
+        if (own) list[nuniq + __popc(bal & lt)] = sl;
+        nuniq += __popc(bal);
+    }
+    for (int base = 128; base < deg; base += 32) {
+        const int j = base + lane;
+        int sl = -1;
+        if (j < deg) {
+            const int n = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+            if (n != v) sl = tab_find(tab, WARP_TAB_LOG2, __ldg(a.b + n));
+        }
+        const bool own = sl >= 0 && tab[sl].w == j;
+        const unsigned bal = __ballot_sync(FULL, own);
+        if (own) list[nuniq + __popc(bal & lt)] = sl;
+        nuniq += __popc(bal);
+    }
+    __syncwarp();
+    // r-side entries of this lane's first unique block (dense regime), also
+    // independent of the proposal
+    int4 e0 = make_int4(-1, 0, 0, 0);
+    int Mrt0 = 0, Mtr0 = 0;
+    double rt0 = 0.0;
+    const int *__restrict__ D = a.m.dense;   // non-null iff DENSE
+    if (lane < nuniq) {
+        e0 = tab[list[lane]];
+        if (DENSE) {
+            Mrt0 = __ldg(D + (size_t)r * B + e0.x);
+            Mtr0 = __ldg(D + (size_t)e0.x * B + r);
+            rt0 = __ldg(a.m.rcp + e0.x);
+        }
+    }
+    // ---- (a1) second half: coin, then the walk
+    int s;
+    if (!a.propose) {
+        s = a.s_in[i];
+    } else if (fast) {
+        const uint32_t du = (uint32_t)(dout_u + din_u);
+        if (coin_random(w.y, (uint32_t)B, du)) {
+            s = (int)pick(w.z, (uint32_t)B);
+        } else {
+            const long long q = (long long)pick(w.z, du);
+            if (q < dout_u) s = __ldg(a.m.col + warp_upper_bound(a.m.cum, rlo, rhi, q));
+            else s = __ldg(a.m.row + warp_upper_bound(a.m.ccum, clo, chi, q - dout_u));
+        }
+    } else {
+        s = propose_warp<WEIGHTED>(a, v, w, deg, tb);
+    }
+    if (a.propose && lane == 0) a.s_out[i] = s;
     double dS = 0.0, H = 1.0;
     bool acc = false;
     if (s != r) {
-        // ---- phase A: histogram of v's neighbour blocks (self-loop excluded)
-        int keep[4];
-#pragma unroll
-        for (int c = 0; c < 4; ++c) {
-            keep[c] = -1;
-            const int j = c * 32 + lane;
-            if (nb[c] >= 0 && nb[c] != v) {
-                const bool out = j < nout;
-                const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
-                const int sl = tab_insert(tab, WARP_TAB_LOG2, tb[c]);
-                atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
-                atomicMin(&tab[sl].w, j);
-                keep[c] = sl;
-            }
-        }
-        for (int j = 128 + lane; j < deg; j += 32) {   // only when B <= 128 (<= B keys)
-            const bool out = j < nout;
-            const int n = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-            if (n == v) continue;
-            const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
-            const int sl = tab_insert(tab, WARP_TAB_LOG2, __ldg(a.b + n));
-            atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
-            atomicMin(&tab[sl].w, j);
-        }
-        __syncwarp();
-        int nuniq = 0;
-#pragma unroll
-        for (int c = 0; c < 4; ++c) {
-            const int sl = keep[c];
-            const bool own = sl >= 0 && tab[sl].w == c * 32 + lane;
-            const unsigned bal = __ballot_sync(FULL, own);
-            if (own) list[nuniq + __popc(bal & lt)] = sl;
-            nuniq += __popc(bal);
-        }
-        for (int base = 128; base < deg; base += 32) {
-            const int j = base + lane;
-            int sl = -1;
-            if (j < deg) {
-                const int n = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-                if (n != v) sl = tab_find(tab, WARP_TAB_LOG2, __ldg(a.b + n));
-            }
-            const bool own = sl >= 0 && tab[sl].w == j;
-            const unsigned bal = __ballot_sync(FULL, own);
-            if (own) list[nuniq + __popc(bal & lt)] = sl;
-            nuniq += __popc(bal);
-        }
-        __syncwarp();
         // ---- core state
         const int slr = tab_find(tab, WARP_TAB_LOG2, r), sls = tab_find(tab, WARP_TAB_LOG2, s);
         const int o_r = slr >= 0 ? tab[slr].y : 0, i_r = slr >= 0 ? tab[slr].z : 0;
@@ -422,8 +465,6 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
         const int kout = __ldg(a.kout + v), kin = __ldg(a.kin + v), l = __ldg(a.selfw + v);
         const int dout_r = __ldg(a.m.dout + r), dout_s = __ldg(a.m.dout + s);
         const int din_r = __ldg(a.m.din + r), din_s = __ldg(a.m.din + s);
-        const int *__restrict__ D = a.m.dense;   // non-null iff DENSE
-        const int B = a.m.B;
         int Mrr, Mrs, Msr, Mss;
         Line Ln[4];   // sparse: row r, row s, column r, column s of M
         if (DENSE) {
@@ -453,7 +494,7 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
         // ---- phase B: one unique neighbour block per lane
         double accS = 0.0, pf = 0.0, pb = 0.0;
         for (int k = lane; k < nuniq; k += 32) {
-            const int4 e = tab[list[k]];
+            const int4 e = k == lane ? e0 : tab[list[k]];
             const int t = e.x, ot = e.y, it = e.z;
             const double cw = (double)(ot + it);
             if (t == r) {
@@ -464,10 +505,18 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
                 pb += cw * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd);
             } else {
                 int Mrt, Mst, Mtr, Mts;
+                double rt;
                 if (DENSE) {
-                    Mrt = __ldg(D + (size_t)r * B + t);
+                    if (k == lane) {
+                        Mrt = Mrt0;
+                        Mtr = Mtr0;
+                        rt = rt0;
+                    } else {
+                        Mrt = __ldg(D + (size_t)r * B + t);
+                        Mtr = __ldg(D + (size_t)t * B + r);
+                        rt = __ldg(rcp + t);
+                    }
                     Mst = __ldg(D + (size_t)s * B + t);
-                    Mtr = __ldg(D + (size_t)t * B + r);
                     Mts = __ldg(D + (size_t)t * B + s);
                 } else {
                     const int yt[4] = {t, t, t, t};
@@ -477,8 +526,8 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
                     Mst = o4[1];
                     Mtr = o4[2];
                     Mts = o4[3];
+                    rt = __ldg(rcp + t);
                 }
-                const double rt = __ldg(rcp + t);
                 accS -= df_t(ft, Mrt, -ot) + df_t(ft, Mst, ot) + df_t(ft, Mtr, -it) + df_t(ft, Mts, it);
                 pf += cw * (double)(Mts + Mst + 1) * rt;
                 pb += cw * (double)(Mtr - it + Mrt - ot + 1) * rt;
@@ -500,14 +549,14 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
         accS = warp_sum(accS);
         pf = warp_sum(pf);
         pb = warp_sum(pb);
-        // leave the table empty: exactly the listed slots were used
-        for (int k = lane; k < nuniq; k += 32) tab[list[k]] = make_int4(-1, 0, 0, 0x7fffffff);
-        __syncwarp();
         dS = accS;
         H = (kout + kin == 0) ? 1.0 : pb / pf;
         const double p = exp(-a.beta * dS) * H;
         acc = ((double)w.w + 0.5) * (1.0 / 4294967296.0) <= p;
     }
+    // leave the table empty: exactly the listed slots were used
+    for (int k = lane; k < nuniq; k += 32) tab[list[k]] = make_int4(-1, 0, 0, 0x7fffffff);
+    __syncwarp();
     if (lane == 0) {
         if (a.dS) a.dS[i] = dS;
         if (a.H) a.H[i] = H;

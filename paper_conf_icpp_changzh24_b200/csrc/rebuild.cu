@@ -194,7 +194,8 @@ __global__ void k_row_stats2(const int *__restrict__ M, const int *__restrict__ 
         const int x = t ? x2 - B : x2;
         const int *__restrict__ R = (t ? Mt : M) + (size_t)x * B;
         int c = 0, s = 0;
-        for (int y0 = 4 * lane; y0 < B; y0 += 128) {
+#pragma unroll 4
+        for (int y0 = 4 * lane; y0 < B; y0 += 128) {   // independent loads: unrolled, in flight together
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
                 const int v = y0 + k < B ? __ldg(R + y0 + k) : 0;
@@ -272,12 +273,16 @@ __global__ void k_row_compact2(const int *__restrict__ M, const int *__restrict_
         int *__restrict__ cum = t ? cumB : cumA;
         int base = (t ? ptrB : ptrA)[x], run = 0;
         if (!t && lane == 0) rcp[x] = 1.0 / ((double)dout[x] + (double)din[x] + (double)B);
+        int nxt[4];   // the next step's entries, loaded one step ahead
+#pragma unroll
+        for (int k = 0; k < 4; ++k) nxt[k] = 4 * lane + k < B ? __ldg(R + 4 * lane + k) : 0;
         for (int y0 = 0; y0 < B; y0 += 128) {
             const int y = y0 + 4 * lane;
             int v[4], nz = 0, sm = 0;
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
-                v[k] = y + k < B ? __ldg(R + y + k) : 0;
+                v[k] = nxt[k];
+                nxt[k] = y + 128 + k < B ? __ldg(R + y + 128 + k) : 0;
                 nz += v[k] != 0;
                 sm += v[k];
             }
@@ -675,8 +680,8 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     k_line_len<<<grid_for(V, 256), 256, 0, c.stream>>>(V, gptr, c.b, c.seg_len);
     ++c.launches;
     device_scan<int>(c.seg_len, ptr, nullptr, B, false, c.scan_tmp, ptr + B, L);
-    k_line_scatter<K><<<grid_for((long long)V * 32, 256), 256, 0, c.stream>>>(V, gptr, gidx, gw, c.b, ptr,
-                                                                             c.seg_cur, seg);
+    k_line_scatter_batched<K><<<grid_for((long long)V, 256), 256, 0, c.stream>>>(V, gptr, gidx, gw, c.b, ptr,
+                                                                                c.seg_cur, seg);
     const LineOut out{cum, end, deg};
     k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, ptr, c.seg_nnz, c.seg_listW, c.seg_listC,
                                                            c.seg_ctr, out, extent);

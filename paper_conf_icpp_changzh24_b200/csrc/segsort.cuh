@@ -5,8 +5,8 @@
 //   1. line lengths: len[b[v]] += deg(v)                  (one atomic per vertex)
 //   2. offsets: exclusive scan of len
 //   3. scatter: each vertex appends the blocks of its neighbours to its line's
-//      segment (one atomic per vertex, coalesced writes; the order inside a
-//      segment is arbitrary, the sort below makes it canonical)
+//      segment (one atomic per vertex, 32 vertices per warp step; the order
+//      inside a segment is arbitrary, the sort below makes it canonical)
 //   4. per segment: sort + run-length encode (a warp for <= 512 entries, a CTA
 //      in shared memory for <= 4096, a CTA in global scratch beyond); the runs
 //      stay at the segment offset (padded CSR: end[x], cum, line sums and
@@ -165,25 +165,88 @@ __global__ void k_line_len(int V, const int *__restrict__ gptr, const int *__res
     }
 }
 
-// 3. scatter neighbour blocks into their line's segment (warp per vertex)
+// 3'. the scatter as warp-batched tasks (task = (side, vertex), sides 0..nsides-1
+// of V vertices each): lane l claims task (base + l)'s slot range with one
+// atomic -- 32 claims in flight instead of one per warp step -- then the warp
+// copies the 32 tasks' entries flattened (lane-parallel over the batch's
+// entries, owner task found by a 5-step search over the lanes' offsets), so
+// every lane has an independent gather in flight.
 template <typename K>
-__global__ void k_line_scatter(int V, const int *__restrict__ gptr, const int *__restrict__ gidx,
-                               const int *__restrict__ gw, const int *__restrict__ b,
-                               const int *__restrict__ off, int *__restrict__ cur, K *__restrict__ seg) {
+struct ScatterSide {
+    const int *__restrict__ gptr;
+    const int *__restrict__ gidx;
+    const int *__restrict__ gw;
+    const int *off;   // written earlier in the same kernel (coop): plain loads
+    int *cur;
+    K *seg;
+};
+
+template <typename K>
+GSAP_DEV void scatter_batched(const ScatterSide<K> &s0, const ScatterSide<K> &s1, int nsides, int V,
+                              const int *__restrict__ b, int gwarp, int gwarps) {
     const int lane = threadIdx.x & 31;
-    for (int v = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < V; v += (gridDim.x * blockDim.x) >> 5) {
-        const int lo = __ldg(gptr + v), n = __ldg(gptr + v + 1) - lo;
-        if (n == 0) continue;
-        const int x = __ldg(b + v);
-        int base = 0;
-        if (lane == 0) base = __ldg(off + x) + atomicAdd(cur + x, n);
-        base = __shfl_sync(FULL, base, 0);
-        for (int j = lane; j < n; j += 32) {
-            const int t = __ldg(b + __ldg(gidx + lo + j));
-            if (sizeof(K) == 8) seg[base + j] = (K)(((unsigned long long)(unsigned)t << 32) | (unsigned)__ldg(gw + lo + j));
-            else seg[base + j] = (K)(unsigned)t;
+    const int ntasks = nsides * V;
+    for (int base = gwarp * 32; base < ntasks; base += gwarps * 32) {
+        const int task = base + lane;
+        int q = 0, lo = 0, n = 0, pos = 0;
+        if (task < ntasks) {
+            q = task >= V;
+            const int v = q ? task - V : task;
+            const int *gptr = q ? s1.gptr : s0.gptr;
+            lo = __ldg(gptr + v);
+            n = __ldg(gptr + v + 1) - lo;
+            if (n) {
+                const int x = __ldg(b + v);
+                pos = (q ? s1.off : s0.off)[x] + atomicAdd((q ? s1.cur : s0.cur) + x, n);
+            }
+        }
+        const int incl = warp_incl_scan(n);
+        const int total = __shfl_sync(FULL, incl, 31);
+        const int excl = incl - n;
+        constexpr int U = 4;   // entries per lane per step: U independent gathers in flight
+        for (int f0 = 0; f0 < total; f0 += 32 * U) {
+            int src[U], dst[U], wq[U], nbr[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int f = f0 + u * 32 + lane;
+                int t = 0;   // the last lane whose offset is <= f owns entry f
+#pragma unroll
+                for (int step = 16; step >= 1; step >>= 1) {
+                    const int cand = t + step;
+                    const int ex = __shfl_sync(FULL, excl, cand & 31);
+                    if (cand < 32 && ex <= f) t = cand;
+                }
+                const int tq = __shfl_sync(FULL, q, t), tlo = __shfl_sync(FULL, lo, t);
+                const int tpos = __shfl_sync(FULL, pos, t), tex = __shfl_sync(FULL, excl, t);
+                wq[u] = f < total ? tq : -1;
+                src[u] = tlo + f - tex;
+                dst[u] = tpos + f - tex;
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) nbr[u] = wq[u] >= 0 ? __ldg((wq[u] ? s1.gidx : s0.gidx) + src[u]) : 0;
+            int blk[U], wt[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                blk[u] = wq[u] >= 0 ? __ldg(b + nbr[u]) : 0;
+                wt[u] = (sizeof(K) == 8 && wq[u] >= 0) ? __ldg((wq[u] ? s1.gw : s0.gw) + src[u]) : 0;
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                if (wq[u] < 0) continue;
+                K *seg = wq[u] ? s1.seg : s0.seg;
+                if (sizeof(K) == 8) seg[dst[u]] = (K)(((unsigned long long)(unsigned)blk[u] << 32) | (unsigned)wt[u]);
+                else seg[dst[u]] = (K)(unsigned)blk[u];
+            }
         }
     }
+}
+
+template <typename K>
+__global__ void k_line_scatter_batched(int V, const int *__restrict__ gptr, const int *__restrict__ gidx,
+                                       const int *__restrict__ gw, const int *__restrict__ b,
+                                       const int *__restrict__ off, int *__restrict__ cur, K *__restrict__ seg) {
+    const ScatterSide<K> sd{gptr, gidx, gw, off, cur, seg};
+    scatter_batched<K>(sd, sd, 1, V, b, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
 }
 
 // 4a. classify lines by segment length
