@@ -72,6 +72,9 @@ typedef struct {
                                  B <= 221 (shared-memory histogram), the multi-kernel path above;
                                  2: the persistent kernel for every dense B (L2 atomics above 221;
                                  slower there on B200); 0: always multi-kernel.  Same result. */
+    int32_t sel_small;        /* 1 (default): merge selection (a4) for B <= 4096 in one CTA (shared
+                                 memory) + 4 grid launches; 0: the multi-kernel selection (radix
+                                 sort, pointer-doubling launches).  Same result. */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */

@@ -921,6 +921,7 @@ void gsap_default_params(gsap_params *p) {
     p->dense_max_B = 0;
     p->sparse_coop = 1;
     p->dense_coop = 1;
+    p->sel_small = 1;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }

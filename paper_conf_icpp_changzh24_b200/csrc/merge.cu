@@ -238,11 +238,174 @@ __global__ void k_relabel(int V, const int *__restrict__ label, int *__restrict_
 
 static inline int g256(long long n) { return (int)std::max<long long>(1, std::min<long long>((n + 255) / 256, 148LL * 32)); }
 
+// ------------------------------------------- selection, one CTA (small B) --
+// The block part of select_merges for B <= SEL_SMALL_B in ONE 1024-thread CTA
+// (shared memory): the same keys (canonical dS bits, id), a bitonic sort on
+// (key, id) -- the order of the stable radix sort --, the same pointer
+// doubling with running max, cycle marks, accepted flags, inclusive scan,
+// applied edges and pointer jumping; writes the roots.  Integer work only: the
+// same result as the multi-kernel path, in one launch instead of ~2 log2(2B) + 20.
+constexpr int SEL_SMALL_B = 4096;
+constexpr int SEL_THREADS = 1024;
+
+GSAP_DEV void sel_cta_scan_incl(int *a, int n, int *sh) {   // in place, inclusive, n <= SEL_SMALL_B
+    const int per = (n + SEL_THREADS - 1) / SEL_THREADS;     // <= 4
+    const int lo = threadIdx.x * per, hi = min(n, lo + per);
+    int sum = 0;
+    for (int i = lo; i < hi; ++i) sum += a[i];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int x = warp_incl_scan(sum);
+    if (lane == 31) sh[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        const int y = warp_incl_scan(sh[lane]);
+        sh[lane] = y;
+    }
+    __syncthreads();
+    int run = (w ? sh[w - 1] : 0) + x - sum;
+    for (int i = lo; i < hi; ++i) {
+        run += a[i];
+        a[i] = run;
+    }
+    __syncthreads();
+}
+
+__global__ void __launch_bounds__(SEL_THREADS) k_select_small(int B, int K, int rounds, const int *__restrict__ best,
+                                                              const double *__restrict__ dS, int *__restrict__ root) {
+    extern __shared__ __align__(16) unsigned char sel_raw[];
+    u64 *key = reinterpret_cast<u64 *>(sel_raw);                 // [N]
+    int *id = reinterpret_cast<int *>(key + SEL_SMALL_B);         // [N]
+    int *rank = id + SEL_SMALL_B;                                 // [B]
+    int *n0 = rank + SEL_SMALL_B, *n1 = n0 + SEL_SMALL_B;         // [B] x 2
+    int *m0 = n1 + SEL_SMALL_B, *m1 = m0 + SEL_SMALL_B;           // [B] x 2
+    int *flag = m1 + SEL_SMALL_B;                                 // [B]
+    int *sh = flag + SEL_SMALL_B;                                 // [32]
+    const int tid = threadIdx.x;
+    int N = 1;
+    while (N < B) N <<= 1;
+    for (int r = tid; r < N; r += SEL_THREADS) {
+        if (r < B) {
+            double d = dS[r];
+            if (d == 0.0) d = 0.0;   // -0.0 == +0.0
+            u64 bits = (u64)__double_as_longlong(d);
+            bits = (bits >> 63) ? ~bits : (bits | 0x8000000000000000ULL);
+            key[r] = bits;
+            id[r] = r;
+        } else {
+            key[r] = ~0ULL;
+            id[r] = 0x7fffffff;
+        }
+    }
+    __syncthreads();
+    // bitonic sort of (key, id) ascending
+    for (int k = 2; k <= N; k <<= 1) {
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            for (int i = tid; i < (N >> 1); i += SEL_THREADS) {
+                const int lo = ((i & ~(j - 1)) << 1) | (i & (j - 1)), hi = lo + j;
+                const bool up = (lo & k) == 0;
+                const u64 ka = key[lo], kb = key[hi];
+                const int ia = id[lo], ib = id[hi];
+                const bool gt = ka > kb || (ka == kb && ia > ib);
+                if (gt == up) {
+                    key[lo] = kb; key[hi] = ka;
+                    id[lo] = ib; id[hi] = ia;
+                }
+            }
+            __syncthreads();
+        }
+    }
+    for (int i = tid; i < B; i += SEL_THREADS) rank[id[i]] = i;
+    __syncthreads();
+    for (int r = tid; r < B; r += SEL_THREADS) {
+        n0[r] = best[r];
+        m0[r] = rank[r];
+        flag[r] = 0;   // oncyc
+    }
+    __syncthreads();
+    for (int q = 0; q < rounds; ++q) {
+        for (int r = tid; r < B; r += SEL_THREADS) {
+            const int n = n0[r];
+            n1[r] = n0[n];
+            m1[r] = max(m0[r], m0[n]);
+        }
+        __syncthreads();
+        int *t = n0; n0 = n1; n1 = t;
+        t = m0; m0 = m1; m1 = t;
+    }
+    for (int r = tid; r < B; r += SEL_THREADS) flag[n0[r]] = 1;   // on a cycle
+    __syncthreads();
+    // accepted flags by rank (into n1: free now), then their inclusive scan
+    for (int i = tid; i < B; i += SEL_THREADS) {
+        const int r = id[i];
+        n1[i] = (flag[r] && m0[r] == rank[r]) ? 0 : 1;
+    }
+    __syncthreads();
+    for (int i = tid; i < B; i += SEL_THREADS) m1[i] = n1[i];
+    __syncthreads();
+    sel_cta_scan_incl(m1, B, sh);
+    for (int i = tid; i < B; i += SEL_THREADS) {
+        const int r = id[i];
+        n0[r] = (n1[i] && m1[i] <= K) ? best[r] : r;
+    }
+    __syncthreads();
+    for (int q = 0; q < rounds; ++q) {
+        for (int r = tid; r < B; r += SEL_THREADS) flag[r] = n0[n0[r]];
+        __syncthreads();
+        for (int r = tid; r < B; r += SEL_THREADS) n0[r] = flag[r];
+        __syncthreads();
+    }
+    for (int r = tid; r < B; r += SEL_THREADS) root[r] = n0[r];
+}
+
+// labels for B <= SEL_SMALL_B in one CTA: exclusive scan of `present`, new B,
+// label[r] = rank of root(r) among the present roots (or -1)
+__global__ void __launch_bounds__(SEL_THREADS) k_labels_small(int B, const int *__restrict__ root,
+                                                              const int *__restrict__ present,
+                                                              int *__restrict__ label, int *__restrict__ newB) {
+    __shared__ int ex[SEL_SMALL_B + 1];
+    __shared__ int sh[32];
+    for (int r = threadIdx.x; r < B; r += SEL_THREADS) ex[r] = present[r];
+    __syncthreads();
+    sel_cta_scan_incl(ex, B, sh);
+    for (int r = threadIdx.x; r < B; r += SEL_THREADS) {
+        const int x = root[r];
+        label[r] = present[x] ? ex[x] - 1 : -1;   // inclusive - 1 = exclusive (present[x] = 1)
+    }
+    if (threadIdx.x == 0) *newB = ex[B - 1];
+}
+
+static void select_merges_small(Ctx &c, const int *best, const double *dS, int K, int rounds) {
+    const int B = c.B, V = c.V;
+    const size_t smem = sizeof(u64) * SEL_SMALL_B + sizeof(int) * (7 * SEL_SMALL_B + 32);
+    static bool attr = false;
+    if (!attr) {
+        GSAP_CUDA(cudaFuncSetAttribute(k_select_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        attr = true;
+    }
+    k_select_small<<<1, SEL_THREADS, smem, c.stream>>>(B, K, rounds, best, dS, c.nxt0);
+    GSAP_CUDA(cudaMemsetAsync(c.present, 0, sizeof(int) * ((size_t)B + 1), c.stream));
+    k_present<<<g256(V), 256, 0, c.stream>>>(V, c.b, c.nxt0, c.present);
+    k_labels_small<<<1, SEL_THREADS, 0, c.stream>>>(B, c.nxt0, c.present, c.label, c.scal_i);
+    k_relabel<<<g256(V), 256, 0, c.stream>>>(V, c.label, c.b);
+    c.launches += 4;
+    GSAP_CHECK_LAUNCH();
+}
+
+
 void select_merges(Ctx &c, const int *best, const double *dS, int K, int *label_out) {
     Launcher L{c.stream, &c.launches};
     const int B = c.B, V = c.V;
     int rounds = 1;
     while ((1LL << rounds) < 2LL * B) ++rounds;
+    if (B <= SEL_SMALL_B && c.prm.sel_small) {
+        select_merges_small(c, best, dS, K, rounds);
+        if (label_out)
+            GSAP_CUDA(cudaMemcpyAsync(label_out, c.label, sizeof(int) * (size_t)B, cudaMemcpyDefault, c.stream));
+        GSAP_CUDA(cudaMemcpyAsync(c.h_int, c.scal_i, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
+        GSAP_CUDA(cudaStreamSynchronize(c.stream));
+        c.B = *c.h_int;
+        return;
+    }
     k_sel_keys<<<g256(B), 256, 0, c.stream>>>(B, dS, c.skey0, c.sval0);
     ++c.launches;
     const int w = radix_sort<u64, int, true>(c.skey0, c.skey1, c.sval0, c.sval1, nullptr, B, 64, c.counts,

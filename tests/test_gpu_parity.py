@@ -140,13 +140,15 @@ def test_merge_proposals_dS_best(G, oracle_mod, gname, regime):
             assert np.all(close(dS, dS_o)), np.max(np.abs(dS - dS_o))
 
 
-@pytest.mark.parametrize("seed", range(12))
-def test_select_merges_bit_exact(G, oracle_mod, seed):
+@pytest.mark.parametrize("sel_small", [1, 0])
+@pytest.mark.parametrize("seed", range(14))
+def test_select_merges_bit_exact(G, oracle_mod, seed, sel_small):
+    """sel_small = 1: one-CTA selection for B <= 4096 (multi-kernel above); 0: multi-kernel."""
     rng = np.random.default_rng(seed)
-    V = 500
-    B = int(rng.integers(2, 400))
-    rowptr, col, _ = dcsbm.random_multigraph(V, 2000, seed)
-    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    V = 500 if seed < 12 else 9000
+    B = int(rng.integers(2, 400)) if seed < 12 else (4096 if seed == 12 else 6000)
+    rowptr, col, _ = dcsbm.random_multigraph(V, 4 * V, seed)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, sel_small=sel_small)
     b = dcsbm.random_partition(V, B, seed)
     if seed % 3 == 0:
         b = np.where(b == 0, 1, b).astype(np.int32)    # an empty block
