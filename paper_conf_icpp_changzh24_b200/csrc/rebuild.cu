@@ -686,8 +686,11 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, ptr, c.seg_nnz, c.seg_listW, c.seg_listC,
                                                            c.seg_ctr, out, extent);
     const int gw_ = (int)std::min<long long>(((long long)B + SEG_WARPS - 1) / SEG_WARPS, 148LL * 16);
-    k_segsort_warp<K><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(ptr, seg, c.seg_listW, c.seg_ctr, idx, cnt,
-                                                           c.seg_nnz, out);
+    k_segsort_warp<K, false><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(ptr, seg, c.seg_listW, c.seg_ctr, idx, cnt,
+                                                                  c.seg_nnz, out);
+    k_segsort_warp<K, true><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(ptr, seg, c.seg_listW, c.seg_ctr, idx, cnt,
+                                                                 c.seg_nnz, out);
+    ++c.launches;
     const int gc = (int)std::min<long long>(std::max(1, B / 4), 148LL * 4);
     k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(ptr, seg, c.seg_listC, c.seg_ctr, bits_for(B), idx, cnt,
                                                c.seg_nnz, out);

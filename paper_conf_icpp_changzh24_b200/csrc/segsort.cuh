@@ -376,36 +376,41 @@ GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict_
     return total;
 }
 
-// 4b. short segments (<= SEG_WARP_MAX): one warp each -- <= 128 entries
-// bitonic + RLE in registers, longer ones bitonic in shared memory
-template <typename K>
+// 4b. short segments (<= SEG_WARP_MAX): one warp each.  MID = false: <= 128
+// entries bitonic + RLE in registers, 257..512 bitonic in shared memory;
+// MID = true: 129..256 entries in registers (8 per lane) -- a separate
+// instantiation so its register footprint does not lower the occupancy of
+// the common case.  Both walk the same line list and skip the other's lines.
+template <typename K, bool MID>
 __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__restrict__ off, K *__restrict__ seg,
                                                                  const int *__restrict__ listW,
                                                                  const int *__restrict__ counters,
                                                                  int *__restrict__ tcol, int *__restrict__ tcnt,
                                                                  int *__restrict__ nnz, LineOut out) {
-    __shared__ K keys[SEG_WARPS][SEG_WARP_MAX];
-    __shared__ int hp[SEG_WARPS][SEG_WARP_MAX];
+    __shared__ K keys[MID ? 1 : SEG_WARPS][MID ? 1 : SEG_WARP_MAX];
+    __shared__ int hp[MID ? 1 : SEG_WARPS][MID ? 1 : SEG_WARP_MAX];
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int n_lines = counters[0];
     for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
         const int x = listW[li];
         const int o = off[x], L = off[x + 1] - o;
-        if (L <= 128) {   // short lines: bitonic + RLE in registers (fewer instructions than shared memory)
-            int u;
+        const bool mid = L > 128 && L <= 256;
+        if (mid != MID) continue;
+        int u;
+        if (MID) {
+            u = warp_segsort_rle<K, 8>(seg + o, L, tcol + o, tcnt + o);
+        } else if (L <= 128) {
             if (L <= 32) u = warp_segsort_rle<K, 1>(seg + o, L, tcol + o, tcnt + o);
             else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, tcol + o, tcnt + o);
             else u = warp_segsort_rle<K, 4>(seg + o, L, tcol + o, tcnt + o);
-            if (lane == 0) nnz[x] = u;
-            if (out.cum) line_epilogue<32>(out, tcnt, o, u, L, x, lane, nullptr);
-            continue;
+        } else {
+            int n = 1;
+            while (n < L) n <<= 1;
+            for (int i = lane; i < n; i += 32) keys[w][i] = i < L ? seg[o + i] : key_max<K>();
+            __syncwarp();
+            bitonic<K, 32>(keys[w], n, lane);
+            u = rle_runs<K, 32>(keys[w], L, hp[w], tcol + o, tcnt + o, lane, nullptr);
         }
-        int n = 1;
-        while (n < L) n <<= 1;
-        for (int i = lane; i < n; i += 32) keys[w][i] = i < L ? seg[o + i] : key_max<K>();
-        __syncwarp();
-        bitonic<K, 32>(keys[w], n, lane);
-        const int u = rle_runs<K, 32>(keys[w], L, hp[w], tcol + o, tcnt + o, lane, nullptr);
         if (lane == 0) nnz[x] = u;
         if (out.cum) line_epilogue<32>(out, tcnt, o, u, L, x, lane, nullptr);
     }

@@ -363,3 +363,51 @@ def test_device_loop_graph_matches_host_loop(G):
         out.append((r["B"], r["mdl"], st["mcmc_itr_total"], r["rounds"], r["b"].tobytes()))
         ctx.close()
     assert out[0] == out[1] == out[2]
+
+
+@pytest.mark.parametrize("regime", list(REGIMES))
+@pytest.mark.parametrize("weighted", [False, True])
+def test_isolated_and_self_loop_vertices_all_regimes(G, oracle_mod, regime, weighted):
+    """Isolated vertices (k_v = 0, R:Z15), self-loops (R:Z26) and empty blocks
+    (R:Z14) through every rebuild path: blockmodel bit-exact, proposals exact,
+    dS / H within the north_star tolerance, and one applied MOVE batch."""
+    rng = np.random.default_rng(11 + weighted)
+    V = 240
+    rp, cl, w = dcsbm.random_multigraph(V, 1500, 5, weighted=weighted)
+    keep = rng.random(V) < 0.8                                # every 5th vertex isolated (on average)
+    src = np.repeat(np.arange(V), np.diff(rp))
+    m = keep[src] & keep[cl]
+    src, cl = src[m], cl[m]
+    w = w[m] if w is not None else None
+    loops = rng.choice(np.flatnonzero(keep), 20, replace=False)
+    src = np.concatenate([src, loops])
+    cl = np.concatenate([cl, loops]).astype(np.int32)
+    if w is not None:
+        w = np.concatenate([w, rng.integers(1, 4, 20)]).astype(np.int32)
+    order = np.argsort(src, kind="stable")
+    src, cl = src[order], cl[order]
+    w = w[order] if w is not None else None
+    rowptr = np.zeros(V + 1, np.int64)
+    np.add.at(rowptr, src + 1, 1)
+    rowptr = np.cumsum(rowptr)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, cl, w, **REGIMES[regime])
+    for B in (3, 40, 200):
+        b = dcsbm.random_partition(V, B, B)
+        b = np.where(b == 1, 0, b).astype(np.int32)          # block 1 empty
+        set_both(ctx, orc, b, B)
+        assert_same_blockmodel(ctx, orc)
+        s = ctx.gsap_propose(G.GSAP_MOVE, 1, 2, 0, V)
+        s_o = orc.propose(1, SEED, 1, 2, 0, V)
+        assert np.array_equal(s, s_o)
+        dS, H, acc = ctx.gsap_delta_mdl(G.GSAP_MOVE, 1, 2, 0, V, s)
+        dS_o, H_o, p_o, acc_o = orc.delta_move(SEED, 1, 2, 0, V, s_o)
+        assert np.all(close(dS, dS_o)) and np.all(close(H, H_o, floor=1e-300))
+        t = ties(oracle_mod, SEED, 1, 2, range(V), p_o)
+        assert np.array_equal(acc[~t], acc_o[~t])
+        sm = ctx.gsap_propose(G.GSAP_MERGE, 1, 0, 0, B)
+        assert np.array_equal(sm, orc.propose(0, SEED, 1, 0, 0, B))
+        ctx.gsap_apply_moves(0, V, s, acc)
+        ctx.gsap_update_blockmodel()
+        orc.apply_moves(0, V, s, acc)
+        orc.rebuild()
+        assert_same_blockmodel(ctx, orc)
