@@ -181,9 +181,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             const LineOut out{sd.cum, sd.end, sd.deg};
             int u;
             if (L <= SegCta<K>::CAP) {
-                for (int i = threadIdx.x; i < L; i += 256) S.cta.keys[0][i] = seg[o + i];
-                __syncthreads();
-                K *keys = cta_radix_sort<K, 256>(S.cta.keys[0], S.cta.keys[1], L, a.col_bits, S.cta.cntp, S.cta.wsum);
+                K *keys = cta_sort(seg + o, L, S.cta.keys[0], S.cta.keys[1], a.col_bits, S.cta.cntp, S.cta.wsum);
                 int *hp = reinterpret_cast<int *>(keys == S.cta.keys[0] ? S.cta.keys[1] : S.cta.keys[0]);
                 u = rle_runs<K, 256>(keys, L, hp, sd.tcol + o, sd.tcnt + o, threadIdx.x, S.cta.sh);
                 line_epilogue<256>(out, sd.tcnt, o, u, L, x, threadIdx.x, S.cta.sh);
