@@ -95,3 +95,23 @@ def test_bench_and_entry_compile():
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     for f in ("bench.py", "__graft_entry__.py"):
         py_compile.compile(os.path.join(root, f), doraise=True)
+
+
+def test_bench_reference_arm_json():
+    """`bench.py --impl reference` (the oracle arm) prints one JSON line with the
+    contract's keys (run on the 1K config so it takes a second)."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--impl", "reference", "--config", "1k",
+                          "--steps", "1", "--warmup", "0"], capture_output=True, text=True, timeout=300, cwd=root)
+    assert out.returncode == 0, out.stderr
+    line = json.loads(out.stdout.strip().splitlines()[-1])
+    for k in ("impl", "metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better",
+              "cpu_baseline", "e2e", "config"):
+        assert k in line, k
+    assert line["impl"] == "reference" and line["value"] > 0
+    assert line["cpu_baseline"]["kind"] == "oracle" and line["cpu_baseline"]["cores"] >= 1
+    assert line["e2e"]["h2d_bytes_per_step"] == 0
