@@ -220,6 +220,15 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
                         const gsap_params *params, const gsap_dist *dist, void *stream) {
     REQUIRE(V >= 1, GSAP_EINVAL, "V must be >= 1");
     REQUIRE(rowptr && (col || true), GSAP_EINVAL, "rowptr is NULL");
+    const bool tm = getenv("GSAP_TIMING") != nullptr;
+    auto t_prev = std::chrono::steady_clock::now();
+    auto mark = [&](const char *what) {
+        if (!tm) return;
+        cudaDeviceSynchronize();
+        const auto t = std::chrono::steady_clock::now();
+        fprintf(stderr, "[gsap] create %-12s %.3f ms\n", what, std::chrono::duration<double, std::milli>(t - t_prev).count());
+        t_prev = t;
+    };
     check_sm100();
     if (params) c.prm = *params;
     else gsap_default_params(&c.prm);
@@ -252,6 +261,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.E = E;
     c.W = W;
     c.weighted = wgt != nullptr;
+    mark("validate");
     if (stream) {
         c.stream = (cudaStream_t)stream;
     } else {
@@ -264,6 +274,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     GSAP_CUDA(cudaGetDevice(&c.dev));
     comm_init(c, dist);
     if (c.nranks > 1) c.prm.cuda_graphs = 0;
+    mark("streams");
     // host-side static info
     c.h_rowptr.resize((size_t)V + 1);
     for (int v = 0; v <= V; ++v) c.h_rowptr[v] = (int)rp[v];
@@ -416,6 +427,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         cut.base = (char *)base;
         carve(cut);
     }
+    mark("arena");
     {   // f-table: f(m) = m ln m in long double, split into double hi + double lo (once per process)
         static std::vector<double2> ft;
         static std::once_flag once;
@@ -434,6 +446,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         GSAP_CUDA(cudaMemsetAsync(c.small_acc, 0, sizeof(int) * SMALL_MAX_B * SMALL_MAX_B, c.stream));
     GSAP_CUDA(cudaMallocHost(&c.h_scal, 8 * sizeof(double)));
     GSAP_CUDA(cudaMallocHost(&c.h_int, 8 * sizeof(int)));
+    mark("ftab+pinned");
     // upload ---------------------------------------------------------------
     GSAP_CUDA(cudaMemcpyAsync(c.rowptr, c.h_rowptr.data(), sizeof(int) * (Vs + 1), cudaMemcpyHostToDevice, c.stream));
     if (E) GSAP_CUDA(cudaMemcpyAsync(c.col, hc.data(), sizeof(int) * (size_t)E, cudaMemcpyHostToDevice, c.stream));
@@ -450,7 +463,9 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
                                   cudaMemcpyHostToDevice, c.stream));
     GSAP_CUDA(cudaMemsetAsync(c.scal, 0, 8 * sizeof(double), c.stream));
     GSAP_CUDA(cudaMemsetAsync(c.scal_i, 0, 8 * sizeof(int), c.stream));
+    mark("upload");
     build_graph_device(c);
+    mark("csc");
     // the singleton partition (P:61 2.1)
     std::vector<int> iota(Vs);
     for (int v = 0; v < V; ++v) iota[v] = v;
@@ -458,6 +473,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     c.B = V;
     rebuild(c);
     GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    mark("rebuild");
 }
 
 // ------------------------------------------------------------- driver --
@@ -1243,7 +1259,11 @@ gsap_status gsap_partition(int32_t V, const int64_t *rowptr, const int32_t *col,
         stats->t_setup = t_setup;
         stats->t_total = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
     }
+    const auto td = std::chrono::steady_clock::now();
     gsap_destroy(ctx);
+    if (getenv("GSAP_TIMING"))
+        fprintf(stderr, "[gsap] partition: create %.3f ms, destroy %.3f ms\n", 1e3 * t_setup,
+                std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - td).count());
     return st;
 }
 
