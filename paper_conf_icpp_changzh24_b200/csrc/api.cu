@@ -357,10 +357,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.flags = A.take<int>(VE);
         c.pos = A.take<int>(VE);
         c.tmpi = A.take<int>(VE);
-        c.rowid = A.take<int>(VE);
         c.rownnz = A.take<int>(Vs + 1);
         c.seg_len = A.take<int>(Vs + 1);
-        c.seg_off = A.take<int>(Vs + 1);
         c.seg_cur = A.take<int>(Vs + 1);
         c.seg_nnz = A.take<int>(Vs + 1);
         c.seg_listW = A.take<int>(Vs + 1);
@@ -370,7 +368,6 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.xl_hp = A.take<int>(2 * Es);
         if (c.coop_ok) {
             c.seg2_len = A.take<int>(Vs + 1);
-            c.seg2_off = A.take<int>(Vs + 1);
             c.seg2_cur = A.take<int>(Vs + 1);
             c.seg2_nnz = A.take<int>(Vs + 1);
             c.seg2_listC = A.take<int>(Vs + 1);

@@ -77,16 +77,16 @@ struct Ctx {
     unsigned long long *keys0 = nullptr, *keys1 = nullptr, *vals64a = nullptr, *vals64b = nullptr;
     unsigned *ukeys0 = nullptr, *ukeys1 = nullptr;
     int *wa = nullptr, *wb = nullptr, *flags = nullptr, *pos = nullptr, *tmpi = nullptr,
-        *rowid = nullptr, *counts = nullptr, *scan_tmp = nullptr, *rownnz = nullptr;
+        *counts = nullptr, *scan_tmp = nullptr, *rownnz = nullptr;
     size_t counts_cap = 0, scan_tmp_cap = 0;
     // segmented rebuild scratch (per line: length, offset, cursor, runs; line lists)
-    int *seg_len = nullptr, *seg_off = nullptr, *seg_cur = nullptr, *seg_nnz = nullptr, *seg_listW = nullptr,
+    int *seg_len = nullptr, *seg_cur = nullptr, *seg_nnz = nullptr, *seg_listW = nullptr,
         *seg_listC = nullptr, *seg_ctr = nullptr, *xl_hp = nullptr;
     unsigned long long *xl_keys = nullptr;   // 2E: long-segment sort scratch
     // persistent sparse rebuild (coop.cuh; small graphs): the column side's
     // line scratch, its long-segment scratch, the grid barrier
     bool coop_ok = false;
-    int *seg2_len = nullptr, *seg2_off = nullptr, *seg2_cur = nullptr, *seg2_nnz = nullptr, *seg2_listC = nullptr;
+    int *seg2_len = nullptr, *seg2_cur = nullptr, *seg2_nnz = nullptr, *seg2_listC = nullptr;
     unsigned long long *xl2_keys = nullptr;
     int *xl2_hp = nullptr;
     unsigned *coop_bar = nullptr;
