@@ -252,7 +252,7 @@ __global__ void k_line_scatter_batched(int V, const int *__restrict__ gptr, cons
 // 4a. classify lines by segment length
 __global__ void k_line_classify(int B, const int *__restrict__ off, int *__restrict__ nnz, int *__restrict__ listW,
                                 int *__restrict__ listC, int *__restrict__ counters, LineOut out,
-                                int *__restrict__ extent) {
+                                int *__restrict__ extent, int warp_max) {
     if (extent && blockIdx.x == 0 && threadIdx.x == 0) *extent = off[B];
     for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < B; x += gridDim.x * blockDim.x) {
         const int L = off[x + 1] - off[x];
@@ -263,8 +263,10 @@ __global__ void k_line_classify(int B, const int *__restrict__ off, int *__restr
                 out.deg[x] = 0;
             }
         }
-        else if (L <= SEG_WARP_MAX) listW[atomicAdd(counters, 1)] = x;
-        else listC[atomicAdd(counters + 1, 1)] = x;
+        else if (L <= 128 || (L > 256 && L <= SEG_WARP_MAX)) listW[atomicAdd(counters, 1)] = x;   // warp mode 0
+        else if (L <= 256) listW[B - 1 - atomicAdd(counters + 2, 1)] = x;                        // warp mode 1
+        else if (L <= warp_max) listC[B - 1 - atomicAdd(counters + 3, 1)] = x;                   // warp mode 2
+        else listC[atomicAdd(counters + 1, 1)] = x;                                               // CTA
     }
 }
 
@@ -376,45 +378,54 @@ GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict_
     return total;
 }
 
-// 4b. short segments (<= SEG_WARP_MAX): one warp each.  MID = false: <= 128
-// entries bitonic + RLE in registers, 257..512 bitonic in shared memory;
-// MID = true: 129..256 entries in registers (8 per lane) -- a separate
-// instantiation so its register footprint does not lower the occupancy of
-// the common case.  Both walk the same line list and skip the other's lines.
-template <typename K, bool MID>
-__global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(const int *__restrict__ off, K *__restrict__ seg,
+// 4b. warp-sized segments: one warp each, three instantiations, each over its
+// own line list (k_line_classify), so that a heavy path does not lower the
+// occupancy of the common one:
+//   MODE 0: <= 128 entries bitonic + RLE in registers, 257..512 bitonic in
+//           static shared memory;
+//   MODE 1: 129..256 entries in registers (8 per lane);
+//   MODE 2: 513..SEG_WARP_MAX_MK entries bitonic in dynamic shared memory.
+constexpr int SEG_WARP_MAX_MK = 1024;   // multi-kernel path: longer lines go to the CTA sorts
+template <typename K, int MODE>
+__global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const int *__restrict__ off, K *__restrict__ seg,
                                                                  const int *__restrict__ listW,
                                                                  const int *__restrict__ counters,
                                                                  int *__restrict__ tcol, int *__restrict__ tcnt,
                                                                  int *__restrict__ nnz, LineOut out) {
-    __shared__ K keys[MID ? 1 : SEG_WARPS][MID ? 1 : SEG_WARP_MAX];
-    __shared__ int hp[MID ? 1 : SEG_WARPS][MID ? 1 : SEG_WARP_MAX];
+    __shared__ K keys[MODE == 0 ? SEG_WARPS : 1][MODE == 0 ? SEG_WARP_MAX : 1];
+    __shared__ int hp[MODE == 0 ? SEG_WARPS : 1][MODE == 0 ? SEG_WARP_MAX : 1];
+    extern __shared__ __align__(16) unsigned char seg_dyn[];   // MODE 2: SEG_WARPS x (keys + heads)
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int n_lines = counters[0];
+    const int n_lines = counters[MODE == 0 ? 0 : MODE == 1 ? 2 : 3];
     for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
-        const int x = listW[li];
+        const int x = MODE == 0 ? listW[li] : listW[B - 1 - li];   // MODE 2: listW is the CTA list (listC)
         const int o = off[x], L = off[x + 1] - o;
-        const bool mid = L > 128 && L <= 256;
-        if (mid != MID) continue;
         int u;
-        if (MID) {
+        if (MODE == 1) {
             u = warp_segsort_rle<K, 8>(seg + o, L, tcol + o, tcnt + o);
-        } else if (L <= 128) {
+        } else if (MODE == 0 && L <= 128) {
             if (L <= 32) u = warp_segsort_rle<K, 1>(seg + o, L, tcol + o, tcnt + o);
             else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, tcol + o, tcnt + o);
             else u = warp_segsort_rle<K, 4>(seg + o, L, tcol + o, tcnt + o);
         } else {
+            K *kw = MODE == 0 ? keys[w] : reinterpret_cast<K *>(seg_dyn) + (size_t)w * SEG_WARP_MAX_MK;
+            int *hw = MODE == 0 ? hp[w]
+                                : reinterpret_cast<int *>(reinterpret_cast<K *>(seg_dyn) + (size_t)SEG_WARPS * SEG_WARP_MAX_MK) +
+                                      (size_t)w * SEG_WARP_MAX_MK;
             int n = 1;
             while (n < L) n <<= 1;
-            for (int i = lane; i < n; i += 32) keys[w][i] = i < L ? seg[o + i] : key_max<K>();
+            for (int i = lane; i < n; i += 32) kw[i] = i < L ? seg[o + i] : key_max<K>();
             __syncwarp();
-            bitonic<K, 32>(keys[w], n, lane);
-            u = rle_runs<K, 32>(keys[w], L, hp[w], tcol + o, tcnt + o, lane, nullptr);
+            bitonic<K, 32>(kw, n, lane);
+            u = rle_runs<K, 32>(kw, L, hw, tcol + o, tcnt + o, lane, nullptr);
         }
         if (lane == 0) nnz[x] = u;
         if (out.cum) line_epilogue<32>(out, tcnt, o, u, L, x, lane, nullptr);
     }
 }
+
+template <typename K>
+constexpr size_t seg_warp2_smem() { return (size_t)SEG_WARPS * SEG_WARP_MAX_MK * (sizeof(K) + sizeof(int)); }
 
 // stable LSD radix sort of a[0, L) by the block bits of the key (key_col),
 // 4-bit digits, NT threads.  Each thread owns a contiguous chunk of an odd
