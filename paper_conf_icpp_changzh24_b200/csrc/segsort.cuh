@@ -385,7 +385,10 @@ GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict_
 //           static shared memory;
 //   MODE 1: 129..256 entries in registers (8 per lane);
 //   MODE 2: 513..SEG_WARP_MAX_MK entries bitonic in dynamic shared memory.
-constexpr int SEG_WARP_MAX_MK = 1024;   // multi-kernel path: longer lines go to the CTA sorts
+#ifndef GSAP_SEG_WARP_MAX_MK
+#define GSAP_SEG_WARP_MAX_MK 1024
+#endif
+constexpr int SEG_WARP_MAX_MK = GSAP_SEG_WARP_MAX_MK;   // multi-kernel path: longer lines go to the CTA sorts
 template <typename K, int MODE>
 __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const int *__restrict__ off, K *__restrict__ seg,
                                                                  const int *__restrict__ listW,
