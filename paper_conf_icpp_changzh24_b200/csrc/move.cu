@@ -137,10 +137,10 @@ GSAP_DEV void group_sum3(double &x, double &y, double &z, double *sh) {
 // binary searches -- each step issues four independent loads, so a lane's
 // dependent-load depth is log2(max len) + 1 instead of four times that
 // (the lines of M live in HBM once the blockmodel outgrows L2)
-GSAP_DEV void lookup4(const Line (&L)[4], const int (&y)[4], int (&out)[4]) {
-    int p[4] = {0, 0, 0, 0}, n[4];
+GSAP_DEV void lookup4_in(const Line (&L)[4], const int (&y)[4], int (&p)[4], int (&n)[4], int (&out)[4]) {
+    bool some[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) n[k] = L[k].len;
+    for (int k = 0; k < 4; ++k) some[k] = n[k] > 0;
     while (n[0] > 1 || n[1] > 1 || n[2] > 1 || n[3] > 1) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
@@ -154,11 +154,46 @@ GSAP_DEV void lookup4(const Line (&L)[4], const int (&y)[4], int (&out)[4]) {
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
         int v = 0;
-        if (L[k].len > 0) {
+        if (some[k]) {
             const int id = __ldg(L[k].idx + p[k]), cn = __ldg(L[k].cnt + p[k]);
             v = id == y[k] ? cn : 0;
         }
         out[k] = v;
+    }
+}
+
+GSAP_DEV void lookup4(const Line (&L)[4], const int (&y)[4], int (&out)[4]) {
+    int p[4] = {0, 0, 0, 0}, n[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) n[k] = L[k].len;
+    lookup4_in(L, y, p, n, out);
+}
+
+// warp path, sparse regime: the 32 lanes of a vertex's warp all search the
+// same four lines, so they first load 32 splitters per line together (lane j:
+// idx[(j len) >> 5], one load level); a lane narrows each key to one of the 32
+// buckets with five shuffles and binary-searches only that bucket -- five
+// dependent load levels fewer per lookup once lines exceed 32 entries
+GSAP_DEV void split4_load(const Line (&L)[4], int lane, int (&sp)[4]) {
+#pragma unroll
+    for (int k = 0; k < 4; ++k) sp[k] = L[k].len > 0 ? __ldg(L[k].idx + ((lane * L[k].len) >> 5)) : 0x7fffffff;
+}
+
+// all 32 lanes: the bucket [p, p + n) of line k that holds key y[k] if present
+// (n = 0: absent); sp[k] are line k's splitters as split4_load left them
+GSAP_DEV void split4_bucket(const Line (&L)[4], const int (&sp)[4], const int (&y)[4], int (&p)[4], int (&n)[4]) {
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        int j = 0;   // the last bucket whose first entry is <= y[k]
+#pragma unroll
+        for (int st = 16; st >= 1; st >>= 1) {
+            const int x = __shfl_sync(0xffffffffu, sp[k], j + st);
+            if (x <= y[k]) j += st;
+        }
+        const int s0 = __shfl_sync(0xffffffffu, sp[k], 0);
+        const int len = L[k].len, lo = (j * len) >> 5;
+        p[k] = lo;
+        n[k] = (len > 0 && s0 <= y[k]) ? (((j + 1) * len) >> 5) - lo : 0;
     }
 }
 
@@ -467,6 +502,7 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
         const int din_r = __ldg(a.m.din + r), din_s = __ldg(a.m.din + s);
         int Mrr, Mrs, Msr, Mss;
         Line Ln[4];   // sparse: row r, row s, column r, column s of M
+        int sp[4];    // sparse: this lane's splitter of each of the four lines
         if (DENSE) {
             Mrr = __ldg(D + (size_t)r * B + r);
             Mrs = __ldg(D + (size_t)r * B + s);
@@ -477,10 +513,13 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
             Ln[1] = row_line(a.m, s);
             Ln[2] = col_line(a.m, r);
             Ln[3] = col_line(a.m, s);
+            split4_load(Ln, lane, sp);
             const Line Lc[4] = {Ln[0], Ln[0], Ln[1], Ln[1]};
+            const int spc[4] = {sp[0], sp[0], sp[1], sp[1]};
             const int yc[4] = {r, s, r, s};
-            int oc[4];
-            lookup4(Lc, yc, oc);
+            int oc[4], pc[4], nc[4];
+            split4_bucket(Lc, spc, yc, pc, nc);
+            lookup4_in(Lc, yc, pc, nc, oc);
             Mrr = oc[0];
             Mrs = oc[1];
             Msr = oc[2];
@@ -493,9 +532,16 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
         const double *__restrict__ rcp = a.m.rcp;
         // ---- phase B: one unique neighbour block per lane
         double accS = 0.0, pf = 0.0, pb = 0.0;
-        for (int k = lane; k < nuniq; k += 32) {
-            const int4 e = k == lane ? e0 : tab[list[k]];
+        for (int base = 0; base < nuniq; base += 32) {   // warp-uniform trips (shuffles below)
+            const int k = base + lane;
+            const int4 e = k >= nuniq ? make_int4(-1, 0, 0, 0) : k == lane ? e0 : tab[list[k]];
             const int t = e.x, ot = e.y, it = e.z;
+            int pb4[4], nb4[4];
+            if (!DENSE) {
+                const int yt[4] = {t, t, t, t};
+                split4_bucket(Ln, sp, yt, pb4, nb4);
+            }
+            if (k >= nuniq) continue;
             const double cw = (double)(ot + it);
             if (t == r) {
                 pf += cw * (double)(Mrs + Msr + 1) * __ldg(rcp + r);
@@ -521,7 +567,7 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
                 } else {
                     const int yt[4] = {t, t, t, t};
                     int o4[4];
-                    lookup4(Ln, yt, o4);
+                    lookup4_in(Ln, yt, pb4, nb4, o4);
                     Mrt = o4[0];
                     Mst = o4[1];
                     Mtr = o4[2];
