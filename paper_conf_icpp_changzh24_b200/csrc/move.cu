@@ -137,6 +137,9 @@ GSAP_DEV void group_sum3(double &x, double &y, double &z, double *sh) {
 // binary searches -- each step issues four independent loads, so a lane's
 // dependent-load depth is log2(max len) + 1 instead of four times that
 // (the lines of M live in HBM once the blockmodel outgrows L2)
+#ifndef GSAP_LOOKUP_CONDCNT
+#define GSAP_LOOKUP_CONDCNT 0
+#endif
 GSAP_DEV void lookup4_in(const Line (&L)[4], const int (&y)[4], int (&p)[4], int (&n)[4], int (&out)[4]) {
     bool some[4];
 #pragma unroll
@@ -155,8 +158,13 @@ GSAP_DEV void lookup4_in(const Line (&L)[4], const int (&y)[4], int (&p)[4], int
     for (int k = 0; k < 4; ++k) {
         int v = 0;
         if (some[k]) {
+#if GSAP_LOOKUP_CONDCNT
+            // the count's sector only for a hit (one more dependent level)
+            if (__ldg(L[k].idx + p[k]) == y[k]) v = __ldg(L[k].cnt + p[k]);
+#else
             const int id = __ldg(L[k].idx + p[k]), cn = __ldg(L[k].cnt + p[k]);
             v = id == y[k] ? cn : 0;
+#endif
         }
         out[k] = v;
     }
