@@ -755,7 +755,10 @@ __global__ void __launch_bounds__(256) k_propose(MoveArgs a) {
 // CTAs take every other vertex of [first, first + count) one warp per vertex.
 // The shared memory is the 8 warp tables, or one CTA table over the same bytes.
 template <bool WEIGHTED>
-__global__ void __launch_bounds__(MOVE_WARPS * 32) k_move_groups(MoveArgs a) {
+#ifndef GSAP_GROUPS_MINB
+#define GSAP_GROUPS_MINB 1
+#endif
+__global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_GROUPS_MINB) k_move_groups(MoveArgs a) {
     __shared__ int4 tabs[CTA_SMEM_SLOTS];
     __shared__ double sh[3 * MOVE_WARPS + 8];   // group sums + the broadcast proposal
     if ((int)blockIdx.x < a.nmid_ctas) {
