@@ -810,8 +810,27 @@ static double mcmc_batch(OState *st, const OParams *pr, uint32_t outer, uint32_t
     return D;
 }
 
-/* MCMC phase; returns the number of iterations run */
-static int32_t mcmc_phase(OState *st, const OParams *pr, uint32_t outer, double thresh, OStats *stats)
+/* The convergence test after MCMC iteration itr (P:141 3; Table 2
+ * "delta_entropy_threshold", "delta_entropy_moving_avg_window"; R:Z19, Z20):
+ * GraphChallenge's slice D[itr-w+1 : itr) -- for the default w = 3 the two
+ * iterations BEFORE itr, not itr itself -- and the MDL of the state AFTER
+ * iteration itr:  stop iff  -mean(slice) < thresh * MDL.  No test before
+ * itr = w - 1; an empty slice (w = 1) has mean 0. */
+static int mcmc_converged(const double *Dh, int32_t itr, int32_t window, double thresh, double mdl)
+{
+    double sum = 0.0, mean;
+    int32_t j, n = 0;
+    if (itr < window - 1) return 0;
+    for (j = itr - window + 1; j < itr; ++j) { sum += Dh[j]; ++n; }
+    mean = n ? sum / n : 0.0;
+    return -mean < thresh * mdl;
+}
+
+/* MCMC phase; returns the number of iterations run.  D_out (nullable,
+ * max_nodal_itr entries): D[itr] = sum of the accepted (stale) dS of
+ * iteration itr, batches in order (R:Z20). */
+static int32_t mcmc_phase(OState *st, const OParams *pr, uint32_t outer, double thresh, OStats *stats,
+                          double *D_out)
 {
     int32_t V = st->g.V, nb = pr->num_batches, itr, k;
     int32_t bs = (V + nb - 1) / nb;
@@ -826,19 +845,24 @@ static int32_t mcmc_phase(OState *st, const OParams *pr, uint32_t outer, double 
             D += mcmc_batch(st, pr, outer, (uint32_t)itr, first, last - first, stats);
         }
         Dh[itr] = D;
+        if (D_out) D_out[itr] = D;
         ran = itr + 1;
-        if (itr >= pr->window - 1) {
-            /* GraphChallenge: -mean(D[itr-w+1 : itr]) < thresh * MDL  (R:Z19, Z20) */
-            double mdl = orc_mdl_of(st, pr->model_term, NULL);
-            double sum = 0.0, mean;
-            int32_t j, n = 0;
-            for (j = itr - pr->window + 1; j < itr; ++j) { sum += Dh[j]; ++n; }
-            mean = n ? sum / n : 0.0;
-            if (-mean < thresh * mdl) break;
-        }
+        if (itr >= pr->window - 1 &&
+            mcmc_converged(Dh, itr, pr->window, thresh, orc_mdl_of(st, pr->model_term, NULL)))
+            break;
     }
     free(Dh);
     return ran;
+}
+
+/* The stopping rule alone against given per-iteration D[] and MDL[] (mock; no
+ * MCMC): the number of iterations mcmc_phase would run (at most n). */
+int32_t orc_mcmc_stop_mock(const double *D, const double *mdl, int32_t n, int32_t window, double thresh)
+{
+    int32_t itr;
+    for (itr = 0; itr < n; ++itr)
+        if (mcmc_converged(D, itr, window, thresh, mdl[itr])) return itr + 1;
+    return n;
 }
 
 /*
@@ -901,7 +925,9 @@ int32_t orc_golden_mock(int32_t V, double rate, const double *mdl_of_B,
     return n;
 }
 
-/* trace rows: [outer, B after merge, mcmc iterations, MDL] per round */
+/* trace rows (ORC_TRACE_COLS): [outer, B after merge, mcmc iterations, MDL,
+ * convergence threshold used, accepted moves] per round */
+#define ORC_TRACE_COLS 6
 int32_t orc_partition(void *h, const OParams *pr, int32_t *b_out, int32_t *B_out,
                       double *mdl_out, OStats *stats, double *trace, int32_t trace_cap)
 {
@@ -928,16 +954,20 @@ int32_t orc_partition(void *h, const OParams *pr, int32_t *b_out, int32_t *B_out
     while (!done && rounds < pr->max_rounds) {
         int bracket = (sS[2] != INFINITY);
         int32_t itrs, B;
-        double S;
+        double S, thresh = bracket ? pr->thresh2 : pr->thresh1;
+        int64_t acc0 = stats ? stats->n_move_acc : 0;
         merge_phase(st, pr, outer, K, stats);
         B = st->B;
-        itrs = mcmc_phase(st, pr, outer, bracket ? pr->thresh2 : pr->thresh1, stats);
+        itrs = mcmc_phase(st, pr, outer, thresh, stats, NULL);
         S = orc_mdl_of(st, pr->model_term, NULL);
         if (trace && rounds < trace_cap) {
-            trace[4 * rounds + 0] = (double)outer;
-            trace[4 * rounds + 1] = (double)B;
-            trace[4 * rounds + 2] = (double)itrs;
-            trace[4 * rounds + 3] = S;
+            double *row = trace + (size_t)ORC_TRACE_COLS * rounds;
+            row[0] = (double)outer;
+            row[1] = (double)B;
+            row[2] = (double)itrs;
+            row[3] = S;
+            row[4] = thresh;
+            row[5] = stats ? (double)(stats->n_move_acc - acc0) : 0.0;
         }
         if (stats) stats->mcmc_itr_total += itrs;
         ++rounds;
@@ -966,11 +996,13 @@ int32_t orc_partition(void *h, const OParams *pr, int32_t *b_out, int32_t *B_out
     return rounds;
 }
 
-/* an MCMC phase alone from the current state (used by lockstep tests) */
-int32_t orc_mcmc_phase(void *h, const OParams *pr, uint32_t outer, double thresh, OStats *stats)
+/* an MCMC phase alone from the current state (used by lockstep tests);
+ * D_out: nullable, max_nodal_itr entries */
+int32_t orc_mcmc_phase(void *h, const OParams *pr, uint32_t outer, double thresh, OStats *stats,
+                       double *D_out)
 {
     if (stats) memset(stats, 0, sizeof(*stats));
-    return mcmc_phase((OState *)h, pr, outer, thresh, stats);
+    return mcmc_phase((OState *)h, pr, outer, thresh, stats, D_out);
 }
 
 /* one merge phase alone from the current state */

@@ -109,7 +109,9 @@ def lib():
                                     C.POINTER(C.c_double), C.POINTER(OStats), _f64p, C.c_int32]
         L.orc_mcmc_phase.restype = C.c_int32
         L.orc_mcmc_phase.argtypes = [C.c_void_p, C.POINTER(OParams), C.c_uint32, C.c_double,
-                                     C.POINTER(OStats)]
+                                     C.POINTER(OStats), C.c_void_p]
+        L.orc_mcmc_stop_mock.restype = C.c_int32
+        L.orc_mcmc_stop_mock.argtypes = [_f64p, _f64p, C.c_int32, C.c_int32, C.c_double]
         L.orc_merge_phase.restype = C.c_int32
         L.orc_merge_phase.argtypes = [C.c_void_p, C.POINTER(OParams), C.c_uint32, C.c_int32]
         L.orc_mcmc_batch.restype = C.c_double
@@ -120,6 +122,20 @@ def lib():
                                       C.POINTER(C.c_int32)]
         _lib = L
     return _lib
+
+
+# orc_partition trace row: [outer, B after merge, MCMC iterations, MDL, threshold used, accepted moves]
+TRACE_COLS = 6
+
+
+def mcmc_stop_mock(D, mdl, window=3, thresh=5e-4):
+    """The MCMC stopping rule alone (the helper mcmc_phase calls) against given
+    per-iteration D[itr] and MDL[itr] (MDL of the state after iteration itr):
+    the number of iterations the phase would run."""
+    D = np.ascontiguousarray(D, np.float64)
+    mdl = np.ascontiguousarray(mdl, np.float64)
+    assert len(D) == len(mdl)
+    return lib().orc_mcmc_stop_mock(D, mdl, len(D), window, thresh)
 
 
 def golden_mock(V, rate, mdl_of_B, cap=1000):
@@ -250,9 +266,13 @@ class Oracle:
     def mcmc_batch(self, params, outer, itr, first, count):
         return lib().orc_mcmc_batch(self.h, C.byref(params), outer, itr, first, count)
 
-    def mcmc_phase(self, params, outer, thresh):
+    def mcmc_phase(self, params, outer, thresh, return_D=False):
+        """One MCMC phase (O.8).  return_D: also D[itr] (sum of accepted dS per iteration)."""
         st = OStats()
-        n = lib().orc_mcmc_phase(self.h, C.byref(params), outer, thresh, C.byref(st))
+        D = np.zeros(params.max_nodal_itr + 1)
+        n = lib().orc_mcmc_phase(self.h, C.byref(params), outer, thresh, C.byref(st), _ptr(D))
+        if return_D:
+            return n, st, D[:n]
         return n, st
 
     def merge_phase(self, params, outer, K):
@@ -264,8 +284,8 @@ class Oracle:
         B = C.c_int32(0)
         mdl = C.c_double(0)
         st = OStats()
-        trace = np.zeros(4 * trace_cap)
+        trace = np.zeros(TRACE_COLS * trace_cap)
         rounds = lib().orc_partition(self.h, C.byref(params), b, C.byref(B), C.byref(mdl),
                                      C.byref(st), trace, trace_cap)
-        tr = trace[:4 * min(rounds, trace_cap)].reshape(-1, 4)
+        tr = trace[:TRACE_COLS * min(rounds, trace_cap)].reshape(-1, TRACE_COLS)
         return dict(b=b[:self.V], B=B.value, mdl=mdl.value, stats=st, trace=tr, rounds=rounds)
