@@ -15,9 +15,13 @@
  *     graph; the context owns all device state and frees it in gsap_destroy.
  *   - Pointer arguments marked "host or device" may point to host memory or
  *     to device memory of the context's GPU (told apart with
- *     cudaPointerGetAttributes).  Host outputs are complete when the call
- *     returns.  Device outputs are written asynchronously on the context's
- *     stream (complete when that stream is synchronised).
+ *     cudaPointerGetAttributes, each pointer separately).  Outputs, host or
+ *     device, are complete when the call returns (the call synchronises the
+ *     context's stream), so a device output may be read on any stream.
+ *     Device INPUTS are read on the context's stream: the caller must have
+ *     completed the work that produced them (e.g. synchronised its stream)
+ *     before the call.  Device id inputs are range-checked on the device
+ *     before any state changes (GSAP_EINVAL otherwise).
  *   - Ids are 0-based.  Vertex ids are int32, edge offsets int64 at the ABI.
  *   - Limits: 1 <= V < 2^31, number of edges and total edge weight < 2^30,
  *     weights >= 1 (GSAP_EUNSUPPORTED / GSAP_EINVAL otherwise).
@@ -94,6 +98,11 @@ typedef struct {
     double k_rebuild_ms, k_rebuild_bytes; int64_t k_rebuild_launches;
     double k_merge_ms, k_merge_bytes; int64_t k_merge_launches;
     double k_mdl_ms; int64_t k_mdl_launches;
+    /* device seconds of the blockmodel rebuilds (Alg. 2) and of
+     * the multi-GPU exchange (both profile = 1, else 0), and the MOVE
+     * proposals actually evaluated (s != b[v]; R:Z13 makes the rest no-ops) */
+    double t_rebuild, t_comm;
+    int64_t n_move_eval;
 } gsap_stats;
 
 typedef struct gsap_ctx gsap_ctx;
@@ -172,7 +181,10 @@ gsap_status gsap_delta_mdl(gsap_ctx *ctx, gsap_phase phase, uint32_t outer, uint
 gsap_status gsap_select_merges(gsap_ctx *ctx, const int32_t *best, const double *dS,
                                int32_t K, int32_t *label_out, int32_t *newB_out);
 
-/* b[first+i] = s[i] where acc[i] != 0 (host or device arrays); no rebuild. */
+/* The "apply" step of a batch (P:141 3, P:176 3.2; R:Z10): b[first+i] = s[i]
+ * where acc[i] != 0.  s[count] int32, acc[count] uint8, each host or device;
+ * accepted s[i] must lie in [0, B) (GSAP_EINVAL, nothing written, otherwise).
+ * No rebuild (call gsap_update_blockmodel). */
 gsap_status gsap_apply_moves(gsap_ctx *ctx, int32_t first, int32_t count,
                              const int32_t *s, const uint8_t *acc);
 
@@ -195,11 +207,23 @@ gsap_status gsap_move_batch(gsap_ctx *ctx, uint32_t outer, uint32_t itr, int32_t
 gsap_status gsap_merge_phase(gsap_ctx *ctx, uint32_t outer, int32_t K,
                              int32_t *best_out, double *dSbest_out);
 
+/*
+ * One MCMC phase (P:141 3, P:176 3.2; Table 2; R:O.8, Z10, Z19,
+ * Z20) from the current state: iterations of num_batches fused batches (ids
+ * in contiguous ranges of ceil(V/num_batches)) until the GraphChallenge test
+ * -mean(D[itr-w+1 : itr)) < thresh * MDL (w = params.window, MDL after the
+ * iteration) or max_nodal_itr stops it.  D_out (host, nullable,
+ * max_nodal_itr doubles): D[itr] = sum of the accepted dS of iteration itr;
+ * itrs_out (host, nullable): iterations run.  outer keys the Philox streams.
+ */
+gsap_status gsap_mcmc_phase(gsap_ctx *ctx, uint32_t outer, double thresh, double *D_out, int32_t *itrs_out);
+
 /* MDL of the current state, Eq. 2 (R:Z1-Z4, Z22); data term S (nullable). Host outputs. */
 gsap_status gsap_mdl(gsap_ctx *ctx, double *mdl_out, double *data_term_out);
 
 /*
- * Blockmodel export (CSR rows ascending column; CSC columns ascending row;
+ * Blockmodel export, the "six arrays" of P:152-159 3.1 (Fig. 3) plus the
+ * block degrees of P:162 (CSR rows ascending column; CSC columns ascending row;
  * cum = inclusive prefix of cnt within a row / column).  *nnz_io (host): in =
  * capacity of the entry arrays, out = nnz.  Any array may be NULL; with all
  * arrays NULL this is a size query.  rowptr/colptr[B+1] int64; col, cnt, cum,
@@ -209,11 +233,13 @@ gsap_status gsap_get_blockmodel(gsap_ctx *ctx, int64_t *nnz_io, int64_t *rowptr,
                                 int32_t *cnt, int32_t *cum, int64_t *colptr, int32_t *row,
                                 int32_t *ccnt, int32_t *ccum, int32_t *dout, int32_t *din);
 
-/* Statistics accumulated since create / the last reset (host). */
+/* Statistics accumulated since create / the last reset (host): the counts
+ * behind the metric of SURVEY 8(d) (proposals, evaluations, accepts) and the
+ * per-phase times of Fig. 11/12 (P:322-330 4.3). */
 gsap_status gsap_get_stats(gsap_ctx *ctx, gsap_stats *out);
 gsap_status gsap_reset_stats(gsap_ctx *ctx);
 
-/* Synchronise the context's stream. */
+/* Synchronise the context's stream (host-side ordering only; no computation). */
 gsap_status gsap_sync(gsap_ctx *ctx);
 
 /*
@@ -222,9 +248,9 @@ gsap_status gsap_sync(gsap_ctx *ctx);
  * trace (host, nullable): GSAP_TRACE_COLS doubles per round, at most
  * trace_cap rows: [outer, B after merge, MCMC iterations, MDL, round seconds,
  * accepted moves, device ms of the move / rebuild / merge kernels (profile = 1,
- * else 0)]; *rounds_out (host, nullable).
+ * else 0), convergence threshold used (R:Z19)]; *rounds_out (host, nullable).
  */
-#define GSAP_TRACE_COLS 9
+#define GSAP_TRACE_COLS 10
 gsap_status gsap_run(gsap_ctx *ctx, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
                      double *trace, int32_t trace_cap, int32_t *rounds_out);
 

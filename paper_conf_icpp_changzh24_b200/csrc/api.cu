@@ -10,6 +10,7 @@
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
+#include <map>
 #include <mutex>
 #include <new>
 #include <vector>
@@ -134,6 +135,19 @@ void kc_resolve(Ctx &c, KClass &k) {
 
 }  // namespace gsap
 
+int gsap::per_device(const void *key, const std::function<int()> &f) {
+    int dev = 0;
+    GSAP_CUDA(cudaGetDevice(&dev));
+    static std::mutex mu;
+    static std::map<std::pair<const void *, int>, int> cache;
+    std::lock_guard<std::mutex> g(mu);
+    const auto it = cache.find({key, dev});
+    if (it != cache.end()) return it->second;
+    const int v = f();
+    cache[{key, dev}] = v;
+    return v;
+}
+
 static bool is_dev(const void *p) {
     if (!p) return false;
     cudaPointerAttributes a;
@@ -144,11 +158,12 @@ static bool is_dev(const void *p) {
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
-// dst: host or device; src: device
+// dst: host or device; src: device.  Complete on return (a device output is
+// then safe on any stream of the caller: no ordering against c.stream needed)
 static void copy_out(Ctx &c, void *dst, const void *src, size_t bytes) {
     if (!dst || !bytes) return;
     GSAP_CUDA(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDefault, c.stream));
-    if (!is_dev(dst)) GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
 }
 
 // src: host or device -> a device pointer (src itself, or staged into `scratch`)
@@ -179,7 +194,7 @@ static void free_ctx(Ctx &c) {
     c.arena = nullptr;
     if (c.h_scal) cudaFreeHost(c.h_scal);
     if (c.h_int) cudaFreeHost(c.h_int);
-    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl}) {
+    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl, &c.k_comm}) {
         for (auto &p : k->pending) {
             cudaEventDestroy(p.first);
             cudaEventDestroy(p.second);
@@ -392,6 +407,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.partials = A.take<double>(VE / 512 + 1024);   // >= max(E, B) / MDL_CHUNK, V / APPLY_CHUNK + ranks
         c.scal = A.take<double>(8);
         c.scal_i = A.take<int>(8);
+        c.n_eval = A.take<unsigned long long>(1);
         c.Dh = A.take<double>((size_t)c.prm.max_nodal_itr + 1);
         c.d_itr = A.take<unsigned>(1);
         c.skey0 = A.take<unsigned long long>(Vs);
@@ -460,6 +476,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
                                   cudaMemcpyHostToDevice, c.stream));
     GSAP_CUDA(cudaMemsetAsync(c.scal, 0, 8 * sizeof(double), c.stream));
     GSAP_CUDA(cudaMemsetAsync(c.scal_i, 0, 8 * sizeof(int), c.stream));
+    GSAP_CUDA(cudaMemsetAsync(c.n_eval, 0, sizeof(unsigned long long), c.stream));
     mark("upload");
     build_graph_device(c);
     mark("csc");
@@ -511,7 +528,7 @@ static void merge_phase(Ctx &c, uint32_t outer, int K, int *best_out, double *dS
 static void move_batch(Ctx &c, uint32_t outer, uint32_t itr, int first, int count, double *dsum) {
     if (c.nranks == 1) {
         launch_move(c, MOVE_FUSED, outer, itr, first, count, c.s, c.dS, nullptr, c.acc);
-        launch_apply(c, first, count, c.s, c.acc, c.dS, dsum, c.scal_i + 1);
+        launch_apply(c, first, count, c.s, c.acc, c.dS, dsum, c.scal_i + 1, c.n_eval);
         rebuild(c);
         c.st.n_move_prop += count;
         return;
@@ -530,7 +547,7 @@ static void move_batch(Ctx &c, uint32_t outer, uint32_t itr, int first, int coun
     comm_allgather(c, c.acc, (size_t)per, 0);
     comm_allgather(c, c.partials, (size_t)pc, 2);
     const int chunks = (count + APPLY_CHUNK_V - 1) / APPLY_CHUNK_V;
-    launch_apply_gathered(c, first, count, c.s, c.acc, c.partials, chunks, dsum, c.scal_i + 1);
+    launch_apply_gathered(c, first, count, c.s, c.acc, c.partials, chunks, dsum, c.scal_i + 1, c.n_eval);
     rebuild(c);
     c.st.n_move_prop += n;
 }
@@ -552,7 +569,7 @@ static bool converged(Ctx &c, const std::vector<double> &D, int itr, double S, d
 // MCMC phase with every iteration (num_batches x (move + apply + rebuild) +
 // the MDL reduction) captured once into a CUDA graph; one graph launch, one
 // 16-byte D2H and one synchronisation per iteration.
-static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh) {
+static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh, std::vector<double> *D_out) {
     const int V = c.V, nb = c.prm.num_batches;
     const int bs = (V + nb - 1) / nb;
     cudaGraph_t graph = nullptr;
@@ -567,7 +584,7 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh) {
             const int first = k * bs, last = std::min(V, first + bs);
             if (first >= last) continue;
             launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
-            launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1);
+            launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
             rebuild(c);
         }
         launch_data_term(c);
@@ -610,6 +627,7 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh) {
     GSAP_CUDA(cudaGraphExecDestroy(exec));
     GSAP_CUDA(cudaGraphDestroy(graph));
     graph_release_events(c);
+    if (D_out) D_out->assign(D.begin(), D.begin() + ran);
     if (getenv("GSAP_TIMING")) {
         const auto tc2 = std::chrono::steady_clock::now();
         fprintf(stderr, "[gsap] mcmc B=%d kernels/itr=%lld capture %.3f ms instantiate %.3f ms %d itrs %.3f ms\n", c.B,
@@ -651,7 +669,7 @@ __global__ void k_mcmc_step(cudaGraphConditionalHandle h, unsigned *d_itr, doubl
 // convergence test or max_nodal_itr stops it -- no host round trip per
 // iteration (N1, P:385 5).  Event nodes are not allowed in conditional
 // bodies, so profile = 1 uses mcmc_phase_graph.
-static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh) {
+static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::vector<double> *D_out) {
     const int V = c.V, nb = c.prm.num_batches;
     const int bs = (V + nb - 1) / nb;
     const long long l0 = c.launches;
@@ -678,7 +696,7 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh) {
                 const int first = k * bs, last = std::min(V, first + bs);
                 if (first >= last) continue;
                 launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
-                launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1);
+                launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
                 rebuild(c);
             }
             launch_data_term(c);
@@ -706,6 +724,11 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh) {
         GSAP_CUDA(cudaMemcpyAsync(c.h_int + 2, c.d_itr, sizeof(unsigned), cudaMemcpyDeviceToHost, c.stream));
         GSAP_CUDA(cudaStreamSynchronize(c.stream));
         const int ran = c.h_int[2];
+        if (D_out) {
+            D_out->resize((size_t)ran);
+            if (ran)
+                GSAP_CUDA(cudaMemcpy(D_out->data(), c.Dh, sizeof(double) * (size_t)ran, cudaMemcpyDeviceToHost));
+        }
         c.launches += kernels * ran;
         c.st.n_move_prop += (long long)V * ran;
         GSAP_CUDA(cudaGraphExecDestroy(exec));
@@ -725,10 +748,11 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh) {
     }
 }
 
-// returns the number of MCMC iterations run (O.8)
-static int mcmc_phase(Ctx &c, uint32_t outer, double thresh) {
-    if (c.prm.cuda_graphs == 2 && !c.prm.profile && c.nranks == 1) return mcmc_phase_device_loop(c, outer, thresh);
-    if (c.prm.cuda_graphs) return mcmc_phase_graph(c, outer, thresh);
+// returns the number of MCMC iterations run (O.8); D_out (nullable): D[itr]
+static int mcmc_phase(Ctx &c, uint32_t outer, double thresh, std::vector<double> *D_out = nullptr) {
+    if (c.prm.cuda_graphs == 2 && !c.prm.profile && c.nranks == 1)
+        return mcmc_phase_device_loop(c, outer, thresh, D_out);
+    if (c.prm.cuda_graphs) return mcmc_phase_graph(c, outer, thresh, D_out);
     const int V = c.V, nb = c.prm.num_batches, w = c.prm.window;
     const int bs = (V + nb - 1) / nb;
     std::vector<double> D((size_t)c.prm.max_nodal_itr + 1, 0.0);
@@ -749,6 +773,10 @@ static int mcmc_phase(Ctx &c, uint32_t outer, double thresh) {
             GSAP_CUDA(cudaStreamSynchronize(c.stream));
             if (converged(c, D, itr, c.h_scal[1], thresh)) break;
         }
+    }
+    if (D_out) {
+        D_out->resize((size_t)ran);
+        if (ran) GSAP_CUDA(cudaMemcpy(D_out->data(), c.Dh, sizeof(double) * (size_t)ran, cudaMemcpyDeviceToHost));
     }
     return ran;
 }
@@ -859,6 +887,7 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
             row[6] = c.k_move.ms - ms0[0];
             row[7] = c.k_rebuild.ms - ms0[1];
             row[8] = c.k_merge.ms - ms0[2];
+            row[9] = bracket ? c.prm.thresh2 : c.prm.thresh1;
         }
         c.st.mcmc_itr_total += itrs;
         ++rounds;
@@ -895,8 +924,14 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
 }
 
 static void fill_stats(Ctx &c, gsap_stats *out) {
-    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl}) kc_resolve(c, *k);
+    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl, &c.k_comm}) kc_resolve(c, *k);
     gsap_stats s = c.st;
+    unsigned long long ne = 0;
+    GSAP_CUDA(cudaMemcpyAsync(&ne, c.n_eval, sizeof(ne), cudaMemcpyDeviceToHost, c.stream));
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    s.n_move_eval = (int64_t)ne;
+    s.t_rebuild = c.k_rebuild.ms * 1e-3;
+    s.t_comm = c.k_comm.ms * 1e-3;
     s.gpu_launches = c.launches;
     s.k_move_ms = c.k_move.ms;
     s.k_move_bytes = c.k_move.bytes;
@@ -970,6 +1005,8 @@ gsap_status gsap_set_partition(gsap_ctx *ctx, const int32_t *b, int32_t B) {
     REQUIRE(B >= 1 && B <= c.V, GSAP_EINVAL, "B must be in [1, V]");
     if (!is_dev(b)) {
         for (int v = 0; v < c.V; ++v) REQUIRE(b[v] >= 0 && b[v] < B, GSAP_EINVAL, "b[v] out of [0, B)");
+    } else {
+        REQUIRE(device_ids_ok(c, c.V, b, nullptr, B, false), GSAP_EINVAL, "b[v] out of [0, B)");
     }
     GSAP_CUDA(cudaMemcpyAsync(c.b, b, sizeof(int) * (size_t)c.V, cudaMemcpyDefault, c.stream));
     c.B = B;
@@ -1048,6 +1085,8 @@ gsap_status gsap_select_merges(gsap_ctx *ctx, const int32_t *best, const double 
     if (!is_dev(best))
         for (int r = 0; r < B; ++r)
             REQUIRE(best[r] >= 0 && best[r] < B && best[r] != r, GSAP_EINVAL, "best[r] must be in [0,B), != r");
+    else
+        REQUIRE(device_ids_ok(c, B, best, nullptr, B, true), GSAP_EINVAL, "best[r] must be in [0,B), != r");
     const int *db = stage_in(c, best, (size_t)B, c.best);
     const double *dd = stage_in(c, dS, (size_t)B, c.dSbest);
     select_merges(c, db, dd, K, nullptr);
@@ -1063,11 +1102,11 @@ gsap_status gsap_apply_moves(gsap_ctx *ctx, int32_t first, int32_t count, const 
     REQUIRE(ctx && s && acc, GSAP_EINVAL, "NULL argument");
     Ctx &c = ctx->c;
     REQUIRE(first >= 0 && count >= 0 && (long long)first + count <= c.V, GSAP_EINVAL, "range out of bounds");
-    if (!is_dev(s))
-        for (int i = 0; i < count; ++i)
-            REQUIRE(!acc[i] || (s[i] >= 0 && s[i] < c.B), GSAP_EINVAL, "s out of [0, B)");
+    // s and acc may each be host or device: both staged to the device, then
+    // range-checked there before anything is written into b
     const int *ds = stage_in(c, s, (size_t)count, c.s);
     const unsigned char *da = stage_in(c, (const unsigned char *)acc, (size_t)count, c.acc);
+    REQUIRE(device_ids_ok(c, count, ds, da, c.B, false), GSAP_EINVAL, "accepted s out of [0, B)");
     launch_apply(c, first, count, ds, da, nullptr, c.scal, nullptr);
     GSAP_CUDA(cudaStreamSynchronize(c.stream));
     API_CATCH
@@ -1089,6 +1128,20 @@ gsap_status gsap_move_batch(gsap_ctx *ctx, uint32_t outer, uint32_t itr, int32_t
         GSAP_CUDA(cudaStreamSynchronize(c.stream));
         *dsum_out = c.h_scal[0];
     }
+    API_CATCH
+}
+
+gsap_status gsap_mcmc_phase(gsap_ctx *ctx, uint32_t outer, double thresh, double *D_out, int32_t *itrs_out) {
+    API_TRY
+    REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
+    Ctx &c = ctx->c;
+    REQUIRE(thresh >= 0.0, GSAP_EINVAL, "thresh must be >= 0");
+    std::vector<double> D;
+    const int ran = mcmc_phase(c, outer, thresh, &D);
+    c.st.mcmc_itr_total += ran;
+    if (D_out && ran) memcpy(D_out, D.data(), sizeof(double) * (size_t)ran);
+    if (itrs_out) *itrs_out = ran;
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
     API_CATCH
 }
 
@@ -1200,12 +1253,14 @@ gsap_status gsap_reset_stats(gsap_ctx *ctx) {
     API_TRY
     REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
     Ctx &c = ctx->c;
-    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl}) {
+    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl, &c.k_comm}) {
         kc_resolve(c, *k);
         k->ms = 0;
         k->bytes = 0;
         k->launches = 0;
     }
+    GSAP_CUDA(cudaMemsetAsync(c.n_eval, 0, sizeof(unsigned long long), c.stream));
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
     c.st = gsap_stats{};
     c.launches = 0;
     API_CATCH

@@ -82,7 +82,10 @@ void comm_allgather(Ctx &c, void *recv, size_t count_per_rank, int dtype) {
     const ncclDataType_t t = dtype == 0 ? ncclInt8 : (dtype == 1 ? ncclInt32 : ncclFloat64);
     const size_t esz = dtype == 0 ? 1 : (dtype == 1 ? 4 : 8);
     const char *send = (const char *)recv + (size_t)c.rank * count_per_rank * esz;
+    cudaEvent_t ev = nullptr;
+    kc_begin(c, c.k_comm, &ev);
     GSAP_NCCL(nccl_api()->AllGather(send, recv, count_per_rank, t, (ncclComm_t)c.nccl_comm, c.stream));
+    kc_end(c, c.k_comm, ev, (double)count_per_rank * esz * c.nranks);
 }
 
 void shard_slice(int n, int chunk, int G, int g, int *first, int *count, int *per_rank) {

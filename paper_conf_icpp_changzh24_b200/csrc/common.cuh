@@ -108,15 +108,6 @@ GSAP_DEV double g2_t(const double2 *__restrict__ ft, long long a, long long c) {
     return g2(a, c);
 }
 
-// legacy exact-math form (tests of the table path compare against it)
-GSAP_DEV double df(long long m, long long d) {
-    if (d == 0) return 0.0;
-    const long long n = m + d;
-    if (m == 0) return fx((double)n);
-    if (n == 0) return -fx((double)m);
-    return (double)d * log((double)n) + (double)m * log1p((double)d / (double)m);
-}
-
 // -------------------------------------------------------------- warps --
 GSAP_DEV unsigned lane_id() { return threadIdx.x & 31u; }
 

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <functional>
 #include <string>
 #include <vector>
 
@@ -102,7 +103,9 @@ struct Ctx {
     double *dSbest = nullptr;    // B
     double *partials = nullptr;  // reduction partials
     double *scal = nullptr;      // device scalars [0] = batch dS sum, [1] = data term
-    int *scal_i = nullptr;       // device int scalars [0] = new B, [1] = accepted moves
+    int *scal_i = nullptr;       // device int scalars [0] = new B, [1] = accepted moves, [4] apply
+                                 // arrivals, [6] argument check flag
+    unsigned long long *n_eval = nullptr;   // device counter: evaluated MOVE proposals (s != b[v])
     double *Dh = nullptr;        // per-iteration sum of accepted dS (max_nodal_itr)
     int *slot_b[3] = {nullptr, nullptr, nullptr};   // golden-section bracket partitions
     // merge selection scratch
@@ -125,7 +128,7 @@ struct Ctx {
 
     // accounting
     long long launches = 0;
-    KClass k_move, k_rebuild, k_merge, k_mdl;
+    KClass k_move, k_rebuild, k_merge, k_mdl, k_comm;
     gsap_stats st{};
     std::vector<double> move_bytes_per_batch;   // algorithmic bytes per MOVE launch
 
@@ -159,6 +162,10 @@ struct Error {
 
 #define GSAP_CHECK_LAUNCH() GSAP_CUDA(cudaGetLastError())
 
+// f() once per (key, current device), result cached under a mutex: kernel
+// attributes (cudaFuncSetAttribute is per device) and occupancy-derived grids
+int per_device(const void *key, const std::function<int()> &f);
+
 // event timing of a kernel class (no-op unless prm.profile)
 void kc_begin(Ctx &c, KClass &k, cudaEvent_t *ev);
 void kc_end(Ctx &c, KClass &k, cudaEvent_t ev, double bytes);
@@ -175,12 +182,15 @@ enum MoveMode { MOVE_FUSED = 0, MOVE_PROPOSE = 1, MOVE_DELTA = 2 };
 void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first, int count,
                  int *s, double *dS, double *H, unsigned char *acc, const unsigned *d_itr = nullptr);
 void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned char *acc,
-                  const double *dS, double *dsum, int *nacc);
+                  const double *dS, double *dsum, int *nacc, unsigned long long *n_eval = nullptr);
+// device-side range check of id arrays (argument validation); synchronises
+bool device_ids_ok(Ctx &c, int n, const int *x, const unsigned char *mask, int B, bool not_self);
 
 void launch_partials(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
                      double *partials);
 void launch_apply_gathered(Ctx &c, int first, int count, const int *s, const unsigned char *acc,
-                           const double *partials, int n, double *dsum, int *nacc);
+                           const double *partials, int n, double *dsum, int *nacc,
+                           unsigned long long *n_eval = nullptr);
 constexpr int APPLY_CHUNK_V = 1024;   // fixed reduction chunk of the accepted-dS sums (move.cu)
 
 // comm.cu: multi-GPU (one process per GPU, NCCL over NVLink, loaded at run time)

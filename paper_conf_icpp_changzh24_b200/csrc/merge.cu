@@ -377,11 +377,10 @@ __global__ void __launch_bounds__(SEL_THREADS) k_labels_small(int B, const int *
 static void select_merges_small(Ctx &c, const int *best, const double *dS, int K, int rounds) {
     const int B = c.B, V = c.V;
     const size_t smem = sizeof(u64) * SEL_SMALL_B + sizeof(int) * (7 * SEL_SMALL_B + 32);
-    static bool attr = false;
-    if (!attr) {
+    per_device((const void *)k_select_small, [&] {
         GSAP_CUDA(cudaFuncSetAttribute(k_select_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        attr = true;
-    }
+        return 1;
+    });
     k_select_small<<<1, SEL_THREADS, smem, c.stream>>>(B, K, rounds, best, dS, c.nxt0);
     GSAP_CUDA(cudaMemsetAsync(c.present, 0, sizeof(int) * ((size_t)B + 1), c.stream));
     k_present<<<g256(V), 256, 0, c.stream>>>(V, c.b, c.nxt0, c.present);

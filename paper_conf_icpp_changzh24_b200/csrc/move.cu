@@ -921,15 +921,14 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         GSAP_CHECK_LAUNCH();
         GSAP_CUDA(cudaEventRecord(c.ev_join, c.side));
     }
-    static bool attr = false;
-    if (!attr) {
+    per_device((const void *)k_move<false, false>, [] {
         const int sm = (int)MOVE_SMEM;
         GSAP_CUDA(cudaFuncSetAttribute(k_move<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
         GSAP_CUDA(cudaFuncSetAttribute(k_move<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
         GSAP_CUDA(cudaFuncSetAttribute(k_move<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
         GSAP_CUDA(cudaFuncSetAttribute(k_move<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
-        attr = true;
-    }
+        return 1;
+    });
     const bool dense = a.m.dense != nullptr;
     if (c.weighted) {
         if (dense) k_move<true, true><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);
@@ -952,16 +951,20 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
 // ---------------------------------------------------------------- apply --
 constexpr int APPLY_CHUNK = 1024;
 
+// n_eval (nullable): += the proposals with s != b[v] (the moves that were
+// evaluated, R:Z13) -- counted before b is written
 __global__ void __launch_bounds__(256) k_apply(int first, int count, const int *__restrict__ s,
                                                const unsigned char *__restrict__ acc,
                                                const double *__restrict__ dS, int *__restrict__ b,
-                                               double *__restrict__ partials, int *__restrict__ nacc) {
+                                               double *__restrict__ partials, int *__restrict__ nacc,
+                                               unsigned long long *__restrict__ n_eval) {
     __shared__ double sh[8];
     const int base = blockIdx.x * APPLY_CHUNK;
     double sum = 0.0;
-    int na = 0;
+    int na = 0, ne = 0;
     for (int k = threadIdx.x; k < APPLY_CHUNK; k += 256) {
         const int i = base + k;
+        if (i < count && n_eval) ne += s[i] != b[first + i];
         if (i < count && acc[i]) {
             if (b) b[first + i] = s[i];
             sum += dS ? dS[i] : 0.0;
@@ -970,6 +973,10 @@ __global__ void __launch_bounds__(256) k_apply(int first, int count, const int *
     }
     na = warp_sum(na);
     if (nacc && (threadIdx.x & 31) == 0 && na) atomicAdd(nacc, na);
+    if (n_eval) {
+        ne = warp_sum(ne);
+        if ((threadIdx.x & 31) == 0 && ne) atomicAdd(n_eval, (unsigned long long)ne);
+    }
     sum = warp_sum(sum);
     if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = sum;
     __syncthreads();
@@ -1003,14 +1010,16 @@ __global__ void __launch_bounds__(256) k_apply_sum(int first, int count, const i
                                                    const unsigned char *__restrict__ acc,
                                                    const double *__restrict__ dS, int *__restrict__ b,
                                                    double *__restrict__ partials, int *__restrict__ nacc,
-                                                   unsigned *__restrict__ arrivals, double *__restrict__ dsum) {
+                                                   unsigned *__restrict__ arrivals, double *__restrict__ dsum,
+                                                   unsigned long long *__restrict__ n_eval) {
     __shared__ double sh[8];
     __shared__ bool last;
     const int base = blockIdx.x * APPLY_CHUNK;
     double sum = 0.0;
-    int na = 0;
+    int na = 0, ne = 0;
     for (int k = threadIdx.x; k < APPLY_CHUNK; k += 256) {
         const int i = base + k;
+        if (i < count && n_eval) ne += s[i] != b[first + i];
         if (i < count && acc[i]) {
             b[first + i] = s[i];
             sum += dS ? dS[i] : 0.0;
@@ -1019,6 +1028,10 @@ __global__ void __launch_bounds__(256) k_apply_sum(int first, int count, const i
     }
     na = warp_sum(na);
     if (nacc && (threadIdx.x & 31) == 0 && na) atomicAdd(nacc, na);
+    if (n_eval) {
+        ne = warp_sum(ne);
+        if ((threadIdx.x & 31) == 0 && ne) atomicAdd(n_eval, (unsigned long long)ne);
+    }
     sum = warp_sum(sum);
     if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = sum;
     __syncthreads();
@@ -1045,12 +1058,36 @@ __global__ void __launch_bounds__(256) k_apply_sum(int first, int count, const i
     }
 }
 
+// argument validation of device inputs (gsap_set_partition, gsap_apply_moves,
+// gsap_select_merges): *bad = 1 if some x[i] (with mask[i] != 0, if a mask is
+// given) lies outside [0, B), or equals i when not_self
+__global__ void k_check_ids(int n, const int *__restrict__ x, const unsigned char *__restrict__ mask, int B,
+                            int not_self, int *__restrict__ bad) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        if (mask && !mask[i]) continue;
+        const int v = x[i];
+        if (v < 0 || v >= B || (not_self && v == i)) *bad = 1;
+    }
+}
+
+bool device_ids_ok(Ctx &c, int n, const int *x, const unsigned char *mask, int B, bool not_self) {
+    if (n <= 0) return true;
+    GSAP_CUDA(cudaMemsetAsync(c.scal_i + 6, 0, sizeof(int), c.stream));
+    const int g = (int)std::min<long long>(((long long)n + 255) / 256, 148LL * 8);
+    k_check_ids<<<g, 256, 0, c.stream>>>(n, x, mask, B, not_self ? 1 : 0, c.scal_i + 6);
+    ++c.launches;
+    GSAP_CHECK_LAUNCH();
+    GSAP_CUDA(cudaMemcpyAsync(c.h_int + 6, c.scal_i + 6, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
+    GSAP_CUDA(cudaStreamSynchronize(c.stream));
+    return c.h_int[6] == 0;
+}
+
 void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
-                  double *dsum, int *nacc) {
+                  double *dsum, int *nacc, unsigned long long *n_eval) {
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
     k_apply_sum<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, c.b, c.partials, nacc,
-                                          reinterpret_cast<unsigned *>(c.scal_i + 4), dsum);
+                                          reinterpret_cast<unsigned *>(c.scal_i + 4), dsum, n_eval);
     c.launches += 1;
     GSAP_CHECK_LAUNCH();
 }
@@ -1061,17 +1098,17 @@ void launch_partials(Ctx &c, int first, int count, const int *s, const unsigned 
                      double *partials) {
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
-    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, nullptr, partials, nullptr);
+    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, nullptr, partials, nullptr, nullptr);
     ++c.launches;
     GSAP_CHECK_LAUNCH();
 }
 
 // sharded batches: apply all gathered moves, then the ordered sum of n partials
 void launch_apply_gathered(Ctx &c, int first, int count, const int *s, const unsigned char *acc,
-                           const double *partials, int n, double *dsum, int *nacc) {
+                           const double *partials, int n, double *dsum, int *nacc, unsigned long long *n_eval) {
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
-    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, nullptr, c.b, nullptr, nacc);
+    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, nullptr, c.b, nullptr, nacc, n_eval);
     k_sum_partials<<<1, 256, 0, c.stream>>>(partials, n, dsum, 1);
     c.launches += 2;
     GSAP_CHECK_LAUNCH();

@@ -303,12 +303,11 @@ int radix_sort(K *k0, K *k1, V *v0, V *v1, const int *d_n, int n_max, int bits, 
     const int nt = tiles_for(n_max);
     if (nt == 0 || bits <= 0) return 0;
     const size_t smem = sizeof(K) * PT_TILE + (HAS_V ? sizeof(V) * PT_TILE : 0);
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaFuncSetAttribute(k_rs_downsweep<K, V, HAS_V>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)smem);
-        attr_set = true;
-    }
+    per_device((const void *)k_rs_downsweep<K, V, HAS_V>, [&] {
+        GSAP_CUDA(cudaFuncSetAttribute(k_rs_downsweep<K, V, HAS_V>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)smem));
+        return 1;
+    });
     int cur = 0;
     for (int shift = 0; shift < bits; shift += 8) {
         K *ks = cur ? k1 : k0;

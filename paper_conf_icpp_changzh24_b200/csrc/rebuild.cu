@@ -597,8 +597,7 @@ static void launch_rebuild_dense_coop(Ctx &c) {
     a.d_nnz = c.d_nnz;
     a.bar = c.coop_bar;
     const size_t smem_max = SMEM ? std::max(DC_TILE_SMEM, sizeof(int) * SMALL_MAX_B * SMALL_MAX_B) : DC_TILE_SMEM;
-    static int grid = 0;
-    if (grid == 0) {
+    const int grid = per_device((const void *)k_rebuild_dense<SMEM>, [&] {
         GSAP_CUDA(cudaFuncSetAttribute(k_rebuild_dense<SMEM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)smem_max));
         int per_sm = 0, sms = 0, dev = 0;
@@ -606,8 +605,8 @@ static void launch_rebuild_dense_coop(Ctx &c) {
                                                                 smem_max));
         GSAP_CUDA(cudaGetDevice(&dev));
         GSAP_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-        grid = std::max(1, std::min(per_sm, SMEM ? 1 : 2) * sms);
-    }
+        return std::max(1, std::min(per_sm, SMEM ? 1 : 2) * sms);
+    });
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = dim3(DC_THREADS);
@@ -630,12 +629,11 @@ static void rebuild_dense(Ctx &c) {
         int dev_sms = 148;
         if (B <= HIST_SMEM_MAX_B) {
             const size_t smem = sizeof(int) * BB;
-            static bool attr = false;
-            if (!attr) {
+            per_device((const void *)k_hist<true>, [] {
                 GSAP_CUDA(cudaFuncSetAttribute(k_hist<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                HIST_SMEM_MAX_B * HIST_SMEM_MAX_B * 4));
-                attr = true;
-            }
+                return 1;
+            });
             const int grid = (int)std::min<long long>(dev_sms, ((long long)E + 1023) / 1024);
             k_hist<true><<<grid, 1024, smem, c.stream>>>(E, c.esrc, c.col, c.wgt, c.b, B, c.dense);
         } else {
@@ -686,12 +684,11 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, ptr, c.seg_nnz, c.seg_listW, c.seg_listC,
                                                            c.seg_ctr, out, extent, SEG_WARP_MAX_MK);
     const int gw_ = (int)std::min<long long>(((long long)B + SEG_WARPS - 1) / SEG_WARPS, 148LL * 16);
-    static bool attr = false;
-    if (!attr) {
+    per_device((const void *)k_segsort_warp<K, 2>, [] {
         GSAP_CUDA(cudaFuncSetAttribute(k_segsort_warp<K, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)seg_warp2_smem<K>()));
-        attr = true;
-    }
+        return 1;
+    });
     k_segsort_warp<K, 0><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, idx, cnt,
                                                               c.seg_nnz, out);
     k_segsort_warp<K, 1><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, idx, cnt,
@@ -733,15 +730,14 @@ static void rebuild_sparse_coop(Ctx &c) {
     a.nlong = c.seg_ctr;
     a.bar = c.coop_bar;
     const size_t smem = sizeof(CoopSmem<K>);
-    static int grid = 0;
-    if (grid == 0) {
+    const int grid = per_device((const void *)k_rebuild_coop<K>, [&] {
         GSAP_CUDA(cudaFuncSetAttribute(k_rebuild_coop<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         int per_sm = 0, sms = 0, dev = 0;
         GSAP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rebuild_coop<K>, 256, smem));
         GSAP_CUDA(cudaGetDevice(&dev));
         GSAP_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-        grid = std::max(3, per_sm * sms);
-    }
+        return std::max(3, per_sm * sms);
+    });
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = dim3(256);

@@ -19,14 +19,14 @@ LIB_PATH = os.environ.get("GSAP_LIB", os.path.join(HERE, "libgsap.so"))
 
 GSAP_OK, GSAP_EINVAL, GSAP_ENOMEM, GSAP_ECUDA, GSAP_ENCCL, GSAP_ESTATE, GSAP_EUNSUPPORTED = range(7)
 GSAP_MERGE, GSAP_MOVE = 0, 1
-TRACE_COLS = 9                  # GSAP_TRACE_COLS (gsap.h)
+TRACE_COLS = 10                 # GSAP_TRACE_COLS (gsap.h)
 STATUS_NAMES = ["GSAP_OK", "GSAP_EINVAL", "GSAP_ENOMEM", "GSAP_ECUDA", "GSAP_ENCCL", "GSAP_ESTATE",
                 "GSAP_EUNSUPPORTED"]
 
 EXPORTED = ["gsap_default_params", "gsap_last_error", "gsap_partition", "gsap_create", "gsap_destroy",
             "gsap_set_partition", "gsap_get_partition", "gsap_update_blockmodel", "gsap_propose",
             "gsap_delta_mdl", "gsap_select_merges", "gsap_apply_moves", "gsap_move_batch",
-            "gsap_merge_phase", "gsap_mdl", "gsap_get_blockmodel", "gsap_get_stats", "gsap_reset_stats",
+            "gsap_merge_phase", "gsap_mcmc_phase", "gsap_mdl", "gsap_get_blockmodel", "gsap_get_stats", "gsap_reset_stats",
             "gsap_sync", "gsap_run", "gsap_nccl_unique_id", "gsap_shard_slice"]
 
 
@@ -54,7 +54,8 @@ class gsap_stats(C.Structure):
                 ("k_rebuild_ms", C.c_double), ("k_rebuild_bytes", C.c_double),
                 ("k_rebuild_launches", C.c_int64),
                 ("k_merge_ms", C.c_double), ("k_merge_bytes", C.c_double), ("k_merge_launches", C.c_int64),
-                ("k_mdl_ms", C.c_double), ("k_mdl_launches", C.c_int64)]
+                ("k_mdl_ms", C.c_double), ("k_mdl_launches", C.c_int64),
+                ("t_rebuild", C.c_double), ("t_comm", C.c_double), ("n_move_eval", C.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -95,6 +96,7 @@ def lib():
         L.gsap_apply_moves.argtypes = [vp, i32, i32, vp, vp]
         L.gsap_move_batch.argtypes = [vp, u32, u32, i32, i32, vp, vp, vp, C.POINTER(C.c_double)]
         L.gsap_merge_phase.argtypes = [vp, u32, i32, vp, vp]
+        L.gsap_mcmc_phase.argtypes = [vp, u32, C.c_double, vp, C.POINTER(i32)]
         L.gsap_mdl.argtypes = [vp, C.POINTER(C.c_double), C.POINTER(C.c_double)]
         L.gsap_get_blockmodel.argtypes = [vp, i64p] + [vp] * 10
         L.gsap_get_stats.argtypes = [vp, C.POINTER(gsap_stats)]
@@ -116,7 +118,9 @@ def _check(status):
 
 
 def _ptr(x, dtype=None):
-    """Raw pointer of a numpy array / torch tensor (None -> NULL)."""
+    """Raw pointer of a numpy array / torch tensor (None -> NULL).  A CUDA
+    tensor is an input the library reads on its own stream (gsap.h): the
+    caller's current stream is synchronised first so its producer finished."""
     if x is None:
         return None
     if isinstance(x, np.ndarray):
@@ -133,6 +137,8 @@ def _ptr(x, dtype=None):
             raise TypeError(f"expected {want}, got {x.dtype}")
         if not x.is_contiguous():
             raise ValueError("tensor must be contiguous")
+        if x.is_cuda:
+            torch.cuda.current_stream(x.device).synchronize()
         return x.data_ptr()
     raise TypeError(f"unsupported array type {type(x)}")
 
@@ -299,6 +305,13 @@ class Context:
         dSb = _out(B, np.float64, device)
         _check(lib().gsap_merge_phase(self.h, outer, int(K), _ptr(best), _ptr(dSb)))
         return best, dSb
+
+    def gsap_mcmc_phase(self, outer, thresh):
+        """One MCMC phase from the current state: (iterations run, D[itr] per iteration)."""
+        D = np.zeros(self.params.max_nodal_itr + 1)
+        n = C.c_int32(0)
+        _check(lib().gsap_mcmc_phase(self.h, outer, float(thresh), D.ctypes.data, C.byref(n)))
+        return n.value, D[:n.value]
 
     def gsap_mdl(self):
         m, d = C.c_double(0), C.c_double(0)

@@ -54,8 +54,10 @@ def test_struct_layout_matches_header():
 #include <stdio.h>
 #include <stddef.h>
 #include "gsap.h"
-int main(void){printf("%zu %zu %zu %zu %zu\n", sizeof(gsap_params), sizeof(gsap_stats), sizeof(gsap_dist),
-  offsetof(gsap_stats, k_move_ms), offsetof(gsap_params, profile));return 0;}
+int main(void){printf("%zu %zu %zu %zu %zu %zu %zu %zu %d\n", sizeof(gsap_params), sizeof(gsap_stats),
+  sizeof(gsap_dist), offsetof(gsap_stats, k_move_ms), offsetof(gsap_params, profile),
+  offsetof(gsap_stats, t_rebuild), offsetof(gsap_stats, t_comm), offsetof(gsap_stats, n_move_eval),
+  GSAP_TRACE_COLS);return 0;}
 '''
     with tempfile.TemporaryDirectory() as d:
         c = os.path.join(d, "t.c")
@@ -64,7 +66,9 @@ int main(void){printf("%zu %zu %zu %zu %zu\n", sizeof(gsap_params), sizeof(gsap_
         subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), c, "-o", exe])
         got = list(map(int, subprocess.check_output([exe]).split()))
     want = [ctypes.sizeof(gsap.gsap_params), ctypes.sizeof(gsap.gsap_stats), ctypes.sizeof(gsap.gsap_dist),
-            gsap.gsap_stats.k_move_ms.offset, gsap.gsap_params.profile.offset]
+            gsap.gsap_stats.k_move_ms.offset, gsap.gsap_params.profile.offset,
+            gsap.gsap_stats.t_rebuild.offset, gsap.gsap_stats.t_comm.offset, gsap.gsap_stats.n_move_eval.offset,
+            gsap.TRACE_COLS]
     assert got == want
 
 
