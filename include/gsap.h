@@ -79,6 +79,11 @@ typedef struct {
     int32_t sel_small;        /* 1 (default): merge selection (a4) for B <= 4096 in one CTA (shared
                                  memory) + 4 grid launches; 0: the multi-kernel selection (radix
                                  sort, pointer-doubling launches).  Same result. */
+    int32_t move_sorted;      /* MOVE batches in the sparse regime: 1 (default) the sorted two-pass
+                                 evaluation (batch grouped by r, then by s) for graphs of
+                                 more than GSAP_COOP_MAX_E edges and batches of >= 2^16 vertices;
+                                 2: always (sparse regime, B > 128); 0: never (one fused pass).
+                                 Same integers; dS sums in another order (1e-9 contract). */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */
@@ -248,9 +253,11 @@ gsap_status gsap_sync(gsap_ctx *ctx);
  * trace (host, nullable): GSAP_TRACE_COLS doubles per round, at most
  * trace_cap rows: [outer, B after merge, MCMC iterations, MDL, round seconds,
  * accepted moves, device ms of the move / rebuild / merge kernels (profile = 1,
- * else 0), convergence threshold used (R:Z19)]; *rounds_out (host, nullable).
+ * else 0), convergence threshold used (R:Z19), B before the merge (the
+ * bracket slot the round restarted from, O.9), merges K requested];
+ * *rounds_out (host, nullable).
  */
-#define GSAP_TRACE_COLS 10
+#define GSAP_TRACE_COLS 12
 gsap_status gsap_run(gsap_ctx *ctx, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
                      double *trace, int32_t trace_cap, int32_t *rounds_out);
 

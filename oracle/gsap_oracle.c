@@ -31,9 +31,19 @@
  *     the kernel's precision.
  *
  * Parity status of each function is listed in DESIGN.md ("Oracle pins").
+ *
+ * Threads: single-threaded by default (the canonical run).  orc_set_threads(n)
+ * lets the per-vertex / per-block loops of a batch or a merge phase (proposals,
+ * Delta S, Hastings, accept) run on n OpenMP threads (SURVEY 8(d) "OpenMP
+ * across the batch"): every id writes only its own outputs from the same
+ * snapshot, so the results are identical for any n; everything else
+ * (rebuild, sums, selection, driver) stays sequential.
  */
 #include <fenv.h>
 #include <math.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -679,12 +689,28 @@ double orc_mdl(void *h, int variant, double *data_out)
     return orc_mdl_of((OState *)h, variant, data_out);
 }
 
+static int g_threads = 1;
+
+/* OpenMP threads of the per-id loops (1 = the canonical single-threaded run);
+ * returns the number in effect (1 if built without OpenMP) */
+int32_t orc_set_threads(int32_t n)
+{
+#ifdef _OPENMP
+    g_threads = n < 1 ? 1 : n;
+#else
+    (void)n;
+    g_threads = 1;
+#endif
+    return g_threads;
+}
+
 /* phase 0 = MERGE (ids are blocks, P draws each), 1 = MOVE (ids are vertices) */
 void orc_propose(void *h, int phase, uint64_t seed, uint32_t outer, uint32_t itr,
                  int32_t first, int32_t count, int32_t P, int32_t *s_out)
 {
     OState *st = (OState *)h;
     int32_t i, j;
+#pragma omp parallel for private(j) schedule(dynamic, 256) num_threads(g_threads) if (g_threads > 1)
     for (i = 0; i < count; ++i) {
         if (phase == 1)
             s_out[i] = propose_move(st, seed, outer, itr, first + i);
@@ -699,22 +725,31 @@ void orc_delta_move(void *h, uint64_t seed, uint32_t outer, uint32_t itr, double
                     double *dS, double *H, double *p, uint8_t *acc)
 {
     OState *st = (OState *)h;
-    DL d = {0, 0, 0};
-    int32_t i;
-    for (i = 0; i < count; ++i)
-        eval_move(st, &d, seed, outer, itr, beta, first + i, s[i], &dS[i], &H[i], &p[i], &acc[i]);
-    free(d.t);
+#pragma omp parallel num_threads(g_threads) if (g_threads > 1)
+    {
+        DL d = {0, 0, 0};   /* scratch per thread */
+        int32_t i;
+#pragma omp for schedule(dynamic, 256)
+        for (i = 0; i < count; ++i)
+            eval_move(st, &d, seed, outer, itr, beta, first + i, s[i], &dS[i], &H[i], &p[i], &acc[i]);
+        free(d.t);
+    }
 }
 
 void orc_delta_merge(void *h, int32_t first, int32_t count, int32_t P,
                      const int32_t *s, double *dS)
 {
     OState *st = (OState *)h;
-    DL d = {0, 0, 0};
-    int64_t i, n = (int64_t)count * P;
-    for (i = 0; i < n; ++i)
-        dS[i] = eval_merge(st, &d, first + (int32_t)(i / P), s[i]);
-    free(d.t);
+    int64_t n = (int64_t)count * P;
+#pragma omp parallel num_threads(g_threads) if (g_threads > 1)
+    {
+        DL d = {0, 0, 0};   /* scratch per thread */
+        int64_t i;
+#pragma omp for schedule(dynamic, 256)
+        for (i = 0; i < n; ++i)
+            dS[i] = eval_merge(st, &d, first + (int32_t)(i / P), s[i]);
+        free(d.t);
+    }
 }
 
 /* best proposal per block: argmin_j with strict <, first j wins (R:Z16) */
@@ -922,6 +957,28 @@ int32_t orc_golden_mock(int32_t V, double rate, const double *mdl_of_B,
         B = sB[restart];
     }
     if (B_final) *B_final = sB[1] ? sB[1] : V;
+    return n;
+}
+
+/* The bracket logic replayed over a given sequence of rounds (B after the
+ * merge, MDL of the round) -- e.g. another implementation's trace: for each
+ * round k, the B the next round restarts from, its number of merges K
+ * (bracket_step above) and whether the bracket is established after round k
+ * (the next round then uses thresh2, R:Z19).  Returns the number of rounds
+ * after which the search stops (n if it would go on). */
+int32_t orc_bracket_replay(int32_t n, const int32_t *B, const double *S, double rate,
+                           int32_t *Bstart_next, int32_t *K_next, int32_t *bracket_next)
+{
+    int32_t sB[3] = {0, 0, 0}, k, K = 0;
+    double sS[3] = {INFINITY, INFINITY, INFINITY};
+    int restart = 1;
+    for (k = 0; k < n; ++k) {
+        int done = bracket_step(NULL, sB, sS, NULL, B[k], S[k], 0, rate, &K, &restart);
+        Bstart_next[k] = sB[restart];
+        K_next[k] = K;
+        bracket_next[k] = sS[2] != INFINITY;
+        if (done) return k + 1;
+    }
     return n;
 }
 

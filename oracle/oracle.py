@@ -67,7 +67,7 @@ def default_params(**kw) -> OParams:
 def build(force: bool = False) -> str:
     """Compile the oracle with gcc (plain -O2, strict IEEE, x87 long double)."""
     if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < os.path.getmtime(SRC):
-        subprocess.check_call(["gcc", "-O2", "-std=c99", "-fPIC", "-shared",
+        subprocess.check_call(["gcc", "-O2", "-std=c99", "-fPIC", "-shared", "-fopenmp",
                                "-o", LIB, SRC, "-lm"])
     return LIB
 
@@ -80,6 +80,8 @@ def lib():
     if _lib is None:
         L = C.CDLL(build())
         L.orc_philox.argtypes = [_u32p, _u32p, _u32p]
+        L.orc_set_threads.restype = C.c_int32
+        L.orc_set_threads.argtypes = [C.c_int32]
         L.orc_create.restype = C.c_void_p
         L.orc_create.argtypes = [C.c_int32, _i64p, _i32p, C.c_void_p]
         L.orc_destroy.argtypes = [C.c_void_p]
@@ -117,6 +119,8 @@ def lib():
         L.orc_mcmc_batch.restype = C.c_double
         L.orc_mcmc_batch.argtypes = [C.c_void_p, C.POINTER(OParams), C.c_uint32, C.c_uint32,
                                      C.c_int32, C.c_int32]
+        L.orc_bracket_replay.restype = C.c_int32
+        L.orc_bracket_replay.argtypes = [C.c_int32, _i32p, _f64p, C.c_double, _i32p, _i32p, _i32p]
         L.orc_golden_mock.restype = C.c_int32
         L.orc_golden_mock.argtypes = [C.c_int32, C.c_double, _f64p, _i32p, C.c_int32,
                                       C.POINTER(C.c_int32)]
@@ -136,6 +140,26 @@ def mcmc_stop_mock(D, mdl, window=3, thresh=5e-4):
     mdl = np.ascontiguousarray(mdl, np.float64)
     assert len(D) == len(mdl)
     return lib().orc_mcmc_stop_mock(D, mdl, len(D), window, thresh)
+
+
+def bracket_replay(B_after_merge, mdl, rate=0.4):
+    """The golden-section bracket logic (O.9) replayed over given rounds:
+    per round the next round's starting B, its K and whether the bracket is
+    established (next round on thresh2); and the number of rounds run."""
+    Bs = np.ascontiguousarray(B_after_merge, np.int32)
+    S = np.ascontiguousarray(mdl, np.float64)
+    n = len(Bs)
+    Bn = np.zeros(max(n, 1), np.int32)
+    Kn = np.zeros(max(n, 1), np.int32)
+    Br = np.zeros(max(n, 1), np.int32)
+    stop = lib().orc_bracket_replay(n, Bs, S, rate, Bn, Kn, Br)
+    return Bn[:n], Kn[:n], Br[:n].astype(bool), stop
+
+
+def set_threads(n: int) -> int:
+    """OpenMP threads of the oracle's per-id loops (1 = canonical single-thread;
+    results are identical for any n).  Returns the number in effect."""
+    return lib().orc_set_threads(int(n))
 
 
 def golden_mock(V, rate, mdl_of_B, cap=1000):

@@ -409,6 +409,12 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.scal_i = A.take<int>(8);
         c.n_eval = A.take<unsigned long long>(1);
         c.Dh = A.take<double>((size_t)c.prm.max_nodal_itr + 1);
+        if (c.prm.move_sorted) {
+            c.mv_cnt = A.take<int>(2 * Vs + 2);
+            c.mv_perm = A.take<int>(2 * Vs);
+            c.mv_part = A.take<double>(3 * Vs);
+            c.mv_scan_tmp = A.take<int>((2 * Vs + 4095) / 4096 + 16);
+        }
         c.d_itr = A.take<unsigned>(1);
         c.skey0 = A.take<unsigned long long>(Vs);
         c.skey1 = A.take<unsigned long long>(Vs);
@@ -855,6 +861,7 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
             acc_before = c.h_int[3];
         }
         auto ta = std::chrono::steady_clock::now();
+        const int B_start = c.B, K_round = K;
         merge_phase(c, outer, K, nullptr, nullptr);
         const int B = c.B;
         auto tb = std::chrono::steady_clock::now();
@@ -888,6 +895,8 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
             row[7] = c.k_rebuild.ms - ms0[1];
             row[8] = c.k_merge.ms - ms0[2];
             row[9] = bracket ? c.prm.thresh2 : c.prm.thresh1;
+            row[10] = (double)B_start;
+            row[11] = (double)K_round;
         }
         c.st.mcmc_itr_total += itrs;
         ++rounds;
@@ -970,6 +979,7 @@ void gsap_default_params(gsap_params *p) {
     p->sparse_coop = 1;
     p->dense_coop = 1;
     p->sel_small = 1;
+    p->move_sorted = 1;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }

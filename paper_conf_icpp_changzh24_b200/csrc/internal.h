@@ -107,6 +107,10 @@ struct Ctx {
                                  // arrivals, [6] argument check flag
     unsigned long long *n_eval = nullptr;   // device counter: evaluated MOVE proposals (s != b[v])
     double *Dh = nullptr;        // per-iteration sum of accepted dS (max_nodal_itr)
+    // sorted two-pass MOVE (move.cu): per-block counts / offsets [2B], the batch
+    // grouped by r then by s [2 count], pass-1 partials [3 count], scan scratch
+    int *mv_cnt = nullptr, *mv_perm = nullptr, *mv_scan_tmp = nullptr;
+    double *mv_part = nullptr;
     int *slot_b[3] = {nullptr, nullptr, nullptr};   // golden-section bracket partitions
     // merge selection scratch
     unsigned long long *skey0 = nullptr, *skey1 = nullptr;

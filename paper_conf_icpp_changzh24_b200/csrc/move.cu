@@ -21,6 +21,7 @@
 #include <cstdlib>
 
 #include "internal.h"
+#include "prims.cuh"
 
 namespace gsap {
 
@@ -66,6 +67,8 @@ struct MoveArgs {
     int4 *gtab;                     // huge role: global tables per CTA, or nullptr (shared)
     int gtab_log2;
     int nhuge_ctas;                 // CTAs [nbig_ctas, nbig_ctas + nhuge_ctas): huge role
+    const int *__restrict__ perm;   // sorted two-pass mode: batch indices in line order
+    double *part;                   // sorted two-pass mode: pass-1 partials, 3 per vertex
 };
 
 GSAP_DEV unsigned hash_slot(int t, int log2cap) {
@@ -140,13 +143,22 @@ GSAP_DEV void group_sum3(double &x, double &y, double &z, double *sh) {
 #ifndef GSAP_LOOKUP_CONDCNT
 #define GSAP_LOOKUP_CONDCNT 0
 #endif
-GSAP_DEV void lookup4_in(const Line (&L)[4], const int (&y)[4], int (&p)[4], int (&n)[4], int (&out)[4]) {
-    bool some[4];
+template <int N>
+GSAP_DEV bool any_open(const int (&n)[N]) {
+    bool o = false;
 #pragma unroll
-    for (int k = 0; k < 4; ++k) some[k] = n[k] > 0;
-    while (n[0] > 1 || n[1] > 1 || n[2] > 1 || n[3] > 1) {
+    for (int k = 0; k < N; ++k) o = o || n[k] > 1;
+    return o;
+}
+
+template <int N>
+GSAP_DEV void lookup4_in(const Line (&L)[N], const int (&y)[N], int (&p)[N], int (&n)[N], int (&out)[N]) {
+    bool some[N];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
+    for (int k = 0; k < N; ++k) some[k] = n[k] > 0;
+    while (any_open<N>(n)) {
+#pragma unroll
+        for (int k = 0; k < N; ++k) {
             if (n[k] > 1) {
                 const int h = n[k] >> 1;
                 p[k] = __ldg(L[k].idx + p[k] + h) <= y[k] ? p[k] + h : p[k];
@@ -155,7 +167,7 @@ GSAP_DEV void lookup4_in(const Line (&L)[4], const int (&y)[4], int (&p)[4], int
         }
     }
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
+    for (int k = 0; k < N; ++k) {
         int v = 0;
         if (some[k]) {
 #if GSAP_LOOKUP_CONDCNT
@@ -182,16 +194,18 @@ GSAP_DEV void lookup4(const Line (&L)[4], const int (&y)[4], int (&out)[4]) {
 // idx[(j len) >> 5], one load level); a lane narrows each key to one of the 32
 // buckets with five shuffles and binary-searches only that bucket -- five
 // dependent load levels fewer per lookup once lines exceed 32 entries
-GSAP_DEV void split4_load(const Line (&L)[4], int lane, int (&sp)[4]) {
+template <int N>
+GSAP_DEV void split4_load(const Line (&L)[N], int lane, int (&sp)[N]) {
 #pragma unroll
-    for (int k = 0; k < 4; ++k) sp[k] = L[k].len > 0 ? __ldg(L[k].idx + ((lane * L[k].len) >> 5)) : 0x7fffffff;
+    for (int k = 0; k < N; ++k) sp[k] = L[k].len > 0 ? __ldg(L[k].idx + ((lane * L[k].len) >> 5)) : 0x7fffffff;
 }
 
 // all 32 lanes: the bucket [p, p + n) of line k that holds key y[k] if present
 // (n = 0: absent); sp[k] are line k's splitters as split4_load left them
-GSAP_DEV void split4_bucket(const Line (&L)[4], const int (&sp)[4], const int (&y)[4], int (&p)[4], int (&n)[4]) {
+template <int N>
+GSAP_DEV void split4_bucket(const Line (&L)[N], const int (&sp)[N], const int (&y)[N], int (&p)[N], int (&n)[N]) {
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
+    for (int k = 0; k < N; ++k) {
         int j = 0;   // the last bucket whose first entry is <= y[k]
 #pragma unroll
         for (int st = 16; st >= 1; st >>= 1) {
@@ -618,6 +632,188 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
     }
 }
 
+// ------------------------------------------------------ sorted two-pass --
+// Large sparse blockmodels (lines of M far outside L2): a vertex move reads
+// four lines of M (rows and columns r and s), and lines fetched per vertex
+// are fetched again by the next vertex of the same block.  Here the batch is
+// evaluated in two passes over the SAME snapshot, each visiting the vertices
+// grouped by one of its two blocks (counting sort of the batch by r = b[v] and
+// by the proposal s), so consecutive warps search the same two lines and a
+// line leaves HBM about once per block and pass:
+//   pass 1 (grouped by r): rows / columns r -- every dS / Hastings term that
+//     reads M_r. or M_.r, the 2x2 core entries M_rr, M_rs, M_sr, the degree
+//     terms and the whole backward law p_bwd (R:Z26);
+//   pass 2 (grouped by s): rows / columns s -- the terms in M_s. / M_.s and
+//     M_ss, then dS, H = p_bwd / p_fwd and the MH decision (Eq. 7, R:O.5).
+// The split follows the decomposition above term by term; only the order of
+// the floating-point sums differs from the fused kernel.  Vertices with more
+// than 128 adjacency entries stay in k_move_groups (fused terms, s given).
+template <bool WEIGHTED, int PASS>
+GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    const int v = a.first + i;
+    const int r = __ldg(a.b + v);
+    const int s = a.s_in[i];
+    if (s == r) {   // R:Z13 (warp-uniform)
+        if (PASS == 2 && lane == 0) {
+            if (a.dS) a.dS[i] = 0.0;
+            if (a.H) a.H[i] = 1.0;
+            if (a.acc) a.acc[i] = 0;
+        }
+        return;
+    }
+    const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
+    const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
+    const int deg = nout + nin;   // <= 128 (the caller routes bigger vertices to k_move_groups)
+    const int B = a.m.B;
+    // the two lines of this pass and their splitters, issued before the histogram
+    Line Ln[2];
+    const int x = PASS == 1 ? r : s;
+    Ln[0] = row_line(a.m, x);
+    Ln[1] = col_line(a.m, x);
+    int sp[2];
+    split4_load<2>(Ln, lane, sp);
+    // ---- phase A: histogram of v's neighbour blocks (self-loop excluded)
+    int keep[4];
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+        keep[c] = -1;
+        const int j = c * 32 + lane;
+        if (j < deg) {
+            const bool out = j < nout;
+            const int n = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+            if (n != v) {
+                const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
+                const int sl = tab_insert(tab, WARP_TAB_LOG2, __ldg(a.b + n));
+                atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
+                atomicMin(&tab[sl].w, j);
+                keep[c] = sl;
+            }
+        }
+    }
+    __syncwarp();
+    int nuniq = 0;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+        const int sl = keep[c];
+        const bool own = sl >= 0 && tab[sl].w == c * 32 + lane;
+        const unsigned bal = __ballot_sync(FULL, own);
+        if (own) list[nuniq + __popc(bal & lt)] = sl;
+        nuniq += __popc(bal);
+    }
+    __syncwarp();
+    const int slr = tab_find(tab, WARP_TAB_LOG2, r), sls = tab_find(tab, WARP_TAB_LOG2, s);
+    const int o_r = slr >= 0 ? tab[slr].y : 0, i_r = slr >= 0 ? tab[slr].z : 0;
+    const int o_s = sls >= 0 ? tab[sls].y : 0, i_s = sls >= 0 ? tab[sls].z : 0;
+    const int kout = __ldg(a.kout + v), kin = __ldg(a.kin + v), l = __ldg(a.selfw + v);
+    const int dout_r = __ldg(a.m.dout + r), dout_s = __ldg(a.m.dout + s);
+    const int din_r = __ldg(a.m.din + r), din_s = __ldg(a.m.din + s);
+    const double Bd = (double)B;
+    const int dr2 = dout_r + din_r - kout - kin, ds2 = dout_s + din_s + kout + kin;
+    const double2 *__restrict__ ft = a.m.ft;
+    const double *__restrict__ rcp = a.m.rcp;
+    // ---- core entries of this pass: pass 1 M_rr, M_rs (row r), M_sr (column r); pass 2 M_ss (row s)
+    int Mrr = 0, Mrs = 0, Msr = 0, Mss = 0;
+    if (PASS == 1) {
+        const Line Lc[3] = {Ln[0], Ln[0], Ln[1]};
+        const int spc[3] = {sp[0], sp[0], sp[1]};
+        const int yc[3] = {r, s, s};
+        int oc[3], pc[3], nc[3];
+        split4_bucket<3>(Lc, spc, yc, pc, nc);
+        lookup4_in<3>(Lc, yc, pc, nc, oc);
+        Mrr = oc[0];
+        Mrs = oc[1];
+        Msr = oc[2];
+    } else {
+        const Line Lc[1] = {Ln[0]};
+        const int spc[1] = {sp[0]};
+        const int yc[1] = {s};
+        int oc[1], pc[1], nc[1];
+        split4_bucket<1>(Lc, spc, yc, pc, nc);
+        lookup4_in<1>(Lc, yc, pc, nc, oc);
+        Mss = oc[0];
+    }
+    const int Mrr2 = Mrr - o_r - i_r - l, Mrs2 = Mrs + i_r - o_s, Msr2 = Msr + o_r - i_s;
+    // ---- phase B: one unique neighbour block per lane, this pass's two lines
+    double accS = 0.0, pf = 0.0, pb = 0.0;
+    for (int base = 0; base < nuniq; base += 32) {   // warp-uniform trips (shuffles below)
+        const int k = base + lane;
+        const int4 e = k >= nuniq ? make_int4(-1, 0, 0, 0) : tab[list[k]];
+        const int t = e.x, ot = e.y, it = e.z;
+        int pb2[2], nb2[2];
+        {
+            const int yt[2] = {t, t};
+            split4_bucket<2>(Ln, sp, yt, pb2, nb2);
+        }
+        if (k >= nuniq) continue;
+        const double cw = (double)(ot + it);
+        if (t == r) {
+            if (PASS == 1) {
+                pf += cw * (double)(Mrs + Msr + 1) * __ldg(rcp + r);
+                pb += cw * (double)(2 * Mrr2 + 1) / ((double)dr2 + Bd);
+            }
+        } else if (t == s) {
+            if (PASS == 1) pb += cw * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd);
+            else pf += cw * (double)(2 * Mss + 1) * __ldg(rcp + s);
+        } else {
+            const int yt[2] = {t, t};
+            int o2[2];
+            lookup4_in<2>(Ln, yt, pb2, nb2, o2);
+            const double rt = __ldg(rcp + t);
+            if (PASS == 1) {   // o2 = {M_rt, M_tr}
+                accS -= df_t(ft, o2[0], -ot) + df_t(ft, o2[1], -it);
+                pb += cw * (double)(o2[1] - it + o2[0] - ot + 1) * rt;
+            } else {           // o2 = {M_st, M_ts}
+                accS -= df_t(ft, o2[0], ot) + df_t(ft, o2[1], it);
+                pf += cw * (double)(o2[1] + o2[0] + 1) * rt;
+            }
+        }
+    }
+    // the 2x2 core, the degree terms and v's self-loop in the proposal laws (R:Z26)
+    if (PASS == 1) {
+        if (lane < 7 && lane != 3) {
+            const int m = lane == 0 ? Mrr : lane == 1 ? Mrs : lane == 2 ? Msr
+                        : lane == 4 ? dout_r : lane == 5 ? dout_s : din_r;
+            const int d = lane == 0 ? -(o_r + i_r + l) : lane == 1 ? i_r - o_s : lane == 2 ? o_r - i_s
+                        : lane == 4 ? -kout : lane == 5 ? kout : -kin;
+            const double y = df_t(ft, m, d);
+            accS += lane < 4 ? -y : y;
+        }
+        if (lane == 7) accS += df_t(ft, din_s, kin);
+        if (lane == 0 && l > 0) {
+            pf += 2.0 * (double)l * (double)(Mrs + Msr + 1) * __ldg(rcp + r);
+            pb += 2.0 * (double)l * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd);
+        }
+    } else if (lane == 3) {
+        accS -= df_t(ft, Mss, o_s + i_s + l);
+    }
+    accS = warp_sum(accS);
+    pf = warp_sum(pf);
+    if (PASS == 1) pb = warp_sum(pb);
+    // leave the table empty: exactly the listed slots were used
+    for (int k = lane; k < nuniq; k += 32) tab[list[k]] = make_int4(-1, 0, 0, 0x7fffffff);
+    __syncwarp();
+    if (lane == 0) {
+        double *pt = a.part + 3 * (size_t)i;
+        if (PASS == 1) {
+            pt[0] = accS;
+            pt[1] = pf;
+            pt[2] = pb;
+        } else {
+            const double dS = pt[0] + accS;
+            const double pft = pt[1] + pf;
+            const double H = (kout + kin == 0) ? 1.0 : pt[2] / pft;
+            const double p = exp(-a.beta * dS) * H;
+            const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
+            const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
+            if (a.dS) a.dS[i] = dS;
+            if (a.H) a.H[i] = H;
+            if (a.acc) a.acc[i] = ((double)w.w + 0.5) * (1.0 / 4294967296.0) <= p ? 1 : 0;
+        }
+    }
+}
+
 // (a2), one G-thread group (64: a quarter CTA, 256: a CTA) per big vertex:
 // every unique block owned by its first adjacency position; threads sum their
 // owned terms in position order.
@@ -818,6 +1014,47 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
     }
 }
 
+// sorted two-pass mode: warp w takes batch index perm[w] (the batch grouped
+// by r in pass 1, by s in pass 2); group vertices are skipped (k_move_groups)
+template <bool WEIGHTED, int PASS>
+__global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move_half(MoveArgs a) {
+    extern __shared__ int4 move_smem[];   // MOVE_SMEM bytes
+    int4 *tabs = move_smem;
+    int *lists = reinterpret_cast<int *>(tabs + MOVE_WARPS * WARP_TAB);
+    const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    int4 *tab = tabs + wl * WARP_TAB;
+    int *list = lists + wl * (WARP_TAB / 2);
+    tab_clear<32>(tab, WARP_TAB, lane);
+    __syncwarp();
+    const int nwarps = gridDim.x * MOVE_WARPS;
+    for (int w = blockIdx.x * MOVE_WARPS + wl; w < a.count; w += nwarps) {
+        const int i = __ldg(a.perm + w);
+        const int v = a.first + i;
+        if ((__ldg(a.rowptr + v + 1) - __ldg(a.rowptr + v)) + (__ldg(a.cscptr + v + 1) - __ldg(a.cscptr + v)) > BIG_THR)
+            continue;
+        move_vertex_half<WEIGHTED, PASS>(a, i, tab, list);
+    }
+}
+
+// counting sort of the batch by r = b[v] (keys [0, B)) and by s (keys [B, 2B)):
+// counts, then (after an exclusive scan of both) the scatter into perm[0, 2 count)
+__global__ void __launch_bounds__(256) k_sort_count(int first, int count, const int *__restrict__ b,
+                                                    const int *__restrict__ s, int B, int *__restrict__ cnt) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < count; i += gridDim.x * blockDim.x) {
+        atomicAdd(cnt + __ldg(b + first + i), 1);
+        atomicAdd(cnt + B + __ldg(s + i), 1);
+    }
+}
+
+__global__ void __launch_bounds__(256) k_sort_scatter(int first, int count, const int *__restrict__ b,
+                                                      const int *__restrict__ s, int B, int *__restrict__ off,
+                                                      int *__restrict__ perm) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < count; i += gridDim.x * blockDim.x) {
+        perm[atomicAdd(off + __ldg(b + first + i), 1)] = i;
+        perm[atomicAdd(off + B + __ldg(s + i), 1)] = i;   // offsets of the s keys start at count
+    }
+}
+
 // ------------------------------------------------------------------ host --
 static int log2_ceil(long long x) {
     int l = 0;
@@ -850,15 +1087,36 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     a.dS = dS; a.H = H; a.acc = acc;
     a.gtab = nullptr;
     a.gtab_log2 = 0;
+    a.perm = nullptr;
+    a.part = nullptr;
     a.propose = mode == MOVE_FUSED ? 1 : 0;
-    if (mode == MOVE_PROPOSE) {   // (a1) alone: thread per vertex
+    // sorted two-pass evaluation of a fused batch (large sparse blockmodels)
+    const bool sorted = mode == MOVE_FUSED && a.m.dense == nullptr && c.B > BIG_THR &&
+                        (c.prm.move_sorted == 2 || (c.prm.move_sorted == 1 && (long long)c.E > GSAP_COOP_MAX_E &&
+                                                    count >= (1 << 16)));
+    if (mode == MOVE_PROPOSE || sorted) {   // (a1) alone: thread per vertex
         const int pg = (int)std::min<long long>(((long long)count + 63) / 64, 148LL * 64);
         if (c.weighted) k_propose<true><<<pg, 64, 0, c.stream>>>(a);
         else k_propose<false><<<pg, 64, 0, c.stream>>>(a);
         ++c.launches;
         GSAP_CHECK_LAUNCH();
-        kc_end(c, c.k_move, ev, 0.0);
-        return;
+        if (!sorted) {
+            kc_end(c, c.k_move, ev, 0.0);
+            return;
+        }
+        // group the batch by r and by s (counting sort; the order inside a
+        // group is irrelevant: every vertex reads the same snapshot)
+        const int B = c.B;
+        Launcher L{c.stream, &c.launches};
+        GSAP_CUDA(cudaMemsetAsync(c.mv_cnt, 0, sizeof(int) * 2 * (size_t)B, c.stream));
+        const int sg = (int)std::min<long long>(((long long)count + 255) / 256, 148LL * 16);
+        k_sort_count<<<sg, 256, 0, c.stream>>>(first, count, c.b, s, B, c.mv_cnt);
+        device_scan<int>(c.mv_cnt, c.mv_cnt, nullptr, 2 * B, false, c.mv_scan_tmp, nullptr, L);
+        k_sort_scatter<<<sg, 256, 0, c.stream>>>(first, count, c.b, s, B, c.mv_cnt, c.mv_perm);
+        c.launches += 2;
+        GSAP_CHECK_LAUNCH();
+        a.propose = 0;          // groups and both passes read the proposals s
+        a.part = c.mv_part;
     }
     a.nbig_ctas = 0;
     a.nhuge_ctas = 0;
@@ -930,14 +1188,35 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         return 1;
     });
     const bool dense = a.m.dense != nullptr;
-    if (c.weighted) {
+    if (sorted) {
+        per_device((const void *)k_move_half<false, 1>, [] {
+            const int sm = (int)MOVE_SMEM;
+            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+            return 1;
+        });
+        MoveArgs a1 = a, a2 = a;
+        a1.perm = c.mv_perm;            // grouped by r
+        a2.perm = c.mv_perm + count;    // grouped by s
+        if (c.weighted) {
+            k_move_half<true, 1><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
+            k_move_half<true, 2><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
+        } else {
+            k_move_half<false, 1><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
+            k_move_half<false, 2><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
+        }
+        c.launches += 2;
+    } else if (c.weighted) {
         if (dense) k_move<true, true><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);
         else k_move<true, false><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);
+        ++c.launches;
     } else {
         if (dense) k_move<false, true><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);
         else k_move<false, false><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);
+        ++c.launches;
     }
-    ++c.launches;
     GSAP_CHECK_LAUNCH();
     if (ggrid > 0) GSAP_CUDA(cudaStreamWaitEvent(c.stream, c.ev_join, 0));
     // algorithmic bytes: adjacency ids (+ weights),

@@ -19,7 +19,7 @@ LIB_PATH = os.environ.get("GSAP_LIB", os.path.join(HERE, "libgsap.so"))
 
 GSAP_OK, GSAP_EINVAL, GSAP_ENOMEM, GSAP_ECUDA, GSAP_ENCCL, GSAP_ESTATE, GSAP_EUNSUPPORTED = range(7)
 GSAP_MERGE, GSAP_MOVE = 0, 1
-TRACE_COLS = 10                 # GSAP_TRACE_COLS (gsap.h)
+TRACE_COLS = 12                 # GSAP_TRACE_COLS (gsap.h)
 STATUS_NAMES = ["GSAP_OK", "GSAP_EINVAL", "GSAP_ENOMEM", "GSAP_ECUDA", "GSAP_ENCCL", "GSAP_ESTATE",
                 "GSAP_EUNSUPPORTED"]
 
@@ -36,7 +36,7 @@ class gsap_params(C.Structure):
                 ("thresh2", C.c_double), ("window", C.c_int32), ("num_batches", C.c_int32),
                 ("model_term", C.c_int32), ("max_rounds", C.c_int32), ("profile", C.c_int32),
                 ("cuda_graphs", C.c_int32), ("dense_max_B", C.c_int32), ("sparse_coop", C.c_int32), ("dense_coop", C.c_int32),
-                ("sel_small", C.c_int32)]
+                ("sel_small", C.c_int32), ("move_sorted", C.c_int32)]
 
 
 class gsap_dist(C.Structure):

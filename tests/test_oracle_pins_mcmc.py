@@ -159,3 +159,43 @@ def test_partition_threshold_slot(oracle_mod):
     assert np.all(tr[k0 + 1:, 4] == p.thresh2)
     # and the rounds' accepted-move column adds up to the run's statistic
     assert int(tr[:, 5].sum()) == res["stats"].n_move_acc
+
+
+def test_bracket_replay_consistent_with_partition_trace(oracle_mod):
+    """The replay entry (used to check another driver's trace) on the oracle's
+    own 1K run: each round's B after its merge is at most the replayed restart
+    B minus K (less only when merged groups held no vertex, R:Z18), the
+    threshold slot of every later round matches the replayed bracket state,
+    and the search stops after exactly the rounds the run did."""
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    p = oracle_mod.default_params()
+    res = oracle_mod.Oracle(rowptr, col).partition_run(p)
+    tr = res["trace"]
+    Bn, Kn, br, stop = oracle_mod.bracket_replay(tr[:, 1].astype(np.int32), tr[:, 3], p.reduction_rate)
+    assert stop == len(tr)
+    assert tr[0, 1] <= cfg.V - int(cfg.V * p.reduction_rate)
+    for k in range(len(tr) - 1):
+        assert 0 < tr[k + 1, 1] <= Bn[k] - Kn[k]
+        assert tr[k + 1, 4] == (p.thresh2 if br[k] else p.thresh1)
+    # mock: a unimodal MDL(B) table replayed round by round ends where golden_mock ends
+    V = 500
+    mdl = np.array([(B - 77) ** 2 + 0.3 * B for B in range(V + 1)], np.float64)
+    vis, Bf = oracle_mod.golden_mock(V, 0.4, mdl)
+    Bn, Kn, br, stop = oracle_mod.bracket_replay(vis, mdl[vis], 0.4)
+    assert stop == len(vis) and Bf == 77
+    assert all(vis[k + 1] == Bn[k] - Kn[k] for k in range(len(vis) - 1))
+
+
+def test_openmp_mode_gives_identical_results(oracle_mod):
+    """The all-core mode changes nothing: same partition, MDL and
+    trace as the single-threaded canonical run."""
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    p = oracle_mod.default_params()
+    try:
+        a = oracle_mod.Oracle(rowptr, col).partition_run(p)
+        assert oracle_mod.set_threads(4) >= 1
+        b = oracle_mod.Oracle(rowptr, col).partition_run(p)
+    finally:
+        oracle_mod.set_threads(1)
+    assert np.array_equal(a["b"], b["b"]) and a["mdl"] == b["mdl"]
+    assert np.array_equal(a["trace"], b["trace"])

@@ -10,7 +10,10 @@ planted partition (§4.4), and the per-round trace
 [outer, B after merge, MCMC iterations, MDL, threshold, accepted moves].
 The GPU layer-3 tests (north_star: MDL within 1 %, P/R within 0.02) read them.
 
-    python tools/oracle_goldens.py 20k 200k
+    python tools/oracle_goldens.py [--threads N] 20k 200k
+
+--threads runs the oracle's per-id loops on N OpenMP threads (identical
+results; orc_set_threads).
 """
 import hashlib
 import json
@@ -48,7 +51,7 @@ def one(name):
         "b_sha256": hashlib.sha256(res["b"].astype("<i4").tobytes()).hexdigest(),
         "trace_cols": ["outer", "B", "itrs", "mdl", "thresh", "accepted"],
         "trace": res["trace"].tolist(),
-        "oracle_seconds_single_thread": dt,
+        "oracle_seconds": dt, "oracle_threads": THREADS,
     }
     path = os.path.join(ROOT, "tests", "golden", f"e2e_{name}.json")
     with open(path, "w") as f:
@@ -56,6 +59,12 @@ def one(name):
     print(name, "B", res["B"], "MDL", res["mdl"], "P/R", prec, rec, f"{dt:.1f} s", flush=True)
 
 
+THREADS = 1
+
 if __name__ == "__main__":
-    for n in sys.argv[1:] or ["20k"]:
+    args = sys.argv[1:]
+    if args and args[0] == "--threads":
+        THREADS = oracle.set_threads(int(args[1]))
+        args = args[2:]
+    for n in args or ["20k"]:
         one(n)
