@@ -108,6 +108,7 @@ union CoopSmem {
     struct {
         K keys[SEG_WARPS][SEG_WARP_MAX];
         int hp[SEG_WARPS][SEG_WARP_MAX];
+        unsigned cntp[SEG_WARPS][8 * 32];
     } warp;
     struct {
         K keys[2][SegCta<K>::CAP];
@@ -227,12 +228,24 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
                 line_epilogue<32>(out, sd.tcnt, o, u, L, x, lane, nullptr);
                 continue;
             }
-            int n = 1;
-            while (n < L) n <<= 1;
-            for (int i = lane; i < n; i += 32) S.warp.keys[wl][i] = i < L ? seg[o + i] : key_max<K>();
-            __syncwarp();
-            bitonic<K, 32>(S.warp.keys[wl], n, lane);
-            const int u = rle_runs<K, 32>(S.warp.keys[wl], L, S.warp.hp[wl], sd.tcol + o, sd.tcnt + o, lane, nullptr);
+            int u;
+            if (sizeof(K) == 4) {
+                // 129..512 entries: the warp LSD radix sort over the block bits,
+                // ping-ponging with the heads buffer (same size for 32-bit keys)
+                K *ka = S.warp.keys[wl], *kb = reinterpret_cast<K *>(S.warp.hp[wl]);
+                for (int i = lane; i < L; i += 32) ka[i] = seg[o + i];
+                __syncwarp();
+                K *keys = cta_radix_sort<K, 32>(ka, kb, L, a.col_bits, S.warp.cntp[wl], nullptr);
+                int *hw = reinterpret_cast<int *>(keys == ka ? kb : ka);
+                u = rle_runs<K, 32>(keys, L, hw, sd.tcol + o, sd.tcnt + o, lane, nullptr);
+            } else {
+                int n = 1;
+                while (n < L) n <<= 1;
+                for (int i = lane; i < n; i += 32) S.warp.keys[wl][i] = i < L ? seg[o + i] : key_max<K>();
+                __syncwarp();
+                bitonic<K, 32>(S.warp.keys[wl], n, lane);
+                u = rle_runs<K, 32>(S.warp.keys[wl], L, S.warp.hp[wl], sd.tcol + o, sd.tcnt + o, lane, nullptr);
+            }
             if (lane == 0) sd.nnz[x] = u;
             line_epilogue<32>(out, sd.tcnt, o, u, L, x, lane, nullptr);
         }

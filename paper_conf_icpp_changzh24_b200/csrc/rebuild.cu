@@ -689,12 +689,14 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
                                        (int)seg_warp2_smem<K>()));
         return 1;
     });
-    k_segsort_warp<K, 0><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, idx, cnt,
+    const int cb = bits_for(B);
+    k_segsort_warp<K, 0><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, cb, idx, cnt,
                                                               c.seg_nnz, out);
-    k_segsort_warp<K, 1><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, idx, cnt,
+    k_segsort_warp<K, 1><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, cb, idx, cnt,
                                                               c.seg_nnz, out);
     k_segsort_warp<K, 2><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(), c.stream>>>(B, ptr, seg, c.seg_listC,
-                                                                                c.seg_ctr, idx, cnt, c.seg_nnz, out);
+                                                                                c.seg_ctr, cb, idx, cnt,
+                                                                                c.seg_nnz, out);
     c.launches += 2;
     const int gc = (int)std::min<long long>(std::max(1, B / 4), 148LL * 4);
     k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(ptr, seg, c.seg_listC, c.seg_ctr, bits_for(B), idx, cnt,

@@ -263,10 +263,10 @@ __global__ void k_line_classify(int B, const int *__restrict__ off, int *__restr
                 out.deg[x] = 0;
             }
         }
-        else if (L <= 128 || (L > 256 && L <= SEG_WARP_MAX)) listW[atomicAdd(counters, 1)] = x;   // warp mode 0
-        else if (L <= 256) listW[B - 1 - atomicAdd(counters + 2, 1)] = x;                        // warp mode 1
-        else if (L <= warp_max) listC[B - 1 - atomicAdd(counters + 3, 1)] = x;                   // warp mode 2
-        else listC[atomicAdd(counters + 1, 1)] = x;                                               // CTA
+        else if (L <= 128) listW[atomicAdd(counters, 1)] = x;                           // warp mode 0
+        else if (L <= 256) listW[B - 1 - atomicAdd(counters + 2, 1)] = x;               // warp mode 1
+        else if (L <= warp_max) listC[B - 1 - atomicAdd(counters + 3, 1)] = x;          // warp mode 2
+        else listC[atomicAdd(counters + 1, 1)] = x;                                      // CTA
     }
 }
 
@@ -381,23 +381,31 @@ GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict_
 // 4b. warp-sized segments: one warp each, three instantiations, each over its
 // own line list (k_line_classify), so that a heavy path does not lower the
 // occupancy of the common one:
-//   MODE 0: <= 128 entries bitonic + RLE in registers, 257..512 bitonic in
-//           static shared memory;
+//   MODE 0: <= 128 entries, bitonic + RLE in registers;
 //   MODE 1: 129..256 entries in registers (8 per lane);
-//   MODE 2: 513..SEG_WARP_MAX_MK entries bitonic in dynamic shared memory.
+//   MODE 2: 257..SEG_WARP_MAX_MK entries: the stable LSD radix sort over the
+//           key's block bits (cta_radix_sort with 32 threads: 4-bit digits,
+//           per-lane packed counters, no atomics; O(L) per pass instead of
+//           bitonic's O(L log^2 L)) in dynamic shared memory, then RLE.
 #ifndef GSAP_SEG_WARP_MAX_MK
 #define GSAP_SEG_WARP_MAX_MK 1024
 #endif
 constexpr int SEG_WARP_MAX_MK = GSAP_SEG_WARP_MAX_MK;   // multi-kernel path: longer lines go to the CTA sorts
+template <typename K>
+constexpr size_t seg_warp2_smem() {
+    return (size_t)SEG_WARPS * (2 * SEG_WARP_MAX_MK * sizeof(K) + 8 * 32 * sizeof(unsigned));
+}
+
+template <typename K, int NT>
+GSAP_DEV K *cta_radix_sort(K *a, K *b, int L, int col_bits, unsigned *cntp, unsigned *wsum);
+
 template <typename K, int MODE>
 __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const int *__restrict__ off, K *__restrict__ seg,
                                                                  const int *__restrict__ listW,
-                                                                 const int *__restrict__ counters,
+                                                                 const int *__restrict__ counters, int col_bits,
                                                                  int *__restrict__ tcol, int *__restrict__ tcnt,
                                                                  int *__restrict__ nnz, LineOut out) {
-    __shared__ K keys[MODE == 0 ? SEG_WARPS : 1][MODE == 0 ? SEG_WARP_MAX : 1];
-    __shared__ int hp[MODE == 0 ? SEG_WARPS : 1][MODE == 0 ? SEG_WARP_MAX : 1];
-    extern __shared__ __align__(16) unsigned char seg_dyn[];   // MODE 2: SEG_WARPS x (keys + heads)
+    extern __shared__ __align__(16) unsigned char seg_dyn[];   // MODE 2: SEG_WARPS x (2 key buffers) + counters
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int n_lines = counters[MODE == 0 ? 0 : MODE == 1 ? 2 : 3];
     for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
@@ -406,29 +414,25 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const in
         int u;
         if (MODE == 1) {
             u = warp_segsort_rle<K, 8>(seg + o, L, tcol + o, tcnt + o);
-        } else if (MODE == 0 && L <= 128) {
+        } else if (MODE == 0) {
             if (L <= 32) u = warp_segsort_rle<K, 1>(seg + o, L, tcol + o, tcnt + o);
             else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, tcol + o, tcnt + o);
             else u = warp_segsort_rle<K, 4>(seg + o, L, tcol + o, tcnt + o);
         } else {
-            K *kw = MODE == 0 ? keys[w] : reinterpret_cast<K *>(seg_dyn) + (size_t)w * SEG_WARP_MAX_MK;
-            int *hw = MODE == 0 ? hp[w]
-                                : reinterpret_cast<int *>(reinterpret_cast<K *>(seg_dyn) + (size_t)SEG_WARPS * SEG_WARP_MAX_MK) +
-                                      (size_t)w * SEG_WARP_MAX_MK;
-            int n = 1;
-            while (n < L) n <<= 1;
-            for (int i = lane; i < n; i += 32) kw[i] = i < L ? seg[o + i] : key_max<K>();
+            K *ka = reinterpret_cast<K *>(seg_dyn) + (size_t)w * 2 * SEG_WARP_MAX_MK;
+            K *kb = ka + SEG_WARP_MAX_MK;
+            unsigned *cntp = reinterpret_cast<unsigned *>(reinterpret_cast<K *>(seg_dyn) +
+                                                          (size_t)SEG_WARPS * 2 * SEG_WARP_MAX_MK) + w * 8 * 32;
+            for (int i = lane; i < L; i += 32) ka[i] = seg[o + i];
             __syncwarp();
-            bitonic<K, 32>(kw, n, lane);
-            u = rle_runs<K, 32>(kw, L, hw, tcol + o, tcnt + o, lane, nullptr);
+            K *keys = cta_radix_sort<K, 32>(ka, kb, L, col_bits, cntp, nullptr);
+            int *hw = reinterpret_cast<int *>(keys == ka ? kb : ka);
+            u = rle_runs<K, 32>(keys, L, hw, tcol + o, tcnt + o, lane, nullptr);
         }
         if (lane == 0) nnz[x] = u;
         if (out.cum) line_epilogue<32>(out, tcnt, o, u, L, x, lane, nullptr);
     }
 }
-
-template <typename K>
-constexpr size_t seg_warp2_smem() { return (size_t)SEG_WARPS * SEG_WARP_MAX_MK * (sizeof(K) + sizeof(int)); }
 
 // stable LSD radix sort of a[0, L) by the block bits of the key (key_col),
 // 4-bit digits, NT threads.  Each thread owns a contiguous chunk of an odd
