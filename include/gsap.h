@@ -84,6 +84,11 @@ typedef struct {
                                  more than GSAP_COOP_MAX_E edges and batches of >= 2^16 vertices;
                                  2: always (sparse regime, B > 128); 0: never (one fused pass).
                                  Same integers; dS sums in another order (1e-9 contract). */
+    int32_t sim_ranks;        /* verification mode (tests): > 1 runs the multi-GPU data path of
+                                 sim_ranks ranks in ONE process on one GPU -- every MOVE batch and
+                                 merge phase cut into the ranks' slices exactly as with NCCL, each
+                                 slice computed in rank order, the all-gathers skipped (the slices
+                                 already sit at their offsets); default 0 = off */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */
@@ -264,9 +269,13 @@ gsap_status gsap_run(gsap_ctx *ctx, int32_t *bmap_out, int32_t *B_out, double *m
 /*
  * Multi-GPU: one process per GPU, every rank passes the same
  * graph and a gsap_dist {nranks, rank, device, nccl_id}; each MOVE batch and
- * each merge phase is split into contiguous slices (whole 1024-vertex chunks
- * / block ranges), whose results are exchanged with ncclAllGather; every rank
- * then applies them identically.  Results are bit-identical for any nranks.
+ * each merge phase is split into contiguous slices (MOVE: edge-balanced runs of
+ * whole 1024-vertex chunks, gsap_shard_plan; MERGE: equal block ranges), whose
+ * results are exchanged in place (one ncclBroadcast per rank in one group: an
+ * all-gather of variable slices); every rank then applies them identically.
+ * Results are bit-identical for any nranks (verified on one GPU with
+ * params.sim_ranks).  Statistics: n_move_prop / n_merge_prop count the
+ * proposals of this rank's slices; n_move_acc / n_move_eval the whole batch.
  * gsap_nccl_unique_id: rank 0 creates the id (host, 128 bytes) and the caller
  * broadcasts it (e.g. with torch.distributed).  NCCL is loaded at run time.
  */
@@ -280,6 +289,16 @@ gsap_status gsap_nccl_unique_id(uint8_t *id_out);
  */
 gsap_status gsap_shard_slice(int32_t n, int32_t chunk, int32_t nranks, int32_t rank, int32_t *first,
                              int32_t *count, int32_t *per_rank);
+
+/*
+ * The slices a MOVE batch [first, first + count) is cut into for nranks ranks
+ * (SURVEY 8(e)): contiguous, whole 1024-vertex chunks from the batch start,
+ * balanced by each chunk's work (adjacency entries + 16 per vertex), the last
+ * rank taking the rest.  Host outputs first_out[nranks] (absolute vertex ids)
+ * and count_out[nranks].  Host-only (the graph's degrees from ctx).
+ */
+gsap_status gsap_shard_plan(gsap_ctx *ctx, int32_t first, int32_t count, int32_t nranks, int32_t *first_out,
+                            int32_t *count_out);
 
 #ifdef __cplusplus
 }

@@ -288,7 +288,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_join, cudaEventDisableTiming));
     GSAP_CUDA(cudaGetDevice(&c.dev));
     comm_init(c, dist);
-    if (c.nranks > 1) c.prm.cuda_graphs = 0;
+    REQUIRE(c.prm.sim_ranks >= 0 && c.prm.sim_ranks <= 64, GSAP_EINVAL, "sim_ranks in [0, 64]");
+    if (c.nranks > 1 || c.prm.sim_ranks > 1) c.prm.cuda_graphs = 0;   // the sliced batch path (move_batch)
     mark("streams");
     // host-side static info
     c.h_rowptr.resize((size_t)V + 1);
@@ -509,21 +510,35 @@ static double mdl_now(Ctx &c) {
     return model_term(c.W, c.V, c.B, c.prm.model_term) + device_data_term(c);
 }
 
+// ranks the batches and merge phases are sliced over: the NCCL ranks, or the
+// ranks one process emulates (params.sim_ranks: every slice computed here in
+// rank order, the exchange skipped -- the sharded data path on one GPU)
+static int ranks_of(const Ctx &c) { return c.nranks > 1 ? c.nranks : std::max(1, c.prm.sim_ranks); }
+
 static void merge_phase(Ctx &c, uint32_t outer, int K, int *best_out, double *dSbest_out) {
     REQUIRE(c.B >= 2, GSAP_ESTATE, "a merge phase needs B >= 2");
     REQUIRE(K >= 0 && K <= c.B / 2, GSAP_EINVAL, "K must be in [0, B/2]");
     const int B = c.B;
-    if (c.nranks == 1) {
+    const int G = ranks_of(c);
+    if (G == 1) {
         launch_merge_props(c, outer, 0, B, true, nullptr, nullptr, c.best, c.dSbest);
         c.st.n_merge_prop += (long long)B * c.prm.num_proposals;
     } else {
-        // each rank proposes for its slice of blocks; winners all-gathered
-        int f, n, per;
-        shard_slice(B, 1, c.nranks, c.rank, &f, &n, &per);
-        launch_merge_props(c, outer, f, n, true, nullptr, nullptr, c.best + f, c.dSbest + f);
-        comm_allgather(c, c.best, (size_t)per, 1);
-        comm_allgather(c, c.dSbest, (size_t)per, 2);
-        c.st.n_merge_prop += (long long)n * c.prm.num_proposals;
+        // each rank proposes for its range of blocks (equal counts); the
+        // winners (12 B per block) are all-gathered; every rank then runs the
+        // identical selection and rebuild.  sim_ranks: all slices here, in order.
+        std::vector<int> f(G), n(G);
+        for (int g = 0; g < G; ++g) {
+            int per;
+            shard_slice(B, 1, G, g, &f[g], &n[g], &per);
+        }
+        const int g0 = c.nranks > 1 ? c.rank : 0, g1 = c.nranks > 1 ? c.rank + 1 : G;
+        for (int g = g0; g < g1; ++g) {
+            if (n[g] > 0) launch_merge_props(c, outer, f[g], n[g], true, nullptr, nullptr, c.best + f[g], c.dSbest + f[g]);
+            c.st.n_merge_prop += (long long)n[g] * c.prm.num_proposals;
+        }
+        comm_allgatherv(c, c.best, f, n, 1);
+        comm_allgatherv(c, c.dSbest, f, n, 2);
     }
     copy_out(c, best_out, c.best, sizeof(int) * (size_t)B);
     copy_out(c, dSbest_out, c.dSbest, sizeof(double) * (size_t)B);
@@ -532,30 +547,45 @@ static void merge_phase(Ctx &c, uint32_t outer, int K, int *best_out, double *dS
 }
 
 static void move_batch(Ctx &c, uint32_t outer, uint32_t itr, int first, int count, double *dsum) {
-    if (c.nranks == 1) {
+    c.batch_count = count;
+    const int G = ranks_of(c);
+    if (G == 1) {
         launch_move(c, MOVE_FUSED, outer, itr, first, count, c.s, c.dS, nullptr, c.acc);
         launch_apply(c, first, count, c.s, c.acc, c.dS, dsum, c.scal_i + 1, c.n_eval);
         rebuild(c);
         c.st.n_move_prop += count;
         return;
     }
-    // this rank's slice of the batch (whole APPLY_CHUNK_V chunks), results and
-    // fixed-chunk dS partials all-gathered, then applied and rebuilt everywhere
-    int f, n, per;
-    shard_slice(count, APPLY_CHUNK_V, c.nranks, c.rank, &f, &n, &per);
-    const int pc = per / APPLY_CHUNK_V;
-    const size_t boff = (size_t)c.rank * per, poff = (size_t)c.rank * pc;
-    if (n > 0) {
-        launch_move(c, MOVE_FUSED, outer, itr, first + f, n, c.s + boff, c.dS + boff, nullptr, c.acc + boff);
-        launch_partials(c, first + f, n, c.s + boff, c.acc + boff, c.dS + boff, c.partials + poff);
+    // the batch cut into G edge-balanced slices of whole APPLY_CHUNK_V chunks;
+    // this rank evaluates its slice (sim_ranks: every slice, in order) and the
+    // fixed-chunk dS partials of its accepted moves; ONE exchange step: the
+    // slices' s, acc and partials all-gathered in place (contiguous, no
+    // padding); then every rank applies the whole batch, sums the partials in
+    // chunk order and rebuilds -- the same operations in the same order as
+    // G = 1, so the trajectory is bit-identical for any G.
+    std::vector<int> f, n;
+    shard_plan(c, first, count, G, f, n);
+    const int CH = APPLY_CHUNK_V;
+    const int g0 = c.nranks > 1 ? c.rank : 0, g1 = c.nranks > 1 ? c.rank + 1 : G;
+    for (int g = g0; g < g1; ++g) {
+        if (n[g] <= 0) continue;
+        launch_move(c, MOVE_FUSED, outer, itr, first + f[g], n[g], c.s + f[g], c.dS + f[g], nullptr, c.acc + f[g]);
+        launch_partials(c, first + f[g], n[g], c.s + f[g], c.acc + f[g], c.dS + f[g], c.partials + f[g] / CH);
+        c.st.n_move_prop += n[g];
     }
-    comm_allgather(c, c.s, (size_t)per, 1);
-    comm_allgather(c, c.acc, (size_t)per, 0);
-    comm_allgather(c, c.partials, (size_t)pc, 2);
-    const int chunks = (count + APPLY_CHUNK_V - 1) / APPLY_CHUNK_V;
+    if (c.nranks > 1) {
+        std::vector<int> pf(G), pn(G);
+        for (int g = 0; g < G; ++g) {
+            pf[g] = f[g] / CH;
+            pn[g] = (n[g] + CH - 1) / CH;
+        }
+        comm_allgatherv(c, c.s, f, n, 1);
+        comm_allgatherv(c, c.acc, f, n, 0);
+        comm_allgatherv(c, c.partials, pf, pn, 2);
+    }
+    const int chunks = (count + CH - 1) / CH;
     launch_apply_gathered(c, first, count, c.s, c.acc, c.partials, chunks, dsum, c.scal_i + 1, c.n_eval);
     rebuild(c);
-    c.st.n_move_prop += n;
 }
 
 static bool converged(Ctx &c, const std::vector<double> &D, int itr, double S, double thresh) {
@@ -589,6 +619,7 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh, std::vector<d
         for (int k = 0; k < nb; ++k) {
             const int first = k * bs, last = std::min(V, first + bs);
             if (first >= last) continue;
+            c.batch_count = last - first;
             launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
             launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
             rebuild(c);
@@ -701,7 +732,8 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::ve
             for (int k = 0; k < nb; ++k) {
                 const int first = k * bs, last = std::min(V, first + bs);
                 if (first >= last) continue;
-                launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
+                c.batch_count = last - first;
+            launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
                 launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
                 rebuild(c);
             }
@@ -980,6 +1012,7 @@ void gsap_default_params(gsap_params *p) {
     p->dense_coop = 1;
     p->sel_small = 1;
     p->move_sorted = 1;
+    p->sim_ranks = 0;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }
@@ -1304,6 +1337,21 @@ gsap_status gsap_shard_slice(int32_t n, int32_t chunk, int32_t nranks, int32_t r
     REQUIRE(n >= 0 && chunk >= 1 && nranks >= 1 && rank >= 0 && rank < nranks && first && count && per_rank,
             GSAP_EINVAL, "bad argument");
     shard_slice(n, chunk, nranks, rank, first, count, per_rank);
+    API_CATCH
+}
+
+gsap_status gsap_shard_plan(gsap_ctx *ctx, int32_t first, int32_t count, int32_t nranks, int32_t *first_out,
+                            int32_t *count_out) {
+    API_TRY
+    REQUIRE(ctx && first_out && count_out && nranks >= 1, GSAP_EINVAL, "bad argument");
+    Ctx &c = ctx->c;
+    REQUIRE(first >= 0 && count >= 0 && (long long)first + count <= c.V, GSAP_EINVAL, "range out of bounds");
+    std::vector<int> f, n;
+    shard_plan(c, first, count, nranks, f, n);
+    for (int g = 0; g < nranks; ++g) {
+        first_out[g] = first + f[g];
+        count_out[g] = n[g];
+    }
     API_CATCH
 }
 

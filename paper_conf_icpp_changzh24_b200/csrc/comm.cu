@@ -21,6 +21,9 @@ struct NcclApi {
     ncclResult_t (*GetUniqueId)(ncclUniqueId *);
     ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int);
     ncclResult_t (*AllGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t);
+    ncclResult_t (*Broadcast)(const void *, void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t);
+    ncclResult_t (*GroupStart)();
+    ncclResult_t (*GroupEnd)();
     ncclResult_t (*CommDestroy)(ncclComm_t);
     const char *(*GetErrorString)(ncclResult_t);
 };
@@ -36,9 +39,13 @@ static NcclApi *nccl_api() {
         api.GetUniqueId = (decltype(api.GetUniqueId))dlsym(h, "ncclGetUniqueId");
         api.CommInitRank = (decltype(api.CommInitRank))dlsym(h, "ncclCommInitRank");
         api.AllGather = (decltype(api.AllGather))dlsym(h, "ncclAllGather");
+        api.Broadcast = (decltype(api.Broadcast))dlsym(h, "ncclBroadcast");
+        api.GroupStart = (decltype(api.GroupStart))dlsym(h, "ncclGroupStart");
+        api.GroupEnd = (decltype(api.GroupEnd))dlsym(h, "ncclGroupEnd");
         api.CommDestroy = (decltype(api.CommDestroy))dlsym(h, "ncclCommDestroy");
         api.GetErrorString = (decltype(api.GetErrorString))dlsym(h, "ncclGetErrorString");
-        ok = api.GetUniqueId && api.CommInitRank && api.AllGather && api.CommDestroy && api.GetErrorString;
+        ok = api.GetUniqueId && api.CommInitRank && api.AllGather && api.Broadcast && api.GroupStart &&
+             api.GroupEnd && api.CommDestroy && api.GetErrorString;
     });
     if (!ok) throw Error{GSAP_ENCCL, "libnccl.so.2 not found (dlopen)"};
     return &api;
@@ -86,6 +93,68 @@ void comm_allgather(Ctx &c, void *recv, size_t count_per_rank, int dtype) {
     kc_begin(c, c.k_comm, &ev);
     GSAP_NCCL(nccl_api()->AllGather(send, recv, count_per_rank, t, (ncclComm_t)c.nccl_comm, c.stream));
     kc_end(c, c.k_comm, ev, (double)count_per_rank * esz * c.nranks);
+}
+
+// variable slices, in place: rank g's cnt[g] elements at buf + off[g] go to
+// every rank (one ncclBroadcast rooted at each rank, in one NCCL group: an
+// all-gather-v without padding, so the gathered array is contiguous)
+void comm_allgatherv(Ctx &c, void *buf, const std::vector<int> &off, const std::vector<int> &cnt, int dtype) {
+    if (c.nranks <= 1) return;
+    const ncclDataType_t t = dtype == 0 ? ncclInt8 : (dtype == 1 ? ncclInt32 : ncclFloat64);
+    const size_t esz = dtype == 0 ? 1 : (dtype == 1 ? 4 : 8);
+    cudaEvent_t ev = nullptr;
+    kc_begin(c, c.k_comm, &ev);
+    NcclApi *api = nccl_api();
+    GSAP_NCCL(api->GroupStart());
+    size_t bytes = 0;
+    for (int g = 0; g < c.nranks; ++g) {
+        if (cnt[g] <= 0) continue;
+        char *p = (char *)buf + (size_t)off[g] * esz;
+        GSAP_NCCL(api->Broadcast(p, p, (size_t)cnt[g], t, g, (ncclComm_t)c.nccl_comm, c.stream));
+        bytes += (size_t)cnt[g] * esz;
+    }
+    GSAP_NCCL(api->GroupEnd());
+    kc_end(c, c.k_comm, ev, (double)bytes);
+}
+
+// the MOVE batch [first, first + count) cut into G contiguous slices of whole
+// APPLY_CHUNK_V chunks (offsets relative to first), balanced by the work of
+// each chunk: adjacency entries + a fixed 16 per vertex (SURVEY 8(e):
+// edge-balanced cut points rounded to the fixed reduction chunk, so every
+// partial sum covers the same vertices for any G).  Same plan on every rank.
+void shard_plan(const Ctx &c, int first, int count, int G, std::vector<int> &off, std::vector<int> &cnt) {
+    const int CH = APPLY_CHUNK_V;
+    const int chunks = (count + CH - 1) / CH;
+    auto work = [&](int v0, int v1) {   // adjacency entries + 16 per vertex of [v0, v1)
+        return (long long)(c.h_rowptr[v1] - c.h_rowptr[v0]) + (c.h_cscptr[v1] - c.h_cscptr[v0]) +
+               16LL * (v1 - v0);
+    };
+    const long long total = work(first, first + count);
+    off.assign(G, count);
+    cnt.assign(G, 0);
+    int k = 0;             // next chunk
+    long long done = 0;    // work of chunks [0, k)
+    for (int g = 0; g < G; ++g) {
+        const int k0 = k;
+        if (g == G - 1) {
+            k = chunks;
+        } else {
+            const long long target = total * (g + 1) / G;
+            while (k < chunks) {
+                const int v0 = first + k * CH, v1 = first + std::min(count, (k + 1) * CH);
+                const long long wk = work(v0, v1);
+                // take chunk k if that ends at or below the target, or overshoots it by less than stopping undershoots
+                if (done + wk <= target || done + wk - target < target - done) {
+                    done += wk;
+                    ++k;
+                } else {
+                    break;
+                }
+            }
+        }
+        off[g] = std::min(count, k0 * CH);
+        cnt[g] = std::min(count, k * CH) - off[g];
+    }
 }
 
 void shard_slice(int n, int chunk, int G, int g, int *first, int *count, int *per_rank) {

@@ -121,9 +121,10 @@ struct Ctx {
     double *h_scal = nullptr;
     int *h_int = nullptr;
 
-    // multi-GPU
+    // multi-GPU (nranks > 1), or one process emulating prm.sim_ranks ranks
     int nranks = 1, rank = 0;
     void *nccl_comm = nullptr;
+    int batch_count = 0;           // the MOVE batch a launch belongs to (mode decisions per batch, not slice)
 
     // CUDA-graph capture of an MCMC iteration (N1: launch overhead, §5)
     unsigned *d_itr = nullptr;     // MCMC iteration read by k_move (device scalar)
@@ -201,6 +202,10 @@ constexpr int APPLY_CHUNK_V = 1024;   // fixed reduction chunk of the accepted-d
 void comm_init(Ctx &c, const gsap_dist *d);
 void comm_destroy(Ctx &c);
 void comm_allgather(Ctx &c, void *recv, size_t count_per_rank, int dtype);   // dtype: 0 int8, 1 int32, 2 f64
+// in place, variable slices (rank g: cnt[g] elements at off[g]); contiguous result
+void comm_allgatherv(Ctx &c, void *buf, const std::vector<int> &off, const std::vector<int> &cnt, int dtype);
+// a MOVE batch cut into G edge-balanced slices of whole APPLY_CHUNK_V chunks (offsets relative to first)
+void shard_plan(const Ctx &c, int first, int count, int G, std::vector<int> &off, std::vector<int> &cnt);
 void comm_unique_id(uint8_t out[128]);
 // the slice of [0, n) that rank g of G owns: whole chunks of `chunk`, contiguous,
 // ceil(ceil(n/chunk)/G) chunks per rank (the last ranks may own less or none)

@@ -648,8 +648,31 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
 // The split follows the decomposition above term by term; only the order of
 // the floating-point sums differs from the fused kernel.  Vertices with more
 // than 128 adjacency entries stay in k_move_groups (fused terms, s given).
+// The pass's two lines (row x, column x) staged in the warp's shared memory
+// (ids only; a hit's count is one global load at the found position), or
+// ok = false when either line is longer than the stage (global searches).
+constexpr int STAGE_CAP = 1024;   // entries per staged line
+struct Stage {
+    const int *row, *col;                            // shared memory copies of the lines' ids
+    const int *__restrict__ rcnt, *__restrict__ ccnt;   // the lines' counts (global)
+    int rlen, clen;
+    bool ok;
+};
+
+// M entry of key y in a staged line: branchless lower bound in shared memory
+GSAP_DEV int stage_get(const int *ids, const int *__restrict__ cnt, int len, int y) {
+    int p = 0, n = len;
+    while (n > 1) {
+        const int h = n >> 1;
+        p = ids[p + h - 1] < y ? p + h : p;
+        n -= h;
+    }
+    if (n == 1 && ids[p] < y) ++p;
+    return (p < len && ids[p] == y) ? __ldg(cnt + p) : 0;
+}
+
 template <bool WEIGHTED, int PASS>
-GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
+GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list, const Stage &st) {
     const int lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
     const int v = a.first + i;
@@ -667,13 +690,17 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
     const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
     const int deg = nout + nin;   // <= 128 (the caller routes bigger vertices to k_move_groups)
     const int B = a.m.B;
-    // the two lines of this pass and their splitters, issued before the histogram
+    // the two lines of this pass: staged in shared memory (st.ok, warp-uniform),
+    // else searched in global memory with warp-shared splitters (issued now,
+    // before the histogram)
     Line Ln[2];
-    const int x = PASS == 1 ? r : s;
-    Ln[0] = row_line(a.m, x);
-    Ln[1] = col_line(a.m, x);
-    int sp[2];
-    split4_load<2>(Ln, lane, sp);
+    int sp[2] = {0, 0};
+    if (!st.ok) {
+        const int x = PASS == 1 ? r : s;
+        Ln[0] = row_line(a.m, x);
+        Ln[1] = col_line(a.m, x);
+        split4_load<2>(Ln, lane, sp);
+    }
     // ---- phase A: histogram of v's neighbour blocks (self-loop excluded)
     int keep[4];
 #pragma unroll
@@ -715,7 +742,15 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
     const double *__restrict__ rcp = a.m.rcp;
     // ---- core entries of this pass: pass 1 M_rr, M_rs (row r), M_sr (column r); pass 2 M_ss (row s)
     int Mrr = 0, Mrs = 0, Msr = 0, Mss = 0;
-    if (PASS == 1) {
+    if (st.ok) {
+        if (PASS == 1) {
+            Mrr = stage_get(st.row, st.rcnt, st.rlen, r);
+            Mrs = stage_get(st.row, st.rcnt, st.rlen, s);
+            Msr = stage_get(st.col, st.ccnt, st.clen, s);
+        } else {
+            Mss = stage_get(st.row, st.rcnt, st.rlen, s);
+        }
+    } else if (PASS == 1) {
         const Line Lc[3] = {Ln[0], Ln[0], Ln[1]};
         const int spc[3] = {sp[0], sp[0], sp[1]};
         const int yc[3] = {r, s, s};
@@ -742,7 +777,7 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
         const int4 e = k >= nuniq ? make_int4(-1, 0, 0, 0) : tab[list[k]];
         const int t = e.x, ot = e.y, it = e.z;
         int pb2[2], nb2[2];
-        {
+        if (!st.ok) {
             const int yt[2] = {t, t};
             split4_bucket<2>(Ln, sp, yt, pb2, nb2);
         }
@@ -757,9 +792,14 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
             if (PASS == 1) pb += cw * (double)(Msr2 + Mrs2 + 1) / ((double)ds2 + Bd);
             else pf += cw * (double)(2 * Mss + 1) * __ldg(rcp + s);
         } else {
-            const int yt[2] = {t, t};
             int o2[2];
-            lookup4_in<2>(Ln, yt, pb2, nb2, o2);
+            if (st.ok) {
+                o2[0] = stage_get(st.row, st.rcnt, st.rlen, t);
+                o2[1] = stage_get(st.col, st.ccnt, st.clen, t);
+            } else {
+                const int yt[2] = {t, t};
+                lookup4_in<2>(Ln, yt, pb2, nb2, o2);
+            }
             const double rt = __ldg(rcp + t);
             if (PASS == 1) {   // o2 = {M_rt, M_tr}
                 accS -= df_t(ft, o2[0], -ot) + df_t(ft, o2[1], -it);
@@ -1014,25 +1054,62 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
     }
 }
 
-// sorted two-pass mode: warp w takes batch index perm[w] (the batch grouped
-// by r in pass 1, by s in pass 2); group vertices are skipped (k_move_groups)
+// sorted two-pass mode: each warp takes chunks of HALF_CHUNK consecutive
+// positions of perm (the batch grouped by r in pass 1, by s in pass 2) and
+// stages the pass's two lines of the current key in its shared memory once
+// per key run (one coalesced copy instead of every vertex's binary searches
+// through L2 / HBM); group vertices are skipped (k_move_groups).
+constexpr int HALF_CHUNK = 16;
+constexpr int HALF_WARPS = 8;
+constexpr size_t HALF_SMEM = (sizeof(int4) * WARP_TAB + sizeof(int) * (WARP_TAB / 2) + sizeof(int) * 2 * STAGE_CAP) *
+                             HALF_WARPS;
 template <bool WEIGHTED, int PASS>
-__global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move_half(MoveArgs a) {
-    extern __shared__ int4 move_smem[];   // MOVE_SMEM bytes
-    int4 *tabs = move_smem;
-    int *lists = reinterpret_cast<int *>(tabs + MOVE_WARPS * WARP_TAB);
+__global__ void __launch_bounds__(HALF_WARPS * 32, 2) k_move_half(MoveArgs a) {
+    extern __shared__ int4 move_smem[];   // HALF_SMEM bytes
     const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    int4 *tab = tabs + wl * WARP_TAB;
-    int *list = lists + wl * (WARP_TAB / 2);
+    int4 *tab = move_smem + wl * WARP_TAB;
+    int *list = reinterpret_cast<int *>(move_smem + HALF_WARPS * WARP_TAB) + wl * (WARP_TAB / 2);
+    int *srow = reinterpret_cast<int *>(move_smem + HALF_WARPS * WARP_TAB) + HALF_WARPS * (WARP_TAB / 2) +
+                wl * 2 * STAGE_CAP;
+    int *scol = srow + STAGE_CAP;
     tab_clear<32>(tab, WARP_TAB, lane);
     __syncwarp();
-    const int nwarps = gridDim.x * MOVE_WARPS;
-    for (int w = blockIdx.x * MOVE_WARPS + wl; w < a.count; w += nwarps) {
-        const int i = __ldg(a.perm + w);
-        const int v = a.first + i;
-        if ((__ldg(a.rowptr + v + 1) - __ldg(a.rowptr + v)) + (__ldg(a.cscptr + v + 1) - __ldg(a.cscptr + v)) > BIG_THR)
-            continue;
-        move_vertex_half<WEIGHTED, PASS>(a, i, tab, list);
+    const int nchunks = (a.count + HALF_CHUNK - 1) / HALF_CHUNK;
+    const int nwarps = gridDim.x * HALF_WARPS;
+    for (int ch = blockIdx.x * HALF_WARPS + wl; ch < nchunks; ch += nwarps) {
+        Stage st;
+        st.row = srow;
+        st.col = scol;
+        st.ok = false;
+        int cur = -1;
+        const int w1 = min(a.count, (ch + 1) * HALF_CHUNK);
+        for (int w = ch * HALF_CHUNK; w < w1; ++w) {
+            const int i = __ldg(a.perm + w);
+            const int v = a.first + i;
+            if ((__ldg(a.rowptr + v + 1) - __ldg(a.rowptr + v)) + (__ldg(a.cscptr + v + 1) - __ldg(a.cscptr + v)) >
+                BIG_THR)
+                continue;
+            const int key = PASS == 1 ? __ldg(a.b + v) : a.s_in[i];
+            if (key != cur) {   // stage row key and column key (ids) of the snapshot
+                cur = key;
+                const int rlo = __ldg(a.m.rowptr + key), rlen = __ldg(a.m.rowend + key) - rlo;
+                const int clo = __ldg(a.m.colptr + key), clen = __ldg(a.m.colend + key) - clo;
+                st.ok = rlen <= STAGE_CAP && clen <= STAGE_CAP;
+                st.rlen = rlen;
+                st.clen = clen;
+                st.rcnt = a.m.cnt + rlo;
+                st.ccnt = a.m.ccnt + clo;
+                __syncwarp();   // the previous key's searches are done
+                if (st.ok) {
+#pragma unroll 4
+                    for (int j = lane; j < rlen; j += 32) srow[j] = __ldg(a.m.col + rlo + j);
+#pragma unroll 4
+                    for (int j = lane; j < clen; j += 32) scol[j] = __ldg(a.m.row + clo + j);
+                }
+                __syncwarp();
+            }
+            move_vertex_half<WEIGHTED, PASS>(a, i, tab, list, st);
+        }
     }
 }
 
@@ -1091,9 +1168,11 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     a.part = nullptr;
     a.propose = mode == MOVE_FUSED ? 1 : 0;
     // sorted two-pass evaluation of a fused batch (large sparse blockmodels)
+    // decided per MOVE batch (c.batch_count), not per slice: the same mode for any number of GPUs
+    const int bc = c.batch_count > 0 ? c.batch_count : count;
     const bool sorted = mode == MOVE_FUSED && a.m.dense == nullptr && c.B > BIG_THR &&
                         (c.prm.move_sorted == 2 || (c.prm.move_sorted == 1 && (long long)c.E > GSAP_COOP_MAX_E &&
-                                                    count >= (1 << 16)));
+                                                    bc >= (1 << 16)));
     if (mode == MOVE_PROPOSE || sorted) {   // (a1) alone: thread per vertex
         const int pg = (int)std::min<long long>(((long long)count + 63) / 64, 148LL * 64);
         if (c.weighted) k_propose<true><<<pg, 64, 0, c.stream>>>(a);
@@ -1190,7 +1269,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     const bool dense = a.m.dense != nullptr;
     if (sorted) {
         per_device((const void *)k_move_half<false, 1>, [] {
-            const int sm = (int)MOVE_SMEM;
+            const int sm = (int)HALF_SMEM;
             GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
             GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
             GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
@@ -1200,12 +1279,15 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         MoveArgs a1 = a, a2 = a;
         a1.perm = c.mv_perm;            // grouped by r
         a2.perm = c.mv_perm + count;    // grouped by s
+        const int hg = (int)std::max<long long>(
+            1, std::min<long long>(((long long)count + HALF_CHUNK * HALF_WARPS - 1) / (HALF_CHUNK * HALF_WARPS),
+                                   148LL * 2));
         if (c.weighted) {
-            k_move_half<true, 1><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
-            k_move_half<true, 2><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
+            k_move_half<true, 1><<<hg, HALF_WARPS * 32, HALF_SMEM, c.stream>>>(a1);
+            k_move_half<true, 2><<<hg, HALF_WARPS * 32, HALF_SMEM, c.stream>>>(a2);
         } else {
-            k_move_half<false, 1><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
-            k_move_half<false, 2><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
+            k_move_half<false, 1><<<hg, HALF_WARPS * 32, HALF_SMEM, c.stream>>>(a1);
+            k_move_half<false, 2><<<hg, HALF_WARPS * 32, HALF_SMEM, c.stream>>>(a2);
         }
         c.launches += 2;
     } else if (c.weighted) {

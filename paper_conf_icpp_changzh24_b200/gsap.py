@@ -27,7 +27,7 @@ EXPORTED = ["gsap_default_params", "gsap_last_error", "gsap_partition", "gsap_cr
             "gsap_set_partition", "gsap_get_partition", "gsap_update_blockmodel", "gsap_propose",
             "gsap_delta_mdl", "gsap_select_merges", "gsap_apply_moves", "gsap_move_batch",
             "gsap_merge_phase", "gsap_mcmc_phase", "gsap_mdl", "gsap_get_blockmodel", "gsap_get_stats", "gsap_reset_stats",
-            "gsap_sync", "gsap_run", "gsap_nccl_unique_id", "gsap_shard_slice"]
+            "gsap_sync", "gsap_run", "gsap_nccl_unique_id", "gsap_shard_slice", "gsap_shard_plan"]
 
 
 class gsap_params(C.Structure):
@@ -36,7 +36,7 @@ class gsap_params(C.Structure):
                 ("thresh2", C.c_double), ("window", C.c_int32), ("num_batches", C.c_int32),
                 ("model_term", C.c_int32), ("max_rounds", C.c_int32), ("profile", C.c_int32),
                 ("cuda_graphs", C.c_int32), ("dense_max_B", C.c_int32), ("sparse_coop", C.c_int32), ("dense_coop", C.c_int32),
-                ("sel_small", C.c_int32), ("move_sorted", C.c_int32)]
+                ("sel_small", C.c_int32), ("move_sorted", C.c_int32), ("sim_ranks", C.c_int32)]
 
 
 class gsap_dist(C.Structure):
@@ -105,6 +105,7 @@ def lib():
         L.gsap_run.argtypes = [vp, vp, C.POINTER(i32), C.POINTER(C.c_double), vp, i32, C.POINTER(i32)]
         L.gsap_nccl_unique_id.argtypes = [vp]
         L.gsap_shard_slice.argtypes = [i32, i32, i32, i32, C.POINTER(i32), C.POINTER(i32), C.POINTER(i32)]
+        L.gsap_shard_plan.argtypes = [vp, i32, i32, i32, vp, vp]
         for name in EXPORTED:
             if name not in ("gsap_default_params", "gsap_last_error", "gsap_destroy"):
                 getattr(L, name).restype = C.c_int
@@ -329,6 +330,19 @@ class Context:
         _check(lib().gsap_get_blockmodel(self.h, C.byref(nnz), *[_ptr(out[k]) for k in (
             "rowptr", "col", "cnt", "cum", "colptr", "row", "ccnt", "ccum", "dout", "din")]))
         return out
+
+    def gsap_blockmodel_nnz(self):
+        """Number of non-zero blockmodel entries (size query of gsap_get_blockmodel)."""
+        nnz = C.c_int64(0)
+        _check(lib().gsap_get_blockmodel(self.h, C.byref(nnz), *([None] * 10)))
+        return nnz.value
+
+    def gsap_shard_plan(self, first, count, nranks):
+        """(first[nranks], count[nranks]): the edge-balanced slices of a MOVE batch."""
+        f = np.zeros(nranks, np.int32)
+        n = np.zeros(nranks, np.int32)
+        _check(lib().gsap_shard_plan(self.h, first, count, nranks, f.ctypes.data, n.ctypes.data))
+        return f, n
 
     def gsap_get_stats(self):
         st = gsap_stats()
