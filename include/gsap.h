@@ -89,6 +89,10 @@ typedef struct {
                                  merge phase cut into the ranks' slices exactly as with NCCL, each
                                  slice computed in rank order, the all-gathers skipped (the slices
                                  already sit at their offsets); default 0 = off */
+    int32_t incremental;      /* N2 (P:250-255 3.4): 1 (default) the rebuild after a MOVE batch in the
+                                 dense regime applies the change of M by the batch's moves to the
+                                 previous M (and skips the compaction when nothing moved); 0: every
+                                 rebuild from scratch.  Same blockmodel bit for bit. */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */

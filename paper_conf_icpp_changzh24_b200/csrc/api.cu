@@ -409,6 +409,11 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.scal = A.take<double>(8);
         c.scal_i = A.take<int>(8);
         c.n_eval = A.take<unsigned long long>(1);
+        if (c.prm.incremental) {
+            c.oldb = A.take<int>(Vs);
+            c.moved = A.take<int>(Vs);
+            c.moved_cnt = A.take<int>(1);
+        }
         c.Dh = A.take<double>((size_t)c.prm.max_nodal_itr + 1);
         if (c.prm.move_sorted) {
             c.mv_cnt = A.take<int>(2 * Vs + 2);
@@ -546,9 +551,19 @@ static void merge_phase(Ctx &c, uint32_t outer, int K, int *best_out, double *dS
     rebuild(c);
 }
 
+// N2: the next rebuild may apply the batch's moves to the dense M of the
+// previous one (the apply logs them); the sparse regime rebuilds in full
+static void announce_batch(Ctx &c, int first, int count) {
+    c.delta.first = first;
+    c.delta.count = count;
+    c.delta.acc = c.acc;
+    c.delta.pending = c.prm.incremental != 0 && c.dense_mode && c.oldb != nullptr;
+}
+
 static void move_batch(Ctx &c, uint32_t outer, uint32_t itr, int first, int count, double *dsum) {
     c.batch_count = count;
     const int G = ranks_of(c);
+    announce_batch(c, first, count);
     if (G == 1) {
         launch_move(c, MOVE_FUSED, outer, itr, first, count, c.s, c.dS, nullptr, c.acc);
         launch_apply(c, first, count, c.s, c.acc, c.dS, dsum, c.scal_i + 1, c.n_eval);
@@ -620,6 +635,7 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh, std::vector<d
             const int first = k * bs, last = std::min(V, first + bs);
             if (first >= last) continue;
             c.batch_count = last - first;
+            announce_batch(c, first, last - first);
             launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
             launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
             rebuild(c);
@@ -733,6 +749,7 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::ve
                 const int first = k * bs, last = std::min(V, first + bs);
                 if (first >= last) continue;
                 c.batch_count = last - first;
+            announce_batch(c, first, last - first);
             launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
                 launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
                 rebuild(c);
@@ -1013,6 +1030,7 @@ void gsap_default_params(gsap_params *p) {
     p->sel_small = 1;
     p->move_sorted = 1;
     p->sim_ranks = 0;
+    p->incremental = 1;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }

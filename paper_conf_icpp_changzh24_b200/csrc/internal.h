@@ -73,6 +73,7 @@ struct Ctx {
     double *rcp = nullptr;         // 1 / (d_x + B), refreshed by every rebuild
     size_t dense_cap = 0;   // elements
     bool dense_mode = false;
+    int dense_B = -1;       // B of the dense M / Mt the last rebuild left (-1: none)
 
     // rebuild scratch
     unsigned long long *keys0 = nullptr, *keys1 = nullptr, *vals64a = nullptr, *vals64b = nullptr;
@@ -125,6 +126,15 @@ struct Ctx {
     int nranks = 1, rank = 0;
     void *nccl_comm = nullptr;
     int batch_count = 0;           // the MOVE batch a launch belongs to (mode decisions per batch, not slice)
+
+    // N2 incremental update (dense regime): the batch a pending rebuild follows;
+    // the apply logs moved vertices and their old blocks, the rebuild applies dM
+    struct DeltaBatch {
+        int first = 0, count = 0;
+        const unsigned char *acc = nullptr;
+        bool pending = false;
+    } delta;
+    int *oldb = nullptr, *moved = nullptr, *moved_cnt = nullptr;
 
     // CUDA-graph capture of an MCMC iteration (N1: launch overhead, §5)
     unsigned *d_itr = nullptr;     // MCMC iteration read by k_move (device scalar)

@@ -648,31 +648,77 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
 // The split follows the decomposition above term by term; only the order of
 // the floating-point sums differs from the fused kernel.  Vertices with more
 // than 128 adjacency entries stay in k_move_groups (fused terms, s given).
-// The pass's two lines (row x, column x) staged in the warp's shared memory
-// (ids only; a hit's count is one global load at the found position), or
-// ok = false when either line is longer than the stage (global searches).
-constexpr int STAGE_CAP = 1024;   // entries per staged line
-struct Stage {
-    const int *row, *col;                            // shared memory copies of the lines' ids
-    const int *__restrict__ rcnt, *__restrict__ ccnt;   // the lines' counts (global)
-    int rlen, clen;
-    bool ok;
-};
-
-// M entry of key y in a staged line: branchless lower bound in shared memory
-GSAP_DEV int stage_get(const int *ids, const int *__restrict__ cnt, int len, int y) {
-    int p = 0, n = len;
-    while (n > 1) {
-        const int h = n >> 1;
-        p = ids[p + h - 1] < y ? p + h : p;
-        n -= h;
-    }
-    if (n == 1 && ids[p] < y) ++p;
-    return (p < len && ids[p] == y) ? __ldg(cnt + p) : 0;
+// wide splitters: K per lane (32 K per line, lane l holds splitters l K ..
+// l K + K - 1: entry floor(g len / (32 K)) for splitter g); a key's bucket is
+// found with 5 + (K - 1) shuffles and holds <= ceil(len / (32 K)) entries,
+// which are then scanned with independent loads (one memory round for
+// lines of <= 256 K entries instead of a dependent binary search)
+template <int N, int K>
+GSAP_DEV void splitw_load(const Line (&L)[N], int lane, int (&sp)[N][K]) {
+#pragma unroll
+    for (int k = 0; k < N; ++k)
+#pragma unroll
+        for (int e = 0; e < K; ++e)
+            sp[k][e] = L[k].len > 0 ? __ldg(L[k].idx + (int)(((long long)(lane * K + e) * L[k].len) / (32 * K)))
+                                    : 0x7fffffff;
 }
 
+template <int N, int K>
+GSAP_DEV void splitw_bucket(const Line (&L)[N], const int (&sp)[N][K], const int (&y)[N], int (&p)[N],
+                            int (&n)[N]) {
+#pragma unroll
+    for (int k = 0; k < N; ++k) {
+        int j = 0;   // the last lane whose first splitter is <= y[k]
+#pragma unroll
+        for (int st = 16; st >= 1; st >>= 1) {
+            const int x = __shfl_sync(0xffffffffu, sp[k][0], j + st);
+            if (x <= y[k]) j += st;
+        }
+        int e = 0;   // the last of lane j's splitters <= y[k]
+#pragma unroll
+        for (int q = 1; q < K; ++q) {
+            const int x = __shfl_sync(0xffffffffu, sp[k][q], j);
+            if (x <= y[k]) e = q;
+        }
+        const int s0 = __shfl_sync(0xffffffffu, sp[k][0], 0);
+        const int len = L[k].len, g = j * K + e;
+        const int lo = (int)(((long long)g * len) / (32 * K)), hi = (int)(((long long)(g + 1) * len) / (32 * K));
+        p[k] = lo;
+        n[k] = (len > 0 && s0 <= y[k]) ? hi - lo : 0;
+    }
+}
+
+// M entry of key y[k] in bucket [p[k], p[k] + n[k]) of line k: binary
+// search down to <= 8 entries, then up to 8 independent id loads; the count
+// only on a hit
+template <int N>
+GSAP_DEV void bucket_get(const Line (&L)[N], const int (&y)[N], int (&p)[N], int (&n)[N], int (&out)[N]) {
+#pragma unroll
+    for (int k = 0; k < N; ++k) {
+        while (n[k] > 8) {
+            const int h = n[k] >> 1;
+            p[k] = __ldg(L[k].idx + p[k] + h) <= y[k] ? p[k] + h : p[k];
+            n[k] -= h;
+        }
+    }
+    int id[N][8];
+#pragma unroll
+    for (int k = 0; k < N; ++k)
+#pragma unroll
+        for (int q = 0; q < 8; ++q) id[k][q] = q < n[k] ? __ldg(L[k].idx + p[k] + q) : -1;
+#pragma unroll
+    for (int k = 0; k < N; ++k) {
+        int hit = -1;
+#pragma unroll
+        for (int q = 0; q < 8; ++q) hit = id[k][q] == y[k] ? q : hit;
+        out[k] = hit >= 0 ? __ldg(L[k].cnt + p[k] + hit) : 0;
+    }
+}
+
+constexpr int HALF_K = 4;   // splitters per lane in the sorted two-pass kernels
+
 template <bool WEIGHTED, int PASS>
-GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list, const Stage &st) {
+GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
     const int lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
     const int v = a.first + i;
@@ -690,17 +736,14 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list, c
     const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
     const int deg = nout + nin;   // <= 128 (the caller routes bigger vertices to k_move_groups)
     const int B = a.m.B;
-    // the two lines of this pass: staged in shared memory (st.ok, warp-uniform),
-    // else searched in global memory with warp-shared splitters (issued now,
-    // before the histogram)
+    // the two lines of this pass and their wide splitters (32 HALF_K per
+    // line, shared by the warp), issued before the histogram
     Line Ln[2];
-    int sp[2] = {0, 0};
-    if (!st.ok) {
-        const int x = PASS == 1 ? r : s;
-        Ln[0] = row_line(a.m, x);
-        Ln[1] = col_line(a.m, x);
-        split4_load<2>(Ln, lane, sp);
-    }
+    const int x = PASS == 1 ? r : s;
+    Ln[0] = row_line(a.m, x);
+    Ln[1] = col_line(a.m, x);
+    int sp[2][HALF_K];
+    splitw_load<2, HALF_K>(Ln, lane, sp);
     // ---- phase A: histogram of v's neighbour blocks (self-loop excluded)
     int keep[4];
 #pragma unroll
@@ -742,31 +785,31 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list, c
     const double *__restrict__ rcp = a.m.rcp;
     // ---- core entries of this pass: pass 1 M_rr, M_rs (row r), M_sr (column r); pass 2 M_ss (row s)
     int Mrr = 0, Mrs = 0, Msr = 0, Mss = 0;
-    if (st.ok) {
-        if (PASS == 1) {
-            Mrr = stage_get(st.row, st.rcnt, st.rlen, r);
-            Mrs = stage_get(st.row, st.rcnt, st.rlen, s);
-            Msr = stage_get(st.col, st.ccnt, st.clen, s);
-        } else {
-            Mss = stage_get(st.row, st.rcnt, st.rlen, s);
-        }
-    } else if (PASS == 1) {
+    if (PASS == 1) {   // row r at r and s, column r at s
         const Line Lc[3] = {Ln[0], Ln[0], Ln[1]};
-        const int spc[3] = {sp[0], sp[0], sp[1]};
+        int spc[3][HALF_K];
+#pragma unroll
+        for (int e = 0; e < HALF_K; ++e) {
+            spc[0][e] = sp[0][e];
+            spc[1][e] = sp[0][e];
+            spc[2][e] = sp[1][e];
+        }
         const int yc[3] = {r, s, s};
-        int oc[3], pc[3], nc[3];
-        split4_bucket<3>(Lc, spc, yc, pc, nc);
-        lookup4_in<3>(Lc, yc, pc, nc, oc);
+        int pc[3], nc[3], oc[3];
+        splitw_bucket<3, HALF_K>(Lc, spc, yc, pc, nc);
+        bucket_get<3>(Lc, yc, pc, nc, oc);
         Mrr = oc[0];
         Mrs = oc[1];
         Msr = oc[2];
-    } else {
+    } else {           // row s at s
         const Line Lc[1] = {Ln[0]};
-        const int spc[1] = {sp[0]};
+        int spc[1][HALF_K];
+#pragma unroll
+        for (int e = 0; e < HALF_K; ++e) spc[0][e] = sp[0][e];
         const int yc[1] = {s};
-        int oc[1], pc[1], nc[1];
-        split4_bucket<1>(Lc, spc, yc, pc, nc);
-        lookup4_in<1>(Lc, yc, pc, nc, oc);
+        int pc[1], nc[1], oc[1];
+        splitw_bucket<1, HALF_K>(Lc, spc, yc, pc, nc);
+        bucket_get<1>(Lc, yc, pc, nc, oc);
         Mss = oc[0];
     }
     const int Mrr2 = Mrr - o_r - i_r - l, Mrs2 = Mrs + i_r - o_s, Msr2 = Msr + o_r - i_s;
@@ -777,9 +820,9 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list, c
         const int4 e = k >= nuniq ? make_int4(-1, 0, 0, 0) : tab[list[k]];
         const int t = e.x, ot = e.y, it = e.z;
         int pb2[2], nb2[2];
-        if (!st.ok) {
+        {
             const int yt[2] = {t, t};
-            split4_bucket<2>(Ln, sp, yt, pb2, nb2);
+            splitw_bucket<2, HALF_K>(Ln, sp, yt, pb2, nb2);
         }
         if (k >= nuniq) continue;
         const double cw = (double)(ot + it);
@@ -793,12 +836,9 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list, c
             else pf += cw * (double)(2 * Mss + 1) * __ldg(rcp + s);
         } else {
             int o2[2];
-            if (st.ok) {
-                o2[0] = stage_get(st.row, st.rcnt, st.rlen, t);
-                o2[1] = stage_get(st.col, st.ccnt, st.clen, t);
-            } else {
+            {
                 const int yt[2] = {t, t};
-                lookup4_in<2>(Ln, yt, pb2, nb2, o2);
+                bucket_get<2>(Ln, yt, pb2, nb2, o2);
             }
             const double rt = __ldg(rcp + t);
             if (PASS == 1) {   // o2 = {M_rt, M_tr}
@@ -992,7 +1032,7 @@ __global__ void __launch_bounds__(256) k_propose(MoveArgs a) {
 // The shared memory is the 8 warp tables, or one CTA table over the same bytes.
 template <bool WEIGHTED>
 #ifndef GSAP_GROUPS_MINB
-#define GSAP_GROUPS_MINB 1
+#define GSAP_GROUPS_MINB 2
 #endif
 __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_GROUPS_MINB) k_move_groups(MoveArgs a) {
     __shared__ int4 tabs[CTA_SMEM_SLOTS];
@@ -1054,62 +1094,28 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
     }
 }
 
-// sorted two-pass mode: each warp takes chunks of HALF_CHUNK consecutive
-// positions of perm (the batch grouped by r in pass 1, by s in pass 2) and
-// stages the pass's two lines of the current key in its shared memory once
-// per key run (one coalesced copy instead of every vertex's binary searches
-// through L2 / HBM); group vertices are skipped (k_move_groups).
-constexpr int HALF_CHUNK = 16;
-constexpr int HALF_WARPS = 8;
-constexpr size_t HALF_SMEM = (sizeof(int4) * WARP_TAB + sizeof(int) * (WARP_TAB / 2) + sizeof(int) * 2 * STAGE_CAP) *
-                             HALF_WARPS;
+// sorted two-pass mode: warp w takes batch index perm[w] (grid-stride), so
+// consecutive warps search the same key's two lines (hits in L1 / L2)
+#ifndef GSAP_HALF_MINB
+#define GSAP_HALF_MINB 4
+#endif
 template <bool WEIGHTED, int PASS>
-__global__ void __launch_bounds__(HALF_WARPS * 32, 2) k_move_half(MoveArgs a) {
-    extern __shared__ int4 move_smem[];   // HALF_SMEM bytes
+__global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_HALF_MINB) k_move_half(MoveArgs a) {
+    extern __shared__ int4 move_smem[];   // MOVE_SMEM bytes
+    int4 *tabs = move_smem;
+    int *lists = reinterpret_cast<int *>(tabs + MOVE_WARPS * WARP_TAB);
     const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    int4 *tab = move_smem + wl * WARP_TAB;
-    int *list = reinterpret_cast<int *>(move_smem + HALF_WARPS * WARP_TAB) + wl * (WARP_TAB / 2);
-    int *srow = reinterpret_cast<int *>(move_smem + HALF_WARPS * WARP_TAB) + HALF_WARPS * (WARP_TAB / 2) +
-                wl * 2 * STAGE_CAP;
-    int *scol = srow + STAGE_CAP;
+    int4 *tab = tabs + wl * WARP_TAB;
+    int *list = lists + wl * (WARP_TAB / 2);
     tab_clear<32>(tab, WARP_TAB, lane);
     __syncwarp();
-    const int nchunks = (a.count + HALF_CHUNK - 1) / HALF_CHUNK;
-    const int nwarps = gridDim.x * HALF_WARPS;
-    for (int ch = blockIdx.x * HALF_WARPS + wl; ch < nchunks; ch += nwarps) {
-        Stage st;
-        st.row = srow;
-        st.col = scol;
-        st.ok = false;
-        int cur = -1;
-        const int w1 = min(a.count, (ch + 1) * HALF_CHUNK);
-        for (int w = ch * HALF_CHUNK; w < w1; ++w) {
-            const int i = __ldg(a.perm + w);
-            const int v = a.first + i;
-            if ((__ldg(a.rowptr + v + 1) - __ldg(a.rowptr + v)) + (__ldg(a.cscptr + v + 1) - __ldg(a.cscptr + v)) >
-                BIG_THR)
-                continue;
-            const int key = PASS == 1 ? __ldg(a.b + v) : a.s_in[i];
-            if (key != cur) {   // stage row key and column key (ids) of the snapshot
-                cur = key;
-                const int rlo = __ldg(a.m.rowptr + key), rlen = __ldg(a.m.rowend + key) - rlo;
-                const int clo = __ldg(a.m.colptr + key), clen = __ldg(a.m.colend + key) - clo;
-                st.ok = rlen <= STAGE_CAP && clen <= STAGE_CAP;
-                st.rlen = rlen;
-                st.clen = clen;
-                st.rcnt = a.m.cnt + rlo;
-                st.ccnt = a.m.ccnt + clo;
-                __syncwarp();   // the previous key's searches are done
-                if (st.ok) {
-#pragma unroll 4
-                    for (int j = lane; j < rlen; j += 32) srow[j] = __ldg(a.m.col + rlo + j);
-#pragma unroll 4
-                    for (int j = lane; j < clen; j += 32) scol[j] = __ldg(a.m.row + clo + j);
-                }
-                __syncwarp();
-            }
-            move_vertex_half<WEIGHTED, PASS>(a, i, tab, list, st);
-        }
+    const int nwarps = gridDim.x * MOVE_WARPS;
+    for (int w = blockIdx.x * MOVE_WARPS + wl; w < a.count; w += nwarps) {
+        const int i = __ldg(a.perm + w);
+        const int v = a.first + i;
+        if ((__ldg(a.rowptr + v + 1) - __ldg(a.rowptr + v)) + (__ldg(a.cscptr + v + 1) - __ldg(a.cscptr + v)) > BIG_THR)
+            continue;
+        move_vertex_half<WEIGHTED, PASS>(a, i, tab, list);
     }
 }
 
@@ -1269,7 +1275,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     const bool dense = a.m.dense != nullptr;
     if (sorted) {
         per_device((const void *)k_move_half<false, 1>, [] {
-            const int sm = (int)HALF_SMEM;
+            const int sm = (int)MOVE_SMEM;
             GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
             GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
             GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
@@ -1279,15 +1285,12 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         MoveArgs a1 = a, a2 = a;
         a1.perm = c.mv_perm;            // grouped by r
         a2.perm = c.mv_perm + count;    // grouped by s
-        const int hg = (int)std::max<long long>(
-            1, std::min<long long>(((long long)count + HALF_CHUNK * HALF_WARPS - 1) / (HALF_CHUNK * HALF_WARPS),
-                                   148LL * 2));
         if (c.weighted) {
-            k_move_half<true, 1><<<hg, HALF_WARPS * 32, HALF_SMEM, c.stream>>>(a1);
-            k_move_half<true, 2><<<hg, HALF_WARPS * 32, HALF_SMEM, c.stream>>>(a2);
+            k_move_half<true, 1><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
+            k_move_half<true, 2><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
         } else {
-            k_move_half<false, 1><<<hg, HALF_WARPS * 32, HALF_SMEM, c.stream>>>(a1);
-            k_move_half<false, 2><<<hg, HALF_WARPS * 32, HALF_SMEM, c.stream>>>(a2);
+            k_move_half<false, 1><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
+            k_move_half<false, 2><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
         }
         c.launches += 2;
     } else if (c.weighted) {
@@ -1312,13 +1315,34 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
 // ---------------------------------------------------------------- apply --
 constexpr int APPLY_CHUNK = 1024;
 
+// N2 (incremental blockmodel update, P:250-255 3.4): when log.oldb is set,
+// every applied move records the vertex's old block (oldb[v]) and appends v
+// to log.moved (warp-aggregated atomics, order irrelevant: the update is
+// integer additions)
+struct MoveLog {
+    int *oldb, *moved, *moved_cnt;
+};
+
+GSAP_DEV void log_move(const MoveLog &lg, bool mv, int v, int old) {
+    const unsigned m = __ballot_sync(FULL, mv);   // warp-uniform call
+    if (!m) return;
+    const int lane = threadIdx.x & 31, leader = __ffs(m) - 1;
+    int base = 0;
+    if (lane == leader) base = atomicAdd(lg.moved_cnt, __popc(m));
+    base = __shfl_sync(FULL, base, leader);
+    if (mv) {
+        lg.oldb[v] = old;
+        lg.moved[base + __popc(m & ((1u << lane) - 1u))] = v;
+    }
+}
+
 // n_eval (nullable): += the proposals with s != b[v] (the moves that were
 // evaluated, R:Z13) -- counted before b is written
 __global__ void __launch_bounds__(256) k_apply(int first, int count, const int *__restrict__ s,
                                                const unsigned char *__restrict__ acc,
                                                const double *__restrict__ dS, int *__restrict__ b,
                                                double *__restrict__ partials, int *__restrict__ nacc,
-                                               unsigned long long *__restrict__ n_eval) {
+                                               unsigned long long *__restrict__ n_eval, MoveLog lg) {
     __shared__ double sh[8];
     const int base = blockIdx.x * APPLY_CHUNK;
     double sum = 0.0;
@@ -1326,6 +1350,10 @@ __global__ void __launch_bounds__(256) k_apply(int first, int count, const int *
     for (int k = threadIdx.x; k < APPLY_CHUNK; k += 256) {
         const int i = base + k;
         if (i < count && n_eval) ne += s[i] != b[first + i];
+        if (lg.oldb) {
+            const bool mv = i < count && acc[i];
+            log_move(lg, mv, first + i, mv ? b[first + i] : 0);
+        }
         if (i < count && acc[i]) {
             if (b) b[first + i] = s[i];
             sum += dS ? dS[i] : 0.0;
@@ -1372,7 +1400,7 @@ __global__ void __launch_bounds__(256) k_apply_sum(int first, int count, const i
                                                    const double *__restrict__ dS, int *__restrict__ b,
                                                    double *__restrict__ partials, int *__restrict__ nacc,
                                                    unsigned *__restrict__ arrivals, double *__restrict__ dsum,
-                                                   unsigned long long *__restrict__ n_eval) {
+                                                   unsigned long long *__restrict__ n_eval, MoveLog lg) {
     __shared__ double sh[8];
     __shared__ bool last;
     const int base = blockIdx.x * APPLY_CHUNK;
@@ -1381,6 +1409,10 @@ __global__ void __launch_bounds__(256) k_apply_sum(int first, int count, const i
     for (int k = threadIdx.x; k < APPLY_CHUNK; k += 256) {
         const int i = base + k;
         if (i < count && n_eval) ne += s[i] != b[first + i];
+        if (lg.oldb) {
+            const bool mv = i < count && acc[i];
+            log_move(lg, mv, first + i, mv ? b[first + i] : 0);
+        }
         if (i < count && acc[i]) {
             b[first + i] = s[i];
             sum += dS ? dS[i] : 0.0;
@@ -1443,12 +1475,24 @@ bool device_ids_ok(Ctx &c, int n, const int *x, const unsigned char *mask, int B
     return c.h_int[6] == 0;
 }
 
+// the move log of the batch for the incremental update (N2): on when the
+// caller announced the batch (c.delta.pending) and the regime keeps dense M
+static MoveLog move_log(Ctx &c) {
+    MoveLog lg{nullptr, nullptr, nullptr};
+    if (c.delta.pending) {
+        GSAP_CUDA(cudaMemsetAsync(c.moved_cnt, 0, sizeof(int), c.stream));
+        lg = MoveLog{c.oldb, c.moved, c.moved_cnt};
+    }
+    return lg;
+}
+
 void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
                   double *dsum, int *nacc, unsigned long long *n_eval) {
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
+    const MoveLog lg = move_log(c);
     k_apply_sum<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, c.b, c.partials, nacc,
-                                          reinterpret_cast<unsigned *>(c.scal_i + 4), dsum, n_eval);
+                                          reinterpret_cast<unsigned *>(c.scal_i + 4), dsum, n_eval, lg);
     c.launches += 1;
     GSAP_CHECK_LAUNCH();
 }
@@ -1459,7 +1503,8 @@ void launch_partials(Ctx &c, int first, int count, const int *s, const unsigned 
                      double *partials) {
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
-    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, nullptr, partials, nullptr, nullptr);
+    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, nullptr, partials, nullptr, nullptr,
+                                      MoveLog{nullptr, nullptr, nullptr});
     ++c.launches;
     GSAP_CHECK_LAUNCH();
 }
@@ -1469,7 +1514,8 @@ void launch_apply_gathered(Ctx &c, int first, int count, const int *s, const uns
                            const double *partials, int n, double *dsum, int *nacc, unsigned long long *n_eval) {
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
-    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, nullptr, c.b, nullptr, nacc, n_eval);
+    const MoveLog lg = move_log(c);
+    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, nullptr, c.b, nullptr, nacc, n_eval, lg);
     k_sum_partials<<<1, 256, 0, c.stream>>>(partials, n, dsum, 1);
     c.launches += 2;
     GSAP_CHECK_LAUNCH();

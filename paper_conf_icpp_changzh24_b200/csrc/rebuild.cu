@@ -186,8 +186,11 @@ __global__ void k_transpose(const int *__restrict__ M, int B, int *__restrict__ 
 // both dense matrices (M: lines x < B, its transpose: lines x >= B) in one
 // launch: non-zeros and sum per line; four consecutive entries per lane per
 // step (128 per warp step, independent loads)
+// skip (nullable): the batch's moved-vertex count; 0 = M unchanged, nothing to do
 __global__ void k_row_stats2(const int *__restrict__ M, const int *__restrict__ Mt, int B, int *__restrict__ nnzA,
-                             int *__restrict__ sumA, int *__restrict__ nnzB, int *__restrict__ sumB) {
+                             int *__restrict__ sumA, int *__restrict__ nnzB, int *__restrict__ sumB,
+                             const int *__restrict__ skip) {
+    if (skip && *skip == 0) return;
     const int lane = threadIdx.x & 31;
     for (int x2 = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x2 < 2 * B; x2 += (gridDim.x * blockDim.x) >> 5) {
         const bool t = x2 >= B;
@@ -213,7 +216,9 @@ __global__ void k_row_stats2(const int *__restrict__ M, const int *__restrict__ 
 }
 
 // two exclusive scans of n <= 32K ints, one CTA each (dense regime: B <= 16384)
-__global__ void __launch_bounds__(1024) k_scan2(const int *a0, int *o0, const int *a1, int *o1, int n) {
+__global__ void __launch_bounds__(1024) k_scan2(const int *a0, int *o0, const int *a1, int *o1, int n,
+                                                const int *__restrict__ skip) {
+    if (skip && *skip == 0) return;
     __shared__ int sh[32];
     const int *in = blockIdx.x ? a1 : a0;
     int *out = blockIdx.x ? o1 : o0;
@@ -261,7 +266,9 @@ __global__ void k_row_compact2(const int *__restrict__ M, const int *__restrict_
                                const int *__restrict__ ptrA, int *__restrict__ idxA, int *__restrict__ cntA,
                                int *__restrict__ cumA, const int *__restrict__ ptrB, int *__restrict__ idxB,
                                int *__restrict__ cntB, int *__restrict__ cumB, const int *__restrict__ dout,
-                               const int *__restrict__ din, double *__restrict__ rcp, int *__restrict__ d_nnz) {
+                               const int *__restrict__ din, double *__restrict__ rcp, int *__restrict__ d_nnz,
+                               const int *__restrict__ skip) {
+    if (skip && *skip == 0) return;
     const int lane = threadIdx.x & 31;
     if (blockIdx.x == 0 && threadIdx.x == 0) *d_nnz = ptrA[B];
     for (int x2 = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x2 < 2 * B; x2 += (gridDim.x * blockDim.x) >> 5) {
@@ -621,6 +628,71 @@ static void launch_rebuild_dense_coop(Ctx &c) {
     ++c.launches;
 }
 
+// N2 (incremental blockmodel update, P:250-255 3.4, Fig. 6): the change of M
+// (and of its transpose) by the batch's applied moves, instead of a histogram
+// of every edge.  One warp per moved vertex v (old block r = oldb[v], new
+// block s = b[v]); an edge u -> w changes from (old b_u, old b_w) to (new b_u,
+// new b_w), each edge counted once: v's out-edges always, its in-edges only
+// from vertices that did not move (a moved source covers the edge with its
+// own out-edges; a self-loop is an out-edge).  Integer additions: the result
+// equals the full histogram exactly.
+__global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ moved, const int *__restrict__ moved_cnt,
+                                                     int first, int count, const unsigned char *__restrict__ acc,
+                                                     const int *__restrict__ oldb, const int *__restrict__ b,
+                                                     const int *__restrict__ rowptr, const int *__restrict__ col,
+                                                     const int *__restrict__ wgt, const int *__restrict__ cscptr,
+                                                     const int *__restrict__ cscsrc, const int *__restrict__ cscwgt,
+                                                     int B, int *__restrict__ M, int *__restrict__ Mt) {
+    const int n = *moved_cnt;
+    const int lane = threadIdx.x & 31;
+    for (int k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < n; k += (gridDim.x * blockDim.x) >> 5) {
+        const int v = moved[k];
+        const int r = oldb[v], s = b[v];
+        const int ro = rowptr[v], nout = rowptr[v + 1] - ro;
+        for (int j = lane; j < nout; j += 32) {
+            const int w = col[ro + j];
+            const int wt = wgt ? wgt[ro + j] : 1;
+            const int bn = b[w];
+            const bool wm = w >= first && w < first + count && acc[w - first];
+            const int bo = wm ? oldb[w] : bn;
+            atomicAdd(M + (size_t)r * B + bo, -wt);
+            atomicAdd(M + (size_t)s * B + bn, wt);
+            atomicAdd(Mt + (size_t)bo * B + r, -wt);
+            atomicAdd(Mt + (size_t)bn * B + s, wt);
+        }
+        const int ci = cscptr[v], nin = cscptr[v + 1] - ci;
+        for (int j = lane; j < nin; j += 32) {
+            const int w = cscsrc[ci + j];
+            if (w >= first && w < first + count && acc[w - first]) continue;   // moved source (incl. v's self-loop)
+            const int wt = cscwgt ? cscwgt[ci + j] : 1;
+            const int bw = b[w];
+            atomicAdd(M + (size_t)bw * B + r, -wt);
+            atomicAdd(M + (size_t)bw * B + s, wt);
+            atomicAdd(Mt + (size_t)r * B + bw, -wt);
+            atomicAdd(Mt + (size_t)s * B + bw, wt);
+        }
+    }
+}
+
+// the dense regime after a MOVE batch whose moves were logged: M and Mt
+// updated in place by k_dense_delta, then the line statistics, offsets and
+// compaction as in the full path (all four skip when no vertex moved)
+static void rebuild_dense_delta(Ctx &c) {
+    const int B = c.B;
+    const int dg = (int)std::min<long long>(((long long)c.delta.count + 7) / 8, 148LL * 8);
+    k_dense_delta<<<std::max(dg, 1), 256, 0, c.stream>>>(c.moved, c.moved_cnt, c.delta.first, c.delta.count,
+                                                        c.delta.acc, c.oldb, c.b, c.rowptr, c.col, c.wgt, c.cscptr,
+                                                        c.cscsrc, c.cscwgt, B, c.dense, c.denseT);
+    const int rg = grid_for(2LL * B * 32, 256);
+    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.rownnz, c.dout, c.tmpi, c.din, c.moved_cnt);
+    k_scan2<<<2, 1024, 0, c.stream>>>(c.rownnz, c.bm_rowptr, c.tmpi, c.bm_colptr, B, c.moved_cnt);
+    k_row_compact2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum,
+                                             c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp,
+                                             c.d_nnz, c.moved_cnt);
+    c.launches += 4;
+    GSAP_CHECK_LAUNCH();
+}
+
 static void rebuild_dense(Ctx &c) {
     const int B = c.B, E = c.E;
     const size_t BB = (size_t)B * B;
@@ -646,11 +718,11 @@ static void rebuild_dense(Ctx &c) {
     dim3 tg((B + 31) / 32, (B + 31) / 32), tb(32, 8);
     k_transpose<<<tg, tb, 0, c.stream>>>(c.dense, B, c.denseT);
     const int rg = grid_for(2LL * B * 32, 256);
-    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.rownnz, c.dout, c.tmpi, c.din);
-    k_scan2<<<2, 1024, 0, c.stream>>>(c.rownnz, c.bm_rowptr, c.tmpi, c.bm_colptr, B);
+    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.rownnz, c.dout, c.tmpi, c.din, nullptr);
+    k_scan2<<<2, 1024, 0, c.stream>>>(c.rownnz, c.bm_rowptr, c.tmpi, c.bm_colptr, B, nullptr);
     k_row_compact2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum,
                                              c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp,
-                                             c.d_nnz);
+                                             c.d_nnz, nullptr);
     c.launches += 4;
     GSAP_CHECK_LAUNCH();
 }
@@ -789,9 +861,12 @@ static void rebuild_sparse(Ctx &c) {
 void rebuild(Ctx &c) {
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_rebuild, &ev);
+    const bool was_dense = c.dense_mode && c.dense_B == c.B;
     c.dense_mode = dense_ok(c, c.B);
     c.padded = false;   // set by the multi-kernel sparse path
-    if (c.dense_mode && c.prm.dense_coop && c.E > 0 && c.B <= SMALL_MAX_B) {
+    if (c.delta.pending && was_dense && c.dense_mode && c.E > 0) {
+        rebuild_dense_delta(c);   // N2: M, Mt of the previous rebuild + the batch's moves
+    } else if (c.dense_mode && c.prm.dense_coop && c.E > 0 && c.B <= SMALL_MAX_B) {
         launch_rebuild_dense_coop<true>(c);
     } else if (c.dense_mode && c.prm.dense_coop == 2 && c.E > 0) {
         launch_rebuild_dense_coop<false>(c);   // measured slower than the multi-kernel path above B = 221
@@ -808,6 +883,8 @@ void rebuild(Ctx &c) {
     // row pointers, b) and the fixed-size outputs (row / column pointers,
     // degrees); the nnz-sized outputs are left out (nnz stays on the device)
     const double bytes = 4.0 * c.E + 8.0 * c.V + 8.0 * (c.B + 1) + 8.0 * c.B;
+    c.dense_B = c.dense_mode ? c.B : -1;
+    c.delta.pending = false;
     kc_end(c, c.k_rebuild, ev, bytes);
 }
 

@@ -614,3 +614,40 @@ def test_fused_move_batch_weighted_hubs_lockstep(G, oracle_mod, regime, weighted
             assert np.array_equal(ctx.gsap_get_partition()[0], orc.partition()[0])
             assert_same_blockmodel(ctx, orc)
     print("MH ties:", nties)
+
+
+@pytest.mark.parametrize("gname,regime", [("1k", "auto"), ("1k", "dense_mk"), ("20k", "auto"), ("20k", "dense_mk"),
+                                          ("20k", "dense_coop2"), ("hubs_w", "auto"), ("hubs_w", "dense_mk")])
+def test_incremental_update_bit_identical(G, oracle_mod, gname, regime):
+    """N2 (§3.4): the rebuild after a MOVE batch applying the batch's
+    change of M to the previous dense M (incremental = 1, the default) gives
+    the same run as rebuilding every blockmodel from scratch: partition, MDL,
+    trace and counters bit for bit; and the blockmodel after a batch equals the
+    oracle's rebuild."""
+    if gname == "hubs_w":
+        rowptr, col, w = _hub_graph(True)
+    else:
+        rowptr, col, truth, cfg = dcsbm.make(gname)
+        w = None
+    runs = []
+    for inc in (1, 0):
+        ctx = G.Context(rowptr, col, w, params=G.gsap_default_params(seed=SEED, incremental=inc, **REGIMES[regime]))
+        r = ctx.gsap_run()
+        st = ctx.gsap_get_stats()
+        runs.append((r["B"], r["mdl"], r["b"].tobytes(), r["trace"][:, [0, 1, 2, 3, 5]].tobytes(),
+                     st["n_move_acc"], st["mcmc_itr_total"]))
+        ctx.close()
+    assert runs[0] == runs[1]
+    # one batch from a dense state, blockmodel vs the oracle's full rebuild
+    V = len(rowptr) - 1
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, **REGIMES[regime])
+    B = min(V, 150)
+    b0 = dcsbm.random_partition(V, B, 17)
+    set_both(ctx, orc, b0, B)
+    bs = (V + 3) // 4
+    for k in range(4):
+        first, count = k * bs, min(V, (k + 1) * bs) - k * bs
+        s, dS, acc, _ = ctx.gsap_move_batch(4, 1, first, count)
+        orc.apply_moves(first, count, s, acc)
+        orc.rebuild()
+        assert_same_blockmodel(ctx, orc)
