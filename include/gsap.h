@@ -93,6 +93,11 @@ typedef struct {
                                  dense regime applies the change of M by the batch's moves to the
                                  previous M (and skips the compaction when nothing moved); 0: every
                                  rebuild from scratch.  Same blockmodel bit for bit. */
+    int32_t proposal_mode;    /* 0 (default): a fresh Philox draw per proposal (R:Z6).  1: the paper-
+                                 literal lookup-table ablation (N4; Alg. 1, Fig. 4):
+                                 ONE weighted neighbour block per block, drawn per merge phase / MOVE
+                                 batch and shared by every proposal that reaches that block (a MERGE
+                                 outcome equal to r is redrawn uniformly over the other blocks) */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */
@@ -164,7 +169,8 @@ gsap_status gsap_update_blockmodel(gsap_ctx *ctx);
  * vertex v in [first, first+count), Philox counter (v, 0, itr, outer<<1|1),
  * s_out[count].  MERGE: num_proposals per block r in [first, first+count),
  * counter (r, j, 0, outer<<1|0), s_out[count*num_proposals] (row-major).
- * s_out: host or device.
+ * proposal_mode = 1 (N4): the shared table is drawn first (MOVE: keyed by
+ * `first`, the batch's first vertex; MERGE: by outer).  s_out: host or device.
  */
 gsap_status gsap_propose(gsap_ctx *ctx, gsap_phase phase, uint32_t outer, uint32_t itr,
                          int32_t first, int32_t count, int32_t *s_out);

@@ -123,6 +123,8 @@ typedef struct {
     int32_t *b;
     int32_t B;
     OBM bm;
+    int table_mode;     /* N4 ablation: 1 = the paper-literal shared lookup table */
+    int32_t *mt;        /* mt[x]: one weighted neighbour block of block x, or -1 */
 } OState;
 
 static void *xmalloc(size_t n)
@@ -293,6 +295,26 @@ static int32_t walk_block(const OBM *m, int32_t u, uint64_t p, int32_t skip)
     return -1; /* unreachable when p < total */
 }
 
+/* ------------------------------------------------------------------------ */
+/* N4 ablation: the paper's lookup tables (P:168 3.2, Fig. 4; Alg. 1 lines   */
+/* 5 and 10): one multinomial draw of a neighbour block per block, */
+/* shared by every proposal of the merge phase / MOVE batch.  The draw for   */
+/* block x uses its own Philox counter (x, TABLE_J | key, itr, outer<<1|ph). */
+/* ------------------------------------------------------------------------ */
+#define ORC_TABLE_J 0x40000000u
+
+static void build_table(OState *st, uint64_t seed, uint32_t j, uint32_t itr, uint32_t outer, uint32_t phase)
+{
+    int32_t x;
+    uint32_t w[4];
+    if (!st->mt) st->mt = (int32_t *)xmalloc(sizeof(int32_t) * (size_t)(st->g.V ? st->g.V : 1));
+    for (x = 0; x < st->B; ++x) {
+        uint64_t d = (uint64_t)deg(&st->bm, x);
+        draws(seed, (uint32_t)x, j, itr, outer, phase, w);
+        st->mt[x] = d ? walk_block(&st->bm, x, pick(w[0], d), -1) : -1;
+    }
+}
+
 static int32_t propose_move(const OState *st, uint64_t seed, uint32_t outer,
                             uint32_t itr, int32_t v)
 {
@@ -318,6 +340,7 @@ static int32_t propose_move(const OState *st, uint64_t seed, uint32_t outer,
     du = (uint64_t)deg(m, u);
     /* x <= B/(B+deg u) -> random block, as an exact integer test (R:Z9) */
     if ((uint64_t)w[1] * (B + du) <= (B << 32)) return (int32_t)pick(w[2], B);
+    if (st->table_mode) return st->mt[u];      /* N4: Alg. 1 line 10 */
     return walk_block(m, u, pick(w[2], du), -1);
 }
 
@@ -330,6 +353,14 @@ static int32_t propose_merge(const OState *st, uint64_t seed, uint32_t outer,
     int32_t u, s;
     draws(seed, (uint32_t)r, j, 0u, outer, 0u, w);
     if (K == 0) goto random;
+    if (st->table_mode) {                      /* N4: Alg. 1 lines 5-10 with the shared table */
+        u = st->mt[r];
+        du = (uint64_t)deg(m, u);
+        if ((uint64_t)w[1] * (B + du) <= (B << 32)) goto random;
+        s = st->mt[u];
+        if (s >= 0 && s != r) return s;
+        goto random;                           /* an outcome equal to r is redrawn (reading N4) */
+    }
     u = walk_block(m, r, pick(w[0], K), -1);
     du = (uint64_t)deg(m, u);
     if ((uint64_t)w[1] * (B + du) <= (B << 32)) goto random;
@@ -622,8 +653,23 @@ void orc_destroy(void *h)
     free(st->g.iptr); free(st->g.isrc); free(st->g.iw);
     free(st->g.kout); free(st->g.kin);
     free(st->b);
+    free(st->mt);
     bm_free(&st->bm);
     free(st);
+}
+
+/* N4 ablation switch: 0 = fresh draws (R:Z6, default), 1 = shared table */
+void orc_set_proposal_mode(void *h, int mode)
+{
+    ((OState *)h)->table_mode = mode == 1;
+}
+
+/* the shared table as the next proposal call would build it (pins) */
+void orc_table(void *h, uint64_t seed, uint32_t j, uint32_t itr, uint32_t outer, uint32_t phase, int32_t *out)
+{
+    OState *st = (OState *)h;
+    build_table(st, seed, j, itr, outer, phase);
+    memcpy(out, st->mt, sizeof(int32_t) * (size_t)st->B);
 }
 
 void orc_set_partition(void *h, const int32_t *b, int32_t B)
@@ -710,6 +756,9 @@ void orc_propose(void *h, int phase, uint64_t seed, uint32_t outer, uint32_t itr
 {
     OState *st = (OState *)h;
     int32_t i, j;
+    if (st->table_mode)   /* N4: the shared table of this MOVE batch (keyed by first) / merge phase */
+        build_table(st, seed, phase == 1 ? (ORC_TABLE_J | ((uint32_t)first & 0x3fffffffu)) : ORC_TABLE_J,
+                    phase == 1 ? itr : 0u, outer, (uint32_t)phase);
 #pragma omp parallel for private(j) schedule(dynamic, 256) num_threads(g_threads) if (g_threads > 1)
     for (i = 0; i < count; ++i) {
         if (phase == 1)

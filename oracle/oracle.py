@@ -82,6 +82,8 @@ def lib():
         L.orc_philox.argtypes = [_u32p, _u32p, _u32p]
         L.orc_set_threads.restype = C.c_int32
         L.orc_set_threads.argtypes = [C.c_int32]
+        L.orc_set_proposal_mode.argtypes = [C.c_void_p, C.c_int]
+        L.orc_table.argtypes = [C.c_void_p, C.c_uint64, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32, _i32p]
         L.orc_create.restype = C.c_void_p
         L.orc_create.argtypes = [C.c_int32, _i64p, _i32p, C.c_void_p]
         L.orc_destroy.argtypes = [C.c_void_p]
@@ -205,6 +207,16 @@ class Oracle:
     # state -----------------------------------------------------------------
     def set_partition(self, b, B):
         lib().orc_set_partition(self.h, np.ascontiguousarray(b, np.int32), int(B))
+
+    def set_proposal_mode(self, mode):
+        """N4 ablation: 0 = fresh Philox draws (default), 1 = the paper's shared lookup table."""
+        lib().orc_set_proposal_mode(self.h, int(mode))
+
+    def table(self, seed, j, itr, outer, phase):
+        """The shared neighbour-block table (N4) for one merge phase / MOVE batch."""
+        out = np.zeros(max(self.B, 1), np.int32)
+        lib().orc_table(self.h, seed, j, itr, outer, phase, out)
+        return out[:self.B]
 
     def set_b_norebuild(self, b, B):
         lib().orc_set_b_norebuild(self.h, np.ascontiguousarray(b, np.int32), int(B))

@@ -289,6 +289,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     GSAP_CUDA(cudaGetDevice(&c.dev));
     comm_init(c, dist);
     REQUIRE(c.prm.sim_ranks >= 0 && c.prm.sim_ranks <= 64, GSAP_EINVAL, "sim_ranks in [0, 64]");
+    REQUIRE(c.prm.proposal_mode == 0 || c.prm.proposal_mode == 1, GSAP_EINVAL, "proposal_mode is 0 or 1");
     if (c.nranks > 1 || c.prm.sim_ranks > 1) c.prm.cuda_graphs = 0;   // the sliced batch path (move_batch)
     mark("streams");
     // host-side static info
@@ -409,6 +410,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.scal = A.take<double>(8);
         c.scal_i = A.take<int>(8);
         c.n_eval = A.take<unsigned long long>(1);
+        if (c.prm.proposal_mode == 1) c.mt = A.take<int>(Vs);
         if (c.prm.incremental) {
             c.oldb = A.take<int>(Vs);
             c.moved = A.take<int>(Vs);
@@ -525,6 +527,7 @@ static void merge_phase(Ctx &c, uint32_t outer, int K, int *best_out, double *dS
     REQUIRE(K >= 0 && K <= c.B / 2, GSAP_EINVAL, "K must be in [0, B/2]");
     const int B = c.B;
     const int G = ranks_of(c);
+    launch_fill_mt(c, TABLE_J, 0, outer, 0);   // N4 ablation only
     if (G == 1) {
         launch_merge_props(c, outer, 0, B, true, nullptr, nullptr, c.best, c.dSbest);
         c.st.n_merge_prop += (long long)B * c.prm.num_proposals;
@@ -564,6 +567,7 @@ static void move_batch(Ctx &c, uint32_t outer, uint32_t itr, int first, int coun
     c.batch_count = count;
     const int G = ranks_of(c);
     announce_batch(c, first, count);
+    launch_fill_mt(c, TABLE_J | ((uint32_t)first & 0x3fffffffu), itr, outer, 1);   // N4 ablation only
     if (G == 1) {
         launch_move(c, MOVE_FUSED, outer, itr, first, count, c.s, c.dS, nullptr, c.acc);
         launch_apply(c, first, count, c.s, c.acc, c.dS, dsum, c.scal_i + 1, c.n_eval);
@@ -636,6 +640,7 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh, std::vector<d
             if (first >= last) continue;
             c.batch_count = last - first;
             announce_batch(c, first, last - first);
+            launch_fill_mt(c, TABLE_J | ((uint32_t)first & 0x3fffffffu), 0, outer, 1, c.d_itr);   // N4 only
             launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
             launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
             rebuild(c);
@@ -750,6 +755,7 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::ve
                 if (first >= last) continue;
                 c.batch_count = last - first;
             announce_batch(c, first, last - first);
+            launch_fill_mt(c, TABLE_J | ((uint32_t)first & 0x3fffffffu), 0, outer, 1, c.d_itr);   // N4 only
             launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
                 launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
                 rebuild(c);
@@ -1031,6 +1037,7 @@ void gsap_default_params(gsap_params *p) {
     p->move_sorted = 1;
     p->sim_ranks = 0;
     p->incremental = 1;
+    p->proposal_mode = 0;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }
@@ -1100,10 +1107,12 @@ gsap_status gsap_propose(gsap_ctx *ctx, gsap_phase phase, uint32_t outer, uint32
     REQUIRE(first >= 0 && count >= 0 && (long long)first + count <= n, GSAP_EINVAL, "range out of bounds");
     if (count == 0) return GSAP_OK;
     if (phase == GSAP_MOVE) {
+        launch_fill_mt(c, TABLE_J | ((uint32_t)first & 0x3fffffffu), itr, outer, 1);   // N4: table keyed by `first`
         launch_move(c, MOVE_PROPOSE, outer, itr, first, count, c.s, nullptr, nullptr, nullptr);
         copy_out(c, s_out, c.s, sizeof(int) * (size_t)count);
     } else {
         REQUIRE(c.B >= 2, GSAP_ESTATE, "merge proposals need B >= 2");
+        launch_fill_mt(c, TABLE_J, 0, outer, 0);   // N4
         launch_merge_props(c, outer, first, count, true, c.s, nullptr, nullptr, nullptr);
         copy_out(c, s_out, c.s, sizeof(int) * (size_t)count * c.prm.num_proposals);
     }

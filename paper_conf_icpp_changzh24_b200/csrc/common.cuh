@@ -152,7 +152,15 @@ struct BM {
     const int *__restrict__ ccum;
     const int *__restrict__ dout;
     const int *__restrict__ din;
+    // N4 ablation (params.proposal_mode = 1, Alg. 1 P:180-200 with the
+    // lookup tables of P:168 Fig. 4): one weighted neighbour block per block,
+    // shared by every proposal of the phase / batch; nullptr otherwise
+    const int *__restrict__ mt;
 };
+
+// the table's key: j word of the Philox counter of block x's table draw
+// (MERGE: one table per merge phase; MOVE: one per batch, keyed by its first vertex)
+constexpr uint32_t TABLE_J = 0x40000000u;
 
 // first index i in [lo, hi) with a[i] > p (upper bound); hi if none
 GSAP_DEV int upper_bound(const int *__restrict__ a, int lo, int hi, long long p) {

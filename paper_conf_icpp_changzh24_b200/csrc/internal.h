@@ -71,6 +71,7 @@ struct Ctx {
     int *dense = nullptr, *denseT = nullptr;
     double2 *ft = nullptr;         // f-table {hi, lo} (FT_N entries)
     double *rcp = nullptr;         // 1 / (d_x + B), refreshed by every rebuild
+    int *mt = nullptr;             // N4: the shared multinomial table (one neighbour block per block)
     size_t dense_cap = 0;   // elements
     bool dense_mode = false;
     int dense_B = -1;       // B of the dense M / Mt the last rebuild left (-1: none)
@@ -158,6 +159,7 @@ struct Ctx {
         m.rowend = padded ? bm_rowend : bm_rowptr + 1;
         m.colend = padded ? bm_colend : bm_colptr + 1;
         m.dout = dout; m.din = din;
+        m.mt = prm.proposal_mode == 1 ? mt : nullptr;
         return m;
     }
 };
@@ -220,6 +222,11 @@ void comm_unique_id(uint8_t out[128]);
 // the slice of [0, n) that rank g of G owns: whole chunks of `chunk`, contiguous,
 // ceil(ceil(n/chunk)/G) chunks per rank (the last ranks may own less or none)
 void shard_slice(int n, int chunk, int G, int g, int *first, int *count, int *per_rank);
+
+// N4 ablation: fill the shared neighbour-block table for a merge phase
+// (phase 0, j = TABLE_J) or a MOVE batch (phase 1, j = TABLE_J | first)
+void launch_fill_mt(Ctx &c, uint32_t j, uint32_t itr, uint32_t outer, uint32_t phase,
+                    const unsigned *d_itr = nullptr);
 
 // merge.cu
 void launch_merge_props(Ctx &c, uint32_t outer, int first, int count, bool propose, int *s,

@@ -31,6 +31,18 @@ GSAP_DEV int propose_merge(const BM &m, int r, uint32_t j, uint64_t seed, uint32
     const uint32_t B = (uint32_t)m.B;
     const uint4 w = draws(seed, (uint32_t)r, j, 0u, outer, 0u);
     const uint32_t K = (uint32_t)bm_deg(m, r);
+    if (m.mt) {   // N4, Alg. 1 lines 2-10 with the shared table; an s = r outcome is redrawn
+        if (K > 0) {
+            const int u = __ldg(m.mt + r);
+            if (!coin_random(w.y, B, (uint32_t)bm_deg(m, u))) {
+                const int s = __ldg(m.mt + u);
+                if (s >= 0 && s != r) return s;
+            }
+        }
+        int s = (int)pick(w.z, B - 1);
+        if (s >= r) ++s;
+        return s;
+    }
     if (K > 0) {
         const int u = bm_walk(m, r, (long long)pick(w.x, K), -1);
         const uint32_t du = (uint32_t)bm_deg(m, u);
@@ -123,6 +135,28 @@ __global__ void __launch_bounds__(MERGE_WARPS * 32) k_merge(MergeArgs a) {
             if (a.dSbest) a.dSbest[i] = bd;
         }
     }
+}
+
+// N4: block x's table entry = a weighted neighbour block of x (the walk of
+// R:O.4 with its own Philox draw), -1 for a block without edges
+__global__ void k_fill_mt(BM m, uint64_t seed, uint32_t j, uint32_t itr, const unsigned *itr_ptr, uint32_t outer,
+                          uint32_t phase, int *__restrict__ mt) {
+    const uint32_t it = itr_ptr ? __ldg(itr_ptr) : itr;
+    for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < m.B; x += gridDim.x * blockDim.x) {
+        const uint32_t d = (uint32_t)bm_deg(m, x);
+        const uint4 w = draws(seed, (uint32_t)x, j, it, outer, phase);
+        mt[x] = d ? bm_walk(m, x, (long long)pick(w.x, d), -1) : -1;
+    }
+}
+
+void launch_fill_mt(Ctx &c, uint32_t j, uint32_t itr, uint32_t outer, uint32_t phase, const unsigned *d_itr) {
+    if (c.prm.proposal_mode != 1) return;
+    BM m = c.bm();
+    m.mt = nullptr;
+    const int g = (int)std::min<long long>(((long long)c.B + 255) / 256, 148LL * 8);
+    k_fill_mt<<<std::max(g, 1), 256, 0, c.stream>>>(m, c.prm.seed, j, itr, d_itr, outer, phase, c.mt);
+    ++c.launches;
+    GSAP_CHECK_LAUNCH();
 }
 
 void launch_merge_props(Ctx &c, uint32_t outer, int first, int count, bool propose, int *s, double *dS,

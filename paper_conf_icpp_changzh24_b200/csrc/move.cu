@@ -367,6 +367,7 @@ GSAP_DEV int propose_move_thread(const MoveArgs &a, int v, uint4 w) {
     const int u = __ldg(a.b + n);
     const uint32_t du = (uint32_t)bm_deg(a.m, u);
     if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
+    if (a.m.mt) return __ldg(a.m.mt + u);   // N4: the shared table entry of u (Alg. 1 line 10)
     return bm_walk(a.m, u, (long long)pick(w.z, du), -1);
 }
 
@@ -386,6 +387,7 @@ GSAP_DEV int propose_warp(const MoveArgs &a, int v, uint4 w, int deg, const int 
     const int u = __shfl_sync(FULL, x, (int)(p & 31u));
     const uint32_t du = (uint32_t)bm_deg(a.m, u);
     if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
+    if (a.m.mt) return __ldg(a.m.mt + u);   // N4
     return bm_walk_warp(a.m, u, (long long)pick(w.z, du));
 }
 
@@ -503,6 +505,8 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
         const uint32_t du = (uint32_t)(dout_u + din_u);
         if (coin_random(w.y, (uint32_t)B, du)) {
             s = (int)pick(w.z, (uint32_t)B);
+        } else if (a.m.mt) {
+            s = __ldg(a.m.mt + u);   // N4: the shared table entry of u (Alg. 1 line 10)
         } else {
             const long long q = (long long)pick(w.z, du);
             if (q < dout_u) s = __ldg(a.m.col + warp_upper_bound(a.m.cum, rlo, rhi, q));
@@ -973,6 +977,7 @@ GSAP_DEV int propose_vertex_warp(const MoveArgs &a, int v, uint4 w, int ro, int 
     const int u = __ldg(a.b + n);
     const uint32_t du = (uint32_t)bm_deg(a.m, u);
     if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
+    if (a.m.mt) return __ldg(a.m.mt + u);   // N4
     return bm_walk_warp(a.m, u, (long long)pick(w.z, du));
 }
 

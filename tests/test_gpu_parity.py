@@ -651,3 +651,59 @@ def test_incremental_update_bit_identical(G, oracle_mod, gname, regime):
         orc.apply_moves(first, count, s, acc)
         orc.rebuild()
         assert_same_blockmodel(ctx, orc)
+
+
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sorted"])
+@pytest.mark.parametrize("gname", ["multi_w", "dcsbm1k"])
+def test_table_mode_proposals_and_batches(G, oracle_mod, gname, regime):
+    """N4 ablation (proposal_mode = 1, the paper's shared lookup tables): MOVE
+    and MERGE proposals bit-exact vs the oracle's table mode, and fused MOVE
+    batches in lockstep (the table drawn inside the batch, keyed by its first
+    vertex)."""
+    rowptr, col, w = GRAPHS[gname]()
+    V = len(rowptr) - 1
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, w, proposal_mode=1, **REGIMES[regime])
+    orc.set_proposal_mode(1)
+    for B, b in _states(V, 21):
+        if B < 2:
+            continue
+        set_both(ctx, orc, b, B)
+        for outer, itr, first in ((0, 0, 0), (3, 5, 75)):
+            count = V - first
+            s = ctx.gsap_propose(G.GSAP_MOVE, outer, itr, first, count)
+            assert np.array_equal(s, orc.propose(1, SEED, outer, itr, first, count)), (B, outer)
+            sm = ctx.gsap_propose(G.GSAP_MERGE, outer, 0, 0, B)
+            assert np.array_equal(sm, orc.propose(0, SEED, outer, 0, 0, B)), (B, outer)
+    b0 = dcsbm.random_partition(V, 40, 8)
+    set_both(ctx, orc, b0, 40)
+    bs = (V + 3) // 4
+    for k in range(4):
+        first, count = k * bs, min(V, (k + 1) * bs) - k * bs
+        s_o = orc.propose(1, SEED, 2, 1, first, count)
+        dS_o, H_o, p_o, acc_o = orc.delta_move(SEED, 2, 1, first, count, s_o)
+        s, dS, acc, _ = ctx.gsap_move_batch(2, 1, first, count)
+        assert np.array_equal(s, s_o)
+        assert np.all(close(dS, dS_o))
+        t = ties(oracle_mod, SEED, 2, 1, range(first, first + count), p_o)
+        assert np.array_equal(acc[~t], acc_o[~t])
+        orc.apply_moves(first, count, s, acc)
+        orc.rebuild()
+        assert_same_blockmodel(ctx, orc)
+
+
+def test_table_mode_end_to_end_1k(G, oracle_mod):
+    """N4 end to end at 1K: layer 3 against the oracle's table-mode run, the
+    driver replay, and one-GPU invariance of the sliced path (sim_ranks)."""
+    from gen import metrics
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, proposal_mode=1)
+    orc.set_proposal_mode(1)
+    res = ctx.gsap_run()
+    ref = orc.partition_run()
+    assert abs(res["mdl"] - ref["mdl"]) <= 0.01 * ref["mdl"]
+    pg, rg = metrics.pairwise_precision_recall(truth, res["b"])
+    po, ro = metrics.pairwise_precision_recall(truth, ref["b"])
+    assert abs(pg - po) <= 0.02 and abs(rg - ro) <= 0.02
+    assert_driver_replay(oracle_mod, res, cfg.V)
+    r2 = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED, proposal_mode=1, sim_ranks=4)).gsap_run()
+    assert r2["B"] == res["B"] and r2["mdl"] == res["mdl"] and np.array_equal(r2["b"], res["b"])
