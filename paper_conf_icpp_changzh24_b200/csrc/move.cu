@@ -719,7 +719,10 @@ GSAP_DEV void bucket_get(const Line (&L)[N], const int (&y)[N], int (&p)[N], int
     }
 }
 
-constexpr int HALF_K = 4;   // splitters per lane in the sorted two-pass kernels
+#ifndef GSAP_HALF_K
+#define GSAP_HALF_K 4
+#endif
+constexpr int HALF_K = GSAP_HALF_K;   // splitters per lane in the sorted two-pass kernels
 
 template <bool WEIGHTED, int PASS>
 GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {

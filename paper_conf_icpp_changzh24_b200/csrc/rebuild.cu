@@ -349,6 +349,7 @@ struct DenseArgs {
     double *rcp;
     int *d_nnz;
     unsigned *bar;
+    const int *skip;   // N2: the batch's moved-vertex count (nullable); 0 = the blockmodel is unchanged
 };
 
 // exclusive scan of in[0, n) into out[0, n], out[n] = total, by one CTA of DC_THREADS
@@ -387,6 +388,7 @@ GSAP_DEV void dc_cta_scan(const int *in, int *out, int n, int *sh) {
 
 template <bool SMEM>
 __global__ void __launch_bounds__(DC_THREADS) k_rebuild_dense(DenseArgs a) {
+    if (a.skip && *a.skip == 0) return;   // every CTA returns before any grid barrier
     extern __shared__ int h[];
     const int B = a.B, E = a.E;
     const size_t BB = (size_t)B * B;
@@ -591,8 +593,9 @@ __global__ void __launch_bounds__(DC_THREADS) k_rebuild_dense(DenseArgs a) {
 }
 
 template <bool SMEM>
-static void launch_rebuild_dense_coop(Ctx &c) {
+static void launch_rebuild_dense_coop(Ctx &c, const int *skip = nullptr) {
     DenseArgs a;
+    a.skip = skip;
     a.E = c.E;
     a.B = c.B;
     a.esrc = c.esrc; a.col = c.col; a.wgt = c.wgt; a.b = c.b;
@@ -864,7 +867,11 @@ void rebuild(Ctx &c) {
     const bool was_dense = c.dense_mode && c.dense_B == c.B;
     c.dense_mode = dense_ok(c, c.B);
     c.padded = false;   // set by the multi-kernel sparse path
-    if (c.delta.pending && was_dense && c.dense_mode && c.E > 0) {
+    if (c.delta.pending && was_dense && c.dense_mode && c.E > 0 && c.prm.dense_coop && c.B <= SMALL_MAX_B) {
+        // N2 at small B: the persistent rebuild (one launch, measured faster than
+        // the delta + compaction here), skipped when the batch moved nothing
+        launch_rebuild_dense_coop<true>(c, c.moved_cnt);
+    } else if (c.delta.pending && was_dense && c.dense_mode && c.E > 0) {
         rebuild_dense_delta(c);   // N2: M, Mt of the previous rebuild + the batch's moves
     } else if (c.dense_mode && c.prm.dense_coop && c.E > 0 && c.B <= SMALL_MAX_B) {
         launch_rebuild_dense_coop<true>(c);

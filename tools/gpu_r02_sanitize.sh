@@ -1,0 +1,11 @@
+#!/bin/bash
+# compute-sanitizer over tools/sanitize_run.py (every kernel family), logs into gpurun_out/
+mkdir -p gpurun_out
+CS=/usr/local/cuda/bin/compute-sanitizer
+for tool in memcheck synccheck racecheck initcheck; do
+  extra=""
+  [ $tool = racecheck ] && extra="--racecheck-report all"
+  timeout 1500 $CS --tool $tool $extra --print-limit 50 python tools/sanitize_run.py > gpurun_out/sanitizer_$tool.txt 2>&1
+  echo "exit=$?" >> gpurun_out/sanitizer_$tool.txt
+  tail -4 gpurun_out/sanitizer_$tool.txt
+done
