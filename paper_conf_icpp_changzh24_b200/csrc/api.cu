@@ -288,6 +288,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_join, cudaEventDisableTiming));
     GSAP_CUDA(cudaGetDevice(&c.dev));
     comm_init(c, dist);
+    if (const char *tg = getenv("GSAP_TEST_GRID")) c.test_grid = std::max(0, atoi(tg));
     REQUIRE(c.prm.sim_ranks >= 0 && c.prm.sim_ranks <= 64, GSAP_EINVAL, "sim_ranks in [0, 64]");
     REQUIRE(c.prm.proposal_mode == 0 || c.prm.proposal_mode == 1, GSAP_EINVAL, "proposal_mode is 0 or 1");
     if (c.nranks > 1 || c.prm.sim_ranks > 1) c.prm.cuda_graphs = 0;   // the sliced batch path (move_batch)

@@ -127,6 +127,7 @@ struct Ctx {
     int nranks = 1, rank = 0;
     void *nccl_comm = nullptr;
     int batch_count = 0;           // the MOVE batch a launch belongs to (mode decisions per batch, not slice)
+    int test_grid = 0;             // tests (env GSAP_TEST_GRID at create): cap of the move kernels' grids
 
     // N2 incremental update (dense regime): the batch a pending rebuild follows;
     // the apply logs moved vertices and their old blocks, the rebuild applies dM

@@ -716,3 +716,27 @@ def test_table_mode_end_to_end_1k(G, oracle_mod):
     po, ro = metrics.pairwise_precision_recall(truth, ref["b"])
     assert abs(pg - po) <= 0.02 and abs(rg - ro) <= 0.02
     assert abs(res["mdl"] - ref["mdl"]) <= 0.01 * ref["mdl"]
+
+
+@pytest.mark.parametrize("regime", ["auto", "sparse", "sorted"])
+def test_move_results_independent_of_launch_shape(G, oracle_mod, regime, monkeypatch):
+    """move.cu's claim: every sum is a fixed tree over a vertex's own entries,
+    so the results do not depend on the grid.  The same fused batches with the
+    move kernels squeezed onto 1 and 3 CTAs (grid-stride over everything; env
+    GSAP_TEST_GRID read at create) give bit-identical s, dS, acc."""
+    rowptr, col, w = _hub_graph(True)
+    V = len(rowptr) - 1
+    b0 = dcsbm.random_partition(V, 700, 3)
+    outs = []
+    for tg in ("0", "1", "3"):
+        monkeypatch.setenv("GSAP_TEST_GRID", tg)
+        ctx = G.Context(rowptr, col, w, params=G.gsap_default_params(seed=SEED, **REGIMES[regime]))
+        ctx.gsap_set_partition(b0, 700)
+        bs = (V + 3) // 4
+        res = []
+        for k in range(4):
+            s, dS, acc, _ = ctx.gsap_move_batch(1, 2, k * bs, min(V, (k + 1) * bs) - k * bs)
+            res.append((s.tobytes(), dS.tobytes(), acc.tobytes()))
+        outs.append(res)
+        ctx.close()
+    assert outs[0] == outs[1] == outs[2]
