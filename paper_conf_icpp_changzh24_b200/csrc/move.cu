@@ -225,37 +225,7 @@ struct MoveCtx {
     long long Mrr, Mrs, Msr, Mss, o_r, i_r, o_s, i_s, kout, kin, l, dr, ds, Mrr2, Mrs2, Msr2, dr2, ds2;
     double Bd;
     Line Rr, Rs, Cr, Cs;
-    const int *spl;   // group path, sparse regime: S splitters of each of the four lines (shared memory)
-    int S;
 };
-
-// M entry of key y in line L with S splitters in shared memory (spl[g] =
-// L.idx[floor(g len / S)]): the bucket by a shared-memory binary search, then
-// <= 8 independent global loads (one memory round instead of a dependent
-// binary search over the whole line); the count only on a hit
-GSAP_DEV int spl_get(const Line &L, const int *spl, int S, int y) {
-    if (L.len == 0 || spl[0] > y) return 0;
-    int g = 0, n = S;
-    while (n > 1) {
-        const int h = n >> 1;
-        g = spl[g + h] <= y ? g + h : g;
-        n -= h;
-    }
-    int p = (int)(((long long)g * L.len) / S);
-    int c = (int)(((long long)(g + 1) * L.len) / S) - p;
-    while (c > 8) {
-        const int h = c >> 1;
-        p = __ldg(L.idx + p + h) <= y ? p + h : p;
-        c -= h;
-    }
-    int id[8];
-#pragma unroll
-    for (int q = 0; q < 8; ++q) id[q] = q < c ? __ldg(L.idx + p + q) : -1;
-    int hit = -1;
-#pragma unroll
-    for (int q = 0; q < 8; ++q) hit = id[q] == y ? q : hit;
-    return hit >= 0 ? __ldg(L.cnt + p + hit) : 0;
-}
 
 // dS / Hastings terms of one unique neighbour block t (out weight ot, in weight it)
 GSAP_DEV void t_terms(const MoveArgs &a, const MoveCtx &q, int t, long long ot, long long it, double &accS,
@@ -276,11 +246,6 @@ GSAP_DEV void t_terms(const MoveArgs &a, const MoveCtx &q, int t, long long ot, 
             Mst = row_at(a.m, q.Rs, q.s, t);
             Mtr = col_at(a.m, q.Cr, q.r, t);
             Mts = col_at(a.m, q.Cs, q.s, t);
-        } else if (q.spl) {
-            Mrt = spl_get(q.Rr, q.spl, q.S, t);
-            Mst = spl_get(q.Rs, q.spl + q.S, q.S, t);
-            Mtr = spl_get(q.Cr, q.spl + 2 * q.S, q.S, t);
-            Mts = spl_get(q.Cs, q.spl + 3 * q.S, q.S, t);
         } else {
             const Line Ln[4] = {q.Rr, q.Rs, q.Cr, q.Cs};
             const int yt[4] = {t, t, t, t};
@@ -324,8 +289,6 @@ GSAP_DEV void move_ctx(const MoveArgs &a, int v, int r, int s, const int4 *tab, 
     q.v = v;
     q.r = r;
     q.s = s;
-    q.spl = nullptr;
-    q.S = 0;
     if (!a.m.dense) {
         q.Rr = row_line(a.m, r);
         q.Rs = row_line(a.m, s);
@@ -663,7 +626,10 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
         const double p = exp(-a.beta * dS) * H;
         acc = ((double)w.w + 0.5) * (1.0 / 4294967296.0) <= p;
     }
-    // leave the table empty: exactly the listed slots were used
+    // leave the table empty: exactly the listed slots were used (after every
+    // lane's last table read: the shuffles above converge the warp but do not
+    // order shared memory, __syncwarp does)
+    __syncwarp();
     for (int k = lane; k < nuniq; k += 32) tab[list[k]] = make_int4(-1, 0, 0, 0x7fffffff);
     __syncwarp();
     if (lane == 0) {
@@ -915,7 +881,10 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
     accS = warp_sum(accS);
     pf = warp_sum(pf);
     if (PASS == 1) pb = warp_sum(pb);
-    // leave the table empty: exactly the listed slots were used
+    // leave the table empty: exactly the listed slots were used (after every
+    // lane's last table read: the shuffles above converge the warp but do not
+    // order shared memory, __syncwarp does)
+    __syncwarp();
     for (int k = lane; k < nuniq; k += 32) tab[list[k]] = make_int4(-1, 0, 0, 0x7fffffff);
     __syncwarp();
     if (lane == 0) {
@@ -963,20 +932,10 @@ GSAP_DEV void group_table(const MoveArgs &a, int v, int ro, int nout, int ci, in
 // first adjacency position; threads sum their owned terms in position order.
 template <int G, bool WEIGHTED>
 GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, int ro, int nout, int ci, int deg,
-                              int4 *tab, int log2cap, double *sh, int *spl, double &dS_out, double &H_out,
-                              bool &acc_out) {
+                              int4 *tab, int log2cap, double *sh, double &dS_out, double &H_out, bool &acc_out) {
     const int gt = threadIdx.x % G;
     MoveCtx q;
     move_ctx(a, v, r, s, tab, log2cap, q);
-    if (!a.m.dense) {   // G splitters of each of the four lines, one load per thread and line
-        const Line L4[4] = {q.Rr, q.Rs, q.Cr, q.Cs};
-#pragma unroll
-        for (int k = 0; k < 4; ++k)
-            spl[k * G + gt] = L4[k].len > 0 ? __ldg(L4[k].idx + (int)(((long long)gt * L4[k].len) / G)) : 0x7fffffff;
-        gsync<G>();
-        q.spl = spl;
-        q.S = G;
-    }
     double accS = 0.0, pf = 0.0, pb = 0.0;
     for (int j = gt; j < deg; j += G) {
         const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
@@ -1038,7 +997,7 @@ GSAP_DEV void tab_clear(int4 *tab, int slots, int gt) {
 
 // outputs of vertex v (index i = v - first) given its proposal s
 template <int G, bool WEIGHTED>
-GSAP_DEV void do_vertex(const MoveArgs &a, int v, int4 *tab, int log2cap, int *list, double *sh, int *spl) {
+GSAP_DEV void do_vertex(const MoveArgs &a, int v, int4 *tab, int log2cap, int *list, double *sh) {
     const int i = v - a.first;
     const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
     const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
@@ -1063,7 +1022,7 @@ GSAP_DEV void do_vertex(const MoveArgs &a, int v, int4 *tab, int log2cap, int *l
     const int s = a.propose ? *sp : a.s_in[i];
     double dS = 0.0, H = 1.0;
     bool acc = false;
-    if (s != r) eval_move_group<G, WEIGHTED>(a, v, r, s, w, ro, nout, ci, deg, tab, log2cap, sh, spl, dS, H, acc);
+    if (s != r) eval_move_group<G, WEIGHTED>(a, v, r, s, w, ro, nout, ci, deg, tab, log2cap, sh, dS, H, acc);
     if ((threadIdx.x & (G - 1)) == 0) {
         if (a.dS) a.dS[i] = dS;
         if (a.H) a.H[i] = H;
@@ -1092,7 +1051,6 @@ template <bool WEIGHTED>
 __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_GROUPS_MINB) k_move_groups(MoveArgs a) {
     __shared__ int4 tabs[CTA_SMEM_SLOTS];
     __shared__ double sh[3 * MOVE_WARPS + 8];   // group sums + the broadcast proposal
-    __shared__ int spl_s[4 * CTA_THREADS];      // line splitters: 4 x 64 per mid group, 4 x 256 per CTA role
     if ((int)blockIdx.x < a.nmid_ctas) {
         // four 64-thread groups per CTA, one mid vertex each
         const int gid = threadIdx.x >> 6, gt = threadIdx.x & 63;
@@ -1100,7 +1058,7 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_GROUPS_MINB) k_move_grou
         for (int li = blockIdx.x * 4 + gid; li < a.mlist_count; li += a.nmid_ctas * 4) {
             tab_clear<64>(tab, MID_TAB, gt);
             gsync<64>();
-            do_vertex<64, WEIGHTED>(a, a.mlist[li], tab, MID_TAB_LOG2, nullptr, sh + gid * 8, spl_s + gid * 256);
+            do_vertex<64, WEIGHTED>(a, a.mlist[li], tab, MID_TAB_LOG2, nullptr, sh + gid * 8);
             gsync<64>();
         }
         return;
@@ -1109,7 +1067,7 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_GROUPS_MINB) k_move_grou
         for (int li = blockIdx.x - a.nmid_ctas; li < a.list_count; li += a.nbig_ctas) {
             tab_clear<CTA_THREADS>(tabs, 1 << a.big_log2, threadIdx.x);
             __syncthreads();
-            do_vertex<CTA_THREADS, WEIGHTED>(a, a.list[li], tabs, a.big_log2, nullptr, sh, spl_s);
+            do_vertex<CTA_THREADS, WEIGHTED>(a, a.list[li], tabs, a.big_log2, nullptr, sh);
             __syncthreads();
         }
         return;
@@ -1120,7 +1078,7 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_GROUPS_MINB) k_move_grou
         for (int li = hb; li < a.hlist_count; li += a.nhuge_ctas) {
             tab_clear<CTA_THREADS>(tab, 1 << a.gtab_log2, threadIdx.x);
             __syncthreads();
-            do_vertex<CTA_THREADS, WEIGHTED>(a, a.hlist[li], tab, a.gtab_log2, nullptr, sh, spl_s);
+            do_vertex<CTA_THREADS, WEIGHTED>(a, a.hlist[li], tab, a.gtab_log2, nullptr, sh);
             __syncthreads();
         }
         }

@@ -5,7 +5,7 @@ CS=/usr/local/cuda/bin/compute-sanitizer
 for tool in memcheck synccheck racecheck initcheck; do
   extra=""
   [ $tool = racecheck ] && extra="--racecheck-report all"
-  timeout 1500 $CS --tool $tool $extra --print-limit 50 python tools/sanitize_run.py > gpurun_out/sanitizer_$tool.txt 2>&1
+  timeout 1500 $CS --tool $tool $extra --print-limit 400 python tools/sanitize_run.py > gpurun_out/sanitizer_$tool.txt 2>&1
   echo "exit=$?" >> gpurun_out/sanitizer_$tool.txt
   tail -4 gpurun_out/sanitizer_$tool.txt
 done
