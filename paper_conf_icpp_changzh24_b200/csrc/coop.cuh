@@ -108,6 +108,7 @@ union CoopSmem {
     struct {
         K keys[SEG_WARPS][SEG_WARP_MAX];
         int hp[SEG_WARPS][SEG_WARP_MAX];
+        unsigned cntp[SEG_WARPS][8 * 32];
     } warp;
     struct {
         K keys[2][SegCta<K>::CAP];
@@ -234,7 +235,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
                 K *ka = S.warp.keys[wl], *kb = reinterpret_cast<K *>(S.warp.hp[wl]);
                 for (int i = lane; i < L; i += 32) ka[i] = seg[o + i];
                 __syncwarp();
-                K *keys = warp_radix_sort<K>(ka, kb, L, a.col_bits);
+                K *keys = cta_radix_sort<K, 32>(ka, kb, L, a.col_bits, S.warp.cntp[wl], nullptr);
                 int *hw = reinterpret_cast<int *>(keys == ka ? kb : ka);
                 u = rle_runs<K, 32>(keys, L, hw, sd.tcol + o, sd.tcnt + o, lane, nullptr);
             } else {

@@ -384,93 +384,20 @@ GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict_
 //   MODE 0: <= 128 entries, bitonic + RLE in registers;
 //   MODE 1: 129..256 entries in registers (8 per lane);
 //   MODE 2: 257..SEG_WARP_MAX_MK entries: the stable LSD radix sort over the
-//           key's block bits (warp_radix_sort: 4-bit digits, register-packed
-//           per-lane counters, no atomics; O(L) per pass instead of bitonic's
-//           O(L log^2 L)) in dynamic shared memory, then RLE.
+//           key's block bits (cta_radix_sort with 32 threads: 4-bit digits,
+//           per-lane packed counters, no atomics; O(L) per pass instead of
+//           bitonic's O(L log^2 L)) in dynamic shared memory, then RLE.
 #ifndef GSAP_SEG_WARP_MAX_MK
 #define GSAP_SEG_WARP_MAX_MK 1024
 #endif
 constexpr int SEG_WARP_MAX_MK = GSAP_SEG_WARP_MAX_MK;   // multi-kernel path: longer lines go to the CTA sorts
 template <typename K>
 constexpr size_t seg_warp2_smem() {
-    return (size_t)SEG_WARPS * 2 * SEG_WARP_MAX_MK * sizeof(K);
+    return (size_t)SEG_WARPS * (2 * SEG_WARP_MAX_MK * sizeof(K) + 8 * 32 * sizeof(unsigned));
 }
 
-// stable LSD radix sort of a[0, L) (L < 2048) by one warp over the key's block
-// bits (4-bit digits), ping-ponging with b; returns the buffer holding the
-// result.  Lane l owns the contiguous chunk [l C, l C + C) (C odd: no bank
-// conflicts on the chunk reads); its 16 digit counters live in REGISTERS,
-// packed 11 bits each, four digits per 64-bit word -- the count and scatter
-// loops have no shared-memory read-modify-write chain, only independent key
-// loads and stores; the per-digit lane prefix is a shuffle scan of the packed
-// words (fields never carry: every count is <= L < 2048).
-GSAP_DEV unsigned long long pk_sel(int w, unsigned long long w0, unsigned long long w1, unsigned long long w2,
-                                   unsigned long long w3) {
-    return w == 0 ? w0 : w == 1 ? w1 : w == 2 ? w2 : w3;
-}
-
-template <typename K>
-GSAP_DEV K *warp_radix_sort(K *a, K *b, int L, int col_bits) {
-    const int lane = threadIdx.x & 31;
-    const int C = ((L + 31) >> 5) | 1;
-    const int lo = min(L, lane * C), hi = min(L, lo + C);
-    for (int sh = 0; sh < col_bits; sh += 4) {
-        unsigned long long c0 = 0, c1 = 0, c2 = 0, c3 = 0;   // own counts, digit d at word d/4, bits 11 (d%4)
-        for (int i = lo; i < hi; ++i) {
-            const int d = (key_col(a[i]) >> sh) & 15;
-            const unsigned long long inc = 1ull << (11 * (d & 3));
-            const int w = d >> 2;
-            c0 += w == 0 ? inc : 0ull;
-            c1 += w == 1 ? inc : 0ull;
-            c2 += w == 2 ? inc : 0ull;
-            c3 += w == 3 ? inc : 0ull;
-        }
-        unsigned long long x0 = c0, x1 = c1, x2 = c2, x3 = c3;   // inclusive lane prefix (packed)
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const unsigned long long t0 = __shfl_up_sync(FULL, x0, o), t1 = __shfl_up_sync(FULL, x1, o);
-            const unsigned long long t2 = __shfl_up_sync(FULL, x2, o), t3 = __shfl_up_sync(FULL, x3, o);
-            if (lane >= o) {
-                x0 += t0;
-                x1 += t1;
-                x2 += t2;
-                x3 += t3;
-            }
-        }
-        const unsigned long long T0 = __shfl_sync(FULL, x0, 31), T1 = __shfl_sync(FULL, x1, 31);
-        const unsigned long long T2 = __shfl_sync(FULL, x2, 31), T3 = __shfl_sync(FULL, x3, 31);
-        // digit bases (exclusive scan over the 16 totals), packed like the counters
-        unsigned long long b0 = 0, b1 = 0, b2 = 0, b3 = 0, run = 0;
-#pragma unroll
-        for (int d = 0; d < 16; ++d) {
-            const unsigned long long Td = (pk_sel(d >> 2, T0, T1, T2, T3) >> (11 * (d & 3))) & 0x7ffull;
-            const unsigned long long f = run << (11 * (d & 3));
-            if ((d >> 2) == 0) b0 |= f;
-            else if ((d >> 2) == 1) b1 |= f;
-            else if ((d >> 2) == 2) b2 |= f;
-            else b3 |= f;
-            run += Td;
-        }
-        // this lane's first slot per digit: base + exclusive lane prefix
-        unsigned long long o0 = b0 + x0 - c0, o1 = b1 + x1 - c1, o2 = b2 + x2 - c2, o3 = b3 + x3 - c3;
-        for (int i = lo; i < hi; ++i) {
-            const K key = a[i];
-            const int d = (key_col(key) >> sh) & 15;
-            const int s11 = 11 * (d & 3), w = d >> 2;
-            b[(int)((pk_sel(w, o0, o1, o2, o3) >> s11) & 0x7ffull)] = key;
-            const unsigned long long inc = 1ull << s11;
-            o0 += w == 0 ? inc : 0ull;
-            o1 += w == 1 ? inc : 0ull;
-            o2 += w == 2 ? inc : 0ull;
-            o3 += w == 3 ? inc : 0ull;
-        }
-        __syncwarp();
-        K *t = a;
-        a = b;
-        b = t;
-    }
-    return a;
-}
+template <typename K, int NT>
+GSAP_DEV K *cta_radix_sort(K *a, K *b, int L, int col_bits, unsigned *cntp, unsigned *wsum);
 
 template <typename K, int MODE>
 __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const int *__restrict__ off, K *__restrict__ seg,
@@ -494,9 +421,11 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const in
         } else {
             K *ka = reinterpret_cast<K *>(seg_dyn) + (size_t)w * 2 * SEG_WARP_MAX_MK;
             K *kb = ka + SEG_WARP_MAX_MK;
+            unsigned *cntp = reinterpret_cast<unsigned *>(reinterpret_cast<K *>(seg_dyn) +
+                                                          (size_t)SEG_WARPS * 2 * SEG_WARP_MAX_MK) + w * 8 * 32;
             for (int i = lane; i < L; i += 32) ka[i] = seg[o + i];
             __syncwarp();
-            K *keys = warp_radix_sort<K>(ka, kb, L, col_bits);
+            K *keys = cta_radix_sort<K, 32>(ka, kb, L, col_bits, cntp, nullptr);
             int *hw = reinterpret_cast<int *>(keys == ka ? kb : ka);
             u = rle_runs<K, 32>(keys, L, hw, tcol + o, tcnt + o, lane, nullptr);
         }
