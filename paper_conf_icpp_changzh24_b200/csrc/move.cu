@@ -263,6 +263,65 @@ GSAP_DEV void t_terms(const MoveArgs &a, const MoveCtx &q, int t, long long ot, 
     }
 }
 
+// the generic (t not in {r, s}) terms of up to GB unique blocks of one group
+// thread, their 4 GB sparse lookups interleaved level by level (one dependent
+// chain of ~log2(line) loads for all of them instead of one per block); the
+// terms are accumulated in the blocks' order (the same sums as one by one)
+constexpr int GB = 4;
+GSAP_DEV void t_terms_batch(const MoveArgs &a, const MoveCtx &q, int n, const int (&bt)[GB], const int (&bo)[GB],
+                            const int (&bi)[GB], double &accS, double &pf, double &pb) {
+    if (n == 0) return;
+    const Line L4[4] = {q.Rr, q.Rs, q.Cr, q.Cs};
+    int p[4][GB], m[4][GB];
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int k = 0; k < GB; ++k) {
+            p[x][k] = 0;
+            m[x][k] = k < n ? L4[x].len : 0;
+        }
+    bool open = true;
+    while (open) {   // every (line, block) search advances one level per round
+        open = false;
+#pragma unroll
+        for (int x = 0; x < 4; ++x)
+#pragma unroll
+            for (int k = 0; k < GB; ++k) {
+                if (m[x][k] > 1) {
+                    const int h = m[x][k] >> 1;
+                    p[x][k] = __ldg(L4[x].idx + p[x][k] + h) <= bt[k] ? p[x][k] + h : p[x][k];
+                    m[x][k] -= h;
+                    open = open || m[x][k] > 1;
+                }
+            }
+    }
+    int o[4][GB];
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int k = 0; k < GB; ++k) {
+            int v = 0;
+            if (m[x][k] > 0) {
+                const int id = __ldg(L4[x].idx + p[x][k]), cn = __ldg(L4[x].cnt + p[x][k]);
+                v = id == bt[k] ? cn : 0;
+            }
+            o[x][k] = v;
+        }
+    const double2 *__restrict__ ft = a.m.ft;
+    const double *__restrict__ rcp = a.m.rcp;
+#pragma unroll
+    for (int k = 0; k < GB; ++k) {
+        if (k < n) {
+            const long long Mrt = o[0][k], Mst = o[1][k], Mtr = o[2][k], Mts = o[3][k];
+            const long long ot = bo[k], it = bi[k];
+            const double c = (double)(ot + it), rt = __ldg(rcp + bt[k]);
+            accS -= df_t(ft, Mrt, -ot) + df_t(ft, Mst, ot) + df_t(ft, Mtr, -it) + df_t(ft, Mts, it);
+            pf += c * (double)(Mts + Mst + 1) * rt;
+            pb += c * (double)(Mtr - it + Mrt - ot + 1) * rt;
+        }
+    }
+}
+
 // the 2x2 core, the four degree terms and the two self-loop terms: term k of 10
 GSAP_DEV void core_term(const MoveArgs &a, const MoveCtx &q, int k, double &accS, double &pf, double &pb) {
     const double2 *__restrict__ ft = a.m.ft;
@@ -937,13 +996,31 @@ GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, i
     MoveCtx q;
     move_ctx(a, v, r, s, tab, log2cap, q);
     double accS = 0.0, pf = 0.0, pb = 0.0;
+    int bt[GB], bo[GB], bi[GB], nbuf = 0;   // sparse regime: generic blocks batched GB at a time
     for (int j = gt; j < deg; j += G) {
         const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
         if (nb == v) continue;
         const int4 e = tab[tab_find(tab, log2cap, __ldg(a.b + nb))];
         if (e.w != j) continue;
-        t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
+        if (a.m.dense || e.x == q.r || e.x == q.s) {
+            t_terms_batch(a, q, nbuf, bt, bo, bi, accS, pf, pb);   // keep the accumulation order
+            nbuf = 0;
+            t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
+        } else {
+#pragma unroll
+            for (int k = 0; k < GB; ++k)   // register slots (no dynamic indexing)
+                if (k == nbuf) {
+                    bt[k] = e.x;
+                    bo[k] = e.y;
+                    bi[k] = e.z;
+                }
+            if (++nbuf == GB) {
+                t_terms_batch(a, q, nbuf, bt, bo, bi, accS, pf, pb);
+                nbuf = 0;
+            }
+        }
     }
+    t_terms_batch(a, q, nbuf, bt, bo, bi, accS, pf, pb);
     if (gt < 10) core_term(a, q, gt, accS, pf, pb);
     group_sum3<G>(accS, pf, pb, sh);
     mh_decide(a, q, w, accS, pf, pb, dS_out, H_out, acc_out);
