@@ -318,9 +318,6 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         } else if (k > 128) {    // move.cu BIG_THR
             c.h_mid.push_back(v);
         }
-        if (k > 128 && k <= 1024) {
-            c.h_midbig.push_back(v);
-        }
     }
     // allocation: one device arena (one cudaMalloc / cudaFree per context),
     // planned in a measuring pass and then carved ---------------------------
@@ -345,7 +342,6 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.selfw = A.take<int>(Vs);
         if (!c.h_big.empty()) c.big = A.take<int>(c.h_big.size());
         if (!c.h_mid.empty()) c.mid = A.take<int>(c.h_mid.size());
-        if (!c.h_midbig.empty()) c.midbig = A.take<int>(c.h_midbig.size());
         if (!c.h_huge.empty()) {
             c.huge = A.take<int>(c.h_huge.size());
             const int log2cap = std::max(log2_ceil_h(2LL * std::min(kmax_big, V)), 5);
@@ -508,9 +504,6 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     if (!c.h_big.empty())
         GSAP_CUDA(cudaMemcpyAsync(c.big, c.h_big.data(), sizeof(int) * c.h_big.size(), cudaMemcpyHostToDevice,
                                   c.stream));
-    if (!c.h_midbig.empty())
-        GSAP_CUDA(cudaMemcpyAsync(c.midbig, c.h_midbig.data(), sizeof(int) * c.h_midbig.size(),
-                                  cudaMemcpyHostToDevice, c.stream));
     if (!c.h_mid.empty())
         GSAP_CUDA(cudaMemcpyAsync(c.mid, c.h_mid.data(), sizeof(int) * c.h_mid.size(), cudaMemcpyHostToDevice,
                                   c.stream));

@@ -263,65 +263,6 @@ GSAP_DEV void t_terms(const MoveArgs &a, const MoveCtx &q, int t, long long ot, 
     }
 }
 
-// the generic (t not in {r, s}) terms of up to GB unique blocks of one group
-// thread, their 4 GB sparse lookups interleaved level by level (one dependent
-// chain of ~log2(line) loads for all of them instead of one per block); the
-// terms are accumulated in the blocks' order (the same sums as one by one)
-constexpr int GB = 4;
-GSAP_DEV void t_terms_batch(const MoveArgs &a, const MoveCtx &q, int n, const int (&bt)[GB], const int (&bo)[GB],
-                            const int (&bi)[GB], double &accS, double &pf, double &pb) {
-    if (n == 0) return;
-    const Line L4[4] = {q.Rr, q.Rs, q.Cr, q.Cs};
-    int p[4][GB], m[4][GB];
-#pragma unroll
-    for (int x = 0; x < 4; ++x)
-#pragma unroll
-        for (int k = 0; k < GB; ++k) {
-            p[x][k] = 0;
-            m[x][k] = k < n ? L4[x].len : 0;
-        }
-    bool open = true;
-    while (open) {   // every (line, block) search advances one level per round
-        open = false;
-#pragma unroll
-        for (int x = 0; x < 4; ++x)
-#pragma unroll
-            for (int k = 0; k < GB; ++k) {
-                if (m[x][k] > 1) {
-                    const int h = m[x][k] >> 1;
-                    p[x][k] = __ldg(L4[x].idx + p[x][k] + h) <= bt[k] ? p[x][k] + h : p[x][k];
-                    m[x][k] -= h;
-                    open = open || m[x][k] > 1;
-                }
-            }
-    }
-    int o[4][GB];
-#pragma unroll
-    for (int x = 0; x < 4; ++x)
-#pragma unroll
-        for (int k = 0; k < GB; ++k) {
-            int v = 0;
-            if (m[x][k] > 0) {
-                const int id = __ldg(L4[x].idx + p[x][k]), cn = __ldg(L4[x].cnt + p[x][k]);
-                v = id == bt[k] ? cn : 0;
-            }
-            o[x][k] = v;
-        }
-    const double2 *__restrict__ ft = a.m.ft;
-    const double *__restrict__ rcp = a.m.rcp;
-#pragma unroll
-    for (int k = 0; k < GB; ++k) {
-        if (k < n) {
-            const long long Mrt = o[0][k], Mst = o[1][k], Mtr = o[2][k], Mts = o[3][k];
-            const long long ot = bo[k], it = bi[k];
-            const double c = (double)(ot + it), rt = __ldg(rcp + bt[k]);
-            accS -= df_t(ft, Mrt, -ot) + df_t(ft, Mst, ot) + df_t(ft, Mtr, -it) + df_t(ft, Mts, it);
-            pf += c * (double)(Mts + Mst + 1) * rt;
-            pb += c * (double)(Mtr - it + Mrt - ot + 1) * rt;
-        }
-    }
-}
-
 // the 2x2 core, the four degree terms and the two self-loop terms: term k of 10
 GSAP_DEV void core_term(const MoveArgs &a, const MoveCtx &q, int k, double &accS, double &pf, double &pb) {
     const double2 *__restrict__ ft = a.m.ft;
@@ -996,31 +937,13 @@ GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, i
     MoveCtx q;
     move_ctx(a, v, r, s, tab, log2cap, q);
     double accS = 0.0, pf = 0.0, pb = 0.0;
-    int bt[GB], bo[GB], bi[GB], nbuf = 0;   // sparse regime: generic blocks batched GB at a time
     for (int j = gt; j < deg; j += G) {
         const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
         if (nb == v) continue;
         const int4 e = tab[tab_find(tab, log2cap, __ldg(a.b + nb))];
         if (e.w != j) continue;
-        if (a.m.dense || e.x == q.r || e.x == q.s) {
-            t_terms_batch(a, q, nbuf, bt, bo, bi, accS, pf, pb);   // keep the accumulation order
-            nbuf = 0;
-            t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
-        } else {
-#pragma unroll
-            for (int k = 0; k < GB; ++k)   // register slots (no dynamic indexing)
-                if (k == nbuf) {
-                    bt[k] = e.x;
-                    bo[k] = e.y;
-                    bi[k] = e.z;
-                }
-            if (++nbuf == GB) {
-                t_terms_batch(a, q, nbuf, bt, bo, bi, accS, pf, pb);
-                nbuf = 0;
-            }
-        }
+        t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
     }
-    t_terms_batch(a, q, nbuf, bt, bo, bi, accS, pf, pb);
     if (gt < 10) core_term(a, q, gt, accS, pf, pb);
     group_sum3<G>(accS, pf, pb, sh);
     mh_decide(a, q, w, accS, pf, pb, dS_out, H_out, acc_out);
@@ -1317,27 +1240,12 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         };
         int nmid = 0, kmid = 0, nbig = 0, kbig = 0, nhuge = 0, khuge = 0;
         const int omid = range(c.h_mid, nmid, kmid);
-        int obig = range(c.h_big, nbig, kbig);
-        // latency mode: few group vertices in the batch (the kernel is as long as
-        // its slowest vertex) -- the 129..256-entry vertices get a whole CTA each
-        // like the bigger ones (1-2 entries per thread instead of 4) instead of
-        // a 64-thread group
-        const bool latency_mode = nmid > 0 && nmid + nbig <= 2 * 148 * GSAP_GROUPS_MINB;
-        if (latency_mode) {
-            int n2 = 0, k2 = 0;
-            const int o2 = range(c.h_midbig, n2, k2);
-            a.list = c.midbig + o2;
-            a.list_count = n2;
-            a.big_log2 = std::max(log2_ceil(2LL * std::min(k2, c.B)), 5);
-            a.nbig_ctas = std::min(n2, c.test_grid > 0 ? c.test_grid : 148 * 16);
-            nmid = 0;
-            nbig = 0;
-        }
         if (nmid > 0) {
             a.mlist = c.mid + omid;
             a.mlist_count = nmid;
             a.nmid_ctas = std::min((nmid + 3) / 4, c.test_grid > 0 ? c.test_grid : 148 * 16);
         }
+        const int obig = range(c.h_big, nbig, kbig);
         const int ohuge = range(c.h_huge, nhuge, khuge);
         if (nbig > 0) {
             a.list = c.big + obig;
