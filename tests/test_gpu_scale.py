@@ -200,3 +200,26 @@ def test_1m_2m_end_to_end_properties(G, oracle_mod, name):
     assert q >= 0.69
     from test_gpu_parity import assert_driver_replay
     assert_driver_replay(oracle_mod, res, cfg.V)
+
+
+def test_bench_tsv_workload(G, tmp_path):
+    """N3: bench.py partitions a GraphChallenge TSV graph (1-based ids) with a
+    truth file and reports NMI / pairwise P/R in `config`."""
+    import json
+    import os
+    import subprocess
+    import sys
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    src = np.repeat(np.arange(cfg.V), np.diff(rowptr))
+    g = tmp_path / "g.tsv"
+    t = tmp_path / "t.tsv"
+    np.savetxt(g, np.stack([src + 1, col + 1], 1), fmt="%d", delimiter="\t")
+    np.savetxt(t, np.stack([np.arange(cfg.V) + 1, truth + 1], 1), fmt="%d", delimiter="\t")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--tsv", str(g), "--truth", str(t),
+                          "--steps", "1", "--warmup", "1", "--no-2m", "--no-cpu-baseline", "--no-e2e"],
+                         capture_output=True, text=True, timeout=600, cwd=root)
+    assert out.returncode == 0, out.stderr[-2000:]
+    line = json.loads([l for l in out.stdout.splitlines() if l.startswith("{")][-1])
+    assert line["config"]["V"] == cfg.V and line["config"]["E"] == cfg.E
+    assert line["config"]["nmi_vs_planted"] > 0.9 and "pairwise_recall" in line["config"]
