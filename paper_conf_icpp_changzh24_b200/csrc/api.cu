@@ -192,7 +192,11 @@ static void check_sm100() {
 static void free_ctx(Ctx &c) {
     if (c.arena) {
         // back to the device's memory pool (kept: the next context reuses it)
+#ifdef GSAP_NO_POOL
+        if (false) {
+#else
         if (c.stream) {
+#endif
             cudaFreeAsync(c.arena, c.stream);
             cudaStreamSynchronize(c.stream);
         } else {
@@ -420,6 +424,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.scal_i = A.take<int>(8);
         c.n_eval = A.take<unsigned long long>(1);
         if (c.prm.proposal_mode == 1) c.mt = A.take<int>(Vs);
+        c.dnnz_r = A.take<int>(Vs + 1);
+        c.dnnz_c = A.take<int>(Vs + 1);
         if (c.prm.incremental) {
             c.oldb = A.take<int>(Vs);
             c.moved = A.take<int>(Vs);
@@ -464,7 +470,11 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
             GSAP_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
             return 1;
         });
+#ifdef GSAP_NO_POOL
+        const cudaError_t e = cudaMalloc(&base, measure.off);
+#else
         const cudaError_t e = cudaMallocAsync(&base, measure.off, c.stream);
+#endif
         if (e == cudaErrorMemoryAllocation) {
             cudaGetLastError();
             throw Error{GSAP_ENOMEM, "cudaMalloc of the context arena failed"};

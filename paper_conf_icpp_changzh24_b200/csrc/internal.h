@@ -137,6 +137,7 @@ struct Ctx {
         bool pending = false;
     } delta;
     int *oldb = nullptr, *moved = nullptr, *moved_cnt = nullptr;
+    int *dnnz_r = nullptr, *dnnz_c = nullptr;   // dense regime: non-zeros per row of M / of Mt (kept for N2)
 
     // CUDA-graph capture of an MCMC iteration (N1: launch overhead, §5)
     unsigned *d_itr = nullptr;     // MCMC iteration read by k_move (device scalar)

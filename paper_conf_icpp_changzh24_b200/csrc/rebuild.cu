@@ -600,7 +600,7 @@ static void launch_rebuild_dense_coop(Ctx &c, const int *skip = nullptr) {
     a.B = c.B;
     a.esrc = c.esrc; a.col = c.col; a.wgt = c.wgt; a.b = c.b;
     a.acc = c.small_acc; a.M = c.dense; a.Mt = c.denseT;
-    a.rownnz = c.rownnz; a.colnnz = c.tmpi; a.dout = c.dout; a.din = c.din;
+    a.rownnz = c.dnnz_r; a.colnnz = c.dnnz_c; a.dout = c.dout; a.din = c.din;   // kept for N2
     a.ptrA = c.bm_rowptr; a.idxA = c.bm_col; a.cntA = c.bm_cnt; a.cumA = c.bm_cum;
     a.ptrB = c.bm_colptr; a.idxB = c.bm_row; a.cntB = c.bm_ccnt; a.cumB = c.bm_ccum;
     a.rcp = c.rcp;
@@ -645,12 +645,34 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
                                                      const int *__restrict__ rowptr, const int *__restrict__ col,
                                                      const int *__restrict__ wgt, const int *__restrict__ cscptr,
                                                      const int *__restrict__ cscsrc, const int *__restrict__ cscwgt,
-                                                     int B, int *__restrict__ M, int *__restrict__ Mt) {
+                                                     int B, int *__restrict__ M, int *__restrict__ Mt,
+                                                     int *__restrict__ rnnz, int *__restrict__ cnnz,
+                                                     int *__restrict__ dout, int *__restrict__ din,
+                                                     const int *__restrict__ kout, const int *__restrict__ kin) {
     const int n = *moved_cnt;
     const int lane = threadIdx.x & 31;
+    // one change of M_xy (and of its transpose entry): the line statistics follow
+    // it -- a non-zero count per row of M (rnnz) and of Mt (cnnz) changes when
+    // the entry goes 0 <-> non-zero (each atomic sees its own old value, so the
+    // transitions of concurrent changes add up to the net one)
+    auto upd = [&](int x, int y, int d) {
+        const int o = atomicAdd(M + (size_t)x * B + y, d);
+        if (o == 0 && o + d != 0) atomicAdd(rnnz + x, 1);
+        else if (o != 0 && o + d == 0) atomicAdd(rnnz + x, -1);
+        const int ot = atomicAdd(Mt + (size_t)y * B + x, d);
+        if (ot == 0 && ot + d != 0) atomicAdd(cnnz + y, 1);
+        else if (ot != 0 && ot + d == 0) atomicAdd(cnnz + y, -1);
+    };
     for (int k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < n; k += (gridDim.x * blockDim.x) >> 5) {
         const int v = moved[k];
         const int r = oldb[v], s = b[v];
+        if (lane == 0) {   // block degrees: v's out / in weight (self-loop in both) moves from r to s
+            const int ko = kout[v], ki = kin[v];
+            atomicAdd(dout + r, -ko);
+            atomicAdd(dout + s, ko);
+            atomicAdd(din + r, -ki);
+            atomicAdd(din + s, ki);
+        }
         const int ro = rowptr[v], nout = rowptr[v + 1] - ro;
         for (int j = lane; j < nout; j += 32) {
             const int w = col[ro + j];
@@ -658,10 +680,8 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
             const int bn = b[w];
             const bool wm = w >= first && w < first + count && acc[w - first];
             const int bo = wm ? oldb[w] : bn;
-            atomicAdd(M + (size_t)r * B + bo, -wt);
-            atomicAdd(M + (size_t)s * B + bn, wt);
-            atomicAdd(Mt + (size_t)bo * B + r, -wt);
-            atomicAdd(Mt + (size_t)bn * B + s, wt);
+            upd(r, bo, -wt);
+            upd(s, bn, wt);
         }
         const int ci = cscptr[v], nin = cscptr[v + 1] - ci;
         for (int j = lane; j < nin; j += 32) {
@@ -669,30 +689,29 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
             if (w >= first && w < first + count && acc[w - first]) continue;   // moved source (incl. v's self-loop)
             const int wt = cscwgt ? cscwgt[ci + j] : 1;
             const int bw = b[w];
-            atomicAdd(M + (size_t)bw * B + r, -wt);
-            atomicAdd(M + (size_t)bw * B + s, wt);
-            atomicAdd(Mt + (size_t)r * B + bw, -wt);
-            atomicAdd(Mt + (size_t)s * B + bw, wt);
+            upd(bw, r, -wt);
+            upd(bw, s, wt);
         }
     }
 }
 
-// the dense regime after a MOVE batch whose moves were logged: M and Mt
-// updated in place by k_dense_delta, then the line statistics, offsets and
-// compaction as in the full path (all four skip when no vertex moved)
+// the dense regime after a MOVE batch whose moves were logged: M, Mt, the
+// line non-zero counts and the block degrees updated in place by
+// k_dense_delta, then the offsets and the compaction as in the full path
+// (both skip when no vertex moved)
 static void rebuild_dense_delta(Ctx &c) {
     const int B = c.B;
     const int dg = (int)std::min<long long>(((long long)c.delta.count + 7) / 8, 148LL * 8);
     k_dense_delta<<<std::max(dg, 1), 256, 0, c.stream>>>(c.moved, c.moved_cnt, c.delta.first, c.delta.count,
                                                         c.delta.acc, c.oldb, c.b, c.rowptr, c.col, c.wgt, c.cscptr,
-                                                        c.cscsrc, c.cscwgt, B, c.dense, c.denseT);
+                                                        c.cscsrc, c.cscwgt, B, c.dense, c.denseT, c.dnnz_r, c.dnnz_c,
+                                                        c.dout, c.din, c.kout, c.kin);
     const int rg = grid_for(2LL * B * 32, 256);
-    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.rownnz, c.dout, c.tmpi, c.din, c.moved_cnt);
-    k_scan2<<<2, 1024, 0, c.stream>>>(c.rownnz, c.bm_rowptr, c.tmpi, c.bm_colptr, B, c.moved_cnt);
+    k_scan2<<<2, 1024, 0, c.stream>>>(c.dnnz_r, c.bm_rowptr, c.dnnz_c, c.bm_colptr, B, c.moved_cnt);
     k_row_compact2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum,
                                              c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp,
                                              c.d_nnz, c.moved_cnt);
-    c.launches += 4;
+    c.launches += 3;
     GSAP_CHECK_LAUNCH();
 }
 
@@ -721,8 +740,10 @@ static void rebuild_dense(Ctx &c) {
     dim3 tg((B + 31) / 32, (B + 31) / 32), tb(32, 8);
     k_transpose<<<tg, tb, 0, c.stream>>>(c.dense, B, c.denseT);
     const int rg = grid_for(2LL * B * 32, 256);
-    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.rownnz, c.dout, c.tmpi, c.din, nullptr);
-    k_scan2<<<2, 1024, 0, c.stream>>>(c.rownnz, c.bm_rowptr, c.tmpi, c.bm_colptr, B, nullptr);
+    // line non-zero counts into the persistent dnnz_r / dnnz_c (the next
+    // rebuild may update them incrementally, N2)
+    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.dnnz_r, c.dout, c.dnnz_c, c.din, nullptr);
+    k_scan2<<<2, 1024, 0, c.stream>>>(c.dnnz_r, c.bm_rowptr, c.dnnz_c, c.bm_colptr, B, nullptr);
     k_row_compact2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum,
                                              c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp,
                                              c.d_nnz, nullptr);
