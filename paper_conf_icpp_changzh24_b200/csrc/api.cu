@@ -190,19 +190,7 @@ static void check_sm100() {
 }
 
 static void free_ctx(Ctx &c) {
-    if (c.arena) {
-        // back to the device's memory pool (kept: the next context reuses it)
-#ifdef GSAP_NO_POOL
-        if (false) {
-#else
-        if (c.stream) {
-#endif
-            cudaFreeAsync(c.arena, c.stream);
-            cudaStreamSynchronize(c.stream);
-        } else {
-            cudaFree(c.arena);
-        }
-    }
+    if (c.arena) cudaFree(c.arena);
     c.arena = nullptr;
     if (c.h_scal) cudaFreeHost(c.h_scal);
     if (c.h_int) cudaFreeHost(c.h_int);
@@ -457,24 +445,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         Arena measure;
         carve(measure);
         void *base = nullptr;
-        // the arena from the device's default memory pool, which keeps freed
-        // memory (release threshold: unlimited): a context created after
-        // another one was destroyed (gsap_partition called repeatedly) maps
-        // no new pages
-        per_device((const void *)&gsap_default_params, [] {
-            int dev = 0;
-            GSAP_CUDA(cudaGetDevice(&dev));
-            cudaMemPool_t pool;
-            GSAP_CUDA(cudaDeviceGetDefaultMemPool(&pool, dev));
-            uint64_t thr = UINT64_MAX;
-            GSAP_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
-            return 1;
-        });
-#ifdef GSAP_NO_POOL
         const cudaError_t e = cudaMalloc(&base, measure.off);
-#else
-        const cudaError_t e = cudaMallocAsync(&base, measure.off, c.stream);
-#endif
         if (e == cudaErrorMemoryAllocation) {
             cudaGetLastError();
             throw Error{GSAP_ENOMEM, "cudaMalloc of the context arena failed"};
