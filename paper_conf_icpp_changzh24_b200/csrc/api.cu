@@ -1259,22 +1259,40 @@ static gsap_status get_blockmodel_padded(Ctx &c, int64_t *nnz_io, int64_t *rowpt
         for (size_t x = 0; x < B; ++x) w[x + 1] = w[x] + (e[x] - p[x]);
         GSAP_CUDA(cudaMemcpy(dst, w.data(), sizeof(int64_t) * (B + 1), cudaMemcpyDefault));
     };
-    auto ent_out = [&](int32_t *dst, const int *src, const std::vector<int> &p, const std::vector<int> &e) {
-        if (!dst) return;
-        const std::vector<int> h = to_host(src, E);
-        std::vector<int> w;
-        w.reserve((size_t)nnz);
-        for (size_t x = 0; x < B; ++x) w.insert(w.end(), h.begin() + p[x], h.begin() + e[x]);
-        if (!w.empty()) GSAP_CUDA(cudaMemcpy(dst, w.data(), sizeof(int) * w.size(), cudaMemcpyDefault));
+    // the entries are compacted on the device (one warp per line) into dst if
+    // it is device memory, else into scratch followed by one nnz-sized copy
+    int *off_r = c.wa, *off_c = c.wb, *stage = reinterpret_cast<int *>(c.keys1);
+    {
+        std::vector<int> orow(B), ocol(B);
+        int a = 0, b2 = 0;
+        for (size_t x = 0; x < B; ++x) {
+            orow[x] = a;
+            ocol[x] = b2;
+            a += re[x] - rp[x];
+            b2 += ce[x] - cp[x];
+        }
+        if (B) {
+            GSAP_CUDA(cudaMemcpy(off_r, orow.data(), sizeof(int) * B, cudaMemcpyHostToDevice));
+            GSAP_CUDA(cudaMemcpy(off_c, ocol.data(), sizeof(int) * B, cudaMemcpyHostToDevice));
+        }
+    }
+    (void)E;
+    auto ent_out = [&](int32_t *dst, const int *src, bool rows) {
+        if (!dst || nnz == 0) return;
+        const bool dev = is_dev(dst);
+        export_lines(c, rows ? c.bm_rowptr : c.bm_colptr, rows ? c.bm_rowend : c.bm_colend, rows ? off_r : off_c,
+                     src, dev ? dst : stage);
+        if (!dev) GSAP_CUDA(cudaMemcpyAsync(dst, stage, sizeof(int) * (size_t)nnz, cudaMemcpyDeviceToHost, c.stream));
+        GSAP_CUDA(cudaStreamSynchronize(c.stream));
     };
     ptr_out(rowptr, rp, re);
     ptr_out(colptr, cp, ce);
-    ent_out(col, c.bm_col, rp, re);
-    ent_out(cnt, c.bm_cnt, rp, re);
-    ent_out(cum, c.bm_cum, rp, re);
-    ent_out(row, c.bm_row, cp, ce);
-    ent_out(ccnt, c.bm_ccnt, cp, ce);
-    ent_out(ccum, c.bm_ccum, cp, ce);
+    ent_out(col, c.bm_col, true);
+    ent_out(cnt, c.bm_cnt, true);
+    ent_out(cum, c.bm_cum, true);
+    ent_out(row, c.bm_row, false);
+    ent_out(ccnt, c.bm_ccnt, false);
+    ent_out(ccum, c.bm_ccum, false);
     if (dout) GSAP_CUDA(cudaMemcpy(dout, c.dout, sizeof(int) * B, cudaMemcpyDefault));
     if (din) GSAP_CUDA(cudaMemcpy(din, c.din, sizeof(int) * B, cudaMemcpyDefault));
     return GSAP_OK;

@@ -194,6 +194,8 @@ void kc_resolve(Ctx &c, KClass &k);
 void build_graph_device(Ctx &c);                 // CSC, esrc, degrees (create time)
 void rebuild(Ctx &c);                            // Alg. 2 from c.b, c.B
 bool dense_ok(const Ctx &c, int B);
+// padded-CSR export: line x's [ptr[x], end[x]) of src to dst[off[x] ..) on the device
+void export_lines(Ctx &c, const int *ptr, const int *end, const int *off, const int *src, int *dst);
 constexpr int SMALL_MAX_B = 221;               // B^2 ints in one CTA's shared memory (195 KB)
 
 // move.cu

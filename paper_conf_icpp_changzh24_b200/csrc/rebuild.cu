@@ -645,34 +645,12 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
                                                      const int *__restrict__ rowptr, const int *__restrict__ col,
                                                      const int *__restrict__ wgt, const int *__restrict__ cscptr,
                                                      const int *__restrict__ cscsrc, const int *__restrict__ cscwgt,
-                                                     int B, int *__restrict__ M, int *__restrict__ Mt,
-                                                     int *__restrict__ rnnz, int *__restrict__ cnnz,
-                                                     int *__restrict__ dout, int *__restrict__ din,
-                                                     const int *__restrict__ kout, const int *__restrict__ kin) {
+                                                     int B, int *__restrict__ M, int *__restrict__ Mt) {
     const int n = *moved_cnt;
     const int lane = threadIdx.x & 31;
-    // one change of M_xy (and of its transpose entry): the line statistics follow
-    // it -- a non-zero count per row of M (rnnz) and of Mt (cnnz) changes when
-    // the entry goes 0 <-> non-zero (each atomic sees its own old value, so the
-    // transitions of concurrent changes add up to the net one)
-    auto upd = [&](int x, int y, int d) {
-        const int o = atomicAdd(M + (size_t)x * B + y, d);
-        if (o == 0 && o + d != 0) atomicAdd(rnnz + x, 1);
-        else if (o != 0 && o + d == 0) atomicAdd(rnnz + x, -1);
-        const int ot = atomicAdd(Mt + (size_t)y * B + x, d);
-        if (ot == 0 && ot + d != 0) atomicAdd(cnnz + y, 1);
-        else if (ot != 0 && ot + d == 0) atomicAdd(cnnz + y, -1);
-    };
     for (int k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < n; k += (gridDim.x * blockDim.x) >> 5) {
         const int v = moved[k];
         const int r = oldb[v], s = b[v];
-        if (lane == 0) {   // block degrees: v's out / in weight (self-loop in both) moves from r to s
-            const int ko = kout[v], ki = kin[v];
-            atomicAdd(dout + r, -ko);
-            atomicAdd(dout + s, ko);
-            atomicAdd(din + r, -ki);
-            atomicAdd(din + s, ki);
-        }
         const int ro = rowptr[v], nout = rowptr[v + 1] - ro;
         for (int j = lane; j < nout; j += 32) {
             const int w = col[ro + j];
@@ -680,8 +658,10 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
             const int bn = b[w];
             const bool wm = w >= first && w < first + count && acc[w - first];
             const int bo = wm ? oldb[w] : bn;
-            upd(r, bo, -wt);
-            upd(s, bn, wt);
+            atomicAdd(M + (size_t)r * B + bo, -wt);
+            atomicAdd(M + (size_t)s * B + bn, wt);
+            atomicAdd(Mt + (size_t)bo * B + r, -wt);
+            atomicAdd(Mt + (size_t)bn * B + s, wt);
         }
         const int ci = cscptr[v], nin = cscptr[v + 1] - ci;
         for (int j = lane; j < nin; j += 32) {
@@ -689,29 +669,32 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
             if (w >= first && w < first + count && acc[w - first]) continue;   // moved source (incl. v's self-loop)
             const int wt = cscwgt ? cscwgt[ci + j] : 1;
             const int bw = b[w];
-            upd(bw, r, -wt);
-            upd(bw, s, wt);
+            atomicAdd(M + (size_t)bw * B + r, -wt);
+            atomicAdd(M + (size_t)bw * B + s, wt);
+            atomicAdd(Mt + (size_t)r * B + bw, -wt);
+            atomicAdd(Mt + (size_t)s * B + bw, wt);
         }
     }
 }
 
-// the dense regime after a MOVE batch whose moves were logged: M, Mt, the
-// line non-zero counts and the block degrees updated in place by
-// k_dense_delta, then the offsets and the compaction as in the full path
-// (both skip when no vertex moved)
+// the dense regime after a MOVE batch whose moves were logged: M and Mt
+// updated in place by k_dense_delta, then the line statistics, offsets and
+// compaction as in the full path (all three skip when no vertex moved; line
+// statistics kept incrementally by returning atomics measured slower: 20K
+// round 5 37.7 vs 35.6 us, round 8 33.4 vs 25.6 us)
 static void rebuild_dense_delta(Ctx &c) {
     const int B = c.B;
     const int dg = (int)std::min<long long>(((long long)c.delta.count + 7) / 8, 148LL * 8);
     k_dense_delta<<<std::max(dg, 1), 256, 0, c.stream>>>(c.moved, c.moved_cnt, c.delta.first, c.delta.count,
                                                         c.delta.acc, c.oldb, c.b, c.rowptr, c.col, c.wgt, c.cscptr,
-                                                        c.cscsrc, c.cscwgt, B, c.dense, c.denseT, c.dnnz_r, c.dnnz_c,
-                                                        c.dout, c.din, c.kout, c.kin);
+                                                        c.cscsrc, c.cscwgt, B, c.dense, c.denseT);
     const int rg = grid_for(2LL * B * 32, 256);
+    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.dnnz_r, c.dout, c.dnnz_c, c.din, c.moved_cnt);
     k_scan2<<<2, 1024, 0, c.stream>>>(c.dnnz_r, c.bm_rowptr, c.dnnz_c, c.bm_colptr, B, c.moved_cnt);
     k_row_compact2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum,
                                              c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp,
                                              c.d_nnz, c.moved_cnt);
-    c.launches += 3;
+    c.launches += 4;
     GSAP_CHECK_LAUNCH();
 }
 
@@ -879,6 +862,23 @@ static void rebuild_sparse(Ctx &c) {
                               c.bm_ccum, c.din, nullptr);
     }
     c.padded = true;
+    GSAP_CHECK_LAUNCH();
+}
+
+// export of a padded CSR / CSC line by line: line x's entries [ptr[x],
+// end[x]) copied to dst[off[x] ..) (one warp per line, coalesced)
+__global__ void k_compact_lines(int B, const int *__restrict__ ptr, const int *__restrict__ end,
+                                const int *__restrict__ off, const int *__restrict__ src, int *__restrict__ dst) {
+    const int lane = threadIdx.x & 31;
+    for (int x = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < B; x += (gridDim.x * blockDim.x) >> 5) {
+        const int p = ptr[x], n = end[x] - p, o = off[x];
+        for (int i = lane; i < n; i += 32) dst[o + i] = src[p + i];
+    }
+}
+
+void export_lines(Ctx &c, const int *ptr, const int *end, const int *off, const int *src, int *dst) {
+    k_compact_lines<<<grid_for(32LL * c.B, 256), 256, 0, c.stream>>>(c.B, ptr, end, off, src, dst);
+    ++c.launches;
     GSAP_CHECK_LAUNCH();
 }
 

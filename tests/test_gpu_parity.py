@@ -740,3 +740,25 @@ def test_move_results_independent_of_launch_shape(G, oracle_mod, regime, monkeyp
         outs.append(res)
         ctx.close()
     assert outs[0] == outs[1] == outs[2]
+
+
+def test_padded_blockmodel_export_device_and_host(G, oracle_mod):
+    """The padded CSR / CSC of the multi-kernel sparse rebuild is compacted on
+    the device for export: device and host destinations give the same arrays,
+    equal to the oracle's blockmodel."""
+    import torch
+    rowptr, col, truth, cfg = dcsbm.make("1k")
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, **SPARSE_MK)
+    b0 = dcsbm.random_partition(cfg.V, 300, 5)
+    set_both(ctx, orc, b0, 300)
+    host = ctx.gsap_get_blockmodel()
+    nnz = ctx.gsap_blockmodel_nnz()
+    dev = {k: torch.zeros(nnz, dtype=torch.int32, device="cuda") for k in ("col", "cnt", "cum", "row", "ccnt", "ccum")}
+    import ctypes as C
+    n = C.c_int64(nnz)
+    G._check(G.lib().gsap_get_blockmodel(ctx.h, C.byref(n), None, dev["col"].data_ptr(), dev["cnt"].data_ptr(),
+                                         dev["cum"].data_ptr(), None, dev["row"].data_ptr(), dev["ccnt"].data_ptr(),
+                                         dev["ccum"].data_ptr(), None, None))
+    for k, t in dev.items():
+        assert np.array_equal(t.cpu().numpy(), host[k]), k
+    assert_same_blockmodel(ctx, orc)
