@@ -765,24 +765,18 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     const int gw_ = (int)std::min<long long>(((long long)B + SEG_WARPS - 1) / SEG_WARPS, 148LL * 16);
     per_device((const void *)k_segsort_warp<K, 2>, [] {
         GSAP_CUDA(cudaFuncSetAttribute(k_segsort_warp<K, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)seg_warp2_smem<K>(SEG_WARP_MAX_MK)));
+                                       (int)seg_warp2_smem<K>()));
         return 1;
     });
     const int cb = bits_for(B);
     k_segsort_warp<K, 0><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, cb, idx, cnt,
-                                                              c.seg_nnz, out, 0, 0);
+                                                              c.seg_nnz, out);
     k_segsort_warp<K, 1><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, cb, idx, cnt,
-                                                              c.seg_nnz, out, 0, 0);
-    // MODE 2 in two length classes: (256, 512] with half-size buffers (more
-    // CTAs per SM), then (512, SEG_WARP_MAX_MK]
-    const int mid = std::min(512, SEG_WARP_MAX_MK);
-    k_segsort_warp<K, 2><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(mid), c.stream>>>(B, ptr, seg, c.seg_listC,
-                                                                                   c.seg_ctr, cb, idx, cnt,
-                                                                                   c.seg_nnz, out, 256, mid);
-    if (SEG_WARP_MAX_MK > mid)
-        k_segsort_warp<K, 2><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(SEG_WARP_MAX_MK), c.stream>>>(
-            B, ptr, seg, c.seg_listC, c.seg_ctr, cb, idx, cnt, c.seg_nnz, out, mid, SEG_WARP_MAX_MK);
-    c.launches += 3;
+                                                              c.seg_nnz, out);
+    k_segsort_warp<K, 2><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(), c.stream>>>(B, ptr, seg, c.seg_listC,
+                                                                                c.seg_ctr, cb, idx, cnt,
+                                                                                c.seg_nnz, out);
+    c.launches += 2;
     const int gc = (int)std::min<long long>(std::max(1, B / 4), 148LL * 4);
     k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(ptr, seg, c.seg_listC, c.seg_ctr, bits_for(B), idx, cnt,
                                                c.seg_nnz, out);

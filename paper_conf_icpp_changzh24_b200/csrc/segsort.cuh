@@ -391,11 +391,9 @@ GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict_
 #define GSAP_SEG_WARP_MAX_MK 1024
 #endif
 constexpr int SEG_WARP_MAX_MK = GSAP_SEG_WARP_MAX_MK;   // multi-kernel path: longer lines go to the CTA sorts
-// MODE 2 is launched once per length class (lo, cap] with buffers of cap
-// keys per warp: the shorter class fits more CTAs per SM
 template <typename K>
-constexpr size_t seg_warp2_smem(int cap) {
-    return (size_t)SEG_WARPS * (2 * (size_t)cap * sizeof(K) + 8 * 32 * sizeof(unsigned));
+constexpr size_t seg_warp2_smem() {
+    return (size_t)SEG_WARPS * (2 * SEG_WARP_MAX_MK * sizeof(K) + 8 * 32 * sizeof(unsigned));
 }
 
 template <typename K, int NT>
@@ -406,14 +404,13 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const in
                                                                  const int *__restrict__ listW,
                                                                  const int *__restrict__ counters, int col_bits,
                                                                  int *__restrict__ tcol, int *__restrict__ tcnt,
-                                                                 int *__restrict__ nnz, LineOut out, int lo, int cap) {
+                                                                 int *__restrict__ nnz, LineOut out) {
     extern __shared__ __align__(16) unsigned char seg_dyn[];   // MODE 2: SEG_WARPS x (2 key buffers) + counters
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int n_lines = counters[MODE == 0 ? 0 : MODE == 1 ? 2 : 3];
     for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
         const int x = MODE == 0 ? listW[li] : listW[B - 1 - li];   // MODE 2: listW is the CTA list (listC)
         const int o = off[x], L = off[x + 1] - o;
-        if (MODE == 2 && (L <= lo || L > cap)) continue;   // another length class's launch
         int u;
         if (MODE == 1) {
             u = warp_segsort_rle<K, 8>(seg + o, L, tcol + o, tcnt + o);
@@ -422,10 +419,10 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const in
             else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, tcol + o, tcnt + o);
             else u = warp_segsort_rle<K, 4>(seg + o, L, tcol + o, tcnt + o);
         } else {
-            K *ka = reinterpret_cast<K *>(seg_dyn) + (size_t)w * 2 * cap;
-            K *kb = ka + cap;
+            K *ka = reinterpret_cast<K *>(seg_dyn) + (size_t)w * 2 * SEG_WARP_MAX_MK;
+            K *kb = ka + SEG_WARP_MAX_MK;
             unsigned *cntp = reinterpret_cast<unsigned *>(reinterpret_cast<K *>(seg_dyn) +
-                                                          (size_t)SEG_WARPS * 2 * cap) + w * 8 * 32;
+                                                          (size_t)SEG_WARPS * 2 * SEG_WARP_MAX_MK) + w * 8 * 32;
             for (int i = lane; i < L; i += 32) ka[i] = seg[o + i];
             __syncwarp();
             K *keys = cta_radix_sort<K, 32>(ka, kb, L, col_bits, cntp, nullptr);
