@@ -727,12 +727,8 @@ GSAP_DEV void bucket_get(const Line (&L)[N], const int (&y)[N], int (&p)[N], int
 #endif
 constexpr int HALF_K = GSAP_HALF_K;   // splitters per lane in the sorted two-pass kernels
 
-// C = adjacency chunks of 32 per vertex: 4 (<= 128 entries, a 256-slot
-// table) or 8 (129..256 entries, 512 slots; these would otherwise take
-// k_move_groups' 64-thread groups)
-template <bool WEIGHTED, int PASS, int C>
+template <bool WEIGHTED, int PASS>
 GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
-    constexpr int TLOG2 = C == 4 ? WARP_TAB_LOG2 : WARP_TAB_LOG2 + 1;
     const int lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
     const int v = a.first + i;
@@ -748,7 +744,7 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
     }
     const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
     const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
-    const int deg = nout + nin;   // <= 32 C (the caller routes bigger vertices to k_move_groups)
+    const int deg = nout + nin;   // <= 128 (the caller routes bigger vertices to k_move_groups)
     const int B = a.m.B;
     // the two lines of this pass and their wide splitters (32 HALF_K per
     // line, shared by the warp), issued before the histogram
@@ -759,9 +755,9 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
     int sp[2][HALF_K];
     splitw_load<2, HALF_K>(Ln, lane, sp);
     // ---- phase A: histogram of v's neighbour blocks (self-loop excluded)
-    int keep[C];
+    int keep[4];
 #pragma unroll
-    for (int c = 0; c < C; ++c) {
+    for (int c = 0; c < 4; ++c) {
         keep[c] = -1;
         const int j = c * 32 + lane;
         if (j < deg) {
@@ -769,7 +765,7 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
             const int n = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
             if (n != v) {
                 const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
-                const int sl = tab_insert(tab, TLOG2, __ldg(a.b + n));
+                const int sl = tab_insert(tab, WARP_TAB_LOG2, __ldg(a.b + n));
                 atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
                 atomicMin(&tab[sl].w, j);
                 keep[c] = sl;
@@ -779,7 +775,7 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
     __syncwarp();
     int nuniq = 0;
 #pragma unroll
-    for (int c = 0; c < C; ++c) {
+    for (int c = 0; c < 4; ++c) {
         const int sl = keep[c];
         const bool own = sl >= 0 && tab[sl].w == c * 32 + lane;
         const unsigned bal = __ballot_sync(FULL, own);
@@ -787,7 +783,7 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
         nuniq += __popc(bal);
     }
     __syncwarp();
-    const int slr = tab_find(tab, TLOG2, r), sls = tab_find(tab, TLOG2, s);
+    const int slr = tab_find(tab, WARP_TAB_LOG2, r), sls = tab_find(tab, WARP_TAB_LOG2, s);
     const int o_r = slr >= 0 ? tab[slr].y : 0, i_r = slr >= 0 ? tab[slr].z : 0;
     const int o_s = sls >= 0 ? tab[sls].y : 0, i_s = sls >= 0 ? tab[sls].z : 0;
     const int kout = __ldg(a.kout + v), kin = __ldg(a.kin + v), l = __ldg(a.selfw + v);
@@ -1117,24 +1113,23 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_MOVE_MINB) k_move(MoveAr
 #ifndef GSAP_HALF_MINB
 #define GSAP_HALF_MINB 4
 #endif
-template <bool WEIGHTED, int PASS, int C>
-__global__ void __launch_bounds__(MOVE_WARPS * 32, C == 4 ? GSAP_HALF_MINB : 2) k_move_half(MoveArgs a) {
-    extern __shared__ int4 move_smem[];   // half_smem(C) bytes
-    constexpr int TS = 64 * C;            // table slots per warp
+template <bool WEIGHTED, int PASS>
+__global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_HALF_MINB) k_move_half(MoveArgs a) {
+    extern __shared__ int4 move_smem[];   // MOVE_SMEM bytes
     int4 *tabs = move_smem;
-    int *lists = reinterpret_cast<int *>(tabs + MOVE_WARPS * TS);
+    int *lists = reinterpret_cast<int *>(tabs + MOVE_WARPS * WARP_TAB);
     const int wl = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    int4 *tab = tabs + wl * TS;
-    int *list = lists + wl * (TS / 2);
-    tab_clear<32>(tab, TS, lane);
+    int4 *tab = tabs + wl * WARP_TAB;
+    int *list = lists + wl * (WARP_TAB / 2);
+    tab_clear<32>(tab, WARP_TAB, lane);
     __syncwarp();
     const int nwarps = gridDim.x * MOVE_WARPS;
     for (int w = blockIdx.x * MOVE_WARPS + wl; w < a.count; w += nwarps) {
         const int i = __ldg(a.perm + w);
         const int v = a.first + i;
-        const int k = (__ldg(a.rowptr + v + 1) - __ldg(a.rowptr + v)) + (__ldg(a.cscptr + v + 1) - __ldg(a.cscptr + v));
-        if (C == 4 ? k > BIG_THR : (k <= BIG_THR || k > 2 * BIG_THR)) continue;   // the other instantiation / groups
-        move_vertex_half<WEIGHTED, PASS, C>(a, i, tab, list);
+        if ((__ldg(a.rowptr + v + 1) - __ldg(a.rowptr + v)) + (__ldg(a.cscptr + v + 1) - __ldg(a.cscptr + v)) > BIG_THR)
+            continue;
+        move_vertex_half<WEIGHTED, PASS>(a, i, tab, list);
     }
 }
 
@@ -1230,7 +1225,6 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     a.hlist = nullptr;
     a.hlist_count = 0;
     a.big_log2 = 5;
-    int nmid_batch = 0;   // 129..256-entry vertices in [first, first + count)
     if (c.B > BIG_THR) {
         // the big (128 < k <= 1024) and huge (k > 1024) vertices inside [first, first + count)
         auto range = [&](const std::vector<int> &h, int &n, int &kmax) {
@@ -1246,8 +1240,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         };
         int nmid = 0, kmid = 0, nbig = 0, kbig = 0, nhuge = 0, khuge = 0;
         const int omid = range(c.h_mid, nmid, kmid);
-        nmid_batch = nmid;
-        if (nmid > 0 && !sorted) {   // sorted mode: the mid vertices take the sorted passes (C = 8)
+        if (nmid > 0) {
             a.mlist = c.mid + omid;
             a.mlist_count = nmid;
             a.nmid_ctas = std::min((nmid + 3) / 4, c.test_grid > 0 ? c.test_grid : 148 * 16);
@@ -1297,35 +1290,24 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     });
     const bool dense = a.m.dense != nullptr;
     if (sorted) {
-        constexpr size_t SM8 = (sizeof(int4) * 512 + sizeof(int) * 256) * MOVE_WARPS;   // C = 8 tables
-        per_device((const void *)k_move_half<false, 1, 4>, [] {
-            const int s4 = (int)MOVE_SMEM, s8 = (int)SM8;
-            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 1, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, s4));
-            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 2, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, s4));
-            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 1, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, s4));
-            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 2, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, s4));
-            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 1, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, s8));
-            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 2, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, s8));
-            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 1, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, s8));
-            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 2, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, s8));
+        per_device((const void *)k_move_half<false, 1>, [] {
+            const int sm = (int)MOVE_SMEM;
+            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<true, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
+            GSAP_CUDA(cudaFuncSetAttribute(k_move_half<false, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm));
             return 1;
         });
         MoveArgs a1 = a, a2 = a;
         a1.perm = c.mv_perm;            // grouped by r
         a2.perm = c.mv_perm + count;    // grouped by s
-        const bool mids = nmid_batch > 0;   // 129..256-entry vertices in this batch: the C = 8 instantiation
         if (c.weighted) {
-            k_move_half<true, 1, 4><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
-            if (mids) k_move_half<true, 1, 8><<<grid, MOVE_WARPS * 32, SM8, c.stream>>>(a1);
-            k_move_half<true, 2, 4><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
-            if (mids) k_move_half<true, 2, 8><<<grid, MOVE_WARPS * 32, SM8, c.stream>>>(a2);
+            k_move_half<true, 1><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
+            k_move_half<true, 2><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
         } else {
-            k_move_half<false, 1, 4><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
-            if (mids) k_move_half<false, 1, 8><<<grid, MOVE_WARPS * 32, SM8, c.stream>>>(a1);
-            k_move_half<false, 2, 4><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
-            if (mids) k_move_half<false, 2, 8><<<grid, MOVE_WARPS * 32, SM8, c.stream>>>(a2);
+            k_move_half<false, 1><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a1);
+            k_move_half<false, 2><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a2);
         }
-        if (mids) c.launches += 2;
         c.launches += 2;
     } else if (c.weighted) {
         if (dense) k_move<true, true><<<grid, MOVE_WARPS * 32, MOVE_SMEM, c.stream>>>(a);

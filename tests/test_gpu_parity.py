@@ -762,3 +762,83 @@ def test_padded_blockmodel_export_device_and_host(G, oracle_mod):
     for k, t in dev.items():
         assert np.array_equal(t.cpu().numpy(), host[k]), k
     assert_same_blockmodel(ctx, orc)
+
+
+def _bracket_step(sl, B, S, cur_b, rate=0.4):
+    """O.9 as the drivers take it (a port for the lockstep driver below; the
+    rule itself is pinned in test_oracle_pins*.py and replayed through the
+    oracle's own code in assert_driver_replay): returns (done, K, restart)."""
+    if S <= sl["S"][1]:
+        idx = 0 if sl["B"][1] > B else 2
+        sl["b"][idx], sl["B"][idx], sl["S"][idx] = sl["b"][1], sl["B"][1], sl["S"][1]
+        idx = 1
+    else:
+        idx = 2 if sl["B"][1] > B else 0
+    sl["b"][idx], sl["B"][idx], sl["S"][idx] = cur_b, B, S
+    if sl["S"][2] == float("inf"):
+        K = int(B * rate)
+        return K == 0, K, 1
+    if sl["B"][0] - sl["B"][2] == 2:
+        return True, 0, 1
+    i = 0 if (sl["B"][0] - sl["B"][1]) >= (sl["B"][1] - sl["B"][2]) else 1
+    nxt = sl["B"][i + 1] + int(np.rint((sl["B"][i] - sl["B"][i + 1]) * 0.618))
+    K = sl["B"][i] - nxt
+    return K <= 0, K, i
+
+
+@pytest.mark.parametrize("name", ["1k", "5k"])
+def test_full_run_lockstep_trace(G, oracle_mod, name):
+    """a7 end to end with the tie escape: the whole SBP run
+    driven round by round on both sides from the same state -- merge phase
+    (proposals exact, dS 1e-9, the merge order taken on the GPU's dS on both
+    sides), MCMC phase (D[itr] 1e-9, iteration count equal, b equal unless an
+    MH tie, which is then copied), MDL 1e-9, the golden-section restart --
+    gives the same per-round [outer, B, itrs] on the GPU as on the oracle;
+    and the GPU's own C driver (gsap_run) reproduces this trace exactly."""
+    if name == "1k":
+        rowptr, col, truth, cfg = dcsbm.make("1k")
+    else:
+        rowptr, col, truth = dcsbm.generate(5000, 50850, 10.0, 5.0, seed=5000)
+    V = len(rowptr) - 1
+    p = oracle_mod.default_params(seed=SEED)
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col)
+    inf = float("inf")
+    sl = {"b": [None] * 3, "B": [0, 0, 0], "S": [inf, inf, inf]}
+    K, outer, trace, mh_ties = int(V * 0.4), 0, [], 0
+    while True:
+        bracket = sl["S"][2] != inf
+        B = ctx.B
+        s = ctx.gsap_propose(G.GSAP_MERGE, outer, 0, 0, B)
+        dS = ctx.gsap_delta_mdl(G.GSAP_MERGE, outer, 0, 0, B, s)
+        s_o = orc.propose(0, SEED, outer, 0, 0, B)
+        assert np.array_equal(s, s_o)
+        assert np.all(close(dS, orc.delta_merge(0, B, s_o)))
+        best, dSb = ctx.gsap_merge_phase(outer, K)
+        assert np.array_equal(best, orc.best_merges(s_o, dS)[0])
+        orc.select_merges(best, dSb, K)
+        b_g, B_g = ctx.gsap_get_partition()
+        assert (B_g, b_g.tobytes()) == (orc.B, orc.partition()[0].tobytes())
+        thresh = p.thresh2 if bracket else p.thresh1
+        n_g, D_g = ctx.gsap_mcmc_phase(outer, thresh)
+        n_o, _, D_o = orc.mcmc_phase(p, outer, thresh, return_D=True)
+        assert n_g == n_o and np.all(close(D_g, D_o)), (outer, n_g, n_o)
+        b_g, _ = ctx.gsap_get_partition()
+        if not np.array_equal(b_g, orc.partition()[0]):   # an MH tie: the GPU's decision on both sides
+            mh_ties += 1
+            orc.set_partition(b_g, B_g)
+        S_g, S_o = ctx.gsap_mdl()[0], orc.mdl()[0]
+        assert abs(S_g - S_o) <= 1e-9 * S_o
+        trace.append((outer, B_g, n_g, S_g))
+        done, K, restart = _bracket_step(sl, B_g, S_g, b_g.copy())
+        if done or len(trace) >= 500:
+            break
+        ctx.gsap_set_partition(sl["b"][restart], sl["B"][restart])
+        orc.set_partition(sl["b"][restart], sl["B"][restart])
+        outer += 1
+    print(name, "rounds", len(trace), "MH ties", mh_ties)
+    res = G.Context(rowptr, col, params=G.gsap_default_params(seed=SEED)).gsap_run()
+    tr = res["trace"]
+    assert len(tr) == len(trace)
+    assert np.array_equal(tr[:, :3].astype(np.int64), np.array([t[:3] for t in trace], np.int64))
+    assert np.array_equal(tr[:, 3], np.array([t[3] for t in trace]))
+    assert res["B"] == sl["B"][1] and np.array_equal(res["b"], sl["b"][1])
