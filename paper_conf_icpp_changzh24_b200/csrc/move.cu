@@ -912,48 +912,17 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
 // owned terms in position order.
 // phase A of a group vertex: its neighbour-block table, built by group
 // threads [t0, G) (t0 = 32 when warp 0 of the group is drawing the proposal)
-// the first GC entries a thread handles (k-th: j = (gt - t0) + k (G - t0)) keep
-// their neighbour's block in registers (-1: the self-loop or past deg), so
-// the evaluation -- which walks the same entries -- does not load them again
-constexpr int GC = 8;
-GSAP_DEV int group_j(int gt, int t0, int G, int k) { return (gt - t0) + k * (G - t0); }
-
-template <int G, bool WEIGHTED>
-GSAP_DEV int group_entry_block(const MoveArgs &a, int v, int ro, int nout, int ci, int j) {
-    const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-    return nb == v ? -1 : __ldg(a.b + nb);   // the self-loop is carried by selfw
-}
-
 template <int G, bool WEIGHTED>
 GSAP_DEV void group_table(const MoveArgs &a, int v, int ro, int nout, int ci, int deg, int4 *tab, int log2cap,
-                          int t0, int (&ct)[GC]) {
-    const int gt = (int)(threadIdx.x % G);
-#pragma unroll
-    for (int k = 0; k < GC; ++k) ct[k] = -1;
-    if (gt < t0) return;
-    int t[GC];
-#pragma unroll
-    for (int k = 0; k < GC; ++k) {   // all loads first (independent), then the inserts
-        const int j = group_j(gt, t0, G, k);
-        t[k] = j < deg ? group_entry_block<G, WEIGHTED>(a, v, ro, nout, ci, j) : -1;
-    }
-#pragma unroll
-    for (int k = 0; k < GC; ++k) {
-        const int j = group_j(gt, t0, G, k);
-        ct[k] = t[k];
-        if (t[k] < 0) continue;
+                          int t0) {
+    for (int j = (int)(threadIdx.x % G) - t0; j < deg; j += G - t0) {
+        if (j < 0) break;
         const bool out = j < nout;
+        const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+        if (nb == v) continue;   // the self-loop is carried by selfw
+        const int t = __ldg(a.b + nb);
         const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
-        const int sl = tab_insert(tab, log2cap, t[k]);
-        atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
-        atomicMin(&tab[sl].w, j);
-    }
-    for (int j = group_j(gt, t0, G, GC); j < deg; j += G - t0) {   // huge vertices: the rest, uncached
-        const int tk = group_entry_block<G, WEIGHTED>(a, v, ro, nout, ci, j);
-        if (tk < 0) continue;
-        const bool out = j < nout;
-        const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
-        const int sl = tab_insert(tab, log2cap, tk);
+        const int sl = tab_insert(tab, log2cap, t);
         atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
         atomicMin(&tab[sl].w, j);
     }
@@ -963,30 +932,17 @@ GSAP_DEV void group_table(const MoveArgs &a, int v, int ro, int nout, int ci, in
 // first adjacency position; threads sum their owned terms in position order.
 template <int G, bool WEIGHTED>
 GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, int ro, int nout, int ci, int deg,
-                              int4 *tab, int log2cap, double *sh, int t0, const int (&ct)[GC], double &dS_out,
-                              double &H_out, bool &acc_out) {
+                              int4 *tab, int log2cap, double *sh, double &dS_out, double &H_out, bool &acc_out) {
     const int gt = threadIdx.x % G;
     MoveCtx q;
     move_ctx(a, v, r, s, tab, log2cap, q);
     double accS = 0.0, pf = 0.0, pb = 0.0;
-    // the entries this thread inserted in phase A, in the same order: the
-    // cached blocks first, the rest (huge vertices) loaded again
-    if (gt >= t0) {
-#pragma unroll
-        for (int k = 0; k < GC; ++k) {
-            if (ct[k] < 0) continue;
-            const int j = group_j(gt, t0, G, k);
-            const int4 e = tab[tab_find(tab, log2cap, ct[k])];
-            if (e.w != j) continue;
-            t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
-        }
-        for (int j = group_j(gt, t0, G, GC); j < deg; j += G - t0) {
-            const int tk = group_entry_block<G, WEIGHTED>(a, v, ro, nout, ci, j);
-            if (tk < 0) continue;
-            const int4 e = tab[tab_find(tab, log2cap, tk)];
-            if (e.w != j) continue;
-            t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
-        }
+    for (int j = gt; j < deg; j += G) {
+        const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
+        if (nb == v) continue;
+        const int4 e = tab[tab_find(tab, log2cap, __ldg(a.b + nb))];
+        if (e.w != j) continue;
+        t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
     }
     if (gt < 10) core_term(a, q, gt, accS, pf, pb);
     group_sum3<G>(accS, pf, pb, sh);
@@ -1053,21 +1009,20 @@ GSAP_DEV void do_vertex(const MoveArgs &a, int v, int4 *tab, int log2cap, int *l
     // phase A beside the proposal: warp 0 of the group draws s (fused mode),
     // the other threads build the neighbour-block table (it does not depend on s)
     int *sp = reinterpret_cast<int *>(sh + 3 * (G / 32));
-    const int t0 = a.propose ? 32 : 0;   // fused mode: warp 0 draws the proposal meanwhile
-    int ct[GC];
-    group_table<G, WEIGHTED>(a, v, ro, nout, ci, deg, tab, log2cap, t0, ct);
     if (a.propose && gt < 32) {
         const int s0 = propose_vertex_warp<WEIGHTED>(a, v, w, ro, nout, ci, deg);
         if (gt == 0) {
             *sp = s0;
             a.s_out[i] = s0;
         }
+    } else {
+        group_table<G, WEIGHTED>(a, v, ro, nout, ci, deg, tab, log2cap, a.propose ? 32 : 0);
     }
     gsync<G>();
     const int s = a.propose ? *sp : a.s_in[i];
     double dS = 0.0, H = 1.0;
     bool acc = false;
-    if (s != r) eval_move_group<G, WEIGHTED>(a, v, r, s, w, ro, nout, ci, deg, tab, log2cap, sh, t0, ct, dS, H, acc);
+    if (s != r) eval_move_group<G, WEIGHTED>(a, v, r, s, w, ro, nout, ci, deg, tab, log2cap, sh, dS, H, acc);
     if ((threadIdx.x & (G - 1)) == 0) {
         if (a.dS) a.dS[i] = dS;
         if (a.H) a.H[i] = H;
