@@ -181,12 +181,16 @@ static std::vector<T> to_host(const T *src, size_t n) {
     return h;
 }
 
+// one attribute query per device (cudaGetDeviceProperties fills the whole
+// struct and was seen taking tens of ms inside gsap_partition's create)
 static void check_sm100() {
-    int dev = 0;
-    GSAP_CUDA(cudaGetDevice(&dev));
-    cudaDeviceProp p;
-    GSAP_CUDA(cudaGetDeviceProperties(&p, dev));
-    REQUIRE(p.major == 10, GSAP_EUNSUPPORTED, "libgsap is built for sm_100a (B200) only");
+    const int major = per_device((const void *)&check_sm100, [] {
+        int dev = 0, mj = 0;
+        GSAP_CUDA(cudaGetDevice(&dev));
+        GSAP_CUDA(cudaDeviceGetAttribute(&mj, cudaDevAttrComputeCapabilityMajor, dev));
+        return mj;
+    });
+    REQUIRE(major == 10, GSAP_EUNSUPPORTED, "libgsap is built for sm_100a (B200) only");
 }
 
 static void free_ctx(Ctx &c) {
@@ -310,6 +314,9 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         } else if (k > 128) {    // move.cu BIG_THR
             c.h_mid.push_back(v);
         }
+        if (k > 128 && k <= 1024) {
+            c.h_midbig.push_back(v);
+        }
     }
     // allocation: one device arena (one cudaMalloc / cudaFree per context),
     // planned in a measuring pass and then carved ---------------------------
@@ -334,6 +341,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.selfw = A.take<int>(Vs);
         if (!c.h_big.empty()) c.big = A.take<int>(c.h_big.size());
         if (!c.h_mid.empty()) c.mid = A.take<int>(c.h_mid.size());
+        if (!c.h_midbig.empty()) c.midbig = A.take<int>(c.h_midbig.size());
         if (!c.h_huge.empty()) {
             c.huge = A.take<int>(c.h_huge.size());
             const int log2cap = std::max(log2_ceil_h(2LL * std::min(kmax_big, V)), 5);
@@ -485,6 +493,9 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     if (!c.h_big.empty())
         GSAP_CUDA(cudaMemcpyAsync(c.big, c.h_big.data(), sizeof(int) * c.h_big.size(), cudaMemcpyHostToDevice,
                                   c.stream));
+    if (!c.h_midbig.empty())
+        GSAP_CUDA(cudaMemcpyAsync(c.midbig, c.h_midbig.data(), sizeof(int) * c.h_midbig.size(),
+                                  cudaMemcpyHostToDevice, c.stream));
     if (!c.h_mid.empty())
         GSAP_CUDA(cudaMemcpyAsync(c.mid, c.h_mid.data(), sizeof(int) * c.h_mid.size(), cudaMemcpyHostToDevice,
                                   c.stream));

@@ -51,7 +51,8 @@ struct Ctx {
     std::vector<int> h_rowptr, h_cscptr;   // host copies (static) for batch accounting
     // vertices whose total degree exceeds the warp path's table (static list)
     int *mid = nullptr, *big = nullptr, *huge = nullptr;   // 128 < k <= 256 / <= 1024 / > 1024 entries
-    std::vector<int> h_mid, h_big, h_huge;
+    int *midbig = nullptr;                                 // 128 < k <= 1024 (latency mode's CTA list)
+    std::vector<int> h_mid, h_big, h_huge, h_midbig;
     size_t big_table_slots = 0;            // per-CTA global table capacity (slots)
     int *big_tables = nullptr;             // global tables for very large vertices
 

@@ -1240,12 +1240,27 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         };
         int nmid = 0, kmid = 0, nbig = 0, kbig = 0, nhuge = 0, khuge = 0;
         const int omid = range(c.h_mid, nmid, kmid);
+        int obig = range(c.h_big, nbig, kbig);
+#ifndef GSAP_GROUPS_LATENCY
+#define GSAP_GROUPS_LATENCY 0
+#endif
+        // latency mode (build flag): few group vertices in the batch -- the
+        // 129..256-entry vertices get a whole CTA each like the bigger ones
+        if (GSAP_GROUPS_LATENCY && nmid > 0 && nmid + nbig <= 2 * 148 * GSAP_GROUPS_MINB) {
+            int n2 = 0, k2 = 0;
+            const int o2 = range(c.h_midbig, n2, k2);
+            a.list = c.midbig + o2;
+            a.list_count = n2;
+            a.big_log2 = std::max(log2_ceil(2LL * std::min(k2, c.B)), 5);
+            a.nbig_ctas = std::min(n2, c.test_grid > 0 ? c.test_grid : 148 * 16);
+            nmid = 0;
+            nbig = 0;
+        }
         if (nmid > 0) {
             a.mlist = c.mid + omid;
             a.mlist_count = nmid;
             a.nmid_ctas = std::min((nmid + 3) / 4, c.test_grid > 0 ? c.test_grid : 148 * 16);
         }
-        const int obig = range(c.h_big, nbig, kbig);
         const int ohuge = range(c.h_huge, nhuge, khuge);
         if (nbig > 0) {
             a.list = c.big + obig;
