@@ -120,6 +120,20 @@ union CoopSmem {
     int scan[8];
 };
 
+#ifdef GSAP_COOP_PROF   // experiment builds only (tools/build_variant.sh): per-phase times by printf
+__device__ unsigned long long g_coop_t[8];
+__device__ unsigned g_coop_done;
+GSAP_DEV unsigned long long coop_now() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+#define COOP_MARK(i) \
+    if (blockIdx.x == 0 && threadIdx.x == 0) g_coop_t[i] = coop_now();
+#else
+#define COOP_MARK(i)
+#endif
+
 template <typename K>
 __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
     extern __shared__ __align__(16) unsigned char coop_raw[];
@@ -128,6 +142,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
     const int gtid = blockIdx.x * blockDim.x + threadIdx.x, gthreads = gridDim.x * blockDim.x;
     const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
     const int gwarp = gtid >> 5, gwarps = gthreads >> 5;
+    COOP_MARK(0)
     // P0
     for (int x = gtid; x <= B; x += gthreads) {
 #pragma unroll
@@ -139,6 +154,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
     }
     if (gtid < 3) a.nlong[gtid] = 0;   // [0, 1] long lines per side, [2] P4a work counter
     grid_sync(a.bar);
+    COOP_MARK(1)
     // P1
     for (int v = gtid; v < V; v += gthreads) {
         const int x = __ldg(a.b + v);
@@ -152,6 +168,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
         if (ki) atomicAdd(a.sd[1].deg + x, ki);
     }
     grid_sync(a.bar);
+    COOP_MARK(2)
     // P2
     if (blockIdx.x < 2) {
         CoopSide &sd = a.sd[blockIdx.x];
@@ -161,6 +178,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             a.rcp[x] = 1.0 / ((double)a.sd[0].deg[x] + (double)a.sd[1].deg[x] + (double)B);
     }
     grid_sync(a.bar);
+    COOP_MARK(3)
     // P3: scatter, 32 (side, vertex) tasks per warp step (segsort.cuh scatter_batched)
     {
         const ScatterSide<K> s0{a.sd[0].gptr, a.sd[0].gidx, a.sd[0].gw, a.sd[0].off, a.sd[0].cur,
@@ -170,6 +188,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
         scatter_batched<K>(s0, s1, 2, V, a.b, gwarp, gwarps);
     }
     grid_sync(a.bar);
+    COOP_MARK(4)
     // P4b: long lines first, one CTA each (static: CTA i takes long lines i, i + grid, ...)
     {
         const int n0 = a.nlong[0], n1 = a.nlong[1];
@@ -195,6 +214,7 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             __syncthreads();
         }
     }
+    COOP_MARK(5)
     __syncthreads();   // the shared memory changes role
     // P4a: short lines, one warp each (bitonic + RLE in registers / shared
     // memory), fetched two at a time from a work counter: warps of CTAs that
@@ -251,6 +271,20 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
         }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *a.d_nnz = a.sd[0].off[B];   // the extent E (padding has cnt 0)
+#ifdef GSAP_COOP_PROF
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        if (atomicAdd(&g_coop_done, 1u) == gridDim.x - 1) {
+            const unsigned long long t6 = coop_now();
+            g_coop_done = 0;
+            printf("COOP B=%d nlong=%d,%d P0 %.2f P1 %.2f P2 %.2f P3 %.2f P4b0 %.2f P4 %.2f total %.2f us\n", B,
+                   a.nlong[0], a.nlong[1], (g_coop_t[1] - g_coop_t[0]) * 1e-3, (g_coop_t[2] - g_coop_t[1]) * 1e-3,
+                   (g_coop_t[3] - g_coop_t[2]) * 1e-3, (g_coop_t[4] - g_coop_t[3]) * 1e-3,
+                   (g_coop_t[5] - g_coop_t[4]) * 1e-3, (t6 - g_coop_t[4]) * 1e-3, (t6 - g_coop_t[0]) * 1e-3);
+        }
+    }
+#endif
 }
 
 }  // namespace gsap

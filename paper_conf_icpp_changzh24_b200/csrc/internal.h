@@ -85,7 +85,7 @@ struct Ctx {
     size_t counts_cap = 0, scan_tmp_cap = 0;
     // segmented rebuild scratch (per line: length, offset, cursor, runs; line lists)
     int *seg_len = nullptr, *seg_cur = nullptr, *seg_nnz = nullptr, *seg_listW = nullptr,
-        *seg_listC = nullptr, *seg_ctr = nullptr, *xl_hp = nullptr;
+        *seg_listC = nullptr, *seg_ctr = nullptr, *xl_hp = nullptr, *seg_listM = nullptr;
     unsigned long long *xl_keys = nullptr;   // 2E: long-segment sort scratch
     // persistent sparse rebuild (coop.cuh; small graphs): the column side's
     // line scratch, its long-segment scratch, the grid barrier

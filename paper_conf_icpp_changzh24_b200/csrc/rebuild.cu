@@ -753,7 +753,7 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     K *seg = reinterpret_cast<K *>(c.keys0);
     GSAP_CUDA(cudaMemsetAsync(c.seg_len, 0, sizeof(int) * (size_t)B, c.stream));
     GSAP_CUDA(cudaMemsetAsync(c.seg_cur, 0, sizeof(int) * (size_t)B, c.stream));
-    GSAP_CUDA(cudaMemsetAsync(c.seg_ctr, 0, 4 * sizeof(int), c.stream));
+    GSAP_CUDA(cudaMemsetAsync(c.seg_ctr, 0, 8 * sizeof(int), c.stream));
     k_line_len<<<grid_for(V, 256), 256, 0, c.stream>>>(V, gptr, c.b, c.seg_len);
     ++c.launches;
     device_scan<int>(c.seg_len, ptr, nullptr, B, false, c.scan_tmp, ptr + B, L);
@@ -761,11 +761,13 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
                                                                                 c.seg_cur, seg);
     const LineOut out{cum, end, deg};
     k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, ptr, c.seg_nnz, c.seg_listW, c.seg_listC,
-                                                           c.seg_ctr, out, extent, SEG_WARP_MAX_MK);
+                                                           c.seg_ctr, out, extent, SEG_WARP_MAX_MK, c.seg_listM);
     const int gw_ = (int)std::min<long long>(((long long)B + SEG_WARPS - 1) / SEG_WARPS, 148LL * 16);
     per_device((const void *)k_segsort_warp<K, 2>, [] {
         GSAP_CUDA(cudaFuncSetAttribute(k_segsort_warp<K, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)seg_warp2_smem<K>()));
+        GSAP_CUDA(cudaFuncSetAttribute(k_segsort_warp<K, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)seg_warp2_smem<K>(512)));
         return 1;
     });
     const int cb = bits_for(B);
@@ -773,10 +775,13 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
                                                               c.seg_nnz, out);
     k_segsort_warp<K, 1><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, cb, idx, cnt,
                                                               c.seg_nnz, out);
+    k_segsort_warp<K, 3><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(512), c.stream>>>(B, ptr, seg, c.seg_listM,
+                                                                                   c.seg_ctr, cb, idx, cnt,
+                                                                                   c.seg_nnz, out);
     k_segsort_warp<K, 2><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(), c.stream>>>(B, ptr, seg, c.seg_listC,
                                                                                 c.seg_ctr, cb, idx, cnt,
                                                                                 c.seg_nnz, out);
-    c.launches += 2;
+    c.launches += 4;
     const int gc = (int)std::min<long long>(std::max(1, B / 4), 148LL * 4);
     k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(ptr, seg, c.seg_listC, c.seg_ctr, bits_for(B), idx, cnt,
                                                c.seg_nnz, out);

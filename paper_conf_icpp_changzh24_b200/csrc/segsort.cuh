@@ -252,7 +252,7 @@ __global__ void k_line_scatter_batched(int V, const int *__restrict__ gptr, cons
 // 4a. classify lines by segment length
 __global__ void k_line_classify(int B, const int *__restrict__ off, int *__restrict__ nnz, int *__restrict__ listW,
                                 int *__restrict__ listC, int *__restrict__ counters, LineOut out,
-                                int *__restrict__ extent, int warp_max) {
+                                int *__restrict__ extent, int warp_max, int *__restrict__ listM) {
     if (extent && blockIdx.x == 0 && threadIdx.x == 0) *extent = off[B];
     for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < B; x += gridDim.x * blockDim.x) {
         const int L = off[x + 1] - off[x];
@@ -265,6 +265,7 @@ __global__ void k_line_classify(int B, const int *__restrict__ off, int *__restr
         }
         else if (L <= 128) listW[atomicAdd(counters, 1)] = x;                           // warp mode 0
         else if (L <= 256) listW[B - 1 - atomicAdd(counters + 2, 1)] = x;               // warp mode 1
+        else if (listM && L <= 512) listM[atomicAdd(counters + 4, 1)] = x;              // warp mode 3
         else if (L <= warp_max) listC[B - 1 - atomicAdd(counters + 3, 1)] = x;          // warp mode 2
         else listC[atomicAdd(counters + 1, 1)] = x;                                      // CTA
     }
@@ -383,7 +384,9 @@ GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict_
 // occupancy of the common one:
 //   MODE 0: <= 128 entries, bitonic + RLE in registers;
 //   MODE 1: 129..256 entries in registers (8 per lane);
-//   MODE 2: 257..SEG_WARP_MAX_MK entries: the stable LSD radix sort over the
+//   MODE 3: 257..512 entries, the MODE 2 sort with half-size buffers (own
+//           list: more CTAs per SM for the shorter lines);
+//   MODE 2: 257 (513 with MODE 3)..SEG_WARP_MAX_MK entries: the stable LSD radix sort over the
 //           key's block bits (cta_radix_sort with 32 threads: 4-bit digits,
 //           per-lane packed counters, no atomics; O(L) per pass instead of
 //           bitonic's O(L log^2 L)) in dynamic shared memory, then RLE.
@@ -392,8 +395,8 @@ GSAP_DEV int warp_segsort_rle(const K *__restrict__ src, int L, int *__restrict_
 #endif
 constexpr int SEG_WARP_MAX_MK = GSAP_SEG_WARP_MAX_MK;   // multi-kernel path: longer lines go to the CTA sorts
 template <typename K>
-constexpr size_t seg_warp2_smem() {
-    return (size_t)SEG_WARPS * (2 * SEG_WARP_MAX_MK * sizeof(K) + 8 * 32 * sizeof(unsigned));
+constexpr size_t seg_warp2_smem(int cap = SEG_WARP_MAX_MK) {
+    return (size_t)SEG_WARPS * (2 * (size_t)cap * sizeof(K) + 8 * 32 * sizeof(unsigned));
 }
 
 template <typename K, int NT>
@@ -405,11 +408,13 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const in
                                                                  const int *__restrict__ counters, int col_bits,
                                                                  int *__restrict__ tcol, int *__restrict__ tcnt,
                                                                  int *__restrict__ nnz, LineOut out) {
-    extern __shared__ __align__(16) unsigned char seg_dyn[];   // MODE 2: SEG_WARPS x (2 key buffers) + counters
+    extern __shared__ __align__(16) unsigned char seg_dyn[];   // MODE 2/3: SEG_WARPS x (2 key buffers) + counters
+    constexpr int CAP = MODE == 3 ? 512 : SEG_WARP_MAX_MK;     // key buffer per warp (MODE 2 / 3)
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int n_lines = counters[MODE == 0 ? 0 : MODE == 1 ? 2 : 3];
+    const int n_lines = counters[MODE == 0 ? 0 : MODE == 1 ? 2 : MODE == 2 ? 3 : 4];
     for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
-        const int x = MODE == 0 ? listW[li] : listW[B - 1 - li];   // MODE 2: listW is the CTA list (listC)
+        // MODE 2: listW is the CTA list (listC), filled from its back; MODE 3: listM, from its front
+        const int x = (MODE == 0 || MODE == 3) ? listW[li] : listW[B - 1 - li];
         const int o = off[x], L = off[x + 1] - o;
         int u;
         if (MODE == 1) {
@@ -419,10 +424,10 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const in
             else if (L <= 64) u = warp_segsort_rle<K, 2>(seg + o, L, tcol + o, tcnt + o);
             else u = warp_segsort_rle<K, 4>(seg + o, L, tcol + o, tcnt + o);
         } else {
-            K *ka = reinterpret_cast<K *>(seg_dyn) + (size_t)w * 2 * SEG_WARP_MAX_MK;
-            K *kb = ka + SEG_WARP_MAX_MK;
+            K *ka = reinterpret_cast<K *>(seg_dyn) + (size_t)w * 2 * CAP;
+            K *kb = ka + CAP;
             unsigned *cntp = reinterpret_cast<unsigned *>(reinterpret_cast<K *>(seg_dyn) +
-                                                          (size_t)SEG_WARPS * 2 * SEG_WARP_MAX_MK) + w * 8 * 32;
+                                                          (size_t)SEG_WARPS * 2 * CAP) + w * 8 * 32;
             for (int i = lane; i < L; i += 32) ka[i] = seg[o + i];
             __syncwarp();
             K *keys = cta_radix_sort<K, 32>(ka, kb, L, col_bits, cntp, nullptr);
