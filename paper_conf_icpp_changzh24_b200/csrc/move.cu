@@ -1370,16 +1370,17 @@ GSAP_DEV void log_move(const MoveLog &lg, bool mv, int v, int old) {
 
 // n_eval (nullable): += the proposals with s != b[v] (the moves that were
 // evaluated, R:Z13) -- counted before b is written
-__global__ void __launch_bounds__(256) k_apply(int first, int count, const int *__restrict__ s,
+__global__ void __launch_bounds__(APPLY_CHUNK) k_apply(int first, int count, const int *__restrict__ s,
                                                const unsigned char *__restrict__ acc,
                                                const double *__restrict__ dS, int *__restrict__ b,
                                                double *__restrict__ partials, int *__restrict__ nacc,
                                                unsigned long long *__restrict__ n_eval, MoveLog lg) {
-    __shared__ double sh[8];
+    __shared__ double sh[APPLY_CHUNK / 32];
     const int base = blockIdx.x * APPLY_CHUNK;
     double sum = 0.0;
     int na = 0, ne = 0;
-    for (int k = threadIdx.x; k < APPLY_CHUNK; k += 256) {
+    {   // one entry of the chunk per thread
+        const int k = threadIdx.x;
         const int i = base + k;
         if (i < count && n_eval) ne += s[i] != b[first + i];
         if (lg.oldb) {
@@ -1403,7 +1404,7 @@ __global__ void __launch_bounds__(256) k_apply(int first, int count, const int *
     __syncthreads();
     if (threadIdx.x == 0 && partials) {
         double t = 0.0;
-        for (int w = 0; w < 8; ++w) t += sh[w];
+        for (int w = 0; w < APPLY_CHUNK / 32; ++w) t += sh[w];
         partials[blockIdx.x] = t;
     }
 }
@@ -1427,18 +1428,19 @@ __global__ void __launch_bounds__(256) k_sum_partials(const double *__restrict__
 // k_apply + the ordered sum of its partials in one launch: the last CTA to
 // finish (arrival counter, reset by that CTA) adds partials[0, nb) in index
 // order to *dsum -- the same fixed-order sum as k_sum_partials
-__global__ void __launch_bounds__(256) k_apply_sum(int first, int count, const int *__restrict__ s,
+__global__ void __launch_bounds__(APPLY_CHUNK) k_apply_sum(int first, int count, const int *__restrict__ s,
                                                    const unsigned char *__restrict__ acc,
                                                    const double *__restrict__ dS, int *__restrict__ b,
                                                    double *__restrict__ partials, int *__restrict__ nacc,
                                                    unsigned *__restrict__ arrivals, double *__restrict__ dsum,
                                                    unsigned long long *__restrict__ n_eval, MoveLog lg) {
-    __shared__ double sh[8];
+    __shared__ double sh[APPLY_CHUNK / 32];
     __shared__ bool last;
     const int base = blockIdx.x * APPLY_CHUNK;
     double sum = 0.0;
     int na = 0, ne = 0;
-    for (int k = threadIdx.x; k < APPLY_CHUNK; k += 256) {
+    {   // one entry of the chunk per thread
+        const int k = threadIdx.x;
         const int i = base + k;
         if (i < count && n_eval) ne += s[i] != b[first + i];
         if (lg.oldb) {
@@ -1462,7 +1464,7 @@ __global__ void __launch_bounds__(256) k_apply_sum(int first, int count, const i
     __syncthreads();
     if (threadIdx.x == 0) {
         double t = 0.0;
-        for (int w = 0; w < 8; ++w) t += sh[w];
+        for (int w = 0; w < APPLY_CHUNK / 32; ++w) t += sh[w];
         partials[blockIdx.x] = t;
         __threadfence();
         last = atomicAdd(arrivals, 1u) == gridDim.x - 1;
@@ -1471,9 +1473,11 @@ __global__ void __launch_bounds__(256) k_apply_sum(int first, int count, const i
     if (!last) return;
     __threadfence();
     double v = 0.0;
-    for (int i = threadIdx.x; i < (int)gridDim.x; i += 256) v += *((volatile double *)(partials + i));
+    // the order of k_sum_partials: 256 strided lanes, warp trees, 8 warp sums
+    if (threadIdx.x < 256)
+        for (int i = threadIdx.x; i < (int)gridDim.x; i += 256) v += *((volatile double *)(partials + i));
     v = warp_sum(v);
-    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = v;
+    if ((threadIdx.x & 31) == 0 && threadIdx.x < 256) sh[threadIdx.x >> 5] = v;
     __syncthreads();
     if (threadIdx.x == 0) {
         double t = 0.0;
@@ -1523,7 +1527,7 @@ void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned cha
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
     const MoveLog lg = move_log(c);
-    k_apply_sum<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, c.b, c.partials, nacc,
+    k_apply_sum<<<nb, APPLY_CHUNK, 0, c.stream>>>(first, count, s, acc, dS, c.b, c.partials, nacc,
                                           reinterpret_cast<unsigned *>(c.scal_i + 4), dsum, n_eval, lg);
     c.launches += 1;
     GSAP_CHECK_LAUNCH();
@@ -1535,7 +1539,7 @@ void launch_partials(Ctx &c, int first, int count, const int *s, const unsigned 
                      double *partials) {
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
-    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, dS, nullptr, partials, nullptr, nullptr,
+    k_apply<<<nb, APPLY_CHUNK, 0, c.stream>>>(first, count, s, acc, dS, nullptr, partials, nullptr, nullptr,
                                       MoveLog{nullptr, nullptr, nullptr});
     ++c.launches;
     GSAP_CHECK_LAUNCH();
@@ -1547,7 +1551,7 @@ void launch_apply_gathered(Ctx &c, int first, int count, const int *s, const uns
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
     const MoveLog lg = move_log(c);
-    k_apply<<<nb, 256, 0, c.stream>>>(first, count, s, acc, nullptr, c.b, nullptr, nacc, n_eval, lg);
+    k_apply<<<nb, APPLY_CHUNK, 0, c.stream>>>(first, count, s, acc, nullptr, c.b, nullptr, nacc, n_eval, lg);
     k_sum_partials<<<1, 256, 0, c.stream>>>(partials, n, dsum, 1);
     c.launches += 2;
     GSAP_CHECK_LAUNCH();
