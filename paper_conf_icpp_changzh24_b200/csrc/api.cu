@@ -120,6 +120,24 @@ static void graph_release_events(Ctx &c) {
     c.graph_ev.clear();
 }
 
+// profile mode outside graph capture: one launch of a role timed on `st`
+// (the MOVE roles run concurrently, so each is measured on its own stream)
+cudaEvent_t role_begin(Ctx &c, KClass &k, cudaStream_t st) {
+    if (!c.prm.profile || c.capturing) return nullptr;
+    cudaEvent_t e = ev_get(k);
+    GSAP_CUDA(cudaEventRecord(e, st));
+    return e;
+}
+
+void role_end(Ctx &c, KClass &k, cudaEvent_t e0, cudaStream_t st) {
+    if (!e0) return;
+    cudaEvent_t e1 = ev_get(k);
+    GSAP_CUDA(cudaEventRecord(e1, st));
+    k.launches += 1;
+    k.pending.emplace_back(e0, e1);
+    if (k.pending.size() > 4096) kc_resolve(c, k);
+}
+
 void kc_resolve(Ctx &c, KClass &k) {
     (void)c;
     for (auto &p : k.pending) {
@@ -244,7 +262,7 @@ static void free_ctx(Ctx &c) {
     c.arena = nullptr;
     if (c.h_scal) cudaFreeHost(c.h_scal);
     if (c.h_int) cudaFreeHost(c.h_int);
-    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl, &c.k_comm}) {
+    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl, &c.k_comm, &c.k_groups, &c.k_warps}) {
         for (auto &p : k->pending) {
             cudaEventDestroy(p.first);
             cudaEventDestroy(p.second);
@@ -1052,7 +1070,12 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
 }
 
 static void fill_stats(Ctx &c, gsap_stats *out) {
-    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl, &c.k_comm}) kc_resolve(c, *k);
+    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl, &c.k_comm, &c.k_groups, &c.k_warps})
+        kc_resolve(c, *k);
+    if (getenv("GSAP_TIMING") && (c.k_groups.launches || c.k_warps.launches))
+        fprintf(stderr, "[gsap] MOVE roles (profile, outside graphs): group role %lld launches %.3f ms, "
+                "warp role %lld launches %.3f ms\n", c.k_groups.launches, c.k_groups.ms, c.k_warps.launches,
+                c.k_warps.ms);
     gsap_stats s = c.st;
     unsigned long long ne = 0;
     GSAP_CUDA(cudaMemcpyAsync(&ne, c.n_eval, sizeof(ne), cudaMemcpyDeviceToHost, c.stream));
@@ -1405,7 +1428,7 @@ gsap_status gsap_reset_stats(gsap_ctx *ctx) {
     API_TRY
     REQUIRE(ctx, GSAP_EINVAL, "NULL ctx");
     Ctx &c = ctx->c;
-    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl, &c.k_comm}) {
+    for (KClass *k : {&c.k_move, &c.k_rebuild, &c.k_merge, &c.k_mdl, &c.k_comm, &c.k_groups, &c.k_warps}) {
         kc_resolve(c, *k);
         k->ms = 0;
         k->bytes = 0;

@@ -148,6 +148,7 @@ struct Ctx {
     // accounting
     long long launches = 0;
     KClass k_move, k_rebuild, k_merge, k_mdl, k_comm;
+    KClass k_groups, k_warps;   // profile mode, outside graphs: the two MOVE roles timed on their own streams
     gsap_stats st{};
     std::vector<double> move_bytes_per_batch;   // algorithmic bytes per MOVE launch
 
@@ -190,6 +191,8 @@ int per_device(const void *key, const std::function<int()> &f);
 void kc_begin(Ctx &c, KClass &k, cudaEvent_t *ev);
 void kc_end(Ctx &c, KClass &k, cudaEvent_t ev, double bytes);
 void kc_resolve(Ctx &c, KClass &k);
+cudaEvent_t role_begin(Ctx &c, KClass &k, cudaStream_t st);
+void role_end(Ctx &c, KClass &k, cudaEvent_t e0, cudaStream_t st);
 
 // rebuild.cu
 void build_graph_device(Ctx &c);                 // CSC, esrc, degrees (create time)

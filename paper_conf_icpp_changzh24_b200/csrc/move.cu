@@ -1289,8 +1289,10 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     if (ggrid > 0) {   // the group roles run beside the warp role (fork / join on the side stream)
         GSAP_CUDA(cudaEventRecord(c.ev_fork, c.stream));
         GSAP_CUDA(cudaStreamWaitEvent(c.side, c.ev_fork, 0));
+        cudaEvent_t rg = role_begin(c, c.k_groups, c.side);
         if (c.weighted) k_move_groups<true><<<ggrid, MOVE_WARPS * 32, 0, c.side>>>(a);
         else k_move_groups<false><<<ggrid, MOVE_WARPS * 32, 0, c.side>>>(a);
+        role_end(c, c.k_groups, rg, c.side);
         ++c.launches;
         GSAP_CHECK_LAUNCH();
         GSAP_CUDA(cudaEventRecord(c.ev_join, c.side));
@@ -1304,6 +1306,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         return 1;
     });
     const bool dense = a.m.dense != nullptr;
+    cudaEvent_t rw = role_begin(c, c.k_warps, c.stream);
     if (sorted) {
         per_device((const void *)k_move_half<false, 1>, [] {
             const int sm = (int)MOVE_SMEM;
@@ -1334,6 +1337,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         ++c.launches;
     }
     GSAP_CHECK_LAUNCH();
+    role_end(c, c.k_warps, rw, c.stream);
     if (ggrid > 0) GSAP_CUDA(cudaStreamWaitEvent(c.stream, c.ev_join, 0));
     // algorithmic bytes: the adjacency ids (+
     // weights), 2 x 16 B of row / column pointers and 13 B of per-vertex
