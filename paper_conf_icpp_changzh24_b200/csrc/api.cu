@@ -415,23 +415,28 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
             }
         }
         c.b = A.take<int>(Vs);
+        c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, (size_t)1 << 24), (size_t)1 << 29);
+        c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
+        if (c.prm.dense_max_B > 0)
+            c.dense_cap = std::min<size_t>(c.dense_cap, (size_t)c.prm.dense_max_B * (size_t)c.prm.dense_max_B);
+        // the lines of M: nnz <= E (sparse, compact or padded by degree) or B^2
+        // (dense regime above SMALL_MAX_B: padded, line x at x B)
+        const size_t Ls = std::max(Es, c.dense_cap);
         c.bm_rowptr = A.take<int>(Vs + 1);
         c.bm_colptr = A.take<int>(Vs + 1);
-        c.bm_col = A.take<int>(Es);
-        c.bm_cnt = A.take<int>(Es);
-        c.bm_cum = A.take<int>(Es);
-        c.bm_row = A.take<int>(Es);
-        c.bm_ccnt = A.take<int>(Es);
-        c.bm_ccum = A.take<int>(Es);
+        c.bm_col = A.take<int>(Ls);
+        c.bm_cnt = A.take<int>(Ls);
+        c.bm_cum = A.take<int>(Ls);
+        c.bm_row = A.take<int>(Ls);
+        c.bm_ccnt = A.take<int>(Ls);
+        c.bm_ccum = A.take<int>(Ls);
         c.dout = A.take<int>(Vs);
         c.din = A.take<int>(Vs);
         c.bm_rowend = A.take<int>(Vs);
         c.bm_colend = A.take<int>(Vs);
         c.d_nnz = A.take<int>(1);
-        c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, (size_t)1 << 24), (size_t)1 << 29);
-        c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
-        if (c.prm.dense_max_B > 0)
-            c.dense_cap = std::min<size_t>(c.dense_cap, (size_t)c.prm.dense_max_B * (size_t)c.prm.dense_max_B);
+        c.line_dirty = A.take<unsigned char>(2 * Vs);
+        c.dl_arrive = A.take<unsigned>(1);
         c.dense = A.take<int>(c.dense_cap);
         c.rcp = A.take<double>(Vs);
         c.ft = A.take<double2>(FT_N);
@@ -480,7 +485,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.acc = A.take<unsigned char>(Vs + pad);
         c.best = A.take<int>(Vs + pad);
         c.dSbest = A.take<double>(Vs + pad);
-        c.partials = A.take<double>(VE / 512 + 1024);   // >= max(E, B) / MDL_CHUNK, V / APPLY_CHUNK + ranks
+        // >= the MDL extent (max(E, B), or B^2 padded dense) / MDL_CHUNK, V / APPLY_CHUNK + ranks
+        c.partials = A.take<double>(std::max(VE, c.dense_cap) / 512 + 1024);
         c.scal = A.take<double>(8);
         c.scal_i = A.take<int>(8);
         c.n_eval = A.take<unsigned long long>(1);
@@ -548,6 +554,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         GSAP_CUDA(cudaMemcpyAsync(c.ft, ft.data(), sizeof(double2) * FT_N, cudaMemcpyHostToDevice, c.stream));
     }
     GSAP_CUDA(cudaMemsetAsync(c.coop_bar, 0, 2 * sizeof(unsigned), c.stream));
+    GSAP_CUDA(cudaMemsetAsync(c.line_dirty, 0, 2 * (size_t)V, c.stream));
+    GSAP_CUDA(cudaMemsetAsync(c.dl_arrive, 0, sizeof(unsigned), c.stream));
     if (c.small_acc)
         GSAP_CUDA(cudaMemsetAsync(c.small_acc, 0, sizeof(int) * SMALL_MAX_B * SMALL_MAX_B, c.stream));
     GSAP_CUDA(cudaMallocHost(&c.h_scal, 8 * sizeof(double)));

@@ -139,6 +139,11 @@ struct Ctx {
     } delta;
     int *oldb = nullptr, *moved = nullptr, *moved_cnt = nullptr;
     int *dnnz_r = nullptr, *dnnz_c = nullptr;   // dense regime: non-zeros per row of M / of Mt (kept for N2)
+    // dense regime above SMALL_MAX_B: the lines of M padded to B entries (line
+    // x at x B); N2 marks the lines a batch changed and re-compacts only those
+    bool dense_padded = false;
+    unsigned char *line_dirty = nullptr;   // [2 B]: rows of M, then rows of Mt
+    unsigned *dl_arrive = nullptr;         // last-CTA counter of k_dense_lines
 
     // CUDA-graph capture of an MCMC iteration (N1: launch overhead, §5)
     unsigned *d_itr = nullptr;     // MCMC iteration read by k_move (device scalar)

@@ -54,7 +54,9 @@ __global__ void __launch_bounds__(256) k_mdl_final(const double *__restrict__ pa
 void launch_data_term(Ctx &c) {
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_mdl, &ev);
-    const long long n = std::max<long long>(std::max<long long>(c.E, c.B), 1);
+    // the extent of the cnt array: nnz <= E, or B^2 for the padded dense lines
+    long long n = std::max<long long>(std::max<long long>(c.E, c.B), 1);
+    if (c.dense_padded) n = std::max(n, (long long)c.B * c.B);
     const int nb = (int)((n + MDL_CHUNK - 1) / MDL_CHUNK);
     k_mdl_partials<<<nb, 256, 0, c.stream>>>(c.bm_cnt, c.d_nnz, c.dout, c.din, c.B, c.partials);
     k_mdl_final<<<1, 256, 0, c.stream>>>(c.partials, nb, c.scal + 1);

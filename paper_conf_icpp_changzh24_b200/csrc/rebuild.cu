@@ -183,134 +183,6 @@ __global__ void k_transpose(const int *__restrict__ M, int B, int *__restrict__ 
 
 
 
-// both dense matrices (M: lines x < B, its transpose: lines x >= B) in one
-// launch: non-zeros and sum per line; four consecutive entries per lane per
-// step (128 per warp step, independent loads)
-// skip (nullable): the batch's moved-vertex count; 0 = M unchanged, nothing to do
-__global__ void k_row_stats2(const int *__restrict__ M, const int *__restrict__ Mt, int B, int *__restrict__ nnzA,
-                             int *__restrict__ sumA, int *__restrict__ nnzB, int *__restrict__ sumB,
-                             const int *__restrict__ skip) {
-    if (skip && *skip == 0) return;
-    const int lane = threadIdx.x & 31;
-    for (int x2 = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x2 < 2 * B; x2 += (gridDim.x * blockDim.x) >> 5) {
-        const bool t = x2 >= B;
-        const int x = t ? x2 - B : x2;
-        const int *__restrict__ R = (t ? Mt : M) + (size_t)x * B;
-        int c = 0, s = 0;
-#pragma unroll 4
-        for (int y0 = 4 * lane; y0 < B; y0 += 128) {   // independent loads: unrolled, in flight together
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-                const int v = y0 + k < B ? __ldg(R + y0 + k) : 0;
-                c += v != 0;
-                s += v;
-            }
-        }
-        c = __reduce_add_sync(FULL, c);
-        s = __reduce_add_sync(FULL, s);
-        if (lane == 0) {
-            (t ? nnzB : nnzA)[x] = c;
-            (t ? sumB : sumA)[x] = s;
-        }
-    }
-}
-
-// two exclusive scans of n <= 32K ints, one CTA each (dense regime: B <= 16384)
-__global__ void __launch_bounds__(1024) k_scan2(const int *a0, int *o0, const int *a1, int *o1, int n,
-                                                const int *__restrict__ skip) {
-    if (skip && *skip == 0) return;
-    __shared__ int sh[32];
-    const int *in = blockIdx.x ? a1 : a0;
-    int *out = blockIdx.x ? o1 : o0;
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    int carry = 0;
-    for (int base = 0; base < n; base += 1024 * 8) {
-        int v[8], sm = 0;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-            const int idx = base + threadIdx.x * 8 + i;
-            v[i] = idx < n ? in[idx] : 0;
-            sm += v[i];
-        }
-        int x = sm;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int t = __shfl_up_sync(FULL, x, o);
-            if (lane >= o) x += t;
-        }
-        if (lane == 31) sh[w] = x;
-        __syncthreads();
-        int wb = 0, tot = 0;
-        for (int i = 0; i < 32; ++i) {
-            const int q = sh[i];
-            if (i < w) wb += q;
-            tot += q;
-        }
-        __syncthreads();
-        int ex = carry + wb + x - sm;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-            const int idx = base + threadIdx.x * 8 + i;
-            if (idx < n) out[idx] = ex;
-            ex += v[i];
-        }
-        carry += tot;
-    }
-    if (threadIdx.x == 0) out[n] = carry;
-}
-
-// compaction of both matrices + nnz + rcp = 1 / (d_x + B): a warp step
-// covers 128 consecutive entries, four per lane (one warp scan of the lane's
-// count and one of its sum per step instead of one per 32 entries)
-__global__ void k_row_compact2(const int *__restrict__ M, const int *__restrict__ Mt, int B,
-                               const int *__restrict__ ptrA, int *__restrict__ idxA, int *__restrict__ cntA,
-                               int *__restrict__ cumA, const int *__restrict__ ptrB, int *__restrict__ idxB,
-                               int *__restrict__ cntB, int *__restrict__ cumB, const int *__restrict__ dout,
-                               const int *__restrict__ din, double *__restrict__ rcp, int *__restrict__ d_nnz,
-                               const int *__restrict__ skip) {
-    if (skip && *skip == 0) return;
-    const int lane = threadIdx.x & 31;
-    if (blockIdx.x == 0 && threadIdx.x == 0) *d_nnz = ptrA[B];
-    for (int x2 = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x2 < 2 * B; x2 += (gridDim.x * blockDim.x) >> 5) {
-        const bool t = x2 >= B;
-        const int x = t ? x2 - B : x2;
-        const int *__restrict__ R = (t ? Mt : M) + (size_t)x * B;
-        int *__restrict__ idx = t ? idxB : idxA;
-        int *__restrict__ cnt = t ? cntB : cntA;
-        int *__restrict__ cum = t ? cumB : cumA;
-        int base = (t ? ptrB : ptrA)[x], run = 0;
-        if (!t && lane == 0) rcp[x] = 1.0 / ((double)dout[x] + (double)din[x] + (double)B);
-        int nxt[4];   // the next step's entries, loaded one step ahead
-#pragma unroll
-        for (int k = 0; k < 4; ++k) nxt[k] = 4 * lane + k < B ? __ldg(R + 4 * lane + k) : 0;
-        for (int y0 = 0; y0 < B; y0 += 128) {
-            const int y = y0 + 4 * lane;
-            int v[4], nz = 0, sm = 0;
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-                v[k] = nxt[k];
-                nxt[k] = y + 128 + k < B ? __ldg(R + y + 128 + k) : 0;
-                nz += v[k] != 0;
-                sm += v[k];
-            }
-            const int nzi = warp_incl_scan(nz), smi = warp_incl_scan(sm);
-            int p = base + nzi - nz, sc = run + smi - sm;
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-                sc += v[k];
-                if (v[k] != 0) {
-                    idx[p] = y + k;
-                    cnt[p] = v[k];
-                    cum[p] = sc;
-                    ++p;
-                }
-            }
-            base += __shfl_sync(FULL, nzi, 31);
-            run += __shfl_sync(FULL, smi, 31);
-        }
-    }
-}
-
 // ------------------------------------------------ dense, one kernel --
 // The whole dense rebuild as ONE persistent cooperative kernel (params.dense_coop).
 // The multi-kernel path (memset, histogram, transpose, stats, scan,
@@ -645,13 +517,22 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
                                                      const int *__restrict__ rowptr, const int *__restrict__ col,
                                                      const int *__restrict__ wgt, const int *__restrict__ cscptr,
                                                      const int *__restrict__ cscsrc, const int *__restrict__ cscwgt,
-                                                     int B, int *__restrict__ M, int *__restrict__ Mt) {
+                                                     int B, int *__restrict__ M, int *__restrict__ Mt,
+                                                     unsigned char *__restrict__ dirty) {
     const int n = *moved_cnt;
     const int lane = threadIdx.x & 31;
     for (int k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < n; k += (gridDim.x * blockDim.x) >> 5) {
         const int v = moved[k];
         const int r = oldb[v], s = b[v];
         const int ro = rowptr[v], nout = rowptr[v + 1] - ro;
+        const int ci = cscptr[v], nin = cscptr[v + 1] - ci;
+        // padded layout (dirty != nullptr): every line whose entries change --
+        // rows r, s (out-edges), columns r, s (in-edges), and the neighbours'
+        // lines marked below
+        if (dirty && lane == 0) {
+            if (nout) dirty[r] = dirty[s] = 1;
+            if (nin) dirty[B + r] = dirty[B + s] = 1;
+        }
         for (int j = lane; j < nout; j += 32) {
             const int w = col[ro + j];
             const int wt = wgt ? wgt[ro + j] : 1;
@@ -662,8 +543,8 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
             atomicAdd(M + (size_t)s * B + bn, wt);
             atomicAdd(Mt + (size_t)bo * B + r, -wt);
             atomicAdd(Mt + (size_t)bn * B + s, wt);
+            if (dirty) dirty[B + bo] = dirty[B + bn] = 1;
         }
-        const int ci = cscptr[v], nin = cscptr[v + 1] - ci;
         for (int j = lane; j < nin; j += 32) {
             const int w = cscsrc[ci + j];
             if (w >= first && w < first + count && acc[w - first]) continue;   // moved source (incl. v's self-loop)
@@ -673,7 +554,97 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
             atomicAdd(M + (size_t)bw * B + s, wt);
             atomicAdd(Mt + (size_t)r * B + bw, -wt);
             atomicAdd(Mt + (size_t)s * B + bw, wt);
+            if (dirty) dirty[bw] = 1;
         }
+    }
+}
+
+// the dense regime's lines in the PADDED layout (line x of M at x B, of Mt at
+// x B in the column arrays; end[x] marks its last run, cnt is zero beyond it):
+// one warp per line compacts the dense row (idx, cnt, in-line prefix cum) and
+// writes its sum (dout / din); DIRTY: only the lines k_dense_delta marked
+// (flag cleared), zeroing the counts its previous version left beyond the new
+// end; else every line (counts pre-zeroed).  The last CTA to finish writes
+// rcp = 1 / (d + B) for every block, the extent B^2 and the end pointer.
+// Integer work: the same runs as the compact layout, at other offsets.
+template <bool DIRTY>
+__global__ void __launch_bounds__(256) k_dense_lines(const int *__restrict__ M, const int *__restrict__ Mt, int B,
+                                                     unsigned char *__restrict__ dirty, int *__restrict__ ptrA,
+                                                     int *__restrict__ endA, int *__restrict__ idxA,
+                                                     int *__restrict__ cntA, int *__restrict__ cumA,
+                                                     int *__restrict__ ptrB, int *__restrict__ endB,
+                                                     int *__restrict__ idxB, int *__restrict__ cntB,
+                                                     int *__restrict__ cumB, int *__restrict__ dout,
+                                                     int *__restrict__ din, double *__restrict__ rcp,
+                                                     int *__restrict__ d_nnz, unsigned *__restrict__ arrive,
+                                                     const int *__restrict__ skip) {
+    if (skip && *skip == 0) return;   // the batch moved nothing: every line as it was
+    __shared__ bool last;
+    const int lane = threadIdx.x & 31;
+    for (int x2 = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x2 < 2 * B; x2 += (gridDim.x * blockDim.x) >> 5) {
+        if (DIRTY && !dirty[x2]) continue;   // warp-uniform
+        const bool t = x2 >= B;
+        const int x = t ? x2 - B : x2;
+        const int *__restrict__ R = (t ? Mt : M) + (size_t)x * B;
+        int *__restrict__ idx = t ? idxB : idxA;
+        int *__restrict__ cnt = t ? cntB : cntA;
+        int *__restrict__ cum = t ? cumB : cumA;
+        int *__restrict__ end = t ? endB : endA;
+        const int lo = x * B;
+        const int old_end = DIRTY ? end[x] : lo;
+        int base = lo, run = 0;
+        int nxt[4];   // the next step's entries, loaded one step ahead
+#pragma unroll
+        for (int k = 0; k < 4; ++k) nxt[k] = 4 * lane + k < B ? __ldg(R + 4 * lane + k) : 0;
+        for (int y0 = 0; y0 < B; y0 += 128) {
+            const int y = y0 + 4 * lane;
+            int v[4], nz = 0, sm = 0;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                v[k] = nxt[k];
+                nxt[k] = y + 128 + k < B ? __ldg(R + y + 128 + k) : 0;
+                nz += v[k] != 0;
+                sm += v[k];
+            }
+            const int nzi = warp_incl_scan(nz), smi = warp_incl_scan(sm);
+            int p = base + nzi - nz, sc = run + smi - sm;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                sc += v[k];
+                if (v[k] != 0) {
+                    idx[p] = y + k;
+                    cnt[p] = v[k];
+                    cum[p] = sc;
+                    ++p;
+                }
+            }
+            base += __shfl_sync(FULL, nzi, 31);
+            run += __shfl_sync(FULL, smi, 31);
+        }
+        if (DIRTY)
+            for (int q = base + lane; q < old_end; q += 32) cnt[q] = 0;   // the previous version's tail
+        if (lane == 0) {
+            (t ? ptrB : ptrA)[x] = lo;
+            end[x] = base;
+            (t ? din : dout)[x] = run;
+            if (DIRTY) dirty[x2] = 0;
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        last = atomicAdd(arrive, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    for (int x = threadIdx.x; x < B; x += blockDim.x)
+        rcp[x] = 1.0 / ((double)__ldcg(dout + x) + (double)__ldcg(din + x) + (double)B);
+    if (threadIdx.x == 0) {
+        ptrA[B] = B * B;
+        ptrB[B] = B * B;
+        *d_nnz = B * B;
+        *arrive = 0u;
     }
 }
 
@@ -682,20 +653,33 @@ __global__ void __launch_bounds__(256) k_dense_delta(const int *__restrict__ mov
 // compaction as in the full path (all three skip when no vertex moved; line
 // statistics kept incrementally by returning atomics measured slower: 20K
 // round 5 37.7 vs 35.6 us, round 8 33.4 vs 25.6 us)
+static void launch_dense_lines(Ctx &c, bool dirty, const int *skip) {
+    const int B = c.B;
+    const int rg = (int)std::min<long long>(((long long)2 * B + 7) / 8, 148LL * 8);
+    if (dirty)
+        k_dense_lines<true><<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.line_dirty, c.bm_rowptr, c.bm_rowend,
+                                                      c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr, c.bm_colend, c.bm_row,
+                                                      c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp, c.d_nnz, c.dl_arrive,
+                                                      skip);
+    else
+        k_dense_lines<false><<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.line_dirty, c.bm_rowptr, c.bm_rowend,
+                                                       c.bm_col, c.bm_cnt, c.bm_cum, c.bm_colptr, c.bm_colend,
+                                                       c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp, c.d_nnz,
+                                                       c.dl_arrive, skip);
+    ++c.launches;
+    GSAP_CHECK_LAUNCH();
+}
+
 static void rebuild_dense_delta(Ctx &c) {
     const int B = c.B;
     const int dg = (int)std::min<long long>(((long long)c.delta.count + 7) / 8, 148LL * 8);
     k_dense_delta<<<std::max(dg, 1), 256, 0, c.stream>>>(c.moved, c.moved_cnt, c.delta.first, c.delta.count,
                                                         c.delta.acc, c.oldb, c.b, c.rowptr, c.col, c.wgt, c.cscptr,
-                                                        c.cscsrc, c.cscwgt, B, c.dense, c.denseT);
-    const int rg = grid_for(2LL * B * 32, 256);
-    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.dnnz_r, c.dout, c.dnnz_c, c.din, c.moved_cnt);
-    k_scan2<<<2, 1024, 0, c.stream>>>(c.dnnz_r, c.bm_rowptr, c.dnnz_c, c.bm_colptr, B, c.moved_cnt);
-    k_row_compact2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum,
-                                             c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp,
-                                             c.d_nnz, c.moved_cnt);
-    c.launches += 4;
-    GSAP_CHECK_LAUNCH();
+                                                        c.cscsrc, c.cscwgt, B, c.dense, c.denseT, c.line_dirty);
+    ++c.launches;
+    launch_dense_lines(c, true, c.moved_cnt);   // the changed lines only, in place
+    c.dense_padded = true;
+    c.padded = true;
 }
 
 static void rebuild_dense(Ctx &c) {
@@ -722,16 +706,14 @@ static void rebuild_dense(Ctx &c) {
     }
     dim3 tg((B + 31) / 32, (B + 31) / 32), tb(32, 8);
     k_transpose<<<tg, tb, 0, c.stream>>>(c.dense, B, c.denseT);
-    const int rg = grid_for(2LL * B * 32, 256);
-    // line non-zero counts into the persistent dnnz_r / dnnz_c (the next
-    // rebuild may update them incrementally, N2)
-    k_row_stats2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.dnnz_r, c.dout, c.dnnz_c, c.din, nullptr);
-    k_scan2<<<2, 1024, 0, c.stream>>>(c.dnnz_r, c.bm_rowptr, c.dnnz_c, c.bm_colptr, B, nullptr);
-    k_row_compact2<<<rg, 256, 0, c.stream>>>(c.dense, c.denseT, B, c.bm_rowptr, c.bm_col, c.bm_cnt, c.bm_cum,
-                                             c.bm_colptr, c.bm_row, c.bm_ccnt, c.bm_ccum, c.dout, c.din, c.rcp,
-                                             c.d_nnz, nullptr);
-    c.launches += 4;
-    GSAP_CHECK_LAUNCH();
+    ++c.launches;
+    // the lines padded to B entries (a later N2 batch re-compacts only the
+    // lines it changed); counts zero beyond each line's end
+    GSAP_CUDA(cudaMemsetAsync(c.bm_cnt, 0, sizeof(int) * BB, c.stream));
+    GSAP_CUDA(cudaMemsetAsync(c.bm_ccnt, 0, sizeof(int) * BB, c.stream));
+    launch_dense_lines(c, false, nullptr);
+    c.dense_padded = true;
+    c.padded = true;
 }
 
 // ---------------------------------------------------------------- sparse --
@@ -891,14 +873,16 @@ void rebuild(Ctx &c) {
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_rebuild, &ev);
     const bool was_dense = c.dense_mode && c.dense_B == c.B;
+    const bool was_padded = c.dense_padded && was_dense;
     c.dense_mode = dense_ok(c, c.B);
-    c.padded = false;   // set by the multi-kernel sparse path
+    c.padded = false;         // set by the multi-kernel sparse path and the padded dense lines
+    c.dense_padded = false;   // set by rebuild_dense (N2 on) and kept by the delta path
     if (c.delta.pending && was_dense && c.dense_mode && c.E > 0 && c.prm.dense_coop && c.B <= SMALL_MAX_B) {
         // N2 at small B: the persistent rebuild (one launch, measured faster than
         // the delta + compaction here), skipped when the batch moved nothing
         launch_rebuild_dense_coop<true>(c, c.moved_cnt);
-    } else if (c.delta.pending && was_dense && c.dense_mode && c.E > 0) {
-        rebuild_dense_delta(c);   // N2: M, Mt of the previous rebuild + the batch's moves
+    } else if (c.delta.pending && was_padded && c.dense_mode && c.E > 0) {
+        rebuild_dense_delta(c);   // N2: M, Mt and the padded lines of the previous rebuild + the batch's moves
     } else if (c.dense_mode && c.prm.dense_coop && c.E > 0 && c.B <= SMALL_MAX_B) {
         launch_rebuild_dense_coop<true>(c);
     } else if (c.dense_mode && c.prm.dense_coop == 2 && c.E > 0) {
