@@ -98,6 +98,10 @@ typedef struct {
                                  ONE weighted neighbour block per block, drawn per merge phase / MOVE
                                  batch and shared by every proposal that reaches that block (a MERGE
                                  outcome equal to r is redrawn uniformly over the other blocks) */
+    int32_t line_sort;        /* multi-kernel sparse rebuild of an unweighted graph: 1 (default) lines of
+                                 129..1024 entries sorted by one bucket pass + insertion sorts inside the
+                                 buckets (k_segsort_bucket); 0: register bitonic / warp radix sorts.
+                                 Same blockmodel bit for bit. */
 } gsap_params;
 
 /* multi-GPU: one process per GPU; NULL or nranks == 1 means single GPU (see gsap_nccl_unique_id) */

@@ -359,6 +359,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     if (const char *tg = getenv("GSAP_TEST_GRID")) c.test_grid = std::max(0, atoi(tg));
     REQUIRE(c.prm.sim_ranks >= 0 && c.prm.sim_ranks <= 64, GSAP_EINVAL, "sim_ranks in [0, 64]");
     REQUIRE(c.prm.proposal_mode == 0 || c.prm.proposal_mode == 1, GSAP_EINVAL, "proposal_mode is 0 or 1");
+    REQUIRE(c.prm.line_sort == 0 || c.prm.line_sort == 1, GSAP_EINVAL, "line_sort is 0 or 1");
     if (c.nranks > 1 || c.prm.sim_ranks > 1) c.prm.cuda_graphs = 0;   // the sliced batch path (move_batch)
     mark("streams");
     // host-side static info
@@ -1133,6 +1134,7 @@ void gsap_default_params(gsap_params *p) {
     p->sim_ranks = 0;
     p->incremental = 1;
     p->proposal_mode = 0;
+    p->line_sort = 1;
 }
 
 const char *gsap_last_error(void) { return g_err.c_str(); }

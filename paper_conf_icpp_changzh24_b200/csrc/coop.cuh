@@ -250,14 +250,17 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
             }
             int u;
             if (sizeof(K) == 4) {
-                // 129..512 entries: the warp LSD radix sort over the block bits,
-                // ping-ponging with the heads buffer (same size for 32-bit keys)
-                K *ka = S.warp.keys[wl], *kb = reinterpret_cast<K *>(S.warp.hp[wl]);
-                for (int i = lane; i < L; i += 32) ka[i] = seg[o + i];
-                __syncwarp();
-                K *keys = cta_radix_sort<K, 32>(ka, kb, L, a.col_bits, S.warp.cntp[wl], nullptr);
-                int *hw = reinterpret_cast<int *>(keys == ka ? kb : ka);
-                u = rle_runs<K, 32>(keys, L, hw, sd.tcol + o, sd.tcnt + o, lane, nullptr);
+                // 129..512 entries: one bucket pass + insertion sorts (segsort.cuh
+                // warp_bucket_line), the padded output written directly
+                u = warp_bucket_line<SEG_WARP_MAX>(reinterpret_cast<const unsigned *>(seg) + o, L, a.col_bits,
+                                                   reinterpret_cast<unsigned *>(S.warp.keys[wl]), S.warp.hp[wl],
+                                                   S.warp.cntp[wl], sd.tcol + o, sd.tcnt + o, sd.cum + o);
+                if (lane == 0) {
+                    sd.nnz[x] = u;
+                    sd.end[x] = o + u;
+                    sd.deg[x] = L;
+                }
+                continue;
             } else {
                 int n = 1;
                 while (n < L) n <<= 1;

@@ -12,6 +12,7 @@
 //          sort and run-length encoding (segsort.cuh), for rows (out-CSR) and
 //          columns (in-CSC) alike.
 #include <algorithm>
+#include <cstdlib>
 
 #include "internal.h"
 #include "prims.cuh"
@@ -722,6 +723,14 @@ __global__ void k_rcp(int B, const int *__restrict__ dout, const int *__restrict
         rcp[x] = 1.0 / ((double)dout[x] + (double)din[x] + (double)B);
 }
 
+static void bucket_attrs() {
+    per_device((const void *)k_segsort_bucket<1024>, [] {
+        GSAP_CUDA(cudaFuncSetAttribute(k_segsort_bucket<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)seg_bucket_smem<1024>()));
+        return 1;
+    });
+}
+
 // one side of the sparse blockmodel: lines (rows of M from the out-CSR, or
 // columns of M from the in-CSC) by counting sort + per-line segment sort,
 // written as a padded CSR: line x's runs stay at its segment offset ptr[x]
@@ -736,11 +745,15 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     GSAP_CUDA(cudaMemsetAsync(c.seg_len, 0, sizeof(int) * (size_t)B, c.stream));
     GSAP_CUDA(cudaMemsetAsync(c.seg_cur, 0, sizeof(int) * (size_t)B, c.stream));
     GSAP_CUDA(cudaMemsetAsync(c.seg_ctr, 0, 8 * sizeof(int), c.stream));
-    k_line_len<<<grid_for(V, 256), 256, 0, c.stream>>>(V, gptr, c.b, c.seg_len);
+    // each vertex's offset inside its line's segment comes back from the
+    // length atomic (vpos), so the scatter has no atomic in its dependent chain
+    static const bool no_vpos = getenv("GSAP_SCATTER_ATOMIC") != nullptr;   // A/B switch
+    int *vpos = no_vpos ? nullptr : c.wa;
+    k_line_len<<<grid_for(V, 256), 256, 0, c.stream>>>(V, gptr, c.b, c.seg_len, vpos);
     ++c.launches;
     device_scan<int>(c.seg_len, ptr, nullptr, B, false, c.scan_tmp, ptr + B, L);
     k_line_scatter_batched<K><<<grid_for((long long)V, 256), 256, 0, c.stream>>>(V, gptr, gidx, gw, c.b, ptr,
-                                                                                c.seg_cur, seg);
+                                                                                c.seg_cur, seg, vpos);
     const LineOut out{cum, end, deg};
     k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, ptr, c.seg_nnz, c.seg_listW, c.seg_listC,
                                                            c.seg_ctr, out, extent, SEG_WARP_MAX_MK, c.seg_listM);
@@ -755,6 +768,18 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     const int cb = bits_for(B);
     k_segsort_warp<K, 0><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, cb, idx, cnt,
                                                               c.seg_nnz, out);
+    if (sizeof(K) == 4 && c.prm.line_sort >= 1) {
+        // unweighted: one bucket pass + insertion sorts (k_segsort_bucket) for 129..1024 entries
+        bucket_attrs();
+        const unsigned *useg = reinterpret_cast<const unsigned *>(seg);
+        k_segsort_bucket<256><<<gw_, SEG_WARPS * 32, seg_bucket_smem<256>(), c.stream>>>(
+            B, ptr, useg, c.seg_listW, 1, c.seg_ctr, 2, cb, idx, cnt, c.seg_nnz, out);
+        k_segsort_bucket<512><<<gw_, SEG_WARPS * 32, seg_bucket_smem<512>(), c.stream>>>(
+            B, ptr, useg, c.seg_listM, 0, c.seg_ctr, 4, cb, idx, cnt, c.seg_nnz, out);
+        k_segsort_bucket<1024><<<gw_, SEG_WARPS * 32, seg_bucket_smem<1024>(), c.stream>>>(
+            B, ptr, useg, c.seg_listC, 1, c.seg_ctr, 3, cb, idx, cnt, c.seg_nnz, out);
+        c.launches += 4;
+    } else {
     k_segsort_warp<K, 1><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, cb, idx, cnt,
                                                               c.seg_nnz, out);
     k_segsort_warp<K, 3><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(512), c.stream>>>(B, ptr, seg, c.seg_listM,
@@ -764,6 +789,7 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
                                                                                 c.seg_ctr, cb, idx, cnt,
                                                                                 c.seg_nnz, out);
     c.launches += 4;
+    }
     const int gc = (int)std::min<long long>(std::max(1, B / 4), 148LL * 4);
     k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(ptr, seg, c.seg_listC, c.seg_ctr, bits_for(B), idx, cnt,
                                                c.seg_nnz, out);

@@ -157,11 +157,15 @@ GSAP_DEV void line_epilogue(const LineOut &out, int *__restrict__ cnt, int o, in
     }
 }
 
-// 1. len[b[v]] += deg(v)
-__global__ void k_line_len(int V, const int *__restrict__ gptr, const int *__restrict__ b, int *__restrict__ len) {
+// 1. len[b[v]] += deg(v); with vpos: the returned old length is v's offset
+// inside its line's segment (vpos[v]), so the scatter places v's entries
+// without an atomic of its own (multi-kernel path)
+__global__ void k_line_len(int V, const int *__restrict__ gptr, const int *__restrict__ b, int *__restrict__ len,
+                           int *__restrict__ vpos) {
     for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
         const int d = gptr[v + 1] - gptr[v];
-        if (d) atomicAdd(len + b[v], d);
+        if (vpos) vpos[v] = d ? atomicAdd(len + b[v], d) : 0;
+        else if (d) atomicAdd(len + b[v], d);
     }
 }
 
@@ -179,6 +183,7 @@ struct ScatterSide {
     const int *off;   // written earlier in the same kernel (coop): plain loads
     int *cur;
     K *seg;
+    const int *vpos;  // nullptr: claim each vertex's slots with an atomic on cur; else vpos[v] (k_line_len)
 };
 
 template <typename K>
@@ -197,7 +202,8 @@ GSAP_DEV void scatter_batched(const ScatterSide<K> &s0, const ScatterSide<K> &s1
             n = __ldg(gptr + v + 1) - lo;
             if (n) {
                 const int x = __ldg(b + v);
-                pos = (q ? s1.off : s0.off)[x] + atomicAdd((q ? s1.cur : s0.cur) + x, n);
+                const ScatterSide<K> &sd = q ? s1 : s0;
+                pos = sd.off[x] + (sd.vpos ? __ldg(sd.vpos + v) : atomicAdd(sd.cur + x, n));
             }
         }
         const int incl = warp_incl_scan(n);
@@ -244,8 +250,9 @@ GSAP_DEV void scatter_batched(const ScatterSide<K> &s0, const ScatterSide<K> &s1
 template <typename K>
 __global__ void k_line_scatter_batched(int V, const int *__restrict__ gptr, const int *__restrict__ gidx,
                                        const int *__restrict__ gw, const int *__restrict__ b,
-                                       const int *__restrict__ off, int *__restrict__ cur, K *__restrict__ seg) {
-    const ScatterSide<K> sd{gptr, gidx, gw, off, cur, seg};
+                                       const int *__restrict__ off, int *__restrict__ cur, K *__restrict__ seg,
+                                       const int *__restrict__ vpos) {
+    const ScatterSide<K> sd{gptr, gidx, gw, off, cur, seg, vpos};
     scatter_batched<K>(sd, sd, 1, V, b, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
 }
 
@@ -436,6 +443,172 @@ __global__ void __launch_bounds__(SEG_WARPS * 32) k_segsort_warp(int B, const in
         }
         if (lane == 0) nnz[x] = u;
         if (out.cum) line_epilogue<32>(out, tcnt, o, u, L, x, lane, nullptr);
+    }
+}
+
+// 4b'. unweighted graphs (32-bit keys = the neighbour block): 129..CAP-entry
+// segments, one warp each, sorted by ONE MSD bucket pass + an insertion sort
+// inside each bucket (O(L) expected work, against bitonic's O(L log^2 L) or
+// the radix sort's ceil(col_bits / 4) passes): the keys stay in registers
+// (striped), nb = pow2 >= L buckets over the line's key range [mn, mx] by the
+// monotone map floor((k - mn) nb / (mx - mn + 1)) in fp32 (monotone: every
+// step rounds monotonically), bucket counts by shared-memory atomics, one
+// warp scan, scatter to bucket start + the key's rank from the counting atomic
+// (order inside a bucket arbitrary), then each lane insertion-sorts the range
+// of its buckets.  A line whose fullest bucket
+// holds > 64 keys (clustered ids) takes the 4-bit radix sort instead.  The
+// RLE is a ballot over the sorted keys; with unit weights a run's count is
+// the distance between heads and cum is the run's end position, so the
+// padded CSR epilogue needs no scan.  Same output as k_segsort_warp.
+constexpr int SEG_BUCKET_FALLBACK = 64;
+template <int CAP>
+constexpr size_t seg_bucket_smem() {
+    return (size_t)SEG_WARPS * (2 * (size_t)CAP * sizeof(unsigned) + 8 * 32 * sizeof(unsigned));
+}
+
+template <typename K, int NT>
+GSAP_DEV K *cta_radix_sort(K *a, K *b, int L, int col_bits, unsigned *cntp, unsigned *wsum);
+
+// one line seg[0, L) (32-bit keys, 129 <= L <= CAP) by one warp: sorted,
+// run-length encoded and written in the padded CSR layout at line offset 0 of
+// tcol / tcnt / cum (the padding's counts zeroed); kb, cb: CAP words of the
+// warp's shared memory each, cntp: 256 words (radix fallback).  Returns the
+// run count.  Warp-uniform.
+template <int CAP>
+GSAP_DEV int warp_bucket_line(const unsigned *__restrict__ seg, int L, int col_bits, unsigned *kb, int *cb,
+                              unsigned *cntp, int *__restrict__ tcol, int *__restrict__ tcnt, int *__restrict__ cum) {
+    constexpr int E = CAP / 32;
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    unsigned k[E];
+    unsigned mn = 0xffffffffu, mx = 0u;
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+        const int i = e * 32 + lane;
+        k[e] = i < L ? seg[i] : 0u;
+        if (i < L) {
+            mn = min(mn, k[e]);
+            mx = max(mx, k[e]);
+        }
+    }
+    mn = __reduce_min_sync(FULL, mn);
+    mx = __reduce_max_sync(FULL, mx);
+    int lp = 0;
+    while ((32 << lp) < L) ++lp;   // nb = 32 << lp buckets, warp-uniform, <= CAP
+    const int nb = 32 << lp, per = 1 << lp;
+    const float scale = (float)nb / ((float)(mx - mn) + 1.0f);
+    // bucket q lives at slot (q mod per) * 32 + q / per: lane l owns the
+    // consecutive buckets l per .. l per + per - 1 for the scan, and the
+    // scan's accesses (all lanes at the same j) hit 32 distinct banks
+    auto slot = [&](unsigned key) {
+        const int q = min(nb - 1, (int)((float)(key - mn) * scale));
+        return ((q & (per - 1)) << 5) | (q >> lp);
+    };
+    for (int j = lane; j < nb; j += 32) cb[j] = 0;
+    __syncwarp();
+    // counts; the returned old count is the key's rank inside its bucket
+    // (two 16-bit ranks per register), so the scatter below needs no atomic
+    unsigned rk[(E + 1) / 2];
+#pragma unroll
+    for (int e = 0; e < (E + 1) / 2; ++e) rk[e] = 0u;
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+        if (e * 32 + lane < L) rk[e >> 1] |= (unsigned)atomicAdd(&cb[slot(k[e])], 1) << ((e & 1) * 16);
+    }
+    __syncwarp();
+    // exclusive scan of the buckets in order
+    int tot = 0, mxc = 0;
+    for (int j = 0; j < per; ++j) {
+        const int cj = cb[(j << 5) | lane];
+        tot += cj;
+        mxc = max(mxc, cj);
+    }
+    int run = warp_incl_scan(tot) - tot;
+    for (int j = 0; j < per; ++j) {
+        const int cj = cb[(j << 5) | lane];
+        cb[(j << 5) | lane] = run;
+        run += cj;
+    }
+    const int fullest = __reduce_max_sync(FULL, mxc);
+    __syncwarp();
+    unsigned *sorted = kb;
+    int *hp = cb;
+    if (fullest > SEG_BUCKET_FALLBACK && mn != mx) {
+#pragma unroll
+        for (int e = 0; e < E; ++e)
+            if (e * 32 + lane < L) kb[e * 32 + lane] = k[e];
+        __syncwarp();
+        sorted = cta_radix_sort<unsigned, 32>(kb, reinterpret_cast<unsigned *>(cb), L, col_bits, cntp, nullptr);
+        hp = reinterpret_cast<int *>(sorted == kb ? reinterpret_cast<unsigned *>(cb) : kb);
+    } else {
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+            if (e * 32 + lane < L) kb[cb[slot(k[e])] + ((rk[e >> 1] >> ((e & 1) * 16)) & 0xffffu)] = k[e];
+        }
+        // lane l's buckets l per .. l per + per - 1 are the contiguous range
+        // [start of bucket l per, start of bucket (l + 1) per) = [cb[l], cb[l + 1])
+        const int s0 = cb[lane], e0 = lane < 31 ? cb[lane + 1] : L;
+        __syncwarp();
+        // one insertion sort over the lane's whole range: the buckets are
+        // already in order, so keys only move inside their bucket (cost =
+        // range + inversions; no per-bucket loop, little divergence)
+        for (int i = s0 + 1; i < e0; ++i) {
+            const unsigned key = kb[i];
+            int q = i - 1;
+            unsigned prev = kb[q];
+            while (prev > key) {
+                kb[q + 1] = prev;
+                if (--q < s0) break;
+                prev = kb[q];
+            }
+            kb[q + 1] = key;
+        }
+        __syncwarp();
+    }
+    // run heads (ballot), then per run: block, count, cum = end position
+    int u = 0;
+    for (int base = 0; base < L; base += 32) {
+        const int i = base + lane;
+        const bool head = i < L && (i == 0 || sorted[i] != sorted[i - 1]);
+        const unsigned bal = __ballot_sync(FULL, head);
+        if (head) hp[u + __popc(bal & lt)] = i;
+        u += __popc(bal);
+    }
+    __syncwarp();
+    for (int q = lane; q < u; q += 32) {
+        const int s0 = hp[q], e0 = q + 1 < u ? hp[q + 1] : L;
+        tcol[q] = (int)sorted[s0];
+        tcnt[q] = e0 - s0;
+        cum[q] = e0;
+    }
+    for (int i = u + lane; i < L; i += 32) tcnt[i] = 0;
+    __syncwarp();   // the buffers are reused by the next line
+    return u;
+}
+
+template <int CAP>
+__global__ void __launch_bounds__(SEG_WARPS * 32, CAP >= 1024 ? 3 : 1) k_segsort_bucket(int B, const int *__restrict__ off,
+                                                                   const unsigned *__restrict__ seg,
+                                                                   const int *__restrict__ list, int from_back,
+                                                                   const int *__restrict__ counters, int ctr,
+                                                                   int col_bits, int *__restrict__ tcol,
+                                                                   int *__restrict__ tcnt, int *__restrict__ nnz,
+                                                                   LineOut out) {
+    extern __shared__ __align__(16) unsigned char seg_dyn[];
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    unsigned *kb = reinterpret_cast<unsigned *>(seg_dyn) + (size_t)w * (2 * CAP + 256);
+    int *cb = reinterpret_cast<int *>(kb + CAP);        // bucket counts -> cursors -> run heads
+    unsigned *cntp = kb + 2 * CAP;                      // radix fallback counters (8 x 32)
+    const int n_lines = counters[ctr];
+    for (int li = blockIdx.x * SEG_WARPS + w; li < n_lines; li += gridDim.x * SEG_WARPS) {
+        const int x = from_back ? list[B - 1 - li] : list[li];
+        const int o = off[x], L = off[x + 1] - o;
+        const int u = warp_bucket_line<CAP>(seg + o, L, col_bits, kb, cb, cntp, tcol + o, tcnt + o, out.cum + o);
+        if (lane == 0) {
+            nnz[x] = u;
+            out.end[x] = o + u;
+            out.deg[x] = L;
+        }
     }
 }
 

@@ -37,7 +37,8 @@ class gsap_params(C.Structure):
                 ("model_term", C.c_int32), ("max_rounds", C.c_int32), ("profile", C.c_int32),
                 ("cuda_graphs", C.c_int32), ("dense_max_B", C.c_int32), ("sparse_coop", C.c_int32), ("dense_coop", C.c_int32),
                 ("sel_small", C.c_int32), ("move_sorted", C.c_int32), ("sim_ranks", C.c_int32),
-                ("incremental", C.c_int32), ("proposal_mode", C.c_int32)]
+                ("incremental", C.c_int32), ("proposal_mode", C.c_int32),
+                ("line_sort", C.c_int32)]
 
 
 class gsap_dist(C.Structure):

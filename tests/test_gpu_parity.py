@@ -421,6 +421,60 @@ def test_rebuild_weighted_long_lines(G, oracle_mod, regime):
     assert np.array_equal(s, orc.propose(1, SEED, 1, 2, 0, 2000))
 
 
+def _line_shapes_graph(seed=11, V=6000, B=1500):
+    """A graph + partition whose rows AND columns of M take every shape the
+    unweighted line sort meets at 129..1100 entries: uniform keys, keys
+    clustered in a narrow id range with one far outlier (the bucket sort's
+    radix fallback), a single key repeated (mn == mx), three heavy keys."""
+    rng = np.random.default_rng(seed)
+    b = dcsbm.random_partition(V, B, seed)
+    members = [np.flatnonzero(b == x) for x in range(B)]
+    src, dst = [], []
+    for shape in range(4):
+        for _ in range(12):
+            x = int(rng.integers(0, B))
+            L = int(rng.integers(258, 2100))
+            if shape == 0:
+                tgt = rng.integers(0, B, L)
+            elif shape == 1:
+                lo = int(rng.integers(0, B - 8))
+                tgt = rng.integers(lo, lo + 6, L)
+                tgt[-1] = B - 1 if lo > 0 else B - 2
+            elif shape == 2:
+                tgt = np.full(L, int(rng.integers(0, B)))
+            else:
+                tgt = rng.choice(rng.integers(0, B, 3), L)
+            for t in tgt:
+                u = int(rng.choice(members[x]))
+                v = int(rng.choice(members[int(t)]))
+                if rng.random() < 0.5:
+                    src.append(u); dst.append(v)        # row x of M
+                else:
+                    src.append(v); dst.append(u)        # column x of M
+    src = np.concatenate([np.array(src), rng.integers(0, V, 20000)])
+    dst = np.concatenate([np.array(dst), rng.integers(0, V, 20000)])
+    order = np.argsort(src, kind="stable")
+    src, dst = src[order], dst[order]
+    rowptr = np.zeros(V + 1, np.int64)
+    np.add.at(rowptr, src + 1, 1)
+    return np.cumsum(rowptr), dst.astype(np.int32), b
+
+
+@pytest.mark.parametrize("line_sort", [1, 0])
+def test_rebuild_line_sort_shapes(G, oracle_mod, line_sort):
+    """Multi-kernel sparse rebuild: lines of 129..1100 entries with uniform,
+    clustered (+ outlier), single-key and few-key contents, rows and columns,
+    through the bucket sort (line_sort = 1) and the bitonic / radix sorts (0)."""
+    rowptr, col, b = _line_shapes_graph()
+    B = int(b.max()) + 1
+    ctx, orc = make_pair(G, oracle_mod, rowptr, col, None, line_sort=line_sort, **SPARSE_MK)
+    set_both(ctx, orc, b, B)
+    assert_same_blockmodel(ctx, orc)
+    m_g, _ = ctx.gsap_mdl()
+    m_o, _ = orc.mdl()
+    assert abs(m_g - m_o) <= 1e-9 * abs(m_o)
+
+
 def test_end_to_end_5k_layer3(G, oracle_mod):
     """5K-LL (Table 1 shape: 50 850 edges, 19 blocks): layer-3 parity."""
     from gen import metrics
