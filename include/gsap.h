@@ -66,9 +66,11 @@ typedef struct {
     int32_t model_term;       /* 0: E h(B^2/E) (Eq. 2); 1: GraphChallenge variant (R:Z3) */
     int32_t max_rounds;       /* guard on merge+MCMC rounds; default 500 */
     int32_t profile;          /* 1: time kernels with CUDA events (gsap_stats k_*) */
-    int32_t cuda_graphs;      /* 0: plain launches; 1: each MCMC iteration one CUDA graph launch
-                                 (default); 2: the whole MCMC phase one graph launch, a device-side
-                                 while loop (conditional node) with the convergence test on the GPU */
+    int32_t cuda_graphs;      /* 0: plain launches; 1: each MCMC iteration one CUDA graph launch;
+                                 2 (default): the whole MCMC phase one graph launch, a device-side
+                                 while loop (conditional node) with the convergence test on the GPU
+                                 (profile = 1 or multi-GPU runs use 1).  Either way the executable
+                                 graph is kept and updated in place by the next round's capture. */
     int32_t dense_max_B;      /* dense blockmodel iff B <= this; 0 = auto (B^2 <= max(4E, 2^24)) */
     int32_t sparse_coop;      /* 1 (default): sparse-regime rebuild as one persistent kernel when
                                  E <= GSAP_COOP_MAX_E; 0: the multi-kernel rebuild (same result) */

@@ -253,7 +253,31 @@ static void arena_give(void *p, size_t bytes, int dev) {
     if (drop) cudaFree(drop);
 }
 
+static void drop_mcmc_exec(Ctx &c) {
+    if (c.mcmc_exec) cudaGraphExecDestroy(c.mcmc_exec);
+    c.mcmc_exec = nullptr;
+    c.mcmc_exec_mode = 0;
+}
+
+// the executable graph of an MCMC phase: the cached one of the previous phase
+// updated in place when the topology matches (kernel parameters, grid sizes,
+// the regime's B all change between rounds; the node structure only with the
+// regime), else a fresh instantiation
+static cudaGraphExec_t mcmc_exec_for(Ctx &c, cudaGraph_t graph, int mode) {
+    static const bool no_update = getenv("GSAP_NO_EXEC_UPDATE") != nullptr;   // A/B switch
+    if (c.mcmc_exec && c.mcmc_exec_mode == mode && !no_update) {
+        cudaGraphExecUpdateResultInfo info;
+        if (cudaGraphExecUpdate(c.mcmc_exec, graph, &info) == cudaSuccess) return c.mcmc_exec;
+        cudaGetLastError();   // clear the update's error state
+    }
+    drop_mcmc_exec(c);
+    GSAP_CUDA(cudaGraphInstantiate(&c.mcmc_exec, graph, 0));
+    c.mcmc_exec_mode = mode;
+    return c.mcmc_exec;
+}
+
 static void free_ctx(Ctx &c) {
+    drop_mcmc_exec(c);
     if (c.arena) {
         if (c.stream) cudaStreamSynchronize(c.stream);
         if (c.side) cudaStreamSynchronize(c.side);
@@ -494,10 +518,15 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         if (c.prm.proposal_mode == 1) c.mt = A.take<int>(Vs);
         c.dnnz_r = A.take<int>(Vs + 1);
         c.dnnz_c = A.take<int>(Vs + 1);
-        if (c.prm.incremental) {
-            c.oldb = A.take<int>(Vs);
-            c.moved = A.take<int>(Vs);
-            c.moved_cnt = A.take<int>(1);
+        // the move log: N2 (dense regime) and the neighbour-block cache's updates
+        c.oldb = A.take<int>(Vs);
+        c.moved = A.take<int>(Vs);
+        c.moved_cnt = A.take<int>(1);
+        if (E > 0) {
+            c.nbo = A.take<int>(Es);
+            c.nbi = A.take<int>(Es);
+            c.csc2csr = A.take<int>(Es);
+            c.csr2csc = A.take<int>(Es);
         }
         c.Dh = A.take<double>((size_t)c.prm.max_nodal_itr + 1);
         if (c.prm.move_sorted) {
@@ -590,6 +619,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     for (int v = 0; v < V; ++v) iota[v] = v;
     GSAP_CUDA(cudaMemcpyAsync(c.b, iota.data(), sizeof(int) * Vs, cudaMemcpyHostToDevice, c.stream));
     c.B = V;
+    b_changed(c);
     rebuild(c);
     GSAP_CUDA(cudaStreamSynchronize(c.stream));
     mark("rebuild");
@@ -602,6 +632,7 @@ static void set_iota(Ctx &c) {
     GSAP_CUDA(cudaMemcpyAsync(c.b, iota.data(), sizeof(int) * (size_t)c.V, cudaMemcpyHostToDevice, c.stream));
     GSAP_CUDA(cudaStreamSynchronize(c.stream));
     c.B = c.V;
+    b_changed(c);
 }
 
 static double mdl_now(Ctx &c) {
@@ -749,7 +780,7 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh, std::vector<d
     const long long kernels = c.launches - l0;
     c.launches = l0;
     const auto tc0 = std::chrono::steady_clock::now();
-    GSAP_CUDA(cudaGraphInstantiate(&exec, graph, 0));
+    exec = mcmc_exec_for(c, graph, 1);
     const auto tc1 = std::chrono::steady_clock::now();
     std::vector<double> D((size_t)c.prm.max_nodal_itr + 1, 0.0);
     int ran = 0;
@@ -768,12 +799,11 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh, std::vector<d
             if (converged(c, D, itr, c.h_scal[1], thresh)) break;
         }
     } catch (...) {
-        cudaGraphExecDestroy(exec);
+        drop_mcmc_exec(c);
         cudaGraphDestroy(graph);
         graph_release_events(c);
         throw;
     }
-    GSAP_CUDA(cudaGraphExecDestroy(exec));
     GSAP_CUDA(cudaGraphDestroy(graph));
     graph_release_events(c);
     if (D_out) D_out->assign(D.begin(), D.begin() + ran);
@@ -868,7 +898,7 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::ve
         const long long kernels = c.launches - l0;
         c.launches = l0;
         const auto tc0 = std::chrono::steady_clock::now();
-        GSAP_CUDA(cudaGraphInstantiate(&exec, graph, 0));
+        exec = mcmc_exec_for(c, graph, 2);
         const auto tc1 = std::chrono::steady_clock::now();
         GSAP_CUDA(cudaMemsetAsync(c.scal, 0, sizeof(double), c.stream));
         GSAP_CUDA(cudaMemsetAsync(c.d_itr, 0, sizeof(unsigned), c.stream));
@@ -883,7 +913,6 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::ve
         }
         c.launches += kernels * ran;
         c.st.n_move_prop += (long long)V * ran;
-        GSAP_CUDA(cudaGraphExecDestroy(exec));
         GSAP_CUDA(cudaGraphDestroy(graph));
         if (getenv("GSAP_TIMING")) {
             const auto tc2 = std::chrono::steady_clock::now();
@@ -894,7 +923,7 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::ve
         }
         return ran;
     } catch (...) {
-        if (exec) cudaGraphExecDestroy(exec);
+        if (exec) drop_mcmc_exec(c);
         cudaGraphDestroy(graph);
         throw;
     }
@@ -1051,6 +1080,7 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
         GSAP_CUDA(cudaMemcpyAsync(c.b, c.slot_b[restart], sizeof(int) * (size_t)c.V, cudaMemcpyDeviceToDevice,
                                   c.stream));
         c.B = br.B[restart];
+        b_changed(c);
         rebuild(c);
         ++outer;
     }
@@ -1062,6 +1092,7 @@ static void run_impl(Ctx &c, int32_t *bmap_out, int32_t *B_out, double *mdl_out,
     // the answer: slot 1
     GSAP_CUDA(cudaMemcpyAsync(c.b, c.slot_b[1], sizeof(int) * (size_t)c.V, cudaMemcpyDeviceToDevice, c.stream));
     c.B = br.B[1];
+    b_changed(c);
     rebuild(c);
     copy_out(c, bmap_out, c.b, sizeof(int) * (size_t)c.V);
     GSAP_CUDA(cudaMemcpyAsync(c.h_int + 1, c.scal_i + 1, sizeof(int), cudaMemcpyDeviceToHost, c.stream));
@@ -1125,7 +1156,7 @@ void gsap_default_params(gsap_params *p) {
     p->model_term = 0;
     p->max_rounds = 500;
     p->profile = 0;
-    p->cuda_graphs = 1;
+    p->cuda_graphs = 2;
     p->dense_max_B = 0;
     p->sparse_coop = 1;
     p->dense_coop = 1;
@@ -1175,6 +1206,7 @@ gsap_status gsap_set_partition(gsap_ctx *ctx, const int32_t *b, int32_t B) {
     }
     GSAP_CUDA(cudaMemcpyAsync(c.b, b, sizeof(int) * (size_t)c.V, cudaMemcpyDefault, c.stream));
     c.B = B;
+    b_changed(c);
     rebuild(c);
     GSAP_CUDA(cudaStreamSynchronize(c.stream));
     API_CATCH

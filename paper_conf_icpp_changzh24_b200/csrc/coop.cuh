@@ -25,7 +25,7 @@ namespace gsap {
 
 struct CoopSide {
     const int *__restrict__ gptr;   // graph lines: out-CSR rowptr / in-CSC cscptr
-    const int *__restrict__ gidx;   // neighbour ids
+    const int *__restrict__ gidx;   // the neighbours' blocks (neighbour-block cache nbo / nbi)
     const int *__restrict__ gw;     // weights or nullptr
     int *len, *cur, *nnz, *listC;   // [B + 1] line scratch
     int *off;                       // out: [B + 1] segment offsets = line pointers (padded)

@@ -59,6 +59,16 @@ struct Ctx {
     // partition
     int *b = nullptr;
     int B = 0;
+    // neighbour-block cache: nbo[p] = b[col[p]] for every out-CSR
+    // position p, nbi[q] = b[cscsrc[q]] for every in-CSC position q, so the
+    // kernels that need the blocks of a vertex's neighbours read them with the
+    // adjacency (coalesced) instead of gathering b per entry.  Kept up to date
+    // by the apply of every MOVE batch (k_nb_update: only the moved vertices'
+    // entries, through the CSC <-> CSR position maps); any other change of b
+    // (create, set_partition, merges, bracket restores) marks it stale and the
+    // next rebuild refreshes it in full (k_nb_refresh).
+    int *nbo = nullptr, *nbi = nullptr, *csc2csr = nullptr, *csr2csc = nullptr;
+    bool nb_stale = true;
 
     // blockmodel (capacity: nnz <= min(E, B^2); B <= V)
     int *bm_rowptr = nullptr, *bm_col = nullptr, *bm_cnt = nullptr, *bm_cum = nullptr;
@@ -147,6 +157,11 @@ struct Ctx {
 
     // CUDA-graph capture of an MCMC iteration (N1: launch overhead, §5)
     unsigned *d_itr = nullptr;     // MCMC iteration read by k_move (device scalar)
+    // the instantiated graph of the last MCMC phase, updated in place
+    // (cudaGraphExecUpdate) by the next phase's capture when the topology is
+    // the same -- one instantiation per regime instead of one per round
+    cudaGraphExec_t mcmc_exec = nullptr;
+    int mcmc_exec_mode = 0;        // 1: one graph per iteration, 2: the device-side loop
     bool capturing = false;
     std::vector<GraphEv> graph_ev;
 
@@ -201,6 +216,8 @@ void role_end(Ctx &c, KClass &k, cudaEvent_t e0, cudaStream_t st);
 
 // rebuild.cu
 void build_graph_device(Ctx &c);                 // CSC, esrc, degrees (create time)
+void nb_refresh(Ctx &c);                         // the neighbour-block cache from b (if stale)
+inline void b_changed(Ctx &c) { c.nb_stale = true; }   // every bulk write of b outside the apply
 void rebuild(Ctx &c);                            // Alg. 2 from c.b, c.B
 bool dense_ok(const Ctx &c, int B);
 // padded-CSR export: line x's [ptr[x], end[x]) of src to dst[off[x] ..) on the device

@@ -420,6 +420,7 @@ static void select_merges_small(Ctx &c, const int *best, const double *dS, int K
     k_present<<<g256(V), 256, 0, c.stream>>>(V, c.b, c.nxt0, c.present);
     k_labels_small<<<1, SEL_THREADS, 0, c.stream>>>(B, c.nxt0, c.present, c.label, c.scal_i);
     k_relabel<<<g256(V), 256, 0, c.stream>>>(V, c.label, c.b);
+    b_changed(c);
     c.launches += 4;
     GSAP_CHECK_LAUNCH();
 }
@@ -472,6 +473,7 @@ void select_merges(Ctx &c, const int *best, const double *dS, int K, int *label_
     device_scan<int>(c.present, c.pos, nullptr, B, false, c.scan_tmp, c.scal_i, L);
     k_labels<<<g256(B), 256, 0, c.stream>>>(B, n0, c.present, c.pos, c.label);
     k_relabel<<<g256(V), 256, 0, c.stream>>>(V, c.label, c.b);
+    b_changed(c);
     c.launches += 2;
     GSAP_CHECK_LAUNCH();
     if (label_out)

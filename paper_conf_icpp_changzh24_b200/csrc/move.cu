@@ -48,6 +48,7 @@ struct MoveArgs {
     const int *__restrict__ rowptr, *__restrict__ col, *__restrict__ wgt;
     const int *__restrict__ cscptr, *__restrict__ cscsrc, *__restrict__ cscwgt;
     const int *__restrict__ kout, *__restrict__ kin, *__restrict__ selfw, *__restrict__ b;
+    const int *__restrict__ nbo, *__restrict__ nbi;   // neighbour-block cache: b[col[p]], b[cscsrc[q]]
     BM m;
     int first, count;
     const int *__restrict__ list;   // big-vertex kernel: sorted vertex ids
@@ -338,6 +339,19 @@ GSAP_DEV void mh_decide(const MoveArgs &a, const MoveCtx &q, uint4 w, double dS,
     acc_out = u <= p;
 }
 
+// the block of v's adjacency entry j (out-CSR entries first, then in-CSC),
+// from the neighbour-block cache (no gather of b)
+GSAP_DEV int nb_block(const MoveArgs &a, int ro, int nout, int ci, int j) {
+    return j < nout ? __ldg(a.nbo + ro + j) : __ldg(a.nbi + ci + (j - nout));
+}
+
+// whether v's adjacency entry j is its self-loop: the neighbour ids are read
+// only for vertices that have one (selfw[v] > 0), the others never load them
+GSAP_DEV bool nb_self(const MoveArgs &a, int v, bool has_self, int ro, int nout, int ci, int j) {
+    if (!has_self) return false;
+    return (j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + (j - nout))) == v;
+}
+
 // (a1) one thread per vertex: the proposal chain is a handful of dependent
 // loads, so 32 vertices per warp keep them in flight (R:O.4).
 template <bool WEIGHTED>
@@ -348,23 +362,23 @@ GSAP_DEV int propose_move_thread(const MoveArgs &a, int v, uint4 w) {
     const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
     const int ci = __ldg(a.cscptr + v);
     const uint32_t p = pick(w.x, K);
-    int n;
+    int j;   // the chosen adjacency entry (out entries, then in entries)
     if (!WEIGHTED) {
-        n = (int)p < nout ? __ldg(a.col + ro + p) : __ldg(a.cscsrc + ci + (p - nout));
+        j = (int)p;
     } else {
         long long acc = 0;
-        n = -1;
-        for (int e = 0; e < nout && n < 0; ++e) {
+        j = -1;
+        for (int e = 0; e < nout && j < 0; ++e) {
             acc += __ldg(a.wgt + ro + e);
-            if ((long long)p < acc) n = __ldg(a.col + ro + e);
+            if ((long long)p < acc) j = e;
         }
         const int nin = __ldg(a.cscptr + v + 1) - ci;
-        for (int e = 0; e < nin && n < 0; ++e) {
+        for (int e = 0; e < nin && j < 0; ++e) {
             acc += __ldg(a.cscwgt + ci + e);
-            if ((long long)p < acc) n = __ldg(a.cscsrc + ci + e);
+            if ((long long)p < acc) j = nout + e;
         }
     }
-    const int u = __ldg(a.b + n);
+    const int u = nb_block(a, ro, nout, ci, j);
     const uint32_t du = (uint32_t)bm_deg(a.m, u);
     if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
     if (a.m.mt) return __ldg(a.m.mt + u);   // N4: the shared table entry of u (Alg. 1 line 10)
@@ -406,14 +420,16 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
     const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
     const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
     const int deg = nout + nin;
-    int nb[4], tb[4];
+    const bool has_self = __ldg(a.selfw + v) > 0;
+    int tb[4];
 #pragma unroll
-    for (int c = 0; c < 4; ++c) {
+    for (int c = 0; c < 4; ++c) {   // the neighbours' blocks, from the cache (no gather of b)
         const int j = c * 32 + lane;
-        nb[c] = j < deg ? (j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout)) : -1;
+        tb[c] = j < deg ? nb_block(a, ro, nout, ci, j) : -1;
     }
+    bool self[4];
 #pragma unroll
-    for (int c = 0; c < 4; ++c) tb[c] = nb[c] >= 0 ? __ldg(a.b + nb[c]) : -1;
+    for (int c = 0; c < 4; ++c) self[c] = c * 32 + lane < deg && nb_self(a, v, has_self, ro, nout, ci, c * 32 + lane);
     const int r = __ldg(a.b + v);
     const uint32_t itr = a.itr_ptr ? __ldg(a.itr_ptr) : a.itr;
     const uint4 w = draws(a.seed, (uint32_t)v, 0u, itr, a.outer, 1u);
@@ -442,7 +458,7 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
     for (int c = 0; c < 4; ++c) {
         keep[c] = -1;
         const int j = c * 32 + lane;
-        if (nb[c] >= 0 && nb[c] != v) {
+        if (tb[c] >= 0 && !self[c]) {
             const bool out = j < nout;
             const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
             const int sl = tab_insert(tab, WARP_TAB_LOG2, tb[c]);
@@ -453,10 +469,9 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
     }
     for (int j = 128 + lane; j < deg; j += 32) {   // only when B <= 128 (<= B keys)
         const bool out = j < nout;
-        const int n = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-        if (n == v) continue;
+        if (nb_self(a, v, has_self, ro, nout, ci, j)) continue;
         const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
-        const int sl = tab_insert(tab, WARP_TAB_LOG2, __ldg(a.b + n));
+        const int sl = tab_insert(tab, WARP_TAB_LOG2, nb_block(a, ro, nout, ci, j));
         atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
         atomicMin(&tab[sl].w, j);
     }
@@ -473,10 +488,8 @@ GSAP_DEV void move_vertex_warp(const MoveArgs &a, int i, int4 *tab, int *list) {
     for (int base = 128; base < deg; base += 32) {
         const int j = base + lane;
         int sl = -1;
-        if (j < deg) {
-            const int n = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-            if (n != v) sl = tab_find(tab, WARP_TAB_LOG2, __ldg(a.b + n));
-        }
+        if (j < deg && !nb_self(a, v, has_self, ro, nout, ci, j))
+            sl = tab_find(tab, WARP_TAB_LOG2, nb_block(a, ro, nout, ci, j));
         const bool own = sl >= 0 && tab[sl].w == j;
         const unsigned bal = __ballot_sync(FULL, own);
         if (own) list[nuniq + __popc(bal & lt)] = sl;
@@ -745,6 +758,7 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
     const int ro = __ldg(a.rowptr + v), nout = __ldg(a.rowptr + v + 1) - ro;
     const int ci = __ldg(a.cscptr + v), nin = __ldg(a.cscptr + v + 1) - ci;
     const int deg = nout + nin;   // <= 128 (the caller routes bigger vertices to k_move_groups)
+    const bool has_self = __ldg(a.selfw + v) > 0;
     const int B = a.m.B;
     // the two lines of this pass and their wide splitters (32 HALF_K per
     // line, shared by the warp), issued before the histogram
@@ -762,10 +776,9 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
         const int j = c * 32 + lane;
         if (j < deg) {
             const bool out = j < nout;
-            const int n = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-            if (n != v) {
+            if (!nb_self(a, v, has_self, ro, nout, ci, j)) {
                 const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
-                const int sl = tab_insert(tab, WARP_TAB_LOG2, __ldg(a.b + n));
+                const int sl = tab_insert(tab, WARP_TAB_LOG2, nb_block(a, ro, nout, ci, j));
                 atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
                 atomicMin(&tab[sl].w, j);
                 keep[c] = sl;
@@ -915,12 +928,12 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
 template <int G, bool WEIGHTED>
 GSAP_DEV void group_table(const MoveArgs &a, int v, int ro, int nout, int ci, int deg, int4 *tab, int log2cap,
                           int t0) {
+    const bool has_self = __ldg(a.selfw + v) > 0;
     for (int j = (int)(threadIdx.x % G) - t0; j < deg; j += G - t0) {
         if (j < 0) break;
         const bool out = j < nout;
-        const int nb = out ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-        if (nb == v) continue;   // the self-loop is carried by selfw
-        const int t = __ldg(a.b + nb);
+        if (nb_self(a, v, has_self, ro, nout, ci, j)) continue;   // the self-loop is carried by selfw
+        const int t = nb_block(a, ro, nout, ci, j);
         const int wt = WEIGHTED ? (out ? __ldg(a.wgt + ro + j) : __ldg(a.cscwgt + ci + j - nout)) : 1;
         const int sl = tab_insert(tab, log2cap, t);
         atomicAdd(out ? &tab[sl].y : &tab[sl].z, wt);
@@ -937,10 +950,10 @@ GSAP_DEV void eval_move_group(const MoveArgs &a, int v, int r, int s, uint4 w, i
     MoveCtx q;
     move_ctx(a, v, r, s, tab, log2cap, q);
     double accS = 0.0, pf = 0.0, pb = 0.0;
+    const bool has_self = q.l > 0;
     for (int j = gt; j < deg; j += G) {
-        const int nb = j < nout ? __ldg(a.col + ro + j) : __ldg(a.cscsrc + ci + j - nout);
-        if (nb == v) continue;
-        const int4 e = tab[tab_find(tab, log2cap, __ldg(a.b + nb))];
+        if (nb_self(a, v, has_self, ro, nout, ci, j)) continue;
+        const int4 e = tab[tab_find(tab, log2cap, nb_block(a, ro, nout, ci, j))];
         if (e.w != j) continue;
         t_terms(a, q, e.x, e.y, e.z, accS, pf, pb);
     }
@@ -959,9 +972,9 @@ GSAP_DEV int propose_vertex_warp(const MoveArgs &a, int v, uint4 w, int ro, int 
     const uint32_t K = (uint32_t)(__ldg(a.kout + v) + __ldg(a.kin + v));
     if (K == 0) return (int)pick(w.z, B);
     const uint32_t p = pick(w.x, K);
-    int n;
+    int n;   // the chosen adjacency entry (out entries, then in entries)
     if (!WEIGHTED) {
-        n = (int)p < nout ? __ldg(a.col + ro + p) : __ldg(a.cscsrc + ci + (p - nout));
+        n = (int)p;
     } else {
         const int lane = threadIdx.x & 31;
         long long base = 0;
@@ -976,14 +989,11 @@ GSAP_DEV int propose_vertex_warp(const MoveArgs &a, int v, uint4 w, int ro, int 
                 if (lane >= o) incl += t;
             }
             const unsigned bal = __ballot_sync(FULL, j < deg && base + incl > (long long)p);
-            if (bal) {
-                const int jj = j0 + __ffs(bal) - 1;
-                n = jj < nout ? __ldg(a.col + ro + jj) : __ldg(a.cscsrc + ci + jj - nout);
-            }
+            if (bal) n = j0 + __ffs(bal) - 1;
             base += __shfl_sync(FULL, incl, 31);
         }
     }
-    const int u = __ldg(a.b + n);
+    const int u = nb_block(a, ro, nout, ci, n);
     const uint32_t du = (uint32_t)bm_deg(a.m, u);
     if (coin_random(w.y, B, du)) return (int)pick(w.z, B);
     if (a.m.mt) return __ldg(a.m.mt + u);   // N4
@@ -1174,6 +1184,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
     a.rowptr = c.rowptr; a.col = c.col; a.wgt = c.wgt;
     a.cscptr = c.cscptr; a.cscsrc = c.cscsrc; a.cscwgt = c.cscwgt;
     a.kout = c.kout; a.kin = c.kin; a.selfw = c.selfw; a.b = c.b;
+    a.nbo = c.nbo; a.nbi = c.nbi;
     a.m = c.bm();
     a.first = first;
     a.count = count;
@@ -1515,11 +1526,41 @@ bool device_ids_ok(Ctx &c, int n, const int *x, const unsigned char *mask, int B
     return c.h_int[6] == 0;
 }
 
-// the move log of the batch for the incremental update (N2): on when the
-// caller announced the batch (c.delta.pending) and the regime keeps dense M
+// the neighbour-block cache after an apply (internal.h Ctx::nbo): every moved
+// vertex v (the apply's move log) rewrites its own entries in its neighbours'
+// lists -- the in-edges u -> v hold v's block at CSR position csc2csr[q] (q in
+// v's CSC range), the out-edges v -> w at CSC position csr2csc[p] (p in v's
+// CSR range); each position belongs to one edge, so the writes never collide.
+// One warp per moved vertex.
+__global__ void __launch_bounds__(256) k_nb_update(const int *__restrict__ moved, const int *__restrict__ moved_cnt,
+                                                   const int *__restrict__ b, const int *__restrict__ rowptr,
+                                                   const int *__restrict__ cscptr, const int *__restrict__ csc2csr,
+                                                   const int *__restrict__ csr2csc, int *__restrict__ nbo,
+                                                   int *__restrict__ nbi) {
+    const int n = *moved_cnt, lane = threadIdx.x & 31;
+    for (int k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < n; k += (gridDim.x * blockDim.x) >> 5) {
+        const int v = moved[k];
+        const int x = b[v];
+        const int q1 = __ldg(cscptr + v + 1), p1 = __ldg(rowptr + v + 1);
+        for (int q = __ldg(cscptr + v) + lane; q < q1; q += 32) nbo[__ldg(csc2csr + q)] = x;
+        for (int p = __ldg(rowptr + v) + lane; p < p1; p += 32) nbi[__ldg(csr2csc + p)] = x;
+    }
+}
+
+static void launch_nb_update(Ctx &c, int count) {
+    if (!c.nbo || c.nb_stale) return;   // a stale cache is refreshed in full by the next rebuild
+    const int g = (int)std::min<long long>(((long long)count + 7) / 8, 148LL * 8);
+    k_nb_update<<<g, 256, 0, c.stream>>>(c.moved, c.moved_cnt, c.b, c.rowptr, c.cscptr, c.csc2csr, c.csr2csc,
+                                         c.nbo, c.nbi);
+    ++c.launches;
+    GSAP_CHECK_LAUNCH();
+}
+
+// the move log of the batch: for the incremental update (N2, when the caller
+// announced the batch and the regime keeps dense M) and the neighbour-block cache
 static MoveLog move_log(Ctx &c) {
     MoveLog lg{nullptr, nullptr, nullptr};
-    if (c.delta.pending) {
+    if (c.delta.pending || c.nbo) {
         GSAP_CUDA(cudaMemsetAsync(c.moved_cnt, 0, sizeof(int), c.stream));
         lg = MoveLog{c.oldb, c.moved, c.moved_cnt};
     }
@@ -1535,6 +1576,7 @@ void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned cha
                                           reinterpret_cast<unsigned *>(c.scal_i + 4), dsum, n_eval, lg);
     c.launches += 1;
     GSAP_CHECK_LAUNCH();
+    launch_nb_update(c, count);
 }
 
 // sharded batches: the fixed-chunk sums of accepted dS over [first, first+count)
@@ -1559,6 +1601,7 @@ void launch_apply_gathered(Ctx &c, int first, int count, const int *s, const uns
     k_sum_partials<<<1, 256, 0, c.stream>>>(partials, n, dsum, 1);
     c.launches += 2;
     GSAP_CHECK_LAUNCH();
+    launch_nb_update(c, count);
 }
 
 }  // namespace gsap

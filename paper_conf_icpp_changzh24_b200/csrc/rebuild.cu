@@ -86,6 +86,31 @@ __global__ void k_ptr_from_ids(const T *__restrict__ ids, const int *d_n, int n_
     }
 }
 
+__global__ void k_invert(int n, const int *__restrict__ p, int *__restrict__ inv) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        inv[p[i]] = (int)i;
+}
+
+// the neighbour-block cache in full: nbo[p] = b[col[p]], nbi[q] = b[cscsrc[q]]
+__global__ void k_nb_refresh(int E, const int *__restrict__ col, const int *__restrict__ cscsrc,
+                             const int *__restrict__ b, int *__restrict__ nbo, int *__restrict__ nbi) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < E; i += (long long)gridDim.x * blockDim.x) {
+        nbo[i] = __ldg(b + __ldg(col + i));
+        nbi[i] = __ldg(b + __ldg(cscsrc + i));
+    }
+}
+
+void nb_refresh(Ctx &c) {
+    if (!c.nb_stale) return;
+    if (c.E > 0) {
+        const int g = (int)std::min<long long>(((long long)c.E + 255) / 256, 148LL * 16);
+        k_nb_refresh<<<g, 256, 0, c.stream>>>(c.E, c.col, c.cscsrc, c.b, c.nbo, c.nbi);
+        ++c.launches;
+        GSAP_CHECK_LAUNCH();
+    }
+    c.nb_stale = false;
+}
+
 __global__ void k_kin(int V, const int *__restrict__ cscptr, const int *__restrict__ cscwgt, int *__restrict__ kin) {
     const int lane = threadIdx.x & 31;
     for (int v = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < V; v += (gridDim.x * blockDim.x) >> 5) {
@@ -115,7 +140,10 @@ void build_graph_device(Ctx &c) {
         const int *idx = which ? c.wb : c.wa;
         k_csc_fill<<<grid_for(E, 256), 256, 0, c.stream>>>(E, idx, c.esrc, c.wgt, c.cscsrc, c.cscwgt);
         k_ptr_from_ids<unsigned><<<grid_for(V + 1, 256), 256, 0, c.stream>>>(keys, nullptr, E, V, c.cscptr);
-        c.launches += 2;
+        // position maps of the neighbour-block cache: CSC position q holds CSR edge idx[q]
+        GSAP_CUDA(cudaMemcpyAsync(c.csc2csr, idx, sizeof(int) * (size_t)E, cudaMemcpyDeviceToDevice, c.stream));
+        k_invert<<<grid_for(E, 256), 256, 0, c.stream>>>(E, idx, c.csr2csc);
+        c.launches += 3;
     } else {
         GSAP_CUDA(cudaMemsetAsync(c.cscptr, 0, sizeof(int) * ((size_t)V + 1), c.stream));
     }
@@ -131,7 +159,7 @@ constexpr int HIST_SMEM_MAX_B = 221;   // B^2 * 4 bytes <= 195 KB of shared memo
 
 // histogram of (b[src], b[dst]) over an edge range; PRIV: privatised in smem
 template <bool PRIV>
-__global__ void __launch_bounds__(1024) k_hist(int E, const int *__restrict__ esrc, const int *__restrict__ col,
+__global__ void __launch_bounds__(1024) k_hist(int E, const int *__restrict__ esrc, const int *__restrict__ nbo,
                                                 const int *__restrict__ wgt, const int *__restrict__ b, int B,
                                                 int *__restrict__ M) {
     extern __shared__ int h[];
@@ -149,7 +177,7 @@ __global__ void __launch_bounds__(1024) k_hist(int E, const int *__restrict__ es
         const long long e = e0 + threadIdx.x;
         int key = -1, w = 0;
         if (e < hi) {
-            key = __ldg(b + __ldg(esrc + e)) * B + __ldg(b + __ldg(col + e));
+            key = __ldg(b + __ldg(esrc + e)) * B + __ldg(nbo + e);
             w = wgt ? __ldg(wgt + e) : 1;
         }
         if (wgt) {
@@ -214,7 +242,7 @@ constexpr size_t DC_TILE_SMEM = sizeof(int) * DC_WARPS * 32 * 33;
 struct DenseArgs {
     int E, B;
     const int *__restrict__ esrc;
-    const int *__restrict__ col;
+    const int *__restrict__ col;   // the block of each edge's destination (the neighbour-block cache nbo)
     const int *__restrict__ wgt;
     const int *__restrict__ b;
     int *acc, *M, *Mt, *rownnz, *colnnz, *dout, *din;
@@ -312,7 +340,7 @@ __global__ void __launch_bounds__(DC_THREADS) k_rebuild_dense(DenseArgs a) {
         }
         int key[4];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) key[k] = src[k] >= 0 ? __ldg(a.b + src[k]) * B + __ldg(a.b + dst[k]) : -1;
+        for (int k = 0; k < 4; ++k) key[k] = src[k] >= 0 ? __ldg(a.b + src[k]) * B + dst[k] : -1;   // dst: block (nbo)
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
             if (a.wgt) {
@@ -471,7 +499,7 @@ static void launch_rebuild_dense_coop(Ctx &c, const int *skip = nullptr) {
     a.skip = skip;
     a.E = c.E;
     a.B = c.B;
-    a.esrc = c.esrc; a.col = c.col; a.wgt = c.wgt; a.b = c.b;
+    a.esrc = c.esrc; a.col = c.nbo; a.wgt = c.wgt; a.b = c.b;   // col: the destinations' blocks
     a.acc = c.small_acc; a.M = c.dense; a.Mt = c.denseT;
     a.rownnz = c.dnnz_r; a.colnnz = c.dnnz_c; a.dout = c.dout; a.din = c.din;   // kept for N2
     a.ptrA = c.bm_rowptr; a.idxA = c.bm_col; a.cntA = c.bm_cnt; a.cumA = c.bm_cum;
@@ -697,10 +725,10 @@ static void rebuild_dense(Ctx &c) {
                 return 1;
             });
             const int grid = (int)std::min<long long>(dev_sms, ((long long)E + 1023) / 1024);
-            k_hist<true><<<grid, 1024, smem, c.stream>>>(E, c.esrc, c.col, c.wgt, c.b, B, c.dense);
+            k_hist<true><<<grid, 1024, smem, c.stream>>>(E, c.esrc, c.nbo, c.wgt, c.b, B, c.dense);
         } else {
             const int grid = (int)std::min<long long>(dev_sms * 8, ((long long)E + 1023) / 1024);
-            k_hist<false><<<grid, 1024, 0, c.stream>>>(E, c.esrc, c.col, c.wgt, c.b, B, c.dense);
+            k_hist<false><<<grid, 1024, 0, c.stream>>>(E, c.esrc, c.nbo, c.wgt, c.b, B, c.dense);
         }
         ++c.launches;
         GSAP_CHECK_LAUNCH();
@@ -737,7 +765,7 @@ static void bucket_attrs() {
 // (= the exclusive scan of the line lengths), end[x] marks their end, cnt is
 // zero in the rest of the segment.  No second scan and no compaction pass.
 template <typename K>
-static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw, int *ptr, int *end, int *idx,
+static void build_lines(Ctx &c, const int *gptr, const int *gblk, const int *gw, int *ptr, int *end, int *idx,
                         int *cnt, int *cum, int *deg, int *extent) {
     Launcher L{c.stream, &c.launches};
     const int B = c.B, V = c.V;
@@ -752,7 +780,7 @@ static void build_lines(Ctx &c, const int *gptr, const int *gidx, const int *gw,
     k_line_len<<<grid_for(V, 256), 256, 0, c.stream>>>(V, gptr, c.b, c.seg_len, vpos);
     ++c.launches;
     device_scan<int>(c.seg_len, ptr, nullptr, B, false, c.scan_tmp, ptr + B, L);
-    k_line_scatter_batched<K><<<grid_for((long long)V, 256), 256, 0, c.stream>>>(V, gptr, gidx, gw, c.b, ptr,
+    k_line_scatter_batched<K><<<grid_for((long long)V, 256), 256, 0, c.stream>>>(V, gptr, gblk, gw, c.b, ptr,
                                                                                 c.seg_cur, seg, vpos);
     const LineOut out{cum, end, deg};
     k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, ptr, c.seg_nnz, c.seg_listW, c.seg_listC,
@@ -811,11 +839,11 @@ static void rebuild_sparse_coop(Ctx &c) {
     a.kout = c.kout;
     a.kin = c.kin;
     CoopSide &r = a.sd[0], &q = a.sd[1];
-    r.gptr = c.rowptr; r.gidx = c.col; r.gw = c.wgt;
+    r.gptr = c.rowptr; r.gidx = c.nbo; r.gw = c.wgt;
     r.len = c.seg_len; r.off = c.bm_rowptr; r.cur = c.seg_cur; r.nnz = c.seg_nnz; r.listC = c.seg_listC;
     r.seg = c.keys0; r.tcol = c.bm_col; r.tcnt = c.bm_cnt; r.xl_keys = c.xl_keys; r.xl_hp = c.xl_hp;
     r.cum = c.bm_cum; r.end = c.bm_rowend; r.deg = c.dout;
-    q.gptr = c.cscptr; q.gidx = c.cscsrc; q.gw = c.cscwgt;
+    q.gptr = c.cscptr; q.gidx = c.nbi; q.gw = c.cscwgt;
     q.len = c.seg2_len; q.off = c.bm_colptr; q.cur = c.seg2_cur; q.nnz = c.seg2_nnz; q.listC = c.seg2_listC;
     q.seg = c.keys1; q.tcol = c.bm_row; q.tcnt = c.bm_ccnt; q.xl_keys = c.xl2_keys; q.xl_hp = c.xl2_hp;
     q.cum = c.bm_ccum; q.end = c.bm_colend; q.deg = c.din;
@@ -864,14 +892,14 @@ static void rebuild_sparse(Ctx &c) {
     }
     // padded CSR / CSC; d_nnz = the extent E the MDL sums cnt over (zeros in the padding)
     if (c.weighted) {
-        build_lines<u64>(c, c.rowptr, c.col, c.wgt, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt, c.bm_cum, c.dout,
+        build_lines<u64>(c, c.rowptr, c.nbo, c.wgt, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt, c.bm_cum, c.dout,
                          c.d_nnz);
-        build_lines<u64>(c, c.cscptr, c.cscsrc, c.cscwgt, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt, c.bm_ccum,
+        build_lines<u64>(c, c.cscptr, c.nbi, c.cscwgt, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt, c.bm_ccum,
                          c.din, nullptr);
     } else {
-        build_lines<unsigned>(c, c.rowptr, c.col, nullptr, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt, c.bm_cum,
+        build_lines<unsigned>(c, c.rowptr, c.nbo, nullptr, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt, c.bm_cum,
                               c.dout, c.d_nnz);
-        build_lines<unsigned>(c, c.cscptr, c.cscsrc, nullptr, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt,
+        build_lines<unsigned>(c, c.cscptr, c.nbi, nullptr, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt,
                               c.bm_ccum, c.din, nullptr);
     }
     c.padded = true;
@@ -896,6 +924,7 @@ void export_lines(Ctx &c, const int *ptr, const int *end, const int *off, const 
 }
 
 void rebuild(Ctx &c) {
+    nb_refresh(c);   // after a bulk change of b (no-op after a MOVE batch: the apply kept it current)
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_rebuild, &ev);
     const bool was_dense = c.dense_mode && c.dense_B == c.B;

@@ -178,7 +178,7 @@ __global__ void k_line_len(int V, const int *__restrict__ gptr, const int *__res
 template <typename K>
 struct ScatterSide {
     const int *__restrict__ gptr;
-    const int *__restrict__ gidx;
+    const int *__restrict__ gblk;   // the neighbours' blocks, parallel to the adjacency (nbo / nbi)
     const int *__restrict__ gw;
     const int *off;   // written earlier in the same kernel (coop): plain loads
     int *cur;
@@ -229,11 +229,11 @@ GSAP_DEV void scatter_batched(const ScatterSide<K> &s0, const ScatterSide<K> &s1
                 dst[u] = tpos + f - tex;
             }
 #pragma unroll
-            for (int u = 0; u < U; ++u) nbr[u] = wq[u] >= 0 ? __ldg((wq[u] ? s1.gidx : s0.gidx) + src[u]) : 0;
+            for (int u = 0; u < U; ++u) nbr[u] = wq[u] >= 0 ? __ldg((wq[u] ? s1.gblk : s0.gblk) + src[u]) : 0;
             int blk[U], wt[U];
 #pragma unroll
             for (int u = 0; u < U; ++u) {
-                blk[u] = wq[u] >= 0 ? __ldg(b + nbr[u]) : 0;
+                blk[u] = nbr[u];   // the neighbour-block cache: no gather of b
                 wt[u] = (sizeof(K) == 8 && wq[u] >= 0) ? __ldg((wq[u] ? s1.gw : s0.gw) + src[u]) : 0;
             }
 #pragma unroll
@@ -248,11 +248,11 @@ GSAP_DEV void scatter_batched(const ScatterSide<K> &s0, const ScatterSide<K> &s1
 }
 
 template <typename K>
-__global__ void k_line_scatter_batched(int V, const int *__restrict__ gptr, const int *__restrict__ gidx,
+__global__ void k_line_scatter_batched(int V, const int *__restrict__ gptr, const int *__restrict__ gblk,
                                        const int *__restrict__ gw, const int *__restrict__ b,
                                        const int *__restrict__ off, int *__restrict__ cur, K *__restrict__ seg,
                                        const int *__restrict__ vpos) {
-    const ScatterSide<K> sd{gptr, gidx, gw, off, cur, seg, vpos};
+    const ScatterSide<K> sd{gptr, gblk, gw, off, cur, seg, vpos};
     scatter_batched<K>(sd, sd, 1, V, b, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
 }
 
