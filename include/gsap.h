@@ -71,7 +71,7 @@ typedef struct {
                                  while loop (conditional node) with the convergence test on the GPU
                                  (profile = 1 or multi-GPU runs use 1).  Either way the executable
                                  graph is kept and updated in place by the next round's capture. */
-    int32_t dense_max_B;      /* dense blockmodel iff B <= this; 0 = auto (B^2 <= max(4E, 2^24)) */
+    int32_t dense_max_B;      /* dense blockmodel iff B <= this; 0 = auto (B^2 <= max(8E, 2^24)) */
     int32_t sparse_coop;      /* 1 (default): sparse-regime rebuild as one persistent kernel when
                                  E <= GSAP_COOP_MAX_E; 0: the multi-kernel rebuild (same result) */
     int32_t dense_coop;       /* dense-regime rebuild: 1 (default) one persistent kernel when

@@ -301,6 +301,8 @@ static void free_ctx(Ctx &c) {
     if (c.side) cudaStreamDestroy(c.side);
     if (c.ev_fork) cudaEventDestroy(c.ev_fork);
     if (c.ev_join) cudaEventDestroy(c.ev_join);
+    if (c.ev_nb) cudaEventDestroy(c.ev_nb);
+    if (c.ev_apply) cudaEventDestroy(c.ev_apply);
 }
 
 // one device allocation per context, carved into aligned sub-buffers
@@ -378,6 +380,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     GSAP_CUDA(cudaStreamCreateWithFlags(&c.side, cudaStreamNonBlocking));
     GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_fork, cudaEventDisableTiming));
     GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_join, cudaEventDisableTiming));
+    GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_nb, cudaEventDisableTiming));
+    GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_apply, cudaEventDisableTiming));
     GSAP_CUDA(cudaGetDevice(&c.dev));
     comm_init(c, dist);
     if (const char *tg = getenv("GSAP_TEST_GRID")) c.test_grid = std::max(0, atoi(tg));
@@ -440,7 +444,13 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
             }
         }
         c.b = A.take<int>(Vs);
-        c.dense_cap = std::min<size_t>(std::max<size_t>(4 * (size_t)E, (size_t)1 << 24), (size_t)1 << 29);
+        {   // dense regime iff B^2 <= max(8 E, 2^24) (density >= 1/8, or M small): experiments may
+            // override the multiplier (GSAP_DENSE_EMULT) and the floor (GSAP_DENSE_FLOOR_LOG2)
+            int fl = 24, em = 8;
+            if (const char *e = getenv("GSAP_DENSE_FLOOR_LOG2")) fl = std::max(16, std::min(29, atoi(e)));
+            if (const char *e = getenv("GSAP_DENSE_EMULT")) em = std::max(1, std::min(64, atoi(e)));
+            c.dense_cap = std::min<size_t>(std::max<size_t>((size_t)em * (size_t)E, (size_t)1 << fl), (size_t)1 << 29);
+        }
         c.dense_cap = std::min<size_t>(c.dense_cap, Vs * Vs);
         if (c.prm.dense_max_B > 0)
             c.dense_cap = std::min<size_t>(c.dense_cap, (size_t)c.prm.dense_max_B * (size_t)c.prm.dense_max_B);
@@ -521,6 +531,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         // the move log: N2 (dense regime) and the neighbour-block cache's updates
         c.oldb = A.take<int>(Vs);
         c.moved = A.take<int>(Vs);
+        c.movedb = A.take<int>(Vs);
         c.moved_cnt = A.take<int>(1);
         if (E > 0) {
             c.nbo = A.take<int>(Es);
@@ -767,6 +778,7 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh, std::vector<d
             launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
             rebuild(c);
         }
+        nb_join(c);   // no side-stream work may stay unjoined in a capture
         launch_data_term(c);
     } catch (...) {
         c.capturing = false;
@@ -881,6 +893,7 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::ve
                 launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
                 rebuild(c);
             }
+            nb_join(c);   // no side-stream work may stay unjoined in a capture
             launch_data_term(c);
             const double model = model_term(c.W, c.V, c.B, c.prm.model_term);
             k_mcmc_step<<<1, 1, 0, c.stream>>>(h, c.d_itr, c.scal, c.Dh, c.prm.max_nodal_itr, c.prm.window, model,

@@ -69,6 +69,11 @@ struct Ctx {
     // next rebuild refreshes it in full (k_nb_refresh).
     int *nbo = nullptr, *nbi = nullptr, *csc2csr = nullptr, *csr2csc = nullptr;
     bool nb_stale = true;
+    // the update after a MOVE batch runs on the side stream beside the dense-regime
+    // rebuild (which does not read the cache); every reader or writer of nbo / nbi
+    // joins it first (nb_join)
+    bool nb_pending = false;
+    cudaEvent_t ev_nb = nullptr, ev_apply = nullptr;
 
     // blockmodel (capacity: nnz <= min(E, B^2); B <= V)
     int *bm_rowptr = nullptr, *bm_col = nullptr, *bm_cnt = nullptr, *bm_cum = nullptr;
@@ -148,6 +153,7 @@ struct Ctx {
         bool pending = false;
     } delta;
     int *oldb = nullptr, *moved = nullptr, *moved_cnt = nullptr;
+    int *movedb = nullptr;                      // the new block of each logged move (k_nb_update)
     int *dnnz_r = nullptr, *dnnz_c = nullptr;   // dense regime: non-zeros per row of M / of Mt (kept for N2)
     // dense regime above SMALL_MAX_B: the lines of M padded to B entries (line
     // x at x B); N2 marks the lines a batch changed and re-compacts only those
@@ -218,6 +224,7 @@ void role_end(Ctx &c, KClass &k, cudaEvent_t e0, cudaStream_t st);
 void build_graph_device(Ctx &c);                 // CSC, esrc, degrees (create time)
 void nb_refresh(Ctx &c);                         // the neighbour-block cache from b (if stale)
 inline void b_changed(Ctx &c) { c.nb_stale = true; }   // every bulk write of b outside the apply
+void nb_join(Ctx &c);                            // the main stream waits for a pending cache update
 void rebuild(Ctx &c);                            // Alg. 2 from c.b, c.B
 bool dense_ok(const Ctx &c, int B);
 // padded-CSR export: line x's [ptr[x], end[x]) of src to dst[off[x] ..) on the device

@@ -17,6 +17,8 @@
 //        relabel to the ranks of the roots present in b (R:Z18).
 #include <algorithm>
 
+#include <cstdlib>
+
 #include "internal.h"
 #include "prims.cuh"
 
@@ -137,6 +139,53 @@ __global__ void __launch_bounds__(MERGE_WARPS * 32) k_merge(MergeArgs a) {
     }
 }
 
+// one warp per (block, proposal j) pair: the P proposals of a block are
+// evaluated in parallel warps instead of one after another by the block's
+// warp (at small B the whole phase was P sequential merge_delta chains long);
+// the same proposal and merge_delta per pair, so the same bits.  Writes s and
+// dS per pair (into the caller's arrays or the context's scratch); k_merge_best
+// then takes the first argmin per block.
+__global__ void __launch_bounds__(MERGE_WARPS * 32) k_merge_pairs(MergeArgs a, int *__restrict__ sbuf,
+                                                                  double *__restrict__ dbuf) {
+    const int lane = threadIdx.x & 31;
+    const long long total = (long long)a.count * a.P;
+    const long long nwarps = (long long)gridDim.x * MERGE_WARPS;
+    for (long long t = (long long)blockIdx.x * MERGE_WARPS + (threadIdx.x >> 5); t < total; t += nwarps) {
+        const int i = (int)(t / a.P), j = (int)(t - (long long)i * a.P);
+        const int r = a.first + i;
+        int s = 0;
+        if (lane == 0) s = a.propose ? propose_merge(a.m, r, (uint32_t)j, a.seed, a.outer) : sbuf[t];
+        s = __shfl_sync(FULL, s, 0);
+        if (!a.dS && !a.best && !a.dSbest) {   // proposals only
+            if (lane == 0) sbuf[t] = s;
+            continue;
+        }
+        const double d = merge_delta(a.m, r, s);
+        if (lane == 0) {
+            if (a.propose) sbuf[t] = s;
+            dbuf[t] = d;
+        }
+    }
+}
+
+// best proposal per block: the first j with the smallest dS (strict <, R:Z16)
+__global__ void k_merge_best(int count, int P, const int *__restrict__ sbuf, const double *__restrict__ dbuf,
+                             int *__restrict__ best, double *__restrict__ dSbest) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < count; i += gridDim.x * blockDim.x) {
+        int bs = sbuf[(size_t)i * P];
+        double bd = dbuf[(size_t)i * P];
+        for (int j = 1; j < P; ++j) {
+            const double d = dbuf[(size_t)i * P + j];
+            if (d < bd) {
+                bd = d;
+                bs = sbuf[(size_t)i * P + j];
+            }
+        }
+        if (best) best[i] = bs;
+        if (dSbest) dSbest[i] = bd;
+    }
+}
+
 // N4: block x's table entry = a weighted neighbour block of x (the walk of
 // R:O.4 with its own Philox draw), -1 for a block without edges
 __global__ void k_fill_mt(BM m, uint64_t seed, uint32_t j, uint32_t itr, const unsigned *itr_ptr, uint32_t outer,
@@ -179,10 +228,25 @@ void launch_merge_props(Ctx &c, uint32_t outer, int first, int count, bool propo
     a.dS = dS;
     a.best = best;
     a.dSbest = dSbest;
-    const long long need = ((long long)count + MERGE_WARPS - 1) / MERGE_WARPS;
-    const int grid = (int)std::min<long long>(need, 148LL * 16);
-    k_merge<<<grid, MERGE_WARPS * 32, 0, c.stream>>>(a);
-    ++c.launches;
+    static const bool block_warps = getenv("GSAP_MERGE_WARP") != nullptr;   // A/B: one warp per block
+    if (block_warps) {
+        const long long need = ((long long)count + MERGE_WARPS - 1) / MERGE_WARPS;
+        const int grid = (int)std::min<long long>(need, 148LL * 16);
+        k_merge<<<grid, MERGE_WARPS * 32, 0, c.stream>>>(a);
+        ++c.launches;
+    } else {
+        int *sbuf = s ? s : c.s;              // [count * P]: the context's proposal / dS scratch
+        double *dbuf = dS ? dS : c.dS;
+        const long long need = ((long long)count * a.P + MERGE_WARPS - 1) / MERGE_WARPS;
+        const int grid = (int)std::min<long long>(need, 148LL * 16);
+        k_merge_pairs<<<grid, MERGE_WARPS * 32, 0, c.stream>>>(a, sbuf, dbuf);
+        ++c.launches;
+        if (best || dSbest) {
+            k_merge_best<<<(int)std::min<long long>((count + 255) / 256, 148LL * 8), 256, 0, c.stream>>>(
+                count, a.P, sbuf, dbuf, best, dSbest);
+            ++c.launches;
+        }
+    }
     GSAP_CHECK_LAUNCH();
     // algorithmic bytes: each proposal reads rows / columns r and s (id + cnt)
     // once; estimated from the mean row length (nnz unknown on the host)

@@ -1172,6 +1172,7 @@ static int log2_ceil(long long x) {
 void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first, int count, int *s, double *dS,
                  double *H, unsigned char *acc, const unsigned *d_itr) {
     if (count <= 0) return;
+    nb_join(c);   // the move kernels read the neighbour-block cache
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_move, &ev);
     MoveArgs a;
@@ -1367,10 +1368,10 @@ constexpr int APPLY_CHUNK = 1024;
 // to log.moved (warp-aggregated atomics, order irrelevant: the update is
 // integer additions)
 struct MoveLog {
-    int *oldb, *moved, *moved_cnt;
+    int *oldb, *moved, *moved_cnt, *movedb;
 };
 
-GSAP_DEV void log_move(const MoveLog &lg, bool mv, int v, int old) {
+GSAP_DEV void log_move(const MoveLog &lg, bool mv, int v, int old, int nw) {
     const unsigned m = __ballot_sync(FULL, mv);   // warp-uniform call
     if (!m) return;
     const int lane = threadIdx.x & 31, leader = __ffs(m) - 1;
@@ -1379,7 +1380,9 @@ GSAP_DEV void log_move(const MoveLog &lg, bool mv, int v, int old) {
     base = __shfl_sync(FULL, base, leader);
     if (mv) {
         lg.oldb[v] = old;
-        lg.moved[base + __popc(m & ((1u << lane) - 1u))] = v;
+        const int k = base + __popc(m & ((1u << lane) - 1u));
+        lg.moved[k] = v;
+        lg.movedb[k] = nw;
     }
 }
 
@@ -1400,7 +1403,7 @@ __global__ void __launch_bounds__(APPLY_CHUNK) k_apply(int first, int count, con
         if (i < count && n_eval) ne += s[i] != b[first + i];
         if (lg.oldb) {
             const bool mv = i < count && acc[i];
-            log_move(lg, mv, first + i, mv ? b[first + i] : 0);
+            log_move(lg, mv, first + i, mv ? b[first + i] : 0, mv ? s[i] : 0);
         }
         if (i < count && acc[i]) {
             if (b) b[first + i] = s[i];
@@ -1460,7 +1463,7 @@ __global__ void __launch_bounds__(APPLY_CHUNK) k_apply_sum(int first, int count,
         if (i < count && n_eval) ne += s[i] != b[first + i];
         if (lg.oldb) {
             const bool mv = i < count && acc[i];
-            log_move(lg, mv, first + i, mv ? b[first + i] : 0);
+            log_move(lg, mv, first + i, mv ? b[first + i] : 0, mv ? s[i] : 0);
         }
         if (i < count && acc[i]) {
             b[first + i] = s[i];
@@ -1533,36 +1536,58 @@ bool device_ids_ok(Ctx &c, int n, const int *x, const unsigned char *mask, int B
 // CSR range); each position belongs to one edge, so the writes never collide.
 // One warp per moved vertex.
 __global__ void __launch_bounds__(256) k_nb_update(const int *__restrict__ moved, const int *__restrict__ moved_cnt,
-                                                   const int *__restrict__ b, const int *__restrict__ rowptr,
+                                                   const int *__restrict__ movedb, const int *__restrict__ rowptr,
                                                    const int *__restrict__ cscptr, const int *__restrict__ csc2csr,
                                                    const int *__restrict__ csr2csc, int *__restrict__ nbo,
                                                    int *__restrict__ nbi) {
     const int n = *moved_cnt, lane = threadIdx.x & 31;
     for (int k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < n; k += (gridDim.x * blockDim.x) >> 5) {
         const int v = moved[k];
-        const int x = b[v];
+        const int x = movedb[k];   // the new block, from the log (not b: the update may run beside later writes of b)
         const int q1 = __ldg(cscptr + v + 1), p1 = __ldg(rowptr + v + 1);
         for (int q = __ldg(cscptr + v) + lane; q < q1; q += 32) nbo[__ldg(csc2csr + q)] = x;
         for (int p = __ldg(rowptr + v) + lane; p < p1; p += 32) nbi[__ldg(csr2csc + p)] = x;
     }
 }
 
+void nb_join(Ctx &c) {
+    if (!c.nb_pending) return;
+    GSAP_CUDA(cudaStreamWaitEvent(c.stream, c.ev_nb, 0));
+    c.nb_pending = false;
+}
+
+// the cache update after an apply.  In the dense regime the rebuild that
+// follows reads b and M only, so the update runs on the side stream beside
+// it and the next reader of nbo / nbi joins it (nb_join); elsewhere in order.
 static void launch_nb_update(Ctx &c, int count) {
     if (!c.nbo || c.nb_stale) return;   // a stale cache is refreshed in full by the next rebuild
+    static const bool in_order = getenv("GSAP_NB_INORDER") != nullptr;   // A/B switch
+    const bool side = !in_order && c.dense_mode && dense_ok(c, c.B) && c.nranks == 1;
+    nb_join(c);
+    cudaStream_t st = c.stream;
+    if (side) {
+        GSAP_CUDA(cudaEventRecord(c.ev_apply, c.stream));
+        GSAP_CUDA(cudaStreamWaitEvent(c.side, c.ev_apply, 0));
+        st = c.side;
+    }
     const int g = (int)std::min<long long>(((long long)count + 7) / 8, 148LL * 8);
-    k_nb_update<<<g, 256, 0, c.stream>>>(c.moved, c.moved_cnt, c.b, c.rowptr, c.cscptr, c.csc2csr, c.csr2csc,
-                                         c.nbo, c.nbi);
+    k_nb_update<<<g, 256, 0, st>>>(c.moved, c.moved_cnt, c.movedb, c.rowptr, c.cscptr, c.csc2csr, c.csr2csc,
+                                   c.nbo, c.nbi);
     ++c.launches;
     GSAP_CHECK_LAUNCH();
+    if (side) {
+        GSAP_CUDA(cudaEventRecord(c.ev_nb, c.side));
+        c.nb_pending = true;
+    }
 }
 
 // the move log of the batch: for the incremental update (N2, when the caller
 // announced the batch and the regime keeps dense M) and the neighbour-block cache
 static MoveLog move_log(Ctx &c) {
-    MoveLog lg{nullptr, nullptr, nullptr};
+    MoveLog lg{nullptr, nullptr, nullptr, nullptr};
     if (c.delta.pending || c.nbo) {
         GSAP_CUDA(cudaMemsetAsync(c.moved_cnt, 0, sizeof(int), c.stream));
-        lg = MoveLog{c.oldb, c.moved, c.moved_cnt};
+        lg = MoveLog{c.oldb, c.moved, c.moved_cnt, c.movedb};
     }
     return lg;
 }
@@ -1586,7 +1611,7 @@ void launch_partials(Ctx &c, int first, int count, const int *s, const unsigned 
     if (count <= 0) return;
     const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
     k_apply<<<nb, APPLY_CHUNK, 0, c.stream>>>(first, count, s, acc, dS, nullptr, partials, nullptr, nullptr,
-                                      MoveLog{nullptr, nullptr, nullptr});
+                                      MoveLog{nullptr, nullptr, nullptr, nullptr});
     ++c.launches;
     GSAP_CHECK_LAUNCH();
 }

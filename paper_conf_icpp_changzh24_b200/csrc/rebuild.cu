@@ -102,6 +102,7 @@ __global__ void k_nb_refresh(int E, const int *__restrict__ col, const int *__re
 
 void nb_refresh(Ctx &c) {
     if (!c.nb_stale) return;
+    nb_join(c);
     if (c.E > 0) {
         const int g = (int)std::min<long long>(((long long)c.E + 255) / 256, 148LL * 16);
         k_nb_refresh<<<g, 256, 0, c.stream>>>(c.E, c.col, c.cscsrc, c.b, c.nbo, c.nbi);
@@ -242,7 +243,7 @@ constexpr size_t DC_TILE_SMEM = sizeof(int) * DC_WARPS * 32 * 33;
 struct DenseArgs {
     int E, B;
     const int *__restrict__ esrc;
-    const int *__restrict__ col;   // the block of each edge's destination (the neighbour-block cache nbo)
+    const int *__restrict__ col;
     const int *__restrict__ wgt;
     const int *__restrict__ b;
     int *acc, *M, *Mt, *rownnz, *colnnz, *dout, *din;
@@ -340,7 +341,7 @@ __global__ void __launch_bounds__(DC_THREADS) k_rebuild_dense(DenseArgs a) {
         }
         int key[4];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) key[k] = src[k] >= 0 ? __ldg(a.b + src[k]) * B + dst[k] : -1;   // dst: block (nbo)
+        for (int k = 0; k < 4; ++k) key[k] = src[k] >= 0 ? __ldg(a.b + src[k]) * B + __ldg(a.b + dst[k]) : -1;
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
             if (a.wgt) {
@@ -499,7 +500,7 @@ static void launch_rebuild_dense_coop(Ctx &c, const int *skip = nullptr) {
     a.skip = skip;
     a.E = c.E;
     a.B = c.B;
-    a.esrc = c.esrc; a.col = c.nbo; a.wgt = c.wgt; a.b = c.b;   // col: the destinations' blocks
+    a.esrc = c.esrc; a.col = c.col; a.wgt = c.wgt; a.b = c.b;   // b gathered: runs beside a pending cache update
     a.acc = c.small_acc; a.M = c.dense; a.Mt = c.denseT;
     a.rownnz = c.dnnz_r; a.colnnz = c.dnnz_c; a.dout = c.dout; a.din = c.din;   // kept for N2
     a.ptrA = c.bm_rowptr; a.idxA = c.bm_col; a.cntA = c.bm_cnt; a.cumA = c.bm_cum;
@@ -712,6 +713,7 @@ static void rebuild_dense_delta(Ctx &c) {
 }
 
 static void rebuild_dense(Ctx &c) {
+    nb_join(c);   // k_hist reads the neighbour-block cache
     const int B = c.B, E = c.E;
     const size_t BB = (size_t)B * B;
     GSAP_CUDA(cudaMemsetAsync(c.dense, 0, sizeof(int) * BB, c.stream));
@@ -876,6 +878,7 @@ static void rebuild_sparse_coop(Ctx &c) {
 }
 
 static void rebuild_sparse(Ctx &c) {
+    nb_join(c);   // the scatters read the neighbour-block cache
     const int B = c.B, E = c.E;
     if (E > 0 && c.coop_ok) {
         if (c.weighted) rebuild_sparse_coop<u64>(c);

@@ -506,14 +506,26 @@ GSAP_DEV int warp_bucket_line(const unsigned *__restrict__ seg, int L, int col_b
     };
     for (int j = lane; j < nb; j += 32) cb[j] = 0;
     __syncwarp();
-    // counts; the returned old count is the key's rank inside its bucket
-    // (two 16-bit ranks per register), so the scatter below needs no atomic
-    unsigned rk[(E + 1) / 2];
+    // counts; the returned old count is the key's rank inside its bucket, so
+    // the scatter below needs no atomic.  CAP <= 512: (slot << 16 | rank) kept
+    // per key; CAP 1024 (register budget): two 16-bit ranks per register, the
+    // slot recomputed
+#ifndef GSAP_BUCKET_PACK
+#define GSAP_BUCKET_PACK 1
+#endif
+    constexpr bool PACK = GSAP_BUCKET_PACK && CAP <= 512;
+    constexpr int NR = PACK ? E : (E + 1) / 2;
+    unsigned rk[NR];
 #pragma unroll
-    for (int e = 0; e < (E + 1) / 2; ++e) rk[e] = 0u;
+    for (int e = 0; e < NR; ++e) rk[e] = 0u;
 #pragma unroll
     for (int e = 0; e < E; ++e) {
-        if (e * 32 + lane < L) rk[e >> 1] |= (unsigned)atomicAdd(&cb[slot(k[e])], 1) << ((e & 1) * 16);
+        if (e * 32 + lane < L) {
+            const int sl = slot(k[e]);
+            const unsigned rank = (unsigned)atomicAdd(&cb[sl], 1);
+            if (PACK) rk[e] = ((unsigned)sl << 16) | rank;
+            else rk[e >> 1] |= rank << ((e & 1) * 16);
+        }
     }
     __syncwarp();
     // exclusive scan of the buckets in order
@@ -543,7 +555,10 @@ GSAP_DEV int warp_bucket_line(const unsigned *__restrict__ seg, int L, int col_b
     } else {
 #pragma unroll
         for (int e = 0; e < E; ++e) {
-            if (e * 32 + lane < L) kb[cb[slot(k[e])] + ((rk[e >> 1] >> ((e & 1) * 16)) & 0xffffu)] = k[e];
+            if (e * 32 + lane < L) {
+                if (PACK) kb[cb[rk[e] >> 16] + (rk[e] & 0xffffu)] = k[e];
+                else kb[cb[slot(k[e])] + ((rk[e >> 1] >> ((e & 1) * 16)) & 0xffffu)] = k[e];
+            }
         }
         // lane l's buckets l per .. l per + per - 1 are the contiguous range
         // [start of bucket l per, start of bucket (l + 1) per) = [cb[l], cb[l + 1])
@@ -565,6 +580,10 @@ GSAP_DEV int warp_bucket_line(const unsigned *__restrict__ seg, int L, int col_b
         }
         __syncwarp();
     }
+#ifndef GSAP_BUCKET_FUSED_RLE
+#define GSAP_BUCKET_FUSED_RLE 0   // measured slower (2M rebuild r4 / r6 1.46 / 1.28 vs 1.40 / 1.19 ms)
+#endif
+#if !GSAP_BUCKET_FUSED_RLE
     // run heads (ballot), then per run: block, count, cum = end position
     int u = 0;
     for (int base = 0; base < L; base += 32) {
@@ -581,13 +600,51 @@ GSAP_DEV int warp_bucket_line(const unsigned *__restrict__ seg, int L, int col_b
         tcnt[q] = e0 - s0;
         cum[q] = e0;
     }
+#else
+    // runs, one 32-key chunk at a time with the next chunk's head ballot in
+    // hand: a head's run ends at the next head (later in its chunk, else the
+    // first head of the next chunk; a run spanning a whole chunk is scanned
+    // for by its lane); per run: block, count, cum = end position (written
+    // directly, consecutive runs to consecutive q)
+    (void)hp;
+    unsigned kc = 0u, hc = 0u;
+    {
+        const bool h = lane < L && (lane == 0 || sorted[lane] != sorted[lane - 1]);
+        kc = lane < L ? sorted[lane] : 0u;
+        hc = __ballot_sync(FULL, h);
+    }
+    int u = 0;
+    for (int base = 0; base < L; base += 32) {
+        const int i = base + lane, in = i + 32;
+        const bool hn_ = in < L && sorted[in] != sorted[in - 1];
+        const unsigned kn = in < L ? sorted[in] : 0u;
+        const unsigned hn = __ballot_sync(FULL, hn_);
+        if ((hc >> lane) & 1u) {
+            const unsigned later = hc & ~((2u << lane) - 1u);   // heads after this lane in the chunk
+            int e;
+            if (later) e = base + __ffs(later) - 1;
+            else if (hn) e = base + 32 + __ffs(hn) - 1;
+            else {   // no head in the next chunk: the run spans it (or the line ends)
+                e = min(L, base + 64);
+                while (e < L && sorted[e] == kc) ++e;
+            }
+            const int q = u + __popc(hc & lt);
+            tcol[q] = (int)kc;
+            tcnt[q] = e - i;
+            cum[q] = e;
+        }
+        u += __popc(hc);
+        hc = hn;
+        kc = kn;
+    }
+#endif
     for (int i = u + lane; i < L; i += 32) tcnt[i] = 0;
     __syncwarp();   // the buffers are reused by the next line
     return u;
 }
 
 template <int CAP>
-__global__ void __launch_bounds__(SEG_WARPS * 32, CAP >= 1024 ? 3 : 1) k_segsort_bucket(int B, const int *__restrict__ off,
+__global__ void __launch_bounds__(SEG_WARPS * 32, CAP >= 512 ? 3 : 1) k_segsort_bucket(int B, const int *__restrict__ off,
                                                                    const unsigned *__restrict__ seg,
                                                                    const int *__restrict__ list, int from_back,
                                                                    const int *__restrict__ counters, int ctr,
