@@ -303,6 +303,8 @@ static void free_ctx(Ctx &c) {
     if (c.ev_join) cudaEventDestroy(c.ev_join);
     if (c.ev_nb) cudaEventDestroy(c.ev_nb);
     if (c.ev_apply) cudaEventDestroy(c.ev_apply);
+    if (c.ev_rb_fork) cudaEventDestroy(c.ev_rb_fork);
+    if (c.ev_rb_join) cudaEventDestroy(c.ev_rb_join);
 }
 
 // one device allocation per context, carved into aligned sub-buffers
@@ -382,6 +384,8 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
     GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_join, cudaEventDisableTiming));
     GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_nb, cudaEventDisableTiming));
     GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_apply, cudaEventDisableTiming));
+    GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_rb_fork, cudaEventDisableTiming));
+    GSAP_CUDA(cudaEventCreateWithFlags(&c.ev_rb_join, cudaEventDisableTiming));
     GSAP_CUDA(cudaGetDevice(&c.dev));
     comm_init(c, dist);
     if (const char *tg = getenv("GSAP_TEST_GRID")) c.test_grid = std::max(0, atoi(tg));
@@ -497,14 +501,17 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.seg_ctr = A.take<int>(8);
         c.xl_keys = A.take<unsigned long long>(2 * Es);
         c.xl_hp = A.take<int>(2 * Es);
-        if (c.coop_ok) {
-            c.seg2_len = A.take<int>(Vs + 1);
-            c.seg2_cur = A.take<int>(Vs + 1);
-            c.seg2_nnz = A.take<int>(Vs + 1);
-            c.seg2_listC = A.take<int>(Vs + 1);
-            c.xl2_keys = A.take<unsigned long long>(2 * Es);
-            c.xl2_hp = A.take<int>(2 * Es);
-        }
+        // the column side of both sparse rebuilds (persistent: its line scratch;
+        // multi-kernel: everything, the two sides run concurrently)
+        c.seg2_len = A.take<int>(Vs + 1);
+        c.seg2_cur = A.take<int>(Vs + 1);
+        c.seg2_nnz = A.take<int>(Vs + 1);
+        c.seg2_listC = A.take<int>(Vs + 1);
+        c.seg2_listW = A.take<int>(Vs + 1);
+        c.seg2_listM = A.take<int>(Vs + 1);
+        c.seg2_ctr = A.take<int>(8);
+        c.xl2_keys = A.take<unsigned long long>(2 * Es);
+        c.xl2_hp = A.take<int>(2 * Es);
         c.coop_bar = A.take<unsigned>(2);
         if (c.prm.dense_coop) c.small_acc = A.take<int>((size_t)SMALL_MAX_B * SMALL_MAX_B);
         const size_t tiles = (VE + 4095) / 4096 + 1;
@@ -512,6 +519,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.counts = A.take<int>(c.counts_cap);
         c.scan_tmp_cap = std::max(c.counts_cap, VE) / 4096 + 16;
         c.scan_tmp = A.take<int>(c.scan_tmp_cap);
+        c.scan_tmp2 = A.take<int>(c.scan_tmp_cap);
         // per-batch / per-phase buffers, padded for the rank-blocked all-gathers
         const size_t pad = 65536;
         c.s = A.take<int>(std::max(Vs * (size_t)P, Vs + pad));

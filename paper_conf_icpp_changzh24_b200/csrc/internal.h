@@ -106,6 +106,9 @@ struct Ctx {
     // line scratch, its long-segment scratch, the grid barrier
     bool coop_ok = false;
     int *seg2_len = nullptr, *seg2_cur = nullptr, *seg2_nnz = nullptr, *seg2_listC = nullptr;
+    // the multi-kernel rebuild's column side (runs beside the rows on the side stream)
+    int *seg2_listW = nullptr, *seg2_listM = nullptr, *seg2_ctr = nullptr, *scan_tmp2 = nullptr;
+    cudaEvent_t ev_rb_fork = nullptr, ev_rb_join = nullptr;
     unsigned long long *xl2_keys = nullptr;
     int *xl2_hp = nullptr;
     unsigned *coop_bar = nullptr;

@@ -761,32 +761,43 @@ static void bucket_attrs() {
     });
 }
 
+// the scratch of one side of the multi-kernel sparse rebuild (the two sides
+// run concurrently: rows on the context stream, columns on the side stream)
+struct LineScratch {
+    cudaStream_t st;
+    int *len, *cur, *ctr, *nnz, *listW, *listC, *listM, *vpos, *scan_tmp;
+    void *seg;
+    unsigned long long *xl_keys;
+    int *xl_hp;
+};
+
 // one side of the sparse blockmodel: lines (rows of M from the out-CSR, or
 // columns of M from the in-CSC) by counting sort + per-line segment sort,
 // written as a padded CSR: line x's runs stay at its segment offset ptr[x]
 // (= the exclusive scan of the line lengths), end[x] marks their end, cnt is
 // zero in the rest of the segment.  No second scan and no compaction pass.
 template <typename K>
-static void build_lines(Ctx &c, const int *gptr, const int *gblk, const int *gw, int *ptr, int *end, int *idx,
-                        int *cnt, int *cum, int *deg, int *extent) {
-    Launcher L{c.stream, &c.launches};
+static void build_lines(Ctx &c, const LineScratch &x, const int *gptr, const int *gblk, const int *gw, int *ptr,
+                        int *end, int *idx, int *cnt, int *cum, int *deg, int *extent) {
+    const cudaStream_t st = x.st;
+    Launcher L{st, &c.launches};
     const int B = c.B, V = c.V;
-    K *seg = reinterpret_cast<K *>(c.keys0);
-    GSAP_CUDA(cudaMemsetAsync(c.seg_len, 0, sizeof(int) * (size_t)B, c.stream));
-    GSAP_CUDA(cudaMemsetAsync(c.seg_cur, 0, sizeof(int) * (size_t)B, c.stream));
-    GSAP_CUDA(cudaMemsetAsync(c.seg_ctr, 0, 8 * sizeof(int), c.stream));
+    K *seg = reinterpret_cast<K *>(x.seg);
+    GSAP_CUDA(cudaMemsetAsync(x.len, 0, sizeof(int) * (size_t)B, st));
+    GSAP_CUDA(cudaMemsetAsync(x.cur, 0, sizeof(int) * (size_t)B, st));
+    GSAP_CUDA(cudaMemsetAsync(x.ctr, 0, 8 * sizeof(int), st));
     // each vertex's offset inside its line's segment comes back from the
     // length atomic (vpos), so the scatter has no atomic in its dependent chain
     static const bool no_vpos = getenv("GSAP_SCATTER_ATOMIC") != nullptr;   // A/B switch
-    int *vpos = no_vpos ? nullptr : c.wa;
-    k_line_len<<<grid_for(V, 256), 256, 0, c.stream>>>(V, gptr, c.b, c.seg_len, vpos);
+    int *vpos = no_vpos ? nullptr : x.vpos;
+    k_line_len<<<grid_for(V, 256), 256, 0, st>>>(V, gptr, c.b, x.len, vpos);
     ++c.launches;
-    device_scan<int>(c.seg_len, ptr, nullptr, B, false, c.scan_tmp, ptr + B, L);
-    k_line_scatter_batched<K><<<grid_for((long long)V, 256), 256, 0, c.stream>>>(V, gptr, gblk, gw, c.b, ptr,
-                                                                                c.seg_cur, seg, vpos);
+    device_scan<int>(x.len, ptr, nullptr, B, false, x.scan_tmp, ptr + B, L);
+    k_line_scatter_batched<K><<<grid_for((long long)V, 256), 256, 0, st>>>(V, gptr, gblk, gw, c.b, ptr,
+                                                                                x.cur, seg, vpos);
     const LineOut out{cum, end, deg};
-    k_line_classify<<<grid_for(B, 256), 256, 0, c.stream>>>(B, ptr, c.seg_nnz, c.seg_listW, c.seg_listC,
-                                                           c.seg_ctr, out, extent, SEG_WARP_MAX_MK, c.seg_listM);
+    k_line_classify<<<grid_for(B, 256), 256, 0, st>>>(B, ptr, x.nnz, x.listW, x.listC,
+                                                           x.ctr, out, extent, SEG_WARP_MAX_MK, x.listM);
     const int gw_ = (int)std::min<long long>(((long long)B + SEG_WARPS - 1) / SEG_WARPS, 148LL * 16);
     per_device((const void *)k_segsort_warp<K, 2>, [] {
         GSAP_CUDA(cudaFuncSetAttribute(k_segsort_warp<K, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -796,35 +807,35 @@ static void build_lines(Ctx &c, const int *gptr, const int *gblk, const int *gw,
         return 1;
     });
     const int cb = bits_for(B);
-    k_segsort_warp<K, 0><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, cb, idx, cnt,
-                                                              c.seg_nnz, out);
+    k_segsort_warp<K, 0><<<gw_, SEG_WARPS * 32, 0, st>>>(B, ptr, seg, x.listW, x.ctr, cb, idx, cnt,
+                                                              x.nnz, out);
     if (sizeof(K) == 4 && c.prm.line_sort >= 1) {
         // unweighted: one bucket pass + insertion sorts (k_segsort_bucket) for 129..1024 entries
         bucket_attrs();
         const unsigned *useg = reinterpret_cast<const unsigned *>(seg);
-        k_segsort_bucket<256><<<gw_, SEG_WARPS * 32, seg_bucket_smem<256>(), c.stream>>>(
-            B, ptr, useg, c.seg_listW, 1, c.seg_ctr, 2, cb, idx, cnt, c.seg_nnz, out);
-        k_segsort_bucket<512><<<gw_, SEG_WARPS * 32, seg_bucket_smem<512>(), c.stream>>>(
-            B, ptr, useg, c.seg_listM, 0, c.seg_ctr, 4, cb, idx, cnt, c.seg_nnz, out);
-        k_segsort_bucket<1024><<<gw_, SEG_WARPS * 32, seg_bucket_smem<1024>(), c.stream>>>(
-            B, ptr, useg, c.seg_listC, 1, c.seg_ctr, 3, cb, idx, cnt, c.seg_nnz, out);
+        k_segsort_bucket<256><<<gw_, SEG_WARPS * 32, seg_bucket_smem<256>(), st>>>(
+            B, ptr, useg, x.listW, 1, x.ctr, 2, cb, idx, cnt, x.nnz, out);
+        k_segsort_bucket<512><<<gw_, SEG_WARPS * 32, seg_bucket_smem<512>(), st>>>(
+            B, ptr, useg, x.listM, 0, x.ctr, 4, cb, idx, cnt, x.nnz, out);
+        k_segsort_bucket<1024><<<gw_, SEG_WARPS * 32, seg_bucket_smem<1024>(), st>>>(
+            B, ptr, useg, x.listC, 1, x.ctr, 3, cb, idx, cnt, x.nnz, out);
         c.launches += 4;
     } else {
-    k_segsort_warp<K, 1><<<gw_, SEG_WARPS * 32, 0, c.stream>>>(B, ptr, seg, c.seg_listW, c.seg_ctr, cb, idx, cnt,
-                                                              c.seg_nnz, out);
-    k_segsort_warp<K, 3><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(512), c.stream>>>(B, ptr, seg, c.seg_listM,
-                                                                                   c.seg_ctr, cb, idx, cnt,
-                                                                                   c.seg_nnz, out);
-    k_segsort_warp<K, 2><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(), c.stream>>>(B, ptr, seg, c.seg_listC,
-                                                                                c.seg_ctr, cb, idx, cnt,
-                                                                                c.seg_nnz, out);
+    k_segsort_warp<K, 1><<<gw_, SEG_WARPS * 32, 0, st>>>(B, ptr, seg, x.listW, x.ctr, cb, idx, cnt,
+                                                              x.nnz, out);
+    k_segsort_warp<K, 3><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(512), st>>>(B, ptr, seg, x.listM,
+                                                                                   x.ctr, cb, idx, cnt,
+                                                                                   x.nnz, out);
+    k_segsort_warp<K, 2><<<gw_, SEG_WARPS * 32, seg_warp2_smem<K>(), st>>>(B, ptr, seg, x.listC,
+                                                                                x.ctr, cb, idx, cnt,
+                                                                                x.nnz, out);
     c.launches += 4;
     }
     const int gc = (int)std::min<long long>(std::max(1, B / 4), 148LL * 4);
-    k_segsort_cta<K><<<gc, 256, 0, c.stream>>>(ptr, seg, c.seg_listC, c.seg_ctr, bits_for(B), idx, cnt,
-                                               c.seg_nnz, out);
-    k_segsort_xl<K><<<gc, 256, 0, c.stream>>>(ptr, seg, c.seg_listC, c.seg_ctr, bits_for(B), idx, cnt,
-                                              c.seg_nnz, reinterpret_cast<K *>(c.xl_keys), c.xl_hp, out);
+    k_segsort_cta<K><<<gc, 256, 0, st>>>(ptr, seg, x.listC, x.ctr, bits_for(B), idx, cnt,
+                                               x.nnz, out);
+    k_segsort_xl<K><<<gc, 256, 0, st>>>(ptr, seg, x.listC, x.ctr, bits_for(B), idx, cnt,
+                                              x.nnz, reinterpret_cast<K *>(x.xl_keys), x.xl_hp, out);
     c.launches += 5;
     GSAP_CHECK_LAUNCH();
 }
@@ -893,17 +904,31 @@ static void rebuild_sparse(Ctx &c) {
         GSAP_CUDA(cudaMemsetAsync(c.d_nnz, 0, sizeof(int), c.stream));
         return;
     }
-    // padded CSR / CSC; d_nnz = the extent E the MDL sums cnt over (zeros in the padding)
+    // padded CSR / CSC; d_nnz = the extent E the MDL sums cnt over (zeros in the padding).
+    // The two sides are independent: columns on the side stream beside the rows.
+    static const bool serial = getenv("GSAP_SIDES_SERIAL") != nullptr;   // A/B switch
+    const LineScratch x0{c.stream, c.seg_len, c.seg_cur, c.seg_ctr, c.seg_nnz, c.seg_listW, c.seg_listC,
+                         c.seg_listM, c.wa, c.scan_tmp, c.keys0, c.xl_keys, c.xl_hp};
+    const LineScratch x1{serial ? c.stream : c.side, c.seg2_len, c.seg2_cur, c.seg2_ctr, c.seg2_nnz, c.seg2_listW,
+                         c.seg2_listC, c.seg2_listM, c.wb, c.scan_tmp2, c.keys1, c.xl2_keys, c.xl2_hp};
+    if (!serial) {
+        GSAP_CUDA(cudaEventRecord(c.ev_rb_fork, c.stream));
+        GSAP_CUDA(cudaStreamWaitEvent(c.side, c.ev_rb_fork, 0));
+    }
     if (c.weighted) {
-        build_lines<u64>(c, c.rowptr, c.nbo, c.wgt, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt, c.bm_cum, c.dout,
-                         c.d_nnz);
-        build_lines<u64>(c, c.cscptr, c.nbi, c.cscwgt, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt, c.bm_ccum,
+        build_lines<u64>(c, x1, c.cscptr, c.nbi, c.cscwgt, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt, c.bm_ccum,
                          c.din, nullptr);
+        build_lines<u64>(c, x0, c.rowptr, c.nbo, c.wgt, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt, c.bm_cum,
+                         c.dout, c.d_nnz);
     } else {
-        build_lines<unsigned>(c, c.rowptr, c.nbo, nullptr, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt, c.bm_cum,
-                              c.dout, c.d_nnz);
-        build_lines<unsigned>(c, c.cscptr, c.nbi, nullptr, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt,
+        build_lines<unsigned>(c, x1, c.cscptr, c.nbi, nullptr, c.bm_colptr, c.bm_colend, c.bm_row, c.bm_ccnt,
                               c.bm_ccum, c.din, nullptr);
+        build_lines<unsigned>(c, x0, c.rowptr, c.nbo, nullptr, c.bm_rowptr, c.bm_rowend, c.bm_col, c.bm_cnt,
+                              c.bm_cum, c.dout, c.d_nnz);
+    }
+    if (!serial) {
+        GSAP_CUDA(cudaEventRecord(c.ev_rb_join, c.side));
+        GSAP_CUDA(cudaStreamWaitEvent(c.stream, c.ev_rb_join, 0));
     }
     c.padded = true;
     GSAP_CHECK_LAUNCH();

@@ -1,0 +1,10 @@
+#!/bin/bash
+# one-launch MDL with table f: full GPU suite, partition timing
+mkdir -p gpurun_out
+o=gpurun_out/s2s.txt; : > $o
+timeout 1500 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_s2s.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_s2s.log
+tail -2 gpurun_out/pytest_s2s.log >> $o
+for i in 1 2; do timeout 180 python tools/partition_ab.py --config 20k --runs 8 >> $o 2>&1; done
+timeout 400 python tools/partition_ab.py --config 200k --runs 3 --warmup 1 >> $o 2>&1
+for i in 1 2; do timeout 600 python bench.py --no-2m --no-cpu-baseline 2>/dev/null | python -c "import json,sys; d=json.loads([l for l in sys.stdin if l.startswith('{')][-1]); print('bench', d['value'], d['ms_per_step'], d['e2e']['value'])" >> $o; done
+cat $o
