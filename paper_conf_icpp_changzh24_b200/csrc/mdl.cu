@@ -3,7 +3,9 @@
 //   S   = -sum_xy f(M_xy) + sum_x f(dout_x) + sum_y f(din_y),  f(m) = m ln m
 //   MDL = E h(B^2/E) + V ln B + S,  h(x) = (1 + x) ln(1 + x) - x ln x.
 // The data term is a fixed-chunk fp64 reduction (chunk = 2048 entries per
-// CTA, then one ordered pass), so it does not depend on the launch shape.
+// CTA, then one ordered pass by the last CTA to finish), so it does not depend
+// on the launch shape.  f(m) for m < FT_N comes from the double-double table
+// (written in long double on the host), a log only beyond it.
 #include <math.h>
 
 #include <algorithm>
@@ -14,17 +16,29 @@ namespace gsap {
 
 constexpr int MDL_CHUNK = 2048;
 
+GSAP_DEV double f_of(const double2 *__restrict__ ft, int m) {
+    if (m <= 0) return 0.0;
+    if (m < FT_N) {
+        const double2 e = __ldg(ft + m);
+        return e.x + e.y;
+    }
+    return fx((double)m);
+}
+
 __global__ void __launch_bounds__(256) k_mdl_partials(const int *__restrict__ cnt, const int *__restrict__ d_nnz,
                                                       const int *__restrict__ dout, const int *__restrict__ din,
-                                                      int B, double *__restrict__ partials) {
+                                                      int B, const double2 *__restrict__ ft,
+                                                      double *__restrict__ partials, unsigned *__restrict__ arrivals,
+                                                      double *__restrict__ out) {
     __shared__ double sh[8];
+    __shared__ bool last;
     const int nnz = *d_nnz;
     const long long base = (long long)blockIdx.x * MDL_CHUNK;
     double acc = 0.0;
     for (int k = threadIdx.x; k < MDL_CHUNK; k += 256) {
         const long long i = base + k;
-        if (i < nnz) acc -= fx((double)cnt[i]);
-        if (i < B) acc += fx((double)dout[i]) + fx((double)din[i]);
+        if (i < nnz) acc -= f_of(ft, cnt[i]);
+        if (i < B) acc += f_of(ft, dout[i]) + f_of(ft, din[i]);
     }
     acc = warp_sum(acc);
     if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = acc;
@@ -33,13 +47,15 @@ __global__ void __launch_bounds__(256) k_mdl_partials(const int *__restrict__ cn
         double t = 0.0;
         for (int w = 0; w < 8; ++w) t += sh[w];
         partials[blockIdx.x] = t;
+        __threadfence();
+        last = atomicAdd(arrivals, 1u) == gridDim.x - 1;
     }
-}
-
-__global__ void __launch_bounds__(256) k_mdl_final(const double *__restrict__ partials, int n, double *out) {
-    __shared__ double sh[8];
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    // the last CTA: one ordered pass over the partials (256 strided lanes, warp trees, 8 warp sums)
     double v = 0.0;
-    for (int i = threadIdx.x; i < n; i += 256) v += partials[i];
+    for (int i = threadIdx.x; i < (int)gridDim.x; i += 256) v += *((volatile double *)(partials + i));
     v = warp_sum(v);
     if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = v;
     __syncthreads();
@@ -47,6 +63,7 @@ __global__ void __launch_bounds__(256) k_mdl_final(const double *__restrict__ pa
         double t = 0.0;
         for (int w = 0; w < 8; ++w) t += sh[w];
         *out = t;
+        *arrivals = 0u;
     }
 }
 
@@ -58,9 +75,9 @@ void launch_data_term(Ctx &c) {
     long long n = std::max<long long>(std::max<long long>(c.E, c.B), 1);
     if (c.dense_padded) n = std::max(n, (long long)c.B * c.B);
     const int nb = (int)((n + MDL_CHUNK - 1) / MDL_CHUNK);
-    k_mdl_partials<<<nb, 256, 0, c.stream>>>(c.bm_cnt, c.d_nnz, c.dout, c.din, c.B, c.partials);
-    k_mdl_final<<<1, 256, 0, c.stream>>>(c.partials, nb, c.scal + 1);
-    c.launches += 2;
+    k_mdl_partials<<<nb, 256, 0, c.stream>>>(c.bm_cnt, c.d_nnz, c.dout, c.din, c.B, c.ft, c.partials,
+                                             reinterpret_cast<unsigned *>(c.scal_i + 5), c.scal + 1);
+    c.launches += 1;
     GSAP_CHECK_LAUNCH();
     kc_end(c, c.k_mdl, ev, 0.0);
 }
