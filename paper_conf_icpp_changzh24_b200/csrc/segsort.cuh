@@ -567,10 +567,17 @@ GSAP_DEV int warp_bucket_line(const unsigned *__restrict__ seg, int L, int col_b
         // one insertion sort over the lane's whole range: the buckets are
         // already in order, so keys only move inside their bucket (cost =
         // range + inversions; no per-bucket loop, little divergence)
+        // (the sorted prefix's maximum is carried in a register: a key not below
+        // it -- the common case -- costs one load and no store)
+        unsigned mxk = s0 < e0 ? kb[s0] : 0u;
         for (int i = s0 + 1; i < e0; ++i) {
             const unsigned key = kb[i];
+            if (key >= mxk) {
+                mxk = key;
+                continue;
+            }
             int q = i - 1;
-            unsigned prev = kb[q];
+            unsigned prev = mxk;
             while (prev > key) {
                 kb[q + 1] = prev;
                 if (--q < s0) break;
@@ -586,12 +593,17 @@ GSAP_DEV int warp_bucket_line(const unsigned *__restrict__ seg, int L, int col_b
 #if !GSAP_BUCKET_FUSED_RLE
     // run heads (ballot), then per run: block, count, cum = end position
     int u = 0;
+    unsigned carry = 0u;   // the previous chunk's last key (lane 31)
     for (int base = 0; base < L; base += 32) {
         const int i = base + lane;
-        const bool head = i < L && (i == 0 || sorted[i] != sorted[i - 1]);
+        const unsigned k0 = i < L ? sorted[i] : 0u;
+        unsigned kp = __shfl_up_sync(FULL, k0, 1);
+        if (lane == 0) kp = carry;
+        const bool head = i < L && (i == 0 || k0 != kp);
         const unsigned bal = __ballot_sync(FULL, head);
         if (head) hp[u + __popc(bal & lt)] = i;
         u += __popc(bal);
+        carry = __shfl_sync(FULL, k0, 31);
     }
     __syncwarp();
     for (int q = lane; q < u; q += 32) {
