@@ -610,7 +610,13 @@ __global__ void __launch_bounds__(256) k_dense_lines(const int *__restrict__ M, 
                                                      const int *__restrict__ skip) {
     if (skip && *skip == 0) return;   // the batch moved nothing: every line as it was
     __shared__ bool last;
+    // each warp stages its line DL_CH entries at a time: all the chunk's loads
+    // in flight at once (one memory latency per 1024 entries instead of one
+    // per 128-entry step), then the compaction from shared memory
+    constexpr int DL_CH = 1024;
+    __shared__ int4 stage[8][DL_CH / 4];
     const int lane = threadIdx.x & 31;
+    int *sb = reinterpret_cast<int *>(stage[threadIdx.x >> 5]);
     for (int x2 = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; x2 < 2 * B; x2 += (gridDim.x * blockDim.x) >> 5) {
         if (DIRTY && !dirty[x2]) continue;   // warp-uniform
         const bool t = x2 >= B;
@@ -623,33 +629,43 @@ __global__ void __launch_bounds__(256) k_dense_lines(const int *__restrict__ M, 
         const int lo = x * B;
         const int old_end = DIRTY ? end[x] : lo;
         int base = lo, run = 0;
-        int nxt[4];   // the next step's entries, loaded one step ahead
+        for (int c0 = 0; c0 < B; c0 += DL_CH) {
+            int tmp[DL_CH / 32];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) nxt[k] = 4 * lane + k < B ? __ldg(R + 4 * lane + k) : 0;
-        for (int y0 = 0; y0 < B; y0 += 128) {
-            const int y = y0 + 4 * lane;
-            int v[4], nz = 0, sm = 0;
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-                v[k] = nxt[k];
-                nxt[k] = y + 128 + k < B ? __ldg(R + y + 128 + k) : 0;
-                nz += v[k] != 0;
-                sm += v[k];
+            for (int j = 0; j < DL_CH / 32; ++j) {
+                const int y = c0 + j * 32 + lane;
+                tmp[j] = y < B ? __ldg(R + y) : 0;
             }
-            const int nzi = warp_incl_scan(nz), smi = warp_incl_scan(sm);
-            int p = base + nzi - nz, sc = run + smi - sm;
 #pragma unroll
-            for (int k = 0; k < 4; ++k) {
-                sc += v[k];
-                if (v[k] != 0) {
-                    idx[p] = y + k;
-                    cnt[p] = v[k];
-                    cum[p] = sc;
-                    ++p;
+            for (int j = 0; j < DL_CH / 32; ++j) sb[j * 32 + lane] = tmp[j];
+            __syncwarp();
+            const int n = min(DL_CH, B - c0);
+            for (int s0 = 0; s0 < n; s0 += 128) {
+                const int y = c0 + s0 + 4 * lane;
+                const int4 q4 = reinterpret_cast<const int4 *>(sb)[(s0 >> 2) + lane];
+                const int v[4] = {q4.x, q4.y, q4.z, q4.w};   // zero beyond B
+                int nz = 0, sm = 0;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    nz += v[k] != 0;
+                    sm += v[k];
                 }
+                const int nzi = warp_incl_scan(nz), smi = warp_incl_scan(sm);
+                int p = base + nzi - nz, sc = run + smi - sm;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    sc += v[k];
+                    if (v[k] != 0) {
+                        idx[p] = y + k;
+                        cnt[p] = v[k];
+                        cum[p] = sc;
+                        ++p;
+                    }
+                }
+                base += __shfl_sync(FULL, nzi, 31);
+                run += __shfl_sync(FULL, smi, 31);
             }
-            base += __shfl_sync(FULL, nzi, 31);
-            run += __shfl_sync(FULL, smi, 31);
+            __syncwarp();   // the stage is rewritten by the next chunk
         }
         if (DIRTY)
             for (int q = base + lane; q < old_end; q += 32) cnt[q] = 0;   // the previous version's tail
