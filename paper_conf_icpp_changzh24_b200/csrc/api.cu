@@ -530,6 +530,7 @@ static void create_impl(Ctx &c, int32_t V, const int64_t *rowptr, const int32_t 
         c.dSbest = A.take<double>(Vs + pad);
         // >= the MDL extent (max(E, B), or B^2 padded dense) / MDL_CHUNK, V / APPLY_CHUNK + ranks
         c.partials = A.take<double>(std::max(VE, c.dense_cap) / 512 + 1024);
+        c.bpart = A.take<double>(Vs / 1024 + 2 * (size_t)std::max(1, c.prm.num_batches) + 16);
         c.scal = A.take<double>(8);
         c.scal_i = A.take<int>(8);
         c.n_eval = A.take<unsigned long long>(1);
@@ -768,6 +769,8 @@ static bool converged(Ctx &c, const std::vector<double> &D, int itr, double S, d
 static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh, std::vector<double> *D_out) {
     const int V = c.V, nb = c.prm.num_batches;
     const int bs = (V + nb - 1) / nb;
+    const int nch = (bs + APPLY_CHUNK_V - 1) / APPLY_CHUNK_V;   // dS chunk partials per full batch
+    DsumSpec ds{c.bpart, 0, nch, nch, 0};
     cudaGraph_t graph = nullptr;
     cudaGraphExec_t exec = nullptr;
     const long long l0 = c.launches;
@@ -783,11 +786,14 @@ static int mcmc_phase_graph(Ctx &c, uint32_t outer, double thresh, std::vector<d
             announce_batch(c, first, last - first);
             launch_fill_mt(c, TABLE_J | ((uint32_t)first & 0x3fffffffu), 0, outer, 1, c.d_itr);   // N4 only
             launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
-            launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
+            launch_apply_deferred(c, first, last - first, c.s, c.acc, c.dS, c.bpart + (size_t)k * ds.stride,
+                                  c.scal_i + 1, c.n_eval);
             rebuild(c);
+            ds.nbat = k + 1;
+            ds.nch_last = (last - first + APPLY_CHUNK_V - 1) / APPLY_CHUNK_V;
         }
         nb_join(c);   // no side-stream work may stay unjoined in a capture
-        launch_data_term(c);
+        launch_data_term(c, &ds);   // the MDL and the iteration's dS sum (c.scal[1], c.scal[0])
     } catch (...) {
         c.capturing = false;
         cudaStreamEndCapture(c.stream, &graph);
@@ -871,6 +877,8 @@ __global__ void k_mcmc_step(cudaGraphConditionalHandle h, unsigned *d_itr, doubl
 static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::vector<double> *D_out) {
     const int V = c.V, nb = c.prm.num_batches;
     const int bs = (V + nb - 1) / nb;
+    const int nch = (bs + APPLY_CHUNK_V - 1) / APPLY_CHUNK_V;   // dS chunk partials per full batch
+    DsumSpec ds{c.bpart, 0, nch, nch, 0};
     const long long l0 = c.launches;
     const auto tcs = std::chrono::steady_clock::now();
     cudaGraph_t graph = nullptr;
@@ -898,11 +906,14 @@ static int mcmc_phase_device_loop(Ctx &c, uint32_t outer, double thresh, std::ve
             announce_batch(c, first, last - first);
             launch_fill_mt(c, TABLE_J | ((uint32_t)first & 0x3fffffffu), 0, outer, 1, c.d_itr);   // N4 only
             launch_move(c, MOVE_FUSED, outer, 0, first, last - first, c.s, c.dS, nullptr, c.acc, c.d_itr);
-                launch_apply(c, first, last - first, c.s, c.acc, c.dS, c.scal, c.scal_i + 1, c.n_eval);
+                launch_apply_deferred(c, first, last - first, c.s, c.acc, c.dS, c.bpart + (size_t)k * ds.stride,
+                                      c.scal_i + 1, c.n_eval);
                 rebuild(c);
+                ds.nbat = k + 1;
+                ds.nch_last = (last - first + APPLY_CHUNK_V - 1) / APPLY_CHUNK_V;
             }
             nb_join(c);   // no side-stream work may stay unjoined in a capture
-            launch_data_term(c);
+            launch_data_term(c, &ds);   // the MDL and the iteration's dS sum (c.scal[1], c.scal[0])
             const double model = model_term(c.W, c.V, c.B, c.prm.model_term);
             k_mcmc_step<<<1, 1, 0, c.stream>>>(h, c.d_itr, c.scal, c.Dh, c.prm.max_nodal_itr, c.prm.window, model,
                                               thresh);

@@ -123,6 +123,7 @@ struct Ctx {
     int *best = nullptr;         // B
     double *dSbest = nullptr;    // B
     double *partials = nullptr;  // reduction partials
+    double *bpart = nullptr;     // MCMC graphs: the accepted-dS chunk partials of every batch of an iteration
     double *scal = nullptr;      // device scalars [0] = batch dS sum, [1] = data term
     int *scal_i = nullptr;       // device int scalars [0] = new B, [1] = accepted moves, [4] apply
                                  // arrivals, [6] argument check flag
@@ -245,6 +246,11 @@ bool device_ids_ok(Ctx &c, int n, const int *x, const unsigned char *mask, int B
 
 void launch_partials(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
                      double *partials);
+// the apply of a batch inside an MCMC graph: b, counters, move log and cache
+// update as launch_apply, the chunk partials into part[] only -- the
+// iteration's ordered sum is taken once by launch_data_term(c, &dsum_spec)
+void launch_apply_deferred(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
+                           double *part, int *nacc, unsigned long long *n_eval);
 void launch_apply_gathered(Ctx &c, int first, int count, const int *s, const unsigned char *acc,
                            const double *partials, int n, double *dsum, int *nacc,
                            unsigned long long *n_eval = nullptr);
@@ -274,7 +280,14 @@ void launch_merge_props(Ctx &c, uint32_t outer, int first, int count, bool propo
 void select_merges(Ctx &c, const int *best, const double *dS, int K, int *label_out);
 
 // mdl.cu
-void launch_data_term(Ctx &c);                   // -> c.scal[1], no synchronisation
+// the iteration's sum of accepted dS from the batches' chunk partials (batch k
+// at part + k stride: nch_first chunks, the last batch nch_last), in the order
+// of k_apply_sum's running sum -> c.scal[0]
+struct DsumSpec {
+    const double *part;
+    int nbat, stride, nch_first, nch_last;
+};
+void launch_data_term(Ctx &c, const DsumSpec *dsum = nullptr);   // -> c.scal[1] (and [0]), no synchronisation
 double device_data_term(Ctx &c);                 // S = -sum f(M) + sum f(dout) + sum f(din)
 double model_term(long long W, int V, int B, int variant);
 

@@ -29,7 +29,7 @@ __global__ void __launch_bounds__(256) k_mdl_partials(const int *__restrict__ cn
                                                       const int *__restrict__ dout, const int *__restrict__ din,
                                                       int B, const double2 *__restrict__ ft,
                                                       double *__restrict__ partials, unsigned *__restrict__ arrivals,
-                                                      double *__restrict__ out) {
+                                                      double *__restrict__ out, DsumSpec ds, double *__restrict__ dsum) {
     __shared__ double sh[8];
     __shared__ bool last;
     const int nnz = *d_nnz;
@@ -65,18 +65,40 @@ __global__ void __launch_bounds__(256) k_mdl_partials(const int *__restrict__ cn
         *out = t;
         *arrivals = 0u;
     }
+    if (ds.nbat == 0) return;
+    // the iteration's dS sum: per batch the ordered pass of k_apply_sum over
+    // its chunk partials (256 strided lanes, warp trees, 8 warp sums), added to
+    // the running sum batch after batch -- the same operations in the same order
+    double run = 0.0;
+    for (int k = 0; k < ds.nbat; ++k) {
+        const int n = k + 1 < ds.nbat ? ds.nch_first : ds.nch_last;
+        double v2 = 0.0;
+        for (int i = threadIdx.x; i < n; i += 256) v2 += ds.part[(size_t)k * ds.stride + i];
+        v2 = warp_sum(v2);
+        __syncthreads();
+        if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = v2;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double t = 0.0;
+            for (int w = 0; w < 8; ++w) t += sh[w];
+            run += t;
+        }
+    }
+    if (threadIdx.x == 0) *dsum = run;
 }
 
 // launches the reduction into c.scal[1] (no synchronisation)
-void launch_data_term(Ctx &c) {
+void launch_data_term(Ctx &c, const DsumSpec *dsum) {
     cudaEvent_t ev = nullptr;
     kc_begin(c, c.k_mdl, &ev);
     // the extent of the cnt array: nnz <= E, or B^2 for the padded dense lines
     long long n = std::max<long long>(std::max<long long>(c.E, c.B), 1);
     if (c.dense_padded) n = std::max(n, (long long)c.B * c.B);
     const int nb = (int)((n + MDL_CHUNK - 1) / MDL_CHUNK);
+    const DsumSpec none{nullptr, 0, 0, 0, 0};
     k_mdl_partials<<<nb, 256, 0, c.stream>>>(c.bm_cnt, c.d_nnz, c.dout, c.din, c.B, c.ft, c.partials,
-                                             reinterpret_cast<unsigned *>(c.scal_i + 5), c.scal + 1);
+                                             reinterpret_cast<unsigned *>(c.scal_i + 5), c.scal + 1,
+                                             dsum ? *dsum : none, c.scal);
     c.launches += 1;
     GSAP_CHECK_LAUNCH();
     kc_end(c, c.k_mdl, ev, 0.0);

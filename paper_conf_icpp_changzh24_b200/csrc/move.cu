@@ -1604,6 +1604,17 @@ void launch_apply(Ctx &c, int first, int count, const int *s, const unsigned cha
     launch_nb_update(c, count);
 }
 
+void launch_apply_deferred(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
+                           double *part, int *nacc, unsigned long long *n_eval) {
+    if (count <= 0) return;
+    const int nb = (count + APPLY_CHUNK - 1) / APPLY_CHUNK;
+    const MoveLog lg = move_log(c);
+    k_apply<<<nb, APPLY_CHUNK, 0, c.stream>>>(first, count, s, acc, dS, c.b, part, nacc, n_eval, lg);
+    c.launches += 1;
+    GSAP_CHECK_LAUNCH();
+    launch_nb_update(c, count);
+}
+
 // sharded batches: the fixed-chunk sums of accepted dS over [first, first+count)
 // (first aligned to APPLY_CHUNK from the batch start) into partials[0, ...)
 void launch_partials(Ctx &c, int first, int count, const int *s, const unsigned char *acc, const double *dS,
