@@ -70,6 +70,30 @@ __global__ void __launch_bounds__(256) k_mdl_partials(const int *__restrict__ cn
     // its chunk partials (256 strided lanes, warp trees, 8 warp sums), added to
     // the running sum batch after batch -- the same operations in the same order
     double run = 0.0;
+    if (ds.nch_first <= 32 && ds.nch_last <= 32 && ds.nbat <= 8) {
+        // <= 32 partials per batch: only warp 0's tree is non-zero (the other
+        // seven warp sums are +0.0), so warp k computes batch k's tree at once
+        const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+        __syncthreads();
+        if (w < ds.nbat) {
+            const int n = w + 1 < ds.nbat ? ds.nch_first : ds.nch_last;
+            double v2 = 0.0;
+            if (lane < n) v2 += ds.part[(size_t)w * ds.stride + lane];
+            v2 = warp_sum(v2);
+            if (lane == 0) sh[w] = v2;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            for (int k = 0; k < ds.nbat; ++k) {
+                double t = 0.0;
+                t += sh[k];
+                for (int q = 1; q < 8; ++q) t += 0.0;
+                run += t;
+            }
+            *dsum = run;
+        }
+        return;
+    }
     for (int k = 0; k < ds.nbat; ++k) {
         const int n = k + 1 < ds.nbat ? ds.nch_first : ds.nch_last;
         double v2 = 0.0;
