@@ -30,7 +30,12 @@ constexpr int WARP_TAB_LOG2 = 8;
 constexpr int BIG_THR = 128;           // warp path iff min(k_v, B) <= BIG_THR
 constexpr int MOVE_WARPS = 8;          // warps per CTA, warp kernel
 constexpr int CTA_THREADS = 256;       // big-vertex role: one CTA per vertex
-constexpr int MID_TAB = 512;           // mid role: 64-thread group tables (<= 256 keys)
+constexpr int MID_TAB = 512;           // mid role: group tables (<= 256 keys)
+#ifndef GSAP_MID_G
+#define GSAP_MID_G 64
+#endif
+constexpr int MID_G = GSAP_MID_G;      // threads per mid-vertex group (64: four per CTA, 128: two)
+constexpr int MID_PER_CTA = MOVE_WARPS * 32 / MID_G;
 constexpr int MID_TAB_LOG2 = 9;
 constexpr int CTA_SMEM_SLOTS = MOVE_WARPS * WARP_TAB;   // big-vertex shared table (<= 1024 keys)
 constexpr size_t MOVE_SMEM = sizeof(int4) * MOVE_WARPS * WARP_TAB + sizeof(int) * MOVE_WARPS * (WARP_TAB / 2);
@@ -1062,14 +1067,15 @@ __global__ void __launch_bounds__(MOVE_WARPS * 32, GSAP_GROUPS_MINB) k_move_grou
     __shared__ int4 tabs[CTA_SMEM_SLOTS];
     __shared__ double sh[3 * MOVE_WARPS + 8];   // group sums + the broadcast proposal
     if ((int)blockIdx.x < a.nmid_ctas) {
-        // four 64-thread groups per CTA, one mid vertex each
-        const int gid = threadIdx.x >> 6, gt = threadIdx.x & 63;
+        // MID_PER_CTA groups of MID_G threads per CTA, one mid vertex each
+        const int gid = threadIdx.x / MID_G, gt = threadIdx.x % MID_G;
         int4 *tab = tabs + gid * MID_TAB;
-        for (int li = blockIdx.x * 4 + gid; li < a.mlist_count; li += a.nmid_ctas * 4) {
-            tab_clear<64>(tab, MID_TAB, gt);
-            gsync<64>();
-            do_vertex<64, WEIGHTED>(a, a.mlist[li], tab, MID_TAB_LOG2, nullptr, sh + gid * 8);
-            gsync<64>();
+        for (int li = blockIdx.x * MID_PER_CTA + gid; li < a.mlist_count; li += a.nmid_ctas * MID_PER_CTA) {
+            tab_clear<MID_G>(tab, MID_TAB, gt);
+            gsync<MID_G>();
+            do_vertex<MID_G, WEIGHTED>(a, a.mlist[li], tab, MID_TAB_LOG2, nullptr,
+                                       sh + gid * ((3 * MOVE_WARPS + 8) / MID_PER_CTA));
+            gsync<MID_G>();
         }
         return;
     }
@@ -1271,7 +1277,7 @@ void launch_move(Ctx &c, MoveMode mode, uint32_t outer, uint32_t itr, int first,
         if (nmid > 0) {
             a.mlist = c.mid + omid;
             a.mlist_count = nmid;
-            a.nmid_ctas = std::min((nmid + 3) / 4, c.test_grid > 0 ? c.test_grid : 148 * 16);
+            a.nmid_ctas = std::min((nmid + MID_PER_CTA - 1) / MID_PER_CTA, c.test_grid > 0 ? c.test_grid : 148 * 16);
         }
         const int ohuge = range(c.h_huge, nhuge, khuge);
         if (nbig > 0) {
