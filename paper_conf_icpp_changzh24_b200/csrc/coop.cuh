@@ -46,6 +46,11 @@ struct CoopArgs {
     int *d_nnz;
     int *nlong;       // [3] long lines per side, short-line work counter
     unsigned *bar;    // [2] barrier: arrivals, generation
+    // the neighbour-block cache update of the MOVE batch before this rebuild
+    // (k_nb_update's work, done in P1 -- before the scatter reads the cache):
+    // moved == nullptr: none pending
+    const int *moved, *moved_cnt, *movedb, *rowptr, *cscptr, *csc2csr, *csr2csc;
+    int *nbo, *nbi;
 };
 
 GSAP_DEV void grid_sync(unsigned *bar) {
@@ -166,6 +171,15 @@ __global__ void __launch_bounds__(256) k_rebuild_coop(CoopArgs a) {
         const int ko = __ldg(a.kout + v), ki = __ldg(a.kin + v);
         if (ko) atomicAdd(a.sd[0].deg + x, ko);
         if (ki) atomicAdd(a.sd[1].deg + x, ki);
+    }
+    if (a.moved) {   // the pending cache update, one warp per moved vertex (as k_nb_update)
+        const int n = *a.moved_cnt;
+        for (int k = gwarp; k < n; k += gwarps) {
+            const int v = a.moved[k], x = a.movedb[k];
+            const int q1 = __ldg(a.cscptr + v + 1), p1 = __ldg(a.rowptr + v + 1);
+            for (int q = __ldg(a.cscptr + v) + lane; q < q1; q += 32) a.nbo[__ldg(a.csc2csr + q)] = x;
+            for (int p = __ldg(a.rowptr + v) + lane; p < p1; p += 32) a.nbi[__ldg(a.csr2csc + p)] = x;
+        }
     }
     grid_sync(a.bar);
     COOP_MARK(2)

@@ -73,6 +73,10 @@ struct Ctx {
     // rebuild (which does not read the cache); every reader or writer of nbo / nbi
     // joins it first (nb_join)
     bool nb_pending = false;
+    // sparse regime with the persistent rebuild: the update after an apply is
+    // deferred into that rebuild's first phase (nb_flush launches it on its own
+    // if anything else needs the cache first)
+    bool nb_deferred = false;
     cudaEvent_t ev_nb = nullptr, ev_apply = nullptr;
 
     // blockmodel (capacity: nnz <= min(E, B^2); B <= V)
@@ -228,7 +232,8 @@ void role_end(Ctx &c, KClass &k, cudaEvent_t e0, cudaStream_t st);
 void build_graph_device(Ctx &c);                 // CSC, esrc, degrees (create time)
 void nb_refresh(Ctx &c);                         // the neighbour-block cache from b (if stale)
 inline void b_changed(Ctx &c) { c.nb_stale = true; }   // every bulk write of b outside the apply
-void nb_join(Ctx &c);                            // the main stream waits for a pending cache update
+void nb_join(Ctx &c, bool flush = true);         // the main stream waits for a pending cache update
+void nb_flush(Ctx &c);                           // a deferred cache update launched now (then joined)
 void rebuild(Ctx &c);                            // Alg. 2 from c.b, c.B
 bool dense_ok(const Ctx &c, int B);
 // padded-CSR export: line x's [ptr[x], end[x]) of src to dst[off[x] ..) on the device

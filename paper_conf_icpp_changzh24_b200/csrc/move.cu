@@ -1556,7 +1556,20 @@ __global__ void __launch_bounds__(256) k_nb_update(const int *__restrict__ moved
     }
 }
 
-void nb_join(Ctx &c) {
+static void launch_nb_update(Ctx &c, int count);
+
+void nb_flush(Ctx &c) {
+    if (!c.nb_deferred) return;
+    c.nb_deferred = false;
+    const int g = 148 * 8;
+    k_nb_update<<<g, 256, 0, c.stream>>>(c.moved, c.moved_cnt, c.movedb, c.rowptr, c.cscptr, c.csc2csr, c.csr2csc,
+                                         c.nbo, c.nbi);
+    ++c.launches;
+    GSAP_CHECK_LAUNCH();
+}
+
+void nb_join(Ctx &c, bool flush) {
+    if (flush) nb_flush(c);
     if (!c.nb_pending) return;
     GSAP_CUDA(cudaStreamWaitEvent(c.stream, c.ev_nb, 0));
     c.nb_pending = false;
@@ -1568,8 +1581,13 @@ void nb_join(Ctx &c) {
 static void launch_nb_update(Ctx &c, int count) {
     if (!c.nbo || c.nb_stale) return;   // a stale cache is refreshed in full by the next rebuild
     static const bool in_order = getenv("GSAP_NB_INORDER") != nullptr;   // A/B switch
+    static const bool no_defer = getenv("GSAP_NB_NODEFER") != nullptr;   // A/B switch
     const bool side = !in_order && c.dense_mode && dense_ok(c, c.B) && c.nranks == 1;
     nb_join(c);
+    if (!no_defer && !dense_ok(c, c.B) && c.coop_ok && c.E > 0) {
+        c.nb_deferred = true;   // done by the persistent sparse rebuild's first phase
+        return;
+    }
     cudaStream_t st = c.stream;
     if (side) {
         GSAP_CUDA(cudaEventRecord(c.ev_apply, c.stream));

@@ -102,6 +102,7 @@ __global__ void k_nb_refresh(int E, const int *__restrict__ col, const int *__re
 
 void nb_refresh(Ctx &c) {
     if (!c.nb_stale) return;
+    c.nb_deferred = false;   // the full refresh covers the deferred update
     nb_join(c);
     if (c.E > 0) {
         const int g = (int)std::min<long long>(((long long)c.E + 255) / 256, 148LL * 16);
@@ -880,6 +881,13 @@ static void rebuild_sparse_coop(Ctx &c) {
     a.d_nnz = c.d_nnz;
     a.nlong = c.seg_ctr;
     a.bar = c.coop_bar;
+    a.moved = nullptr;
+    if (c.nb_deferred) {   // the MOVE batch's cache update, in P1
+        c.nb_deferred = false;
+        a.moved = c.moved; a.moved_cnt = c.moved_cnt; a.movedb = c.movedb;
+        a.rowptr = c.rowptr; a.cscptr = c.cscptr; a.csc2csr = c.csc2csr; a.csr2csc = c.csr2csc;
+        a.nbo = c.nbo; a.nbi = c.nbi;
+    }
     const size_t smem = sizeof(CoopSmem<K>);
     const int grid = per_device((const void *)k_rebuild_coop<K>, [&] {
         GSAP_CUDA(cudaFuncSetAttribute(k_rebuild_coop<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -905,8 +913,10 @@ static void rebuild_sparse_coop(Ctx &c) {
 }
 
 static void rebuild_sparse(Ctx &c) {
-    nb_join(c);   // the scatters read the neighbour-block cache
     const int B = c.B, E = c.E;
+    // the scatters read the neighbour-block cache: a side-stream update is
+    // joined; a deferred one is done by the persistent kernel's first phase
+    nb_join(c, !(E > 0 && c.coop_ok));
     if (E > 0 && c.coop_ok) {
         if (c.weighted) rebuild_sparse_coop<u64>(c);
         else rebuild_sparse_coop<unsigned>(c);
