@@ -240,15 +240,16 @@ static void *arena_take(int dev, size_t need, size_t *got) {
 }
 
 static void arena_give(void *p, size_t bytes, int dev) {
-    void *drop = p;
+    void *drop = nullptr;
     {
         std::lock_guard<std::mutex> g(g_arena_mu);
-        if (!g_arena_cache.p || g_arena_cache.dev != dev || g_arena_cache.bytes < bytes) {
-            drop = g_arena_cache.p;   // keep the larger / newer one
-            g_arena_cache.p = p;
-            g_arena_cache.bytes = bytes;
-            g_arena_cache.dev = dev;
-        }
+        // keep the newest: the next create is most likely the same workload (keeping
+        // the larger one made every later create of a smaller graph pay a
+        // cudaMalloc + cudaFree -- e.g. the bench's 20K e2e calls after its 2M states)
+        drop = g_arena_cache.p;
+        g_arena_cache.p = p;
+        g_arena_cache.bytes = bytes;
+        g_arena_cache.dev = dev;
     }
     if (drop) cudaFree(drop);
 }
