@@ -714,28 +714,29 @@ GSAP_DEV void splitw_bucket(const Line (&L)[N], const int (&sp)[N][K], const int
 }
 
 // M entry of key y[k] in bucket [p[k], p[k] + n[k]) of line k: binary
-// search down to <= 8 entries, then up to 8 independent id loads; the count
-// only on a hit
-template <int N>
+// search down to <= W entries, then up to W independent id loads; the count
+// only on a hit (W = 8 for 128 splitters per line, 4 for 256: the bucket of a
+// line of <= 1024 entries never needs the search)
+template <int N, int W = 8>
 GSAP_DEV void bucket_get(const Line (&L)[N], const int (&y)[N], int (&p)[N], int (&n)[N], int (&out)[N]) {
 #pragma unroll
     for (int k = 0; k < N; ++k) {
-        while (n[k] > 8) {
+        while (n[k] > W) {
             const int h = n[k] >> 1;
             p[k] = __ldg(L[k].idx + p[k] + h) <= y[k] ? p[k] + h : p[k];
             n[k] -= h;
         }
     }
-    int id[N][8];
+    int id[N][W];
 #pragma unroll
     for (int k = 0; k < N; ++k)
 #pragma unroll
-        for (int q = 0; q < 8; ++q) id[k][q] = q < n[k] ? __ldg(L[k].idx + p[k] + q) : -1;
+        for (int q = 0; q < W; ++q) id[k][q] = q < n[k] ? __ldg(L[k].idx + p[k] + q) : -1;
 #pragma unroll
     for (int k = 0; k < N; ++k) {
         int hit = -1;
 #pragma unroll
-        for (int q = 0; q < 8; ++q) hit = id[k][q] == y[k] ? q : hit;
+        for (int q = 0; q < W; ++q) hit = id[k][q] == y[k] ? q : hit;
         out[k] = hit >= 0 ? __ldg(L[k].cnt + p[k] + hit) : 0;
     }
 }
@@ -744,6 +745,7 @@ GSAP_DEV void bucket_get(const Line (&L)[N], const int (&y)[N], int (&p)[N], int
 #define GSAP_HALF_K 4
 #endif
 constexpr int HALF_K = GSAP_HALF_K;   // splitters per lane in the sorted two-pass kernels
+constexpr int HALF_W = HALF_K >= 8 ? 4 : 8;   // bucket scan width (bucket_get)
 
 template <bool WEIGHTED, int PASS>
 GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
@@ -825,7 +827,7 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
         const int yc[3] = {r, s, s};
         int pc[3], nc[3], oc[3];
         splitw_bucket<3, HALF_K>(Lc, spc, yc, pc, nc);
-        bucket_get<3>(Lc, yc, pc, nc, oc);
+        bucket_get<3, HALF_W>(Lc, yc, pc, nc, oc);
         Mrr = oc[0];
         Mrs = oc[1];
         Msr = oc[2];
@@ -837,7 +839,7 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
         const int yc[1] = {s};
         int pc[1], nc[1], oc[1];
         splitw_bucket<1, HALF_K>(Lc, spc, yc, pc, nc);
-        bucket_get<1>(Lc, yc, pc, nc, oc);
+        bucket_get<1, HALF_W>(Lc, yc, pc, nc, oc);
         Mss = oc[0];
     }
     const int Mrr2 = Mrr - o_r - i_r - l, Mrs2 = Mrs + i_r - o_s, Msr2 = Msr + o_r - i_s;
@@ -866,7 +868,7 @@ GSAP_DEV void move_vertex_half(const MoveArgs &a, int i, int4 *tab, int *list) {
             int o2[2];
             {
                 const int yt[2] = {t, t};
-                bucket_get<2>(Ln, yt, pb2, nb2, o2);
+                bucket_get<2, HALF_W>(Ln, yt, pb2, nb2, o2);
             }
             const double rt = __ldg(rcp + t);
             if (PASS == 1) {   // o2 = {M_rt, M_tr}
